@@ -1,0 +1,214 @@
+"""fp64 CPU oracle for the KDE range-selectivity hot path (Heimel, Kiefer, Markl, SIGMOD 2015).
+
+TEST INFRASTRUCTURE ONLY.  Only ``tests/``, ``__graft_entry__.smoke()`` and the
+``cpu_baseline`` / ``--impl reference`` legs of ``bench.py`` may import this
+package.  The product package ``paper_conf_sigmod_heimelkm15_b200`` never
+imports it and shares no code with it.
+
+The arithmetic lives in ``kde_oracle.c`` (plain C, fp64, libm ``erf``); this
+module only marshals numpy arrays through ctypes.  Every function names the
+PAPER.md passage it follows; see the C file for the readings R1-R6.
+
+Parity status:
+  point_mass / contributions / estimate      pinned (tests/test_oracle_pins.py)
+  estimate_grad / loss_and_grad              pinned (finite differences, mpmath)
+  loss                                       pinned (finite differences, kinks)
+  scott                                      pinned (numpy population std)
+  empty_region_threshold                     pinned (eq. 19 centre point, boundary max)
+  karma_update                               pinned (brute-force leave-one-out)
+  online_apply (Listing 1 reconstruction)    PARITY UNPINNED (listing missing from PAPER.md)
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "kde_oracle.c")
+_LIB_PATH = os.path.join(_HERE, "liboracle.so")
+
+LOSS_SQUARED, LOSS_ABSOLUTE, LOSS_RELATIVE, LOSS_SQUARED_RELATIVE, LOSS_SQUARED_Q = range(5)
+
+
+def build(force: bool = False) -> str:
+    """Compile kde_oracle.c into liboracle.so (gcc, -O2, OpenMP, strict IEEE)."""
+    if force or not os.path.exists(_LIB_PATH) or os.path.getmtime(_LIB_PATH) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-o", _LIB_PATH, _SRC, "-lm"])
+    return _LIB_PATH
+
+
+_lib = None
+
+
+def _L():
+    global _lib
+    if _lib is None:
+        _lib = ctypes.CDLL(build())
+        P = ctypes.c_void_p
+        i64, i32, f64 = ctypes.c_int64, ctypes.c_int32, ctypes.c_double
+        sig = {
+            "oracle_point_mass": (f64, [P, i32, P, P, P]),
+            "oracle_contributions": (None, [P, i64, i32, P, P, P, P]),
+            "oracle_estimate": (None, [P, i64, i32, P, P, P, i64, P]),
+            "oracle_estimate_grad": (None, [P, i64, i32, P, P, P, i64, P, P]),
+            "oracle_loss": (None, [i32, f64, f64, f64, P, P]),
+            "oracle_loss_and_grad": (None, [P, i64, i32, P, P, P, P, i64, i32, f64, i32, P, P, P]),
+            "oracle_scott": (None, [P, i64, i32, P]),
+            "oracle_empty_region_threshold": (f64, [i32, P, P, P, P]),
+            "oracle_karma_update": (i64, [P, i64, f64, f64, i32, f64, f64, f64, f64, P, P, i64]),
+            "oracle_online_accumulate": (None, [i32, P, P]),
+            "oracle_online_apply": (None, [i32, i32, f64, f64, f64, f64, f64, i32, P, P, P, P, P]),
+        }
+        for name, (res, args) in sig.items():
+            fn = getattr(_lib, name)
+            fn.restype = res
+            fn.argtypes = args
+    return _lib
+
+
+def _f32(a):
+    return np.ascontiguousarray(a, dtype=np.float32)
+
+
+def _f64(a):
+    return np.ascontiguousarray(a, dtype=np.float64)
+
+
+def _p(a):
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+def set_threads(n: int) -> None:
+    """Set the OpenMP thread count used by estimate/estimate_grad (0 = default)."""
+    os.environ["OMP_NUM_THREADS"] = str(n)
+    try:
+        libgomp = ctypes.CDLL("libgomp.so.1")
+        libgomp.omp_set_num_threads(ctypes.c_int(n))
+    except OSError:
+        pass
+
+
+def point_mass(t, h, lo, hi) -> float:
+    """eq. (13): one point's mass in the box [lo, hi]."""
+    t, lo, hi, h = _f32(t), _f32(lo), _f32(hi), _f64(h)
+    return _L().oracle_point_mass(_p(t), len(h), _p(h), _p(lo), _p(hi))
+
+
+def contributions(sample, h, lo, hi) -> np.ndarray:
+    """eq. (13) for every sample point of one query (the retained buffer)."""
+    sample, h, lo, hi = _f32(sample), _f64(h), _f32(lo).ravel(), _f32(hi).ravel()
+    n, d = sample.shape
+    out = np.empty(n, dtype=np.float64)
+    _L().oracle_contributions(_p(sample), n, d, _p(h), _p(lo), _p(hi), _p(out))
+    return out
+
+
+def estimate(sample, h, lo, hi) -> np.ndarray:
+    """eq. (2): p_hat for each of the q boxes lo/hi [q, d]."""
+    sample, h = _f32(sample), _f64(h)
+    lo, hi = _f32(np.atleast_2d(lo)), _f32(np.atleast_2d(hi))
+    n, d = sample.shape
+    q = lo.shape[0]
+    out = np.empty(q, dtype=np.float64)
+    _L().oracle_estimate(_p(sample), n, d, _p(h), _p(lo), _p(hi), q, _p(out))
+    return out
+
+
+def estimate_grad(sample, h, lo, hi):
+    """eq. (2) and eq. (17): (p_hat[q], dp_hat/dh[q, d])."""
+    sample, h = _f32(sample), _f64(h)
+    lo, hi = _f32(np.atleast_2d(lo)), _f32(np.atleast_2d(hi))
+    n, d = sample.shape
+    q = lo.shape[0]
+    est = np.empty(q, dtype=np.float64)
+    g = np.empty((q, d), dtype=np.float64)
+    _L().oracle_estimate_grad(_p(sample), n, d, _p(h), _p(lo), _p(hi), q, _p(est), _p(g))
+    return est, g
+
+
+def loss(kind: int, lam: float, phat: float, p: float):
+    """Appendix C.1: (L(p_hat, p), dL/dp_hat)."""
+    L = ctypes.c_double()
+    dL = ctypes.c_double()
+    _L().oracle_loss(kind, lam, phat, p, ctypes.byref(L), ctypes.byref(dL))
+    return L.value, dL.value
+
+
+def loss_and_grad(sample, h, lo, hi, true_sel, kind: int, lam: float, log_bw: bool):
+    """eq. (5), (14), (18): (loss, grad[d], est[q])."""
+    sample, h = _f32(sample), _f64(h)
+    lo, hi = _f32(np.atleast_2d(lo)), _f32(np.atleast_2d(hi))
+    ts = _f64(true_sel)
+    n, d = sample.shape
+    q = lo.shape[0]
+    lo_ = ctypes.c_double()
+    g = np.empty(d, dtype=np.float64)
+    est = np.empty(q, dtype=np.float64)
+    _L().oracle_loss_and_grad(_p(sample), n, d, _p(h), _p(lo), _p(hi), _p(ts), q, kind, lam,
+                              int(bool(log_bw)), ctypes.byref(lo_), _p(g), _p(est))
+    return lo_.value, g, est
+
+
+def scott(sample) -> np.ndarray:
+    """eq. (3), P:L129 with population sigma."""
+    sample = _f32(sample)
+    n, d = sample.shape
+    h = np.empty(d, dtype=np.float64)
+    _L().oracle_scott(_p(sample), n, d, _p(h))
+    return h
+
+
+def empty_region_threshold(h, lo, hi):
+    """eq. (19)-(20): (thr_20, p_max); thr = +inf when disabled."""
+    h, lo, hi = _f64(h), _f32(lo).ravel(), _f32(hi).ravel()
+    pmax = ctypes.c_double()
+    thr = _L().oracle_empty_region_threshold(len(h), _p(h), _p(lo), _p(hi), ctypes.byref(pmax))
+    return thr, pmax.value
+
+
+def karma_update(c, phat, p, kind, lam, k_max, tau, thr20, karma):
+    """eq. (6)-(8) and the flag rule of P:L250.  Updates ``karma`` in place
+    (fp64 array) and returns the ascending array of flagged indices."""
+    c = _f64(c)
+    n = c.shape[0]
+    assert karma.dtype == np.float64 and karma.flags.c_contiguous and karma.shape == (n,)
+    idx = np.empty(n, dtype=np.int64)
+    nf = _L().oracle_karma_update(_p(c), n, phat, p, kind, lam, k_max, tau, thr20, _p(karma), _p(idx), n)
+    return idx[:nf].copy()
+
+
+class OnlineState:
+    """Listing 1 state (reconstructed; PARITY UNPINNED): acc, ms, lr, gprev, count."""
+
+    def __init__(self, d: int, lr0: float = 0.1):
+        self.acc = np.zeros(d)
+        self.ms = np.zeros(d)
+        self.lr = np.full(d, float(lr0))
+        self.gprev = np.zeros(d)
+        self.count = 0
+
+    def copy(self):
+        s = OnlineState(len(self.acc))
+        s.acc, s.ms, s.lr, s.gprev, s.count = self.acc.copy(), self.ms.copy(), self.lr.copy(), self.gprev.copy(), self.count
+        return s
+
+
+def online_step(state: OnlineState, h: np.ndarray, grad, batch=10, alpha=0.9, lr_min=1e-6,
+                lr_max=50.0, lr_inc=1.2, lr_dec=0.5, log_bw=True) -> bool:
+    """Listing 1: add one query's loss gradient to the
+    mini-batch; when ``batch`` gradients are collected, update ``h`` in place.
+    Returns True when ``h`` changed."""
+    g = _f64(grad)
+    d = len(h)
+    assert h.dtype == np.float64 and h.flags.c_contiguous
+    _L().oracle_online_accumulate(d, _p(g), _p(state.acc))
+    state.count += 1
+    if state.count < batch:
+        return False
+    _L().oracle_online_apply(d, batch, alpha, lr_min, lr_max, lr_inc, lr_dec, int(bool(log_bw)),
+                             _p(h), _p(state.acc), _p(state.ms), _p(state.lr), _p(state.gprev))
+    state.count = 0
+    return True

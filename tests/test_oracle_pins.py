@@ -1,0 +1,349 @@
+"""Pins the fp64 oracle to things other than itself (CPU only, ``-m "not gpu"``).
+
+Each test names the PAPER.md passage ("P:L<n>") and what fixes the expected
+value: an independent mpmath quadrature fixture, a closed form, an invariant,
+a limit, finite differences, or brute force.  A plausible slip in the oracle
+(dropped 1/2^d, wrong sign on the l-term of eq. 17, swapped u/l, sample- vs
+population sigma, wrong leave-one-out denominator, ...) fails at least one.
+"""
+import json
+import math
+import os
+
+import mpmath as mp
+import numpy as np
+import pytest
+
+import oracle
+
+GOLD = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "micro_example.json")))
+INF = np.float32(np.inf)
+
+
+def _micro():
+    S = np.array(GOLD["sample"], np.float32)
+    h = np.array(GOLD["h"], np.float64)
+    lo = np.array([GOLD["lo"]], np.float32)
+    hi = np.array([GOLD["hi"]], np.float32)
+    return S, h, lo, hi
+
+
+def _close(a, b, rel=1e-13, abs_=1e-15):
+    a = np.asarray(a, np.float64)
+    b = np.asarray([float(x) for x in np.atleast_1d(b)], np.float64)
+    assert np.all(np.abs(a - b) <= abs_ + rel * np.abs(b)), (a, b)
+
+
+# --- golden micro example (independent 50-digit quadrature) -----------------
+
+def test_micro_contributions_and_estimate():
+    """eq. (13) vs quadrature of eq. (12); eq. (2)."""
+    S, h, lo, hi = _micro()
+    _close(oracle.contributions(S, h, lo[0], hi[0]), GOLD["contributions"])
+    _close(oracle.estimate(S, h, lo, hi), [GOLD["estimate"]])
+
+
+def test_micro_gradient_and_loss():
+    """eq. (17), eq. (18), eq. (14) + C.1 L2."""
+    S, h, lo, hi = _micro()
+    est, g = oracle.estimate_grad(S, h, lo, hi)
+    _close(g[0], GOLD["dpdh"], rel=1e-12)
+    L, gL, e2 = oracle.loss_and_grad(S, h, lo, hi, [GOLD["true_sel"]], oracle.LOSS_SQUARED, 0.0, False)
+    _close([L], [GOLD["l2_loss"]])
+    _close(gL, GOLD["l2_grad"], rel=1e-12)
+    _, gl, _ = oracle.loss_and_grad(S, h, lo, hi, [GOLD["true_sel"]], oracle.LOSS_SQUARED, 0.0, True)
+    _close(gl, [float(GOLD["l2_grad"][j]) * h[j] for j in range(2)], rel=1e-12)
+    _close(g[0] * h, GOLD["dpdlnh"], rel=1e-12)
+
+
+def test_micro_karma_and_threshold():
+    """eq. (6)-(7) and eq. (19)-(20) vs quadrature."""
+    S, h, lo, hi = _micro()
+    c = oracle.contributions(S, h, lo[0], hi[0])
+    est = oracle.estimate(S, h, lo, hi)[0]
+    karma = np.zeros(3)
+    oracle.karma_update(c, est, GOLD["true_sel"], oracle.LOSS_ABSOLUTE, 0.0, 4.0, -1e9, np.inf, karma)
+    _close(karma, GOLD["karma_delta_l1"], rel=1e-12)
+    thr, pmax = oracle.empty_region_threshold(h, lo[0], hi[0])
+    _close([pmax], [GOLD["p_max"]])
+    _close([thr], [GOLD["thr20"]])
+
+
+def test_micro_scott():
+    """eq. (3) with population sigma."""
+    S, _, _, _ = _micro()
+    _close(oracle.scott(S), GOLD["scott_h"])
+
+
+# --- closed forms and limits -------------------------------------------------
+
+@pytest.mark.parametrize("t,h,l,u", [(0.3, 0.7, -1.0, 2.0), (5.0, 0.1, 4.8, 5.05), (-2.0, 3.0, 1.0, 9.0),
+                                     (0.0, 1.0, -np.inf, 0.5), (1.0, 2.0, 0.0, np.inf)])
+def test_d1_closed_form_vs_mpmath_ncdf(t, h, l, u):
+    """d = 1, N = 1: eq. (13) is Phi((u-t)/h) - Phi((l-t)/h)."""
+    mp.mp.dps = 40
+    ref = mp.ncdf((mp.mpf(float(np.float32(u))) - mp.mpf(float(np.float32(t)))) / h) - \
+        mp.ncdf((mp.mpf(float(np.float32(l))) - mp.mpf(float(np.float32(t)))) / h)
+    got = oracle.point_mass(np.array([t], np.float32), [h], np.array([l], np.float32), np.array([u], np.float32))
+    assert abs(got - float(ref)) <= 2e-16 + 1e-14 * abs(float(ref))
+
+
+def test_unbounded_query_is_exactly_one():
+    """erf(+-inf) = +-1 makes every factor of eq. (13) exactly 1; eq. (17) is exactly 0."""
+    rng = np.random.default_rng(1)
+    S = rng.normal(size=(200, 4)).astype(np.float32)
+    h = rng.uniform(0.1, 2, 4)
+    lo = np.full((1, 4), -INF, np.float32)
+    hi = np.full((1, 4), INF, np.float32)
+    est, g = oracle.estimate_grad(S, h, lo, hi)
+    assert est[0] == 1.0
+    assert np.all(g == 0.0)
+
+
+def test_product_factorisation_and_marginalisation():
+    """Product kernel: with all other dims unbounded, the d-dim estimate
+    equals the 1-D estimate on column j; for N = 1 the mass is the product of 1-D masses."""
+    rng = np.random.default_rng(2)
+    S = rng.normal(size=(64, 3)).astype(np.float32)
+    h = np.array([0.3, 0.8, 1.7])
+    lo = np.array([-0.4, 0.1, -2.0], np.float32)
+    hi = np.array([0.9, 1.1, 0.5], np.float32)
+    for j in range(3):
+        l2 = np.full(3, -INF, np.float32)
+        u2 = np.full(3, INF, np.float32)
+        l2[j], u2[j] = lo[j], hi[j]
+        a = oracle.estimate(S, h, l2[None], u2[None])[0]
+        b = oracle.estimate(S[:, j:j + 1], h[j:j + 1], lo[None, j:j + 1], hi[None, j:j + 1])[0]
+        assert a == pytest.approx(b, rel=1e-15, abs=1e-16)
+    t = S[0]
+    prod = np.prod([oracle.point_mass(t[j:j + 1], h[j:j + 1], lo[j:j + 1], hi[j:j + 1]) for j in range(3)])
+    assert oracle.point_mass(t, h, lo, hi) == pytest.approx(prod, rel=1e-14)
+
+
+def test_additivity_along_a_dimension():
+    """The box integral eq. (12) is additive: [l,c] + [c,u] = [l,u] on any axis."""
+    rng = np.random.default_rng(3)
+    S = rng.normal(size=(128, 3)).astype(np.float32)
+    h = np.array([0.5, 0.25, 1.5])
+    lo = np.array([-1.0, -0.5, -2.0], np.float32)
+    hi = np.array([1.0, 0.75, 0.25], np.float32)
+    for j in range(3):
+        c = np.float32(0.125)
+        hi1 = hi.copy(); hi1[j] = c
+        lo2 = lo.copy(); lo2[j] = c
+        a = oracle.estimate(S, h, lo[None], hi1[None])[0] + oracle.estimate(S, h, lo2[None], hi[None])[0]
+        b = oracle.estimate(S, h, lo[None], hi[None])[0]
+        assert a == pytest.approx(b, rel=1e-13, abs=1e-16)
+
+
+def test_lower_equals_upper_gives_zero():
+    """An empty interval has zero mass (eq. 12 integral over (l, l))."""
+    S = np.array([[0.0, 1.0], [2.0, -1.0]], np.float32)
+    est = oracle.estimate(S, [1.0, 1.0], np.array([[0.5, -3]], np.float32), np.array([[0.5, 3]], np.float32))
+    assert est[0] == 0.0
+
+
+def test_invariances():
+    """Translation of (t, l, u), joint scaling of (t, l, u, h) by 2 (exact in fp32),
+    and reflection t -> -t, (l, u) -> (-u, -l) leave eq. (13) unchanged."""
+    rng = np.random.default_rng(4)
+    # values on a 2^-10 grid so that adding 8 and scaling by 2 are exact in fp32
+    S = (np.round(rng.normal(size=(100, 2)) * 1024) / 1024).astype(np.float32)
+    h = np.array([0.4, 0.9])
+    lo = np.array([[-0.5, -1.0]], np.float32)
+    hi = np.array([[0.75, 0.5]], np.float32)
+    base = oracle.estimate(S, h, lo, hi)[0]
+    shift = np.float32(8.0)
+    assert oracle.estimate(S + shift, h, lo + shift, hi + shift)[0] == pytest.approx(base, rel=1e-12)
+    assert oracle.estimate(S * 2, h * 2, lo * 2, hi * 2)[0] == pytest.approx(base, rel=1e-14)
+    assert oracle.estimate(-S, h, -hi, -lo)[0] == pytest.approx(base, rel=1e-14)
+
+
+def test_small_bandwidth_limit_is_exact_count():
+    """h -> 0 degrades to counting: with every point >= 10h from every
+    face, each erf is exactly +-1 in fp64, so p_hat == count/N exactly."""
+    rng = np.random.default_rng(5)
+    S = rng.integers(-50, 50, size=(500, 3)).astype(np.float32)
+    h = np.full(3, 0.01)
+    lo = np.array([[-20.5, -10.5, -30.5]], np.float32)
+    hi = np.array([[15.5, 30.5, 5.5]], np.float32)
+    inside = np.all((S > lo) & (S < hi), axis=1).sum()
+    assert oracle.estimate(S, h, lo, hi)[0] == inside / 500.0
+
+
+# --- gradient: finite differences ---------------------------------------------
+
+@pytest.mark.parametrize("log_bw", [False, True])
+def test_gradient_matches_central_differences(log_bw):
+    """eq. (17) and eq. (18) vs central FD of eq. (2)+(13)."""
+    rng = np.random.default_rng(6)
+    S = rng.normal(size=(50, 3)).astype(np.float32)
+    h = np.array([0.3, 0.6, 1.1])
+    lo = np.array([[-0.5, -1.0, -np.inf]], np.float32)
+    hi = np.array([[0.8, 0.4, 0.9]], np.float32)
+    est, g = oracle.estimate_grad(S, h, lo, hi)
+    for j in range(3):
+        if log_bw:
+            dl = 1e-6
+            hp, hm = h.copy(), h.copy()
+            hp[j] = h[j] * math.exp(dl); hm[j] = h[j] * math.exp(-dl)
+            fd = (oracle.estimate(S, hp, lo, hi)[0] - oracle.estimate(S, hm, lo, hi)[0]) / (2 * dl)
+            ana = g[0, j] * h[j]
+        else:
+            dh = 1e-6 * h[j]
+            hp, hm = h.copy(), h.copy()
+            hp[j] += dh; hm[j] -= dh
+            fd = (oracle.estimate(S, hp, lo, hi)[0] - oracle.estimate(S, hm, lo, hi)[0]) / (2 * dh)
+            ana = g[0, j]
+        assert ana == pytest.approx(fd, rel=1e-7, abs=1e-12)
+
+
+@pytest.mark.parametrize("kind", range(5))
+def test_loss_derivatives_match_finite_differences(kind):
+    """C.1 derivatives vs central FD of the listed loss, away from kinks."""
+    lam = 1e-3
+    for phat, p in [(0.3, 0.1), (0.05, 0.2), (0.6, 0.61)]:
+        L, dL = oracle.loss(kind, lam, phat, p)
+        e = 1e-7
+        fd = (oracle.loss(kind, lam, phat + e, p)[0] - oracle.loss(kind, lam, phat - e, p)[0]) / (2 * e)
+        assert dL == pytest.approx(fd, rel=1e-6)
+
+
+def test_loss_values_and_kinks():
+    """C.1 values and the printed 0 derivative at equality for L1/relative."""
+    lam = 0.01
+    assert oracle.loss(0, lam, 0.3, 0.1)[0] == pytest.approx(0.04)
+    assert oracle.loss(1, lam, 0.3, 0.1)[0] == pytest.approx(0.2)
+    assert oracle.loss(2, lam, 0.3, 0.1)[0] == pytest.approx(0.2 / 0.11)
+    assert oracle.loss(3, lam, 0.3, 0.1)[0] == pytest.approx((0.2 / 0.11) ** 2)
+    assert oracle.loss(4, lam, 0.3, 0.1)[0] == pytest.approx((math.log(0.31) - math.log(0.11)) ** 2)
+    assert oracle.loss(1, lam, 0.2, 0.2)[1] == 0.0
+    assert oracle.loss(2, lam, 0.2, 0.2)[1] == 0.0
+    assert oracle.loss(1, lam, 0.1, 0.2)[1] == -1.0
+    assert oracle.loss(2, lam, 0.3, 0.2)[1] == pytest.approx(1 / 0.21)
+
+
+def test_loss_and_grad_averages_over_queries():
+    """eq. (5): loss and gradient are means over the q training queries."""
+    rng = np.random.default_rng(7)
+    S = rng.normal(size=(40, 2)).astype(np.float32)
+    h = np.array([0.5, 0.7])
+    lo = np.array([[-1, -1], [0, -0.5], [-2, 0.2]], np.float32)
+    hi = np.array([[0.5, 1], [1, 0.5], [0, 2]], np.float32)
+    p = np.array([0.2, 0.1, 0.3])
+    L, g, est = oracle.loss_and_grad(S, h, lo, hi, p, 0, 0.0, False)
+    Ls, gs = [], []
+    for k in range(3):
+        l1, g1, _ = oracle.loss_and_grad(S, h, lo[k:k + 1], hi[k:k + 1], p[k:k + 1], 0, 0.0, False)
+        Ls.append(l1); gs.append(g1)
+    assert L == pytest.approx(np.mean(Ls), rel=1e-14)
+    assert np.allclose(g, np.mean(gs, axis=0), rtol=1e-13)
+
+
+# --- Scott ----------------------------------------------------------------------
+
+def test_scott_matches_numpy_population_std():
+    """eq. (3), population sigma == numpy std(ddof=0)."""
+    rng = np.random.default_rng(8)
+    S = (rng.normal(size=(1000, 5)) * [1, 2, 3, 0.5, 10] + 1e3).astype(np.float32)
+    ref = 1000 ** (-1 / 9) * S.astype(np.float64).std(axis=0, ddof=0)
+    assert np.allclose(oracle.scott(S), ref, rtol=1e-12)
+
+
+# --- karma ------------------------------------------------------------------------
+
+def test_leave_one_out_matches_brute_force():
+    """eq. (6) equals re-estimating on S \\ {t_i}."""
+    rng = np.random.default_rng(9)
+    S = rng.normal(size=(12, 2)).astype(np.float32)
+    h = np.array([0.4, 0.6])
+    lo = np.array([-0.5, -0.2], np.float32)
+    hi = np.array([0.7, 1.0], np.float32)
+    c = oracle.contributions(S, h, lo, hi)
+    est = oracle.estimate(S, h, lo[None], hi[None])[0]
+    p = 0.3
+    karma = np.zeros(12)
+    oracle.karma_update(c, est, p, oracle.LOSS_SQUARED, 0.0, 1e9, -1e9, np.inf, karma)
+    for i in range(12):
+        loo = oracle.estimate(np.delete(S, i, axis=0), h, lo[None], hi[None])[0]
+        assert karma[i] == pytest.approx((loo - p) ** 2 - (est - p) ** 2, rel=1e-9, abs=1e-15)
+
+
+def test_karma_saturation_and_threshold_by_hand():
+    """eq. (8) min(K + dK, K_max) and the strict threshold of P:L204/L250, N = 4."""
+    c = np.array([0.9, 0.1, 0.0, 0.5])
+    n = 4
+    phat = c.mean()
+    p = 0.2
+    # L1: L(p_hat) = |0.375 - 0.2| = 0.175; p^-(i) = (1.5 - c_i)/3
+    loo = (phat * n - c) / (n - 1)
+    dK = np.abs(loo - p) - abs(phat - p)
+    karma = np.array([3.99, 0.0, -0.05, 0.0])
+    k_max, tau = 4.0, -0.02
+    idx = oracle.karma_update(c, phat, p, oracle.LOSS_ABSOLUTE, 0.0, k_max, tau, np.inf, karma)
+    expect = np.minimum(np.array([3.99, 0.0, -0.05, 0.0]) + dK, k_max)
+    assert np.allclose(karma, expect, rtol=0, atol=1e-15)
+    assert list(idx) == [i for i in range(4) if expect[i] < tau]
+    assert karma[0] <= k_max
+
+
+def test_empty_region_rule_flags_only_inside_points():
+    """P:L250 + eq. (20): with true selectivity 0 a point is flagged when its
+    contribution reaches thr_20; such points are always inside the box."""
+    rng = np.random.default_rng(10)
+    for trial in range(30):
+        d = rng.integers(1, 5)
+        h = rng.uniform(0.05, 1.0, d)
+        lo = rng.uniform(-1, 0, d).astype(np.float32)
+        hi = (lo + rng.uniform(0.05, 2.0, d)).astype(np.float32)
+        S = rng.uniform(-2, 2, size=(4000, d)).astype(np.float32)
+        c = oracle.contributions(S, h, lo, hi)
+        thr, pmax = oracle.empty_region_threshold(h, lo, hi)
+        karma = np.zeros(len(S))
+        idx = oracle.karma_update(c, c.mean(), 0.0, oracle.LOSS_ABSOLUTE, 0.0, 4.0, -1e300, thr, karma)
+        inside = np.all((S >= lo) & (S <= hi), axis=1)
+        assert inside[idx].all()
+        assert c.max() <= pmax * (1 + 1e-12)
+
+
+def test_eq19_centre_and_eq20_boundary_points():
+    """eq. (19): the box centre attains p_max; eq. (20): the threshold is the
+    largest mass among the centre moved to a face along one dimension."""
+    h = np.array([0.3, 1.2, 0.7])
+    lo = np.array([-1.0, 0.0, 2.0], np.float32)
+    hi = np.array([0.5, 3.0, 2.5], np.float32)
+    centre = ((lo.astype(np.float64) + hi) / 2).astype(np.float32)
+    thr, pmax = oracle.empty_region_threshold(h, lo, hi)
+    assert oracle.point_mass(centre, h, lo, hi) == pytest.approx(pmax, rel=1e-14)
+    faces = []
+    for j in range(3):
+        t = centre.copy(); t[j] = lo[j]
+        faces.append(oracle.point_mass(t, h, lo, hi))
+    assert thr == pytest.approx(max(faces), rel=1e-13)
+    # zero width disables the shortcut
+    thr0, _ = oracle.empty_region_threshold(h, lo, lo)
+    assert thr0 == np.inf
+
+
+# --- Listing 1 (reconstruction, PARITY UNPINNED): sanity property only -----------
+
+def test_online_update_reduces_training_loss():
+    """Sanity property for the reconstructed Listing 1: on a static
+    workload, SGD with the RMSprop-style step lowers the L2 loss from Scott's h."""
+    rng = np.random.default_rng(11)
+    R = np.concatenate([rng.normal(0, 0.3, (3000, 2)), rng.normal(3, 0.5, (3000, 2))]).astype(np.float32)
+    S = R[rng.choice(len(R), 256, replace=False)]
+    h = oracle.scott(S)
+    c = R[rng.choice(len(R), 200)]
+    w = rng.uniform(0.2, 1.0, (200, 2))
+    lo = (c - w / 2).astype(np.float32)
+    hi = (c + w / 2).astype(np.float32)
+    p = np.array([np.all((R >= lo[k]) & (R <= hi[k]), axis=1).mean() for k in range(200)])
+    L0, _, _ = oracle.loss_and_grad(S, h, lo, hi, p, 0, 0.0, True)
+    st = oracle.OnlineState(2, lr0=0.1)
+    for epoch in range(3):
+        for k in range(200):
+            _, g, _ = oracle.loss_and_grad(S, h, lo[k:k + 1], hi[k:k + 1], p[k:k + 1], 0, 0.0, True)
+            oracle.online_step(st, h, g, log_bw=True)
+    L1, _, _ = oracle.loss_and_grad(S, h, lo, hi, p, 0, 0.0, True)
+    assert L1 < L0
