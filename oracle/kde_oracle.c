@@ -24,6 +24,9 @@
  *   R4 karma threshold compare is strict (<), after the update
  *   R5 eq. 20 is applied only when the true selectivity == 0 and
  *      every box width is > 0 (a zero width makes eq. 19 vanish)
+ *   R7 squared-relative loss: the printed derivative lacks the
+ *      square of (lambda + p); the true derivative of the printed loss
+ *      is used (pinned by finite differences)
  *   R6 Listing 1 (adaptive bandwidth) is missing from the text; the
  *      update is reconstructed from the prose P:L179-183, L561.
  *      PARITY UNPINNED by the paper (no listing, no trace).
@@ -138,7 +141,9 @@ void oracle_loss(int32_t kind, double lambda, double phat, double p,
     case 1: *L = fabs(phat - p);                       *dL = sgn3(phat, p); break;
     case 2: *L = fabs(phat - p) / (lambda + p);        *dL = sgn3(phat, p) / (lambda + p); break;
     case 3: *L = ((phat - p) / (lambda + p)) * ((phat - p) / (lambda + p));
-            *dL = 2.0 * (phat - p) / (lambda + p); break;
+            /* R7: P:L520 prints 2(p_hat-p)/(lambda+p), which is not the derivative of the
+             * loss printed on the same line; the derivative of that loss is used. */
+            *dL = 2.0 * (phat - p) / ((lambda + p) * (lambda + p)); break;
     default: {
             double r = log(lambda + phat) - log(lambda + p);
             *L = r * r;
