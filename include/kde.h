@@ -1,0 +1,244 @@
+/*
+ * kde.h -- C ABI of the B200-native KDE range-selectivity hot path.
+ *
+ * Method: Heimel, Kiefer, Markl, "Self-Tuning, GPU-Accelerated Kernel Density
+ * Models for Multidimensional Selectivity Estimation", SIGMOD 2015.
+ * Citations "P:L<n>" are line numbers of the paper text.
+ *
+ * A model owns a d-dimensional fp32 data sample S = {t^(1..s)} resident in
+ * device memory (structure-of-arrays columns), a diagonal Gaussian bandwidth
+ * H = diag(h_1..h_d), per-point cumulative karma K_i (eq. 8) and the
+ * retained per-point contributions of the last single-query scan.
+ *
+ * Conventions for every entry point
+ *  - Return value: KDE_OK or an error code; nothing throws across the ABI.
+ *    kde_last_error() returns a thread-local message for the last failure.
+ *  - Validation happens before any device work, so KDE_EINVAL leaves the
+ *    model unchanged.  A CUDA / NCCL failure after launch poisons the model:
+ *    every later call returns KDE_ESTATE (only kde_destroy is valid).
+ *  - Host pointers: the library copies inputs during the call; outputs go to
+ *    caller-allocated buffers; the caller keeps ownership of everything.
+ *    Host-pointer calls are synchronous (they return after results landed).
+ *  - "_dev" variants take DEVICE pointers (on the model's device) and a CUDA
+ *    stream (cudaStream_t passed as void*, NULL = the model's own stream);
+ *    they only enqueue work: results are valid once that stream reaches the
+ *    end of the enqueued work.  Device buffers must stay alive until then.
+ *  - Box queries are hyper-rectangles Omega = (l_1,u_1) x ... x (l_d,u_d)
+ *    over real-valued attributes, passed as row-major fp32 arrays
+ *    lo[q][d], hi[q][d].  lo <= hi is required (lo == hi gives 0);
+ *    +-infinity is allowed (half-open / unbounded boxes); NaN is rejected.
+ *  - Sharded models (one process per GPU): every rank calls every function
+ *    collectively with identical query arguments; point indices are GLOBAL.
+ *  - A model is externally synchronised (one thread at a time).
+ */
+#ifndef KDE_H
+#define KDE_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define KDE_ABI_VERSION 1
+#define KDE_MAX_DIM 16          /* d in [1, KDE_MAX_DIM] */
+#define KDE_NCCL_ID_BYTES 128   /* sizeof(ncclUniqueId) */
+
+typedef struct kde_model kde_model;
+
+typedef enum {
+    KDE_OK = 0,
+    KDE_EINVAL = 1,   /* invalid argument; model unchanged                    */
+    KDE_ENOMEM = 2,   /* device or pinned host allocation failed              */
+    KDE_ECUDA = 3,    /* CUDA runtime error (model poisoned)                  */
+    KDE_ENCCL = 4,    /* NCCL error (model poisoned)                          */
+    KDE_ESTATE = 5,   /* model poisoned by an earlier failure, or bad state   */
+    KDE_ETRUNC = 6    /* output truncated (more results than capacity)        */
+} kde_status;
+
+/* Loss functions of Appendix C.1, argument order L(p_hat, p).
+ * lambda is the smoothing constant of footnote 6; it must be > 0 for
+ * RELATIVE, SQUARED_RELATIVE and SQUARED_Q.  SQUARED_RELATIVE uses the true
+ * derivative of the printed loss, 2(p_hat-p)/(lambda+p)^2 (R7). */
+typedef enum {
+    KDE_LOSS_SQUARED = 0,
+    KDE_LOSS_ABSOLUTE = 1,
+    KDE_LOSS_RELATIVE = 2,
+    KDE_LOSS_SQUARED_RELATIVE = 3,
+    KDE_LOSS_SQUARED_Q = 4
+} kde_loss;
+
+/* Karma-based sample maintenance, Section 4.2 and P:L250.
+ *   loss, lambda : the loss L of eq. (7)
+ *   k_max        : saturation constant of eq. (8); the paper uses 4
+ *   k_init       : karma given to a (re)placed point (reading R8: 0)
+ *   threshold    : a point is flagged when K_i < threshold after the update
+ *                  ("a given threshold"; no value in the paper)
+ *   empty_region : 1 = also flag points with p^(i) >= thr_20 when the true
+ *                  selectivity is exactly 0 (eq. 20, Appendix E)   */
+typedef struct {
+    int32_t loss;
+    int32_t empty_region;
+    double lambda;
+    double k_max;
+    double k_init;
+    double threshold;
+} kde_karma_params;
+
+/* Adaptive bandwidth (Section 4.1; Listing 1 reconstructed, see
+ * DESIGN.md R6).  Defaults: minibatch 10, alpha 0.9,
+ * lr_min 1e-6, lr_max 50, lr_inc 1.2, lr_dec 0.5.  lr0 is unspecified in the
+ * paper (reading: 0.1).  log_bandwidth selects eq. (18) updates. */
+typedef struct {
+    int32_t minibatch;
+    int32_t log_bandwidth;
+    int32_t loss;
+    int32_t _pad;
+    double lambda;
+    double alpha;
+    double lr_min;
+    double lr_max;
+    double lr_inc;
+    double lr_dec;
+    double lr0;
+} kde_online_params;
+
+/* ---------------------------------------------------------------- misc */
+int32_t     kde_abi_version(void);
+const char *kde_last_error(void);                 /* thread-local, never NULL */
+const char *kde_status_string(kde_status s);
+
+/* ---------------------------------------------------------------- model */
+/* kde_create -- build a model on the current CUDA device.
+ *   sample : host, row-major n x d fp32 (copied).  Finite values only.
+ *   n      : number of sample points s, n >= 2 (eq. 6 divides by s-1).
+ *   d      : dimensionality, 1 <= d <= KDE_MAX_DIM.
+ *   h      : host, d bandwidths, each finite in [1e-30, 1e30]; or NULL for
+ *            Scott's rule, eq. (3) with population sigma,
+ *            computed on the device in fp64.
+ *   out    : receives the model handle (set only on KDE_OK).
+ * Errors: KDE_EINVAL (arguments, non-finite sample), KDE_ENOMEM, KDE_ECUDA. */
+kde_status kde_create(const float *sample, int64_t n, int32_t d, const double *h, kde_model **out);
+
+/* kde_create_sharded -- collective over `world` processes, one GPU each.
+ * This rank holds global rows [row_offset, row_offset + n_local) of a sample
+ * of n_global rows.  nccl_id: KDE_NCCL_ID_BYTES bytes from
+ * kde_get_unique_id() on rank 0, broadcast by the caller.  h == NULL runs
+ * Scott's rule over the GLOBAL sample (per-rank moments merged in rank order).
+ * world == 1 is valid and equivalent to kde_create.
+ * Errors: as kde_create, plus KDE_ENCCL. */
+kde_status kde_create_sharded(const float *local_rows, int64_t n_local, int64_t row_offset,
+                              int64_t n_global, int32_t d, const double *h,
+                              const void *nccl_id, int32_t rank, int32_t world, kde_model **out);
+
+/* kde_get_unique_id -- writes an ncclUniqueId (KDE_NCCL_ID_BYTES bytes). */
+kde_status kde_get_unique_id(void *nccl_id_out);
+
+/* kde_destroy -- frees all device and host resources; NULL is a no-op. */
+void kde_destroy(kde_model *m);
+
+/* kde_get_info -- any output pointer may be NULL. */
+kde_status kde_get_info(const kde_model *m, int64_t *n_local, int64_t *n_global, int32_t *d,
+                        int32_t *rank, int32_t *world);
+
+/* kde_get_bandwidth / kde_set_bandwidth -- host fp64 h[d].  set validates
+ * every h_j finite in [1e-30, 1e30]; it invalidates retained contributions. */
+kde_status kde_get_bandwidth(kde_model *m, double *h);
+kde_status kde_set_bandwidth(kde_model *m, const double *h);
+
+/* kde_set_retain -- on != 0: single-query scans (q == 1) also store the
+ * per-point contributions p^(i) (fp32, 4 B/point) for a following
+ * kde_karma_update on the same box ("we do not discard the temporary
+ * buffer").  Default off. */
+kde_status kde_set_retain(kde_model *m, int32_t on);
+
+/* ---------------------------------------------------------------- hot path */
+/* kde_estimate_batch -- selectivity estimates for q boxes, eq. (2)+(13):
+ *   est[k]        = p_hat_H(Omega_k) = (1/s) sum_i prod_j [Phi((u_kj - t_ij)/h_j) - Phi((l_kj - t_ij)/h_j)]
+ *   dest_dh[k*d+j] = d p_hat(Omega_k) / d h_j, eq. (17); NULL = skip.
+ * lo, hi: host row-major q x d fp32.  est: host q fp64.  dest_dh: host q*d fp64.
+ * q == 0 is a no-op.  Per-point arithmetic is fp32, all sums fp64,
+ * deterministic (fixed reduction order for a given device and world size). */
+kde_status kde_estimate_batch(kde_model *m, const float *lo, const float *hi, int64_t q,
+                              double *est, double *dest_dh);
+kde_status kde_estimate_batch_dev(kde_model *m, const float *d_lo, const float *d_hi, int64_t q,
+                                  double *d_est, double *d_dest_dh, void *stream);
+
+/* kde_loss_and_grad -- batch objective of eq. (5) and its gradient (eq. 14):
+ *   loss    = (1/q) sum_k L(p_hat_k, p_k)
+ *   grad[j] = (1/q) sum_k L'(p_hat_k, p_k) * d p_hat_k / d h_j
+ *             (times h_j when log_bandwidth != 0, eq. 18)
+ * true_sel: host q fp64 in [0, 1].  loss_out: 1 fp64.  grad_out: d fp64.
+ * est_out: q fp64 or NULL.  q >= 1.
+ * Errors: KDE_EINVAL (bounds, true_sel, loss kind, lambda <= 0 where needed). */
+kde_status kde_loss_and_grad(kde_model *m, const float *lo, const float *hi, const double *true_sel,
+                             int64_t q, int32_t loss, double lambda, int32_t log_bandwidth,
+                             double *loss_out, double *grad_out, double *est_out);
+kde_status kde_loss_and_grad_dev(kde_model *m, const float *d_lo, const float *d_hi,
+                                 const double *d_true_sel, int64_t q, int32_t loss, double lambda,
+                                 int32_t log_bandwidth, double *d_loss, double *d_grad, double *d_est,
+                                 void *stream);
+
+/* kde_karma_update -- one query's feedback (true selectivity p) for sample
+ * maintenance: for every point, eq. (6) leave-one-out estimate,
+ * eq. (7) karma delta, eq. (8) saturating update of K_i, then flag K_i <
+ * threshold, or (empty_region && p == 0 && p^(i) >= thr_20 of eq. 20).
+ * Reuses the retained contributions when the previous single-query scan was
+ * on the same box with unchanged h and sample; otherwise rescans (same
+ * result).  idx_out receives the ascending GLOBAL indices of flagged points
+ * (at most idx_cap of them); *n_flagged = total flagged.  Returns
+ * KDE_ETRUNC (karma still updated) when total > idx_cap.  lo/hi: host d fp32. */
+kde_status kde_karma_update(kde_model *m, const float *lo, const float *hi, double true_sel,
+                            const kde_karma_params *kp, int64_t *idx_out, int64_t idx_cap,
+                            int64_t *n_flagged);
+
+/* kde_online_update -- adaptive bandwidth step (Section 4.1, Fig. 3 steps
+ * 5-8): L'(p_hat, p) * d p_hat/d h (x h in log mode) is added to the
+ * mini-batch; when `minibatch` gradients are collected the RMSprop/Rprop step
+ * of Listing 1 (reconstructed, R6) updates h ON THE DEVICE.  Uses
+ * the retained estimate+gradient of a preceding kde_estimate_batch(q == 1,
+ * dest_dh != NULL) on the same box, else rescans.  *updated = 1 when h
+ * changed (may be NULL).  lo/hi: host d fp32. */
+kde_status kde_online_update(kde_model *m, const float *lo, const float *hi, double true_sel,
+                             const kde_online_params *op, int32_t *updated);
+
+/* kde_replace_points -- write k rows (host row-major k x d fp32) to the GLOBAL
+ * indices idx[k] (unique, in [0, n_global)), reset their karma to k_init
+ * (P:L248 reservoir inserts, P:L250 karma replacement).  Invalidates retained
+ * contributions.  Errors: KDE_EINVAL on duplicates, range, non-finite rows. */
+kde_status kde_replace_points(kde_model *m, const int64_t *idx, const float *rows, int64_t k,
+                              double k_init);
+
+/* ---------------------------------------------------------------- inspection */
+kde_status kde_get_karma(kde_model *m, double *karma);   /* local n fp64          */
+kde_status kde_set_karma(kde_model *m, const double *karma); /* local n fp64      */
+kde_status kde_get_sample(kde_model *m, float *rows);    /* local n x d row-major */
+/* last retained per-point contributions (local n fp32); KDE_ESTATE if none. */
+kde_status kde_get_contributions(kde_model *m, float *c);
+/* online (Listing 1) state, each d fp64 (any may be NULL), and batch count. */
+kde_status kde_get_online_state(kde_model *m, double *acc, double *ms, double *lr, double *gprev,
+                                int32_t *count);
+kde_status kde_set_online_state(kde_model *m, const double *acc, const double *ms, const double *lr,
+                                const double *gprev, int32_t count);
+/* wait for all work enqueued on the model's stream. */
+kde_status kde_synchronize(kde_model *m);
+
+/* kde_set_profiling -- on != 0: record CUDA events around every scan kernel
+ * launch (on the stream it is launched on) and count every kernel launch.
+ * Resets the counters.  kde_get_profile synchronises the device and returns
+ * the summed scan-kernel time (ms), the number of scan launches and of all
+ * kernel launches since the last reset, then resets them. */
+kde_status kde_set_profiling(kde_model *m, int32_t on);
+kde_status kde_get_profile(kde_model *m, double *scan_ms, int64_t *scan_launches, int64_t *launches);
+
+/* ---------------------------------------------------------------- harness */
+/* kde_count_in_box_dev -- NOT part of the estimator: the exact feedback the
+ * DBMS would return.  counts[k] = |{ r : l_kj < R_rj < u_kj  for all j }|
+ * over a device row-major R[n][d] fp32.  All pointers are device pointers. */
+kde_status kde_count_in_box_dev(const float *d_rows, int64_t n, int32_t d, const float *d_lo,
+                                const float *d_hi, int64_t q, int64_t *d_counts, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* KDE_H */

@@ -54,6 +54,7 @@ def _L():
             "oracle_contributions": (None, [P, i64, i32, P, P, P, P]),
             "oracle_estimate": (None, [P, i64, i32, P, P, P, i64, P]),
             "oracle_estimate_grad": (None, [P, i64, i32, P, P, P, i64, P, P]),
+            "oracle_grad_abs_scale": (None, [P, i64, i32, P, P, P, i64, P]),
             "oracle_loss": (None, [i32, f64, f64, f64, P, P]),
             "oracle_loss_and_grad": (None, [P, i64, i32, P, P, P, P, i64, i32, f64, i32, P, P, P]),
             "oracle_scott": (None, [P, i64, i32, P]),
@@ -127,6 +128,18 @@ def estimate_grad(sample, h, lo, hi):
     g = np.empty((q, d), dtype=np.float64)
     _L().oracle_estimate_grad(_p(sample), n, d, _p(h), _p(lo), _p(hi), q, _p(est), _p(g))
     return est, g
+
+
+def grad_abs_scale(sample, h, lo, hi):
+    """Tolerance scale for gradient parity: eq. (17) with per-point terms in
+    absolute value, [q, d] (test infrastructure, not a paper quantity)."""
+    sample, h = _f32(sample), _f64(h)
+    lo, hi = _f32(np.atleast_2d(lo)), _f32(np.atleast_2d(hi))
+    n, d = sample.shape
+    q = lo.shape[0]
+    g = np.empty((q, d), dtype=np.float64)
+    _L().oracle_grad_abs_scale(_p(sample), n, d, _p(h), _p(lo), _p(hi), q, _p(g))
+    return g
 
 
 def loss(kind: int, lam: float, phat: float, p: float):

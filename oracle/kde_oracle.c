@@ -126,6 +126,38 @@ void oracle_estimate_grad(const float *sample, int64_t n, int32_t d, const doubl
     }
 }
 
+/* Gradient magnitude scale used by the parity tolerance (test infrastructure):
+ *   m_ij = sqrt2 / (sqrtpi h_i^2 2^d s) * sum_j | [bracket of eq. 17] * prod_{k != i} [...] |
+ * i.e. eq. (17) with every per-point term taken in absolute value. */
+void oracle_grad_abs_scale(const float *sample, int64_t n, int32_t d, const double *h,
+                           const float *lo, const float *hi, int64_t q, double *mabs)
+{
+    #pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t qq = 0; qq < q; ++qq) {
+        const float *l = lo + qq * d, *u = hi + qq * d;
+        double gsum[64];
+        for (int32_t i = 0; i < d; ++i) gsum[i] = 0.0;
+        for (int64_t j = 0; j < n; ++j) {
+            const float *t = sample + j * d;
+            for (int32_t i = 0; i < d; ++i) {
+                double li = (double)l[i] - (double)t[i];
+                double ui = (double)u[i] - (double)t[i];
+                double bracket = xexp(li, h[i]) - xexp(ui, h[i]);
+                double prod = 1.0;
+                for (int32_t k = 0; k < d; ++k) {
+                    if (k == i) continue;
+                    prod *= erf(((double)u[k] - (double)t[k]) / (OR_SQRT2 * h[k]))
+                          - erf(((double)l[k] - (double)t[k]) / (OR_SQRT2 * h[k]));
+                }
+                gsum[i] += fabs(bracket * prod);
+            }
+        }
+        for (int32_t i = 0; i < d; ++i)
+            mabs[qq * d + i] = OR_SQRT2 / (OR_SQRTPI * h[i] * h[i] * pow(2.0, (double)d) * (double)n)
+                               * gsum[i];
+    }
+}
+
 /* ---------------------------------------------------------------------
  * Appendix C.1: loss L(p_hat, p) and dL/dp_hat.
  * kind: 0 quadratic, 1 absolute, 2 relative, 3 squared relative, 4 squared Q.

@@ -1,0 +1,83 @@
+// common.cuh -- internal types shared by the KDE kernels and the C-ABI runtime.
+// Citations "P:L<n>" refer to lines of the paper text.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#ifndef KDE_MAX_DIM
+#define KDE_MAX_DIM 16
+#endif
+
+namespace kde {
+
+constexpr int kMaxDim = KDE_MAX_DIM;
+constexpr int kColAlign = 1024;  // columns padded to a multiple of this many points
+
+// Per-dimension constants derived from the fp64 bandwidth h (device resident
+// so that an on-device bandwidth update needs no host round trip).
+//   ap[j]     = sqrt(log2 e) / (sqrt(2) h_j)      y' = (b - t) * ap[j] = z_j sqrt(log2 e),
+//                                                  z = (b - t)/(sqrt2 h) is the erf argument of eq. (13)
+//   gconst[j] = 1 / (sqrt(pi) sqrt(log2 e) h_j)   so that d p^(i)/d h_j = gconst[j] * w_j * prod_{k!=j} D_k,
+//                                                  w_j = y'_l E_l - y'_u E_u (eq. 17 rewritten in z)
+struct DevConsts {
+  double h[kMaxDim];
+  double gconst[kMaxDim];
+  float ap[kMaxDim];
+};
+
+// Listing 1 state (reconstruction, R6), device resident.
+struct OnlineState {
+  double acc[kMaxDim];
+  double ms[kMaxDim];
+  double lr[kMaxDim];
+  double gprev[kMaxDim];
+  int32_t count;
+  int32_t updated;  // 1 when the last kde_online_update changed h
+};
+
+struct OnlineParamsDev {
+  int32_t minibatch, log_bw, loss;
+  double lambda, alpha, lr_min, lr_max, lr_inc, lr_dec;
+};
+
+struct KarmaParamsDev {
+  int32_t loss, empty_region;
+  double lambda, k_max, threshold;
+};
+
+// scan over the sample for ONE box (q == 1): HBM-streaming reduction.
+struct ScanSingleArgs {
+  const float* cols;      // [d][ld] fp32 SoA sample
+  int64_t ld;             // padded column length (multiple of kColAlign)
+  int64_t n;              // valid points in this shard
+  const float* lo;        // device, d floats
+  const float* hi;        // device, d floats
+  const DevConsts* consts;
+  float* c_out;           // nullable: retained p^(i) (fp32) per point
+  double* block_partials; // [gridDim.x][1+d]
+  unsigned* counter;      // zero on entry; the last block resets it to zero
+  double* sums_out;       // [1+d] raw sums S_0 = sum_i p^(i), S_j = sum_i w_j prod_{k!=j} D_k
+  double* fin_out;        // nullable: [1+d] finalised (p_hat, dp_hat/dh_j) for world == 1
+  double n_global;        // s (results are divided by s, so s ones give exactly 1)
+};
+
+// scan for many boxes: sample tiles staged in shared memory by TMA bulk
+// copies, each thread keeps QT boxes in registers.
+struct ScanBatchedArgs {
+  const float* cols;
+  int64_t ld, n;
+  const float* lo;        // device [q][d]
+  const float* hi;        // device [q][d]
+  int64_t q;
+  const DevConsts* consts;
+  int64_t split_len;      // points per split (multiple of the tile size)
+  double* partials;       // [splits][1+d][q]
+};
+
+// host-side launchers (scan_inst_*.cu)
+cudaError_t launch_scan_single(int d, bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s);
+cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int num_sms, int* splits_out,
+                                cudaStream_t s, bool dry_run);
+int scan_single_grid(int d, int64_t n, int num_sms);
+
+}  // namespace kde

@@ -1,0 +1,980 @@
+// kde_api.cu -- the C ABI (include/kde.h) and the kde_model runtime:
+// device buffers, stream, argument validation, dispatch between the
+// single-box streaming scan and the tiled batched scan, NCCL combine of
+// per-shard partial sums, retained state for feedback, error handling.
+//
+// Every numeric step runs in the kernels of scan.cuh / kernels.cu; this file
+// only moves arguments, validates them and orders launches on one stream.
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include "../../include/kde.h"
+#include "common.cuh"
+#include "kernels.cuh"
+
+using namespace kde;
+
+// ------------------------------------------------------------------ errors
+static thread_local char g_err[512] = "";
+
+static kde_status fail(kde_status st, const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof(g_err), fmt, ap);
+  va_end(ap);
+  return st;
+}
+
+struct kde_model {
+  int device = 0;
+  int num_sms = 148;
+  cudaStream_t stream = nullptr;
+  int32_t d = 0;
+  int64_t n = 0;         // local points
+  int64_t n_global = 0;  // s
+  int64_t row_offset = 0;
+  int64_t ld = 0;        // padded column length
+  int rank = 0, world = 1;
+  ncclComm_t comm = nullptr;
+  bool poisoned = false;
+
+  float* cols = nullptr;       // [d][ld]
+  double* karma = nullptr;     // [n]
+  float* cret = nullptr;       // [ld] retained contributions
+  DevConsts* consts = nullptr;
+  OnlineState* online = nullptr;
+
+  // scratch
+  double* block_partials = nullptr;  // single-scan block partials
+  unsigned* counter = nullptr;
+  double* ret = nullptr;             // [1 + d] retained (p_hat, dp/dh)
+  double* single_sums = nullptr;     // [1 + d]
+  float* qbuf = nullptr;             // device bounds staging [2][qcap][d]
+  int64_t qcap = 0;
+  double* obuf = nullptr;            // device outputs: est [qcap], dpdh [qcap*d], sums [qcap*(1+d)], true [qcap], loss, grad
+  int64_t ocap = 0;
+  double* partials = nullptr;
+  size_t partials_cap = 0;           // bytes
+  double* gather = nullptr;          // [world][q][1+d]
+  size_t gather_cap = 0;
+  uint32_t* bitmap = nullptr;
+  int32_t* block_counts = nullptr;
+  int64_t* offsets = nullptr;
+  int64_t* idx_dev = nullptr;
+  int64_t idx_cap = 0;
+  int32_t* bad = nullptr;            // device flag
+  void* pinned = nullptr;            // pinned host staging
+  size_t pinned_cap = 0;
+
+  // retained single-box state
+  bool retain = false;
+  bool ret_valid = false, ret_has_c = false, ret_has_grad = false;
+  float ret_lo[kMaxDim], ret_hi[kMaxDim];
+  uint64_t gen = 1;      // bumped whenever h or the sample changes
+  uint64_t ret_gen = 0;
+  bool online_init = false;
+
+  // profiling (kde_set_profiling): CUDA events around every scan launch on its
+  // own stream, and a count of every kernel this model launched
+  bool prof = false;
+  std::vector<cudaEvent_t> ev;  // pairs (start, end)
+  size_t ev_used = 0;
+  int64_t scan_launches = 0;
+  int64_t launches = 0;
+};
+
+#define CU(call)                                                                                     \
+  do {                                                                                               \
+    cudaError_t e_ = (call);                                                                         \
+    if (e_ != cudaSuccess) {                                                                         \
+      if (m) m->poisoned = true;                                                                     \
+      return fail(KDE_ECUDA, "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    }                                                                                                \
+  } while (0)
+
+#define CUL(call)   \
+  do {              \
+    ++m->launches;  \
+    CU(call);       \
+  } while (0)
+
+#define NC(call)                                                                                     \
+  do {                                                                                               \
+    ncclResult_t r_ = (call);                                                                        \
+    if (r_ != ncclSuccess) {                                                                         \
+      if (m) m->poisoned = true;                                                                     \
+      return fail(KDE_ENCCL, "%s failed: %s", #call, ncclGetErrorString(r_));                       \
+    }                                                                                                \
+  } while (0)
+
+#define CHECK_MODEL(m)                                                                     \
+  do {                                                                                     \
+    if (!(m)) return fail(KDE_EINVAL, "model is NULL");                                   \
+    if ((m)->poisoned) return fail(KDE_ESTATE, "model poisoned by an earlier CUDA/NCCL error"); \
+  } while (0)
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) == cudaSuccess && prev != dev) cudaSetDevice(dev);
+    else prev = -1;
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+static bool h_ok(double h) { return std::isfinite(h) && h >= 1e-30 && h <= 1e30; }
+
+static kde_status validate_bounds(const float* lo, const float* hi, int64_t q, int d) {
+  if (q < 0) return fail(KDE_EINVAL, "q < 0");
+  if (q > 0 && (!lo || !hi)) return fail(KDE_EINVAL, "lo/hi is NULL");
+  for (int64_t i = 0; i < q * d; ++i) {
+    if (std::isnan(lo[i]) || std::isnan(hi[i])) return fail(KDE_EINVAL, "NaN in query bounds (element %lld)", (long long)i);
+    if (lo[i] > hi[i]) return fail(KDE_EINVAL, "lo > hi in query bounds (element %lld)", (long long)i);
+  }
+  return KDE_OK;
+}
+
+static kde_status validate_loss(int32_t loss, double lambda) {
+  if (loss < 0 || loss > 4) return fail(KDE_EINVAL, "unknown loss kind %d", loss);
+  if (!std::isfinite(lambda) || lambda < 0.0) return fail(KDE_EINVAL, "lambda must be finite and >= 0");
+  if (loss >= 2 && !(lambda > 0.0)) return fail(KDE_EINVAL, "lambda must be > 0 for relative / Q losses");
+  return KDE_OK;
+}
+
+// ------------------------------------------------------------------ buffers
+static kde_status ensure_pinned(kde_model* m, size_t bytes) {
+  if (m->pinned_cap >= bytes) return KDE_OK;
+  if (m->pinned) cudaFreeHost(m->pinned);
+  m->pinned = nullptr;
+  m->pinned_cap = 0;
+  size_t cap = std::max<size_t>(bytes, 1 << 16);
+  if (cudaMallocHost(&m->pinned, cap) != cudaSuccess) return fail(KDE_ENOMEM, "pinned host allocation of %zu bytes failed", cap);
+  m->pinned_cap = cap;
+  return KDE_OK;
+}
+
+static kde_status ensure_q(kde_model* m, int64_t q) {
+  const int d = m->d;
+  if (m->qcap < q) {
+    if (m->qbuf) cudaFree(m->qbuf);
+    m->qbuf = nullptr;
+    int64_t cap = std::max<int64_t>(q, 64);
+    if (cudaMalloc(&m->qbuf, sizeof(float) * 2 * cap * d) != cudaSuccess) return fail(KDE_ENOMEM, "bounds buffer");
+    m->qcap = cap;
+  }
+  if (m->ocap < q) {
+    if (m->obuf) cudaFree(m->obuf);
+    m->obuf = nullptr;
+    int64_t cap = std::max<int64_t>(q, 64);
+    // est[cap] dpdh[cap*d] sums[cap*(1+d)] true[cap] loss[1] grad[d]
+    size_t elems = cap + cap * d + cap * (1 + d) + cap + 1 + d;
+    if (cudaMalloc(&m->obuf, sizeof(double) * elems) != cudaSuccess) return fail(KDE_ENOMEM, "output buffer");
+    m->ocap = cap;
+  }
+  return KDE_OK;
+}
+static double* o_est(kde_model* m) { return m->obuf; }
+static double* o_dpdh(kde_model* m) { return m->obuf + m->ocap; }
+static double* o_sums(kde_model* m) { return m->obuf + m->ocap * (1 + m->d); }
+static double* o_true(kde_model* m) { return m->obuf + m->ocap * (2 + 2 * m->d); }
+static double* o_loss(kde_model* m) { return m->obuf + m->ocap * (3 + 2 * m->d); }
+static double* o_grad(kde_model* m) { return o_loss(m) + 1; }
+
+static kde_status ensure_bytes(void** p, size_t* cap, size_t bytes) {
+  if (*cap >= bytes) return KDE_OK;
+  if (*p) cudaFree(*p);
+  *p = nullptr;
+  *cap = 0;
+  if (cudaMalloc(p, bytes) != cudaSuccess) return fail(KDE_ENOMEM, "device allocation of %zu bytes failed", bytes);
+  *cap = bytes;
+  return KDE_OK;
+}
+
+// ------------------------------------------------------------------ profiling
+static kde_status prof_begin(kde_model* m, cudaStream_t s, cudaEvent_t* e1, cudaEvent_t* e2) {
+  ++m->scan_launches;
+  if (!m->prof) return KDE_OK;
+  while (m->ev.size() < m->ev_used + 2) {
+    cudaEvent_t e;
+    CU(cudaEventCreate(&e));
+    m->ev.push_back(e);
+  }
+  *e1 = m->ev[m->ev_used];
+  *e2 = m->ev[m->ev_used + 1];
+  m->ev_used += 2;
+  CU(cudaEventRecord(*e1, s));
+  return KDE_OK;
+}
+
+// ------------------------------------------------------------------ scans
+// Raw sums for q boxes (device bounds) -> sums[q][na] combined over ranks.
+// For q == 1 also retains c (if c_out) and writes the finalised values to fin.
+static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, int64_t q, bool grad, float* c_out,
+                            double* d_sums, cudaStream_t s) {
+  const int d = m->d;
+  const int na = grad ? d + 1 : 1;
+  if (q == 1) {
+    ScanSingleArgs a;
+    a.cols = m->cols;
+    a.ld = m->ld;
+    a.n = m->n;
+    a.lo = d_lo;
+    a.hi = d_hi;
+    a.consts = m->consts;
+    a.c_out = c_out;
+    a.block_partials = m->block_partials;
+    a.counter = m->counter;
+    a.sums_out = d_sums;
+    a.fin_out = nullptr;
+    a.n_global = (double)m->n_global;
+    const int grid = scan_single_grid(d, m->n, m->num_sms);
+    cudaEvent_t e1 = nullptr, e2 = nullptr;
+    kde_status pst = prof_begin(m, s, &e1, &e2);
+    if (pst != KDE_OK) return pst;
+    CUL(launch_scan_single(d, grad, a, grid, s));
+    if (e2) CU(cudaEventRecord(e2, s));
+  } else {
+    ScanBatchedArgs a;
+    a.cols = m->cols;
+    a.ld = m->ld;
+    a.n = m->n;
+    a.lo = d_lo;
+    a.hi = d_hi;
+    a.q = q;
+    a.consts = m->consts;
+    a.split_len = 0;
+    a.partials = nullptr;
+    int splits = 1;
+    CU(launch_scan_batched(d, grad, a, m->num_sms, &splits, s, true));
+    kde_status st = ensure_bytes((void**)&m->partials, &m->partials_cap, sizeof(double) * (size_t)splits * na * q);
+    if (st != KDE_OK) return st;
+    a.partials = m->partials;
+    cudaEvent_t e1 = nullptr, e2 = nullptr;
+    st = prof_begin(m, s, &e1, &e2);
+    if (st != KDE_OK) return st;
+    CUL(launch_scan_batched(d, grad, a, m->num_sms, &splits, s, false));
+    if (e2) CU(cudaEventRecord(e2, s));
+    CUL(launch_reduce_splits(m->partials, splits, q, na, d_sums, s));
+  }
+  if (m->world > 1) {
+    const size_t bytes = sizeof(double) * (size_t)m->world * q * na;
+    kde_status st = ensure_bytes((void**)&m->gather, &m->gather_cap, bytes);
+    if (st != KDE_OK) return st;
+    NC(ncclAllGather(d_sums, m->gather, (size_t)q * na, ncclDouble, m->comm, s));
+    CUL(launch_combine_ranks(m->gather, m->world, q, na, d_sums, s));
+  }
+  return KDE_OK;
+}
+
+// est/dpdh (device) for q boxes with device bounds.
+static kde_status estimate_dev(kde_model* m, const float* d_lo, const float* d_hi, int64_t q, double* d_est,
+                               double* d_dpdh, cudaStream_t s, bool retain_c) {
+  const bool grad = d_dpdh != nullptr;
+  const int na = grad ? m->d + 1 : 1;
+  kde_status st = ensure_q(m, q);
+  if (st != KDE_OK) return st;
+  double* sums = o_sums(m);
+  st = scan_sums(m, d_lo, d_hi, q, grad, (q == 1 && retain_c) ? m->cret : nullptr, sums, s);
+  if (st != KDE_OK) return st;
+  CUL(launch_finalize(sums, q, m->d, na, m->consts, (double)m->n_global, d_est, d_dpdh, s));
+  return KDE_OK;
+}
+
+// ------------------------------------------------------------------ ABI: misc
+extern "C" int32_t kde_abi_version(void) { return KDE_ABI_VERSION; }
+extern "C" const char* kde_last_error(void) { return g_err; }
+extern "C" const char* kde_status_string(kde_status s) {
+  switch (s) {
+    case KDE_OK: return "KDE_OK";
+    case KDE_EINVAL: return "KDE_EINVAL";
+    case KDE_ENOMEM: return "KDE_ENOMEM";
+    case KDE_ECUDA: return "KDE_ECUDA";
+    case KDE_ENCCL: return "KDE_ENCCL";
+    case KDE_ESTATE: return "KDE_ESTATE";
+    case KDE_ETRUNC: return "KDE_ETRUNC";
+  }
+  return "KDE_UNKNOWN";
+}
+
+extern "C" kde_status kde_get_unique_id(void* id_out) {
+  kde_model* m = nullptr;
+  if (!id_out) return fail(KDE_EINVAL, "id_out is NULL");
+  ncclUniqueId id;
+  NC(ncclGetUniqueId(&id));
+  memcpy(id_out, &id, sizeof(id));
+  return KDE_OK;
+}
+
+static void free_model(kde_model* m) {
+  if (!m) return;
+  DeviceGuard g(m->device);
+  if (m->stream) cudaStreamSynchronize(m->stream);
+  cudaFree(m->cols);
+  cudaFree(m->karma);
+  cudaFree(m->cret);
+  cudaFree(m->consts);
+  cudaFree(m->online);
+  cudaFree(m->block_partials);
+  cudaFree(m->counter);
+  cudaFree(m->ret);
+  cudaFree(m->single_sums);
+  cudaFree(m->qbuf);
+  cudaFree(m->obuf);
+  cudaFree(m->partials);
+  cudaFree(m->gather);
+  cudaFree(m->bitmap);
+  cudaFree(m->block_counts);
+  cudaFree(m->offsets);
+  cudaFree(m->idx_dev);
+  cudaFree(m->bad);
+  if (m->pinned) cudaFreeHost(m->pinned);
+  for (cudaEvent_t e : m->ev) cudaEventDestroy(e);
+  if (m->comm) ncclCommDestroy(m->comm);
+  if (m->stream) cudaStreamDestroy(m->stream);
+  delete m;
+}
+
+extern "C" void kde_destroy(kde_model* m) { free_model(m); }
+
+// ------------------------------------------------------------------ ABI: create
+static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_offset, int64_t n_global, int32_t d,
+                              const double* h, const void* nccl_id, int32_t rank, int32_t world, kde_model** out) {
+  if (!out) return fail(KDE_EINVAL, "out is NULL");
+  if (d < 1 || d > KDE_MAX_DIM) return fail(KDE_EINVAL, "d = %d outside [1, %d]", d, KDE_MAX_DIM);
+  if (world < 1 || rank < 0 || rank >= world) return fail(KDE_EINVAL, "bad rank/world %d/%d", rank, world);
+  if (n_global < 2) return fail(KDE_EINVAL, "n = %lld < 2 (eq. 6 divides by n - 1)", (long long)n_global);
+  if (n_local < 1 || row_offset < 0 || row_offset + n_local > n_global)
+    return fail(KDE_EINVAL, "shard [%lld, %lld) outside [0, %lld) or empty", (long long)row_offset,
+                (long long)(row_offset + n_local), (long long)n_global);
+  if (!rows) return fail(KDE_EINVAL, "sample is NULL");
+  if (world > 1 && !nccl_id) return fail(KDE_EINVAL, "nccl_id is NULL for world > 1");
+  if (h)
+    for (int j = 0; j < d; ++j)
+      if (!h_ok(h[j])) return fail(KDE_EINVAL, "h[%d] = %g not finite in [1e-30, 1e30]", j, h[j]);
+
+  kde_model* m = new (std::nothrow) kde_model();
+  if (!m) return fail(KDE_ENOMEM, "host allocation failed");
+  kde_status st = KDE_OK;
+  auto bail = [&](kde_status s2) {
+    free_model(m);
+    return s2;
+  };
+  if (cudaGetDevice(&m->device) != cudaSuccess) return bail(fail(KDE_ECUDA, "no CUDA device"));
+  cudaDeviceGetAttribute(&m->num_sms, cudaDevAttrMultiProcessorCount, m->device);
+  m->d = d;
+  m->n = n_local;
+  m->n_global = n_global;
+  m->row_offset = row_offset;
+  m->rank = rank;
+  m->world = world;
+  m->ld = (n_local + kColAlign - 1) / kColAlign * kColAlign;
+#define CUB(call)                                                                                   \
+  do {                                                                                              \
+    cudaError_t e_ = (call);                                                                        \
+    if (e_ != cudaSuccess)                                                                          \
+      return bail(fail(e_ == cudaErrorMemoryAllocation ? KDE_ENOMEM : KDE_ECUDA, "%s: %s", #call,   \
+                       cudaGetErrorString(e_)));                                                    \
+  } while (0)
+  CUB(cudaStreamCreateWithFlags(&m->stream, cudaStreamNonBlocking));
+  CUB(cudaMalloc(&m->cols, sizeof(float) * (size_t)d * m->ld));
+  CUB(cudaMalloc(&m->karma, sizeof(double) * (size_t)n_local));
+  CUB(cudaMalloc(&m->cret, sizeof(float) * (size_t)m->ld));
+  CUB(cudaMalloc(&m->consts, sizeof(DevConsts)));
+  CUB(cudaMalloc(&m->online, sizeof(OnlineState)));
+  CUB(cudaMalloc(&m->block_partials, sizeof(double) * (size_t)m->num_sms * 4 * (kMaxDim + 1)));
+  CUB(cudaMalloc(&m->counter, sizeof(unsigned)));
+  CUB(cudaMalloc(&m->ret, sizeof(double) * (kMaxDim + 1)));
+  CUB(cudaMalloc(&m->single_sums, sizeof(double) * (kMaxDim + 1)));
+  CUB(cudaMalloc(&m->bad, sizeof(int32_t)));
+  const int nkb = karma_blocks(n_local);
+  CUB(cudaMalloc(&m->bitmap, sizeof(uint32_t) * (size_t)nkb * (kKarmaPts / 32)));
+  CUB(cudaMalloc(&m->block_counts, sizeof(int32_t) * (size_t)nkb));
+  CUB(cudaMalloc(&m->offsets, sizeof(int64_t) * (size_t)(nkb + 1)));
+  cudaStream_t s = m->stream;
+  CUB(cudaMemsetAsync(m->cols, 0, sizeof(float) * (size_t)d * m->ld, s));
+  CUB(cudaMemsetAsync(m->karma, 0, sizeof(double) * (size_t)n_local, s));
+  CUB(cudaMemsetAsync(m->cret, 0, sizeof(float) * (size_t)m->ld, s));
+  CUB(cudaMemsetAsync(m->consts, 0, sizeof(DevConsts), s));
+  CUB(cudaMemsetAsync(m->online, 0, sizeof(OnlineState), s));
+  CUB(cudaMemsetAsync(m->counter, 0, sizeof(unsigned), s));
+  CUB(cudaMemsetAsync(m->bad, 0, sizeof(int32_t), s));
+
+  if (world > 1) {
+    ncclUniqueId id;
+    memcpy(&id, nccl_id, sizeof(id));
+    ncclResult_t r = ncclCommInitRank(&m->comm, world, id, rank);
+    if (r != ncclSuccess) return bail(fail(KDE_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r)));
+  }
+
+  // sample: host row-major -> device (chunked through a pinned buffer) -> SoA columns
+  {
+    const int64_t chunk_rows = std::max<int64_t>(1, (64ll << 20) / (4ll * d));
+    float* d_rows = nullptr;
+    const int64_t cr = std::min<int64_t>(chunk_rows, n_local);
+    CUB(cudaMalloc(&d_rows, sizeof(float) * (size_t)cr * d));
+    st = ensure_pinned(m, sizeof(float) * (size_t)cr * d);
+    if (st != KDE_OK) {
+      cudaFree(d_rows);
+      return bail(st);
+    }
+    for (int64_t r0 = 0; r0 < n_local; r0 += cr) {
+      const int64_t k = std::min<int64_t>(cr, n_local - r0);
+      memcpy(m->pinned, rows + r0 * d, sizeof(float) * (size_t)k * d);
+      cudaError_t e = cudaMemcpyAsync(d_rows, m->pinned, sizeof(float) * (size_t)k * d, cudaMemcpyHostToDevice, s);
+      if (e == cudaSuccess) e = launch_rows_to_cols(d_rows, k, d, m->cols + r0, m->ld, m->bad, s);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(s);  // pinned buffer reuse
+      if (e != cudaSuccess) {
+        cudaFree(d_rows);
+        return bail(fail(KDE_ECUDA, "sample upload: %s", cudaGetErrorString(e)));
+      }
+    }
+    cudaFree(d_rows);
+    int32_t bad = 0;
+    CUB(cudaMemcpy(&bad, m->bad, sizeof(int32_t), cudaMemcpyDeviceToHost));
+    if (bad) return bail(fail(KDE_EINVAL, "non-finite value in sample"));
+  }
+
+  // bandwidth: caller's h, or Scott's rule (eq. 3) over the global sample
+  if (h) {
+    CUB(launch_set_consts(h, d, m->consts, s));
+  } else {
+    const int nb = moments_blocks(n_local);
+    double* part = nullptr;
+    CUB(cudaMalloc(&part, sizeof(double) * ((size_t)nb * d * 3 + (size_t)d * 3 * (world + 1))));
+    double* mom = part + (size_t)nb * d * 3;
+    double* gath = mom + (size_t)d * 3;
+    cudaError_t e = launch_moments(m->cols, m->ld, n_local, d, part, mom, s);
+    if (e == cudaSuccess && world > 1) {
+      ncclResult_t r = ncclAllGather(mom, gath, (size_t)d * 3, ncclDouble, m->comm, s);
+      if (r != ncclSuccess) {
+        cudaFree(part);
+        return bail(fail(KDE_ENCCL, "moments allgather: %s", ncclGetErrorString(r)));
+      }
+      e = launch_moments_merge_ranks(gath, world, d, mom, s);
+    }
+    if (e == cudaSuccess) e = launch_scott(mom, d, m->consts, m->bad, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    cudaFree(part);
+    if (e != cudaSuccess) return bail(fail(KDE_ECUDA, "Scott bandwidth: %s", cudaGetErrorString(e)));
+    int32_t bad = 0;
+    CUB(cudaMemcpy(&bad, m->bad, sizeof(int32_t), cudaMemcpyDeviceToHost));
+    if (bad) return bail(fail(KDE_EINVAL, "Scott's rule gives h outside [1e-30, 1e30] (constant column?)"));
+  }
+  CUB(cudaStreamSynchronize(s));
+#undef CUB
+  *out = m;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_create(const float* sample, int64_t n, int32_t d, const double* h, kde_model** out) {
+  return create_impl(sample, n, 0, n, d, h, nullptr, 0, 1, out);
+}
+
+extern "C" kde_status kde_create_sharded(const float* local_rows, int64_t n_local, int64_t row_offset,
+                                         int64_t n_global, int32_t d, const double* h, const void* nccl_id,
+                                         int32_t rank, int32_t world, kde_model** out) {
+  return create_impl(local_rows, n_local, row_offset, n_global, d, h, nccl_id, rank, world, out);
+}
+
+extern "C" kde_status kde_get_info(const kde_model* m, int64_t* n_local, int64_t* n_global, int32_t* d,
+                                   int32_t* rank, int32_t* world) {
+  if (!m) return fail(KDE_EINVAL, "model is NULL");
+  if (n_local) *n_local = m->n;
+  if (n_global) *n_global = m->n_global;
+  if (d) *d = m->d;
+  if (rank) *rank = m->rank;
+  if (world) *world = m->world;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_get_bandwidth(kde_model* m, double* h) {
+  CHECK_MODEL(m);
+  if (!h) return fail(KDE_EINVAL, "h is NULL");
+  DeviceGuard g(m->device);
+  DevConsts c;
+  CU(cudaMemcpyAsync(&c, m->consts, sizeof(DevConsts), cudaMemcpyDeviceToHost, m->stream));
+  CU(cudaStreamSynchronize(m->stream));
+  for (int j = 0; j < m->d; ++j) h[j] = c.h[j];
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_set_bandwidth(kde_model* m, const double* h) {
+  CHECK_MODEL(m);
+  if (!h) return fail(KDE_EINVAL, "h is NULL");
+  for (int j = 0; j < m->d; ++j)
+    if (!h_ok(h[j])) return fail(KDE_EINVAL, "h[%d] = %g not finite in [1e-30, 1e30]", j, h[j]);
+  DeviceGuard g(m->device);
+  CUL(launch_set_consts(h, m->d, m->consts, m->stream));
+  CU(cudaStreamSynchronize(m->stream));
+  ++m->gen;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_set_retain(kde_model* m, int32_t on) {
+  CHECK_MODEL(m);
+  m->retain = on != 0;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_synchronize(kde_model* m) {
+  CHECK_MODEL(m);
+  DeviceGuard g(m->device);
+  CU(cudaStreamSynchronize(m->stream));
+  return KDE_OK;
+}
+
+// ------------------------------------------------------------------ ABI: estimates
+// Stage host bounds into m->qbuf (lo at [0, q*d), hi at [q*d, 2*q*d)).
+static kde_status stage_bounds(kde_model* m, const float* lo, const float* hi, int64_t q) {
+  const size_t bytes = sizeof(float) * (size_t)q * m->d;
+  kde_status st = ensure_q(m, q);
+  if (st != KDE_OK) return st;
+  st = ensure_pinned(m, 2 * bytes);
+  if (st != KDE_OK) return st;
+  memcpy(m->pinned, lo, bytes);
+  memcpy((char*)m->pinned + bytes, hi, bytes);
+  CU(cudaMemcpyAsync(m->qbuf, m->pinned, 2 * bytes, cudaMemcpyHostToDevice, m->stream));
+  return KDE_OK;
+}
+
+static void note_retained(kde_model* m, const float* lo, const float* hi, bool has_c, bool has_grad) {
+  m->ret_valid = true;
+  m->ret_has_c = has_c;
+  m->ret_has_grad = has_grad;
+  m->ret_gen = m->gen;
+  memcpy(m->ret_lo, lo, sizeof(float) * m->d);
+  memcpy(m->ret_hi, hi, sizeof(float) * m->d);
+}
+
+extern "C" kde_status kde_estimate_batch(kde_model* m, const float* lo, const float* hi, int64_t q, double* est,
+                                         double* dest_dh) {
+  CHECK_MODEL(m);
+  kde_status st = validate_bounds(lo, hi, q, m->d);
+  if (st != KDE_OK) return st;
+  if (q > 0 && !est) return fail(KDE_EINVAL, "est is NULL");
+  if (q == 0) return KDE_OK;
+  DeviceGuard g(m->device);
+  st = stage_bounds(m, lo, hi, q);
+  if (st != KDE_OK) return st;
+  const float* d_lo = m->qbuf;
+  const float* d_hi = m->qbuf + q * m->d;
+  const bool grad = dest_dh != nullptr;
+  const bool retain_c = m->retain && q == 1;
+  double* d_est = q == 1 ? m->ret : o_est(m);
+  double* d_dpdh = grad ? (q == 1 ? m->ret + 1 : o_dpdh(m)) : nullptr;
+  st = estimate_dev(m, d_lo, d_hi, q, d_est, d_dpdh, m->stream, retain_c);
+  if (st != KDE_OK) return st;
+  if (q == 1) {
+    CU(cudaMemcpyAsync(est, m->ret, sizeof(double), cudaMemcpyDeviceToHost, m->stream));
+    if (grad) CU(cudaMemcpyAsync(dest_dh, m->ret + 1, sizeof(double) * m->d, cudaMemcpyDeviceToHost, m->stream));
+  } else {
+    CU(cudaMemcpyAsync(est, d_est, sizeof(double) * q, cudaMemcpyDeviceToHost, m->stream));
+    if (grad) CU(cudaMemcpyAsync(dest_dh, d_dpdh, sizeof(double) * q * m->d, cudaMemcpyDeviceToHost, m->stream));
+  }
+  CU(cudaStreamSynchronize(m->stream));
+  if (q == 1) note_retained(m, lo, hi, retain_c, grad);
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_estimate_batch_dev(kde_model* m, const float* d_lo, const float* d_hi, int64_t q,
+                                             double* d_est, double* d_dest_dh, void* stream) {
+  CHECK_MODEL(m);
+  if (q < 0) return fail(KDE_EINVAL, "q < 0");
+  if (q == 0) return KDE_OK;
+  if (!d_lo || !d_hi || !d_est) return fail(KDE_EINVAL, "NULL device pointer");
+  DeviceGuard g(m->device);
+  cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
+  m->ret_valid = false;  // bounds are device-side; no retained-state bookkeeping
+  return estimate_dev(m, d_lo, d_hi, q, d_est, d_dest_dh, s, m->retain && q == 1);
+}
+
+static kde_status loss_grad_dev_impl(kde_model* m, const float* d_lo, const float* d_hi, const double* d_true,
+                                     int64_t q, int32_t loss, double lambda, int32_t log_bw, double* d_loss,
+                                     double* d_grad, double* d_est_out, cudaStream_t s) {
+  kde_status st = ensure_q(m, q);
+  if (st != KDE_OK) return st;
+  double* d_est = d_est_out ? d_est_out : o_est(m);
+  double* d_dpdh = o_dpdh(m);
+  st = estimate_dev(m, d_lo, d_hi, q, d_est, d_dpdh, s, false);
+  if (st != KDE_OK) return st;
+  CUL(launch_loss_epilogue(d_est, d_dpdh, d_true, q, m->d, loss, lambda, log_bw, m->consts, d_loss, d_grad, s));
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_loss_and_grad(kde_model* m, const float* lo, const float* hi, const double* true_sel,
+                                        int64_t q, int32_t loss, double lambda, int32_t log_bandwidth,
+                                        double* loss_out, double* grad_out, double* est_out) {
+  CHECK_MODEL(m);
+  if (q < 1) return fail(KDE_EINVAL, "q must be >= 1");
+  kde_status st = validate_bounds(lo, hi, q, m->d);
+  if (st != KDE_OK) return st;
+  st = validate_loss(loss, lambda);
+  if (st != KDE_OK) return st;
+  if (!true_sel || !loss_out || !grad_out) return fail(KDE_EINVAL, "NULL output/true_sel pointer");
+  for (int64_t k = 0; k < q; ++k)
+    if (!(true_sel[k] >= 0.0 && true_sel[k] <= 1.0)) return fail(KDE_EINVAL, "true_sel[%lld] outside [0, 1]", (long long)k);
+  DeviceGuard g(m->device);
+  st = stage_bounds(m, lo, hi, q);
+  if (st != KDE_OK) return st;
+  CU(cudaMemcpyAsync(o_true(m), true_sel, sizeof(double) * q, cudaMemcpyHostToDevice, m->stream));
+  st = loss_grad_dev_impl(m, m->qbuf, m->qbuf + q * m->d, o_true(m), q, loss, lambda, log_bandwidth, o_loss(m),
+                          o_grad(m), o_est(m), m->stream);
+  if (st != KDE_OK) return st;
+  CU(cudaMemcpyAsync(loss_out, o_loss(m), sizeof(double), cudaMemcpyDeviceToHost, m->stream));
+  CU(cudaMemcpyAsync(grad_out, o_grad(m), sizeof(double) * m->d, cudaMemcpyDeviceToHost, m->stream));
+  if (est_out) CU(cudaMemcpyAsync(est_out, o_est(m), sizeof(double) * q, cudaMemcpyDeviceToHost, m->stream));
+  CU(cudaStreamSynchronize(m->stream));
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_loss_and_grad_dev(kde_model* m, const float* d_lo, const float* d_hi,
+                                            const double* d_true_sel, int64_t q, int32_t loss, double lambda,
+                                            int32_t log_bandwidth, double* d_loss, double* d_grad, double* d_est,
+                                            void* stream) {
+  CHECK_MODEL(m);
+  if (q < 1) return fail(KDE_EINVAL, "q must be >= 1");
+  kde_status st = validate_loss(loss, lambda);
+  if (st != KDE_OK) return st;
+  if (!d_lo || !d_hi || !d_true_sel || !d_loss || !d_grad) return fail(KDE_EINVAL, "NULL device pointer");
+  DeviceGuard g(m->device);
+  cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
+  m->ret_valid = false;
+  return loss_grad_dev_impl(m, d_lo, d_hi, d_true_sel, q, loss, lambda, log_bandwidth, d_loss, d_grad, d_est, s);
+}
+
+// ------------------------------------------------------------------ ABI: feedback
+static bool retained_matches(kde_model* m, const float* lo, const float* hi, bool need_c, bool need_grad) {
+  if (!m->ret_valid || m->ret_gen != m->gen) return false;
+  if (need_c && !m->ret_has_c) return false;
+  if (need_grad && !m->ret_has_grad) return false;
+  return memcmp(m->ret_lo, lo, sizeof(float) * m->d) == 0 && memcmp(m->ret_hi, hi, sizeof(float) * m->d) == 0;
+}
+
+// Make sure m->ret (p_hat, dp/dh) and (need_c) m->cret hold this box's values.
+static kde_status ensure_retained(kde_model* m, const float* lo, const float* hi, bool need_c, bool need_grad) {
+  if (retained_matches(m, lo, hi, need_c, need_grad)) {
+    // bounds of the retained query are still needed on the device (karma eq. 20)
+    kde_status st = stage_bounds(m, lo, hi, 1);
+    return st;
+  }
+  kde_status st = stage_bounds(m, lo, hi, 1);
+  if (st != KDE_OK) return st;
+  const bool grad = need_grad;
+  st = estimate_dev(m, m->qbuf, m->qbuf + m->d, 1, m->ret, grad ? m->ret + 1 : nullptr, m->stream, true);
+  if (st != KDE_OK) return st;
+  note_retained(m, lo, hi, true, grad);
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_karma_update(kde_model* m, const float* lo, const float* hi, double true_sel,
+                                       const kde_karma_params* kp, int64_t* idx_out, int64_t idx_cap,
+                                       int64_t* n_flagged) {
+  CHECK_MODEL(m);
+  kde_status st = validate_bounds(lo, hi, 1, m->d);
+  if (st != KDE_OK) return st;
+  if (!kp || !n_flagged) return fail(KDE_EINVAL, "NULL karma params / n_flagged");
+  if (idx_cap < 0 || (idx_cap > 0 && !idx_out)) return fail(KDE_EINVAL, "bad idx_out / idx_cap");
+  if (!(true_sel >= 0.0 && true_sel <= 1.0)) return fail(KDE_EINVAL, "true_sel outside [0, 1]");
+  st = validate_loss(kp->loss, kp->lambda);
+  if (st != KDE_OK) return st;
+  if (std::isnan(kp->k_max) || std::isnan(kp->threshold)) return fail(KDE_EINVAL, "NaN k_max / threshold");
+  DeviceGuard g(m->device);
+  st = ensure_retained(m, lo, hi, true, false);
+  if (st != KDE_OK) return st;
+  // index output buffer: local flags at most n
+  const int64_t local_cap = m->n;
+  if (m->idx_cap < local_cap) {
+    cudaFree(m->idx_dev);
+    m->idx_dev = nullptr;
+    if (cudaMalloc(&m->idx_dev, sizeof(int64_t) * (size_t)local_cap) != cudaSuccess) return fail(KDE_ENOMEM, "idx buffer");
+    m->idx_cap = local_cap;
+  }
+  KarmaParamsDev kd;
+  kd.loss = kp->loss;
+  kd.empty_region = kp->empty_region;
+  kd.lambda = kp->lambda;
+  kd.k_max = kp->k_max;
+  kd.threshold = kp->threshold;
+  const int nkb = karma_blocks(m->n);
+  m->launches += 2;  // karma + scan_counts + compact
+  CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, true_sel, kd, m->qbuf, m->qbuf + m->d, m->d,
+                  m->consts, m->bitmap, m->block_counts, m->offsets, m->row_offset, m->idx_dev, local_cap,
+                  m->stream));
+  int64_t local_total = 0;
+  CU(cudaMemcpyAsync(&local_total, m->offsets + nkb, sizeof(int64_t), cudaMemcpyDeviceToHost, m->stream));
+  CU(cudaStreamSynchronize(m->stream));
+  if (m->world == 1) {
+    const int64_t ncopy = std::min(local_total, idx_cap);
+    if (ncopy > 0) CU(cudaMemcpy(idx_out, m->idx_dev, sizeof(int64_t) * ncopy, cudaMemcpyDeviceToHost));
+    *n_flagged = local_total;
+    return local_total > idx_cap ? fail(KDE_ETRUNC, "%lld flagged > idx_cap %lld", (long long)local_total, (long long)idx_cap)
+                                 : KDE_OK;
+  }
+  // world > 1: gather counts, then the (ascending, rank-ordered) index lists
+  std::vector<int64_t> counts(m->world);
+  {
+    int64_t* d_cnt = nullptr;
+    CU(cudaMalloc(&d_cnt, sizeof(int64_t) * (m->world + 1)));
+    CU(cudaMemcpyAsync(d_cnt + m->world, &local_total, sizeof(int64_t), cudaMemcpyHostToDevice, m->stream));
+    ncclResult_t r = ncclAllGather(d_cnt + m->world, d_cnt, 1, ncclInt64, m->comm, m->stream);
+    if (r != ncclSuccess) {
+      cudaFree(d_cnt);
+      m->poisoned = true;
+      return fail(KDE_ENCCL, "karma count allgather: %s", ncclGetErrorString(r));
+    }
+    CU(cudaMemcpyAsync(counts.data(), d_cnt, sizeof(int64_t) * m->world, cudaMemcpyDeviceToHost, m->stream));
+    CU(cudaStreamSynchronize(m->stream));
+    cudaFree(d_cnt);
+  }
+  int64_t maxc = 0, total = 0;
+  for (int64_t c : counts) {
+    maxc = std::max(maxc, c);
+    total += c;
+  }
+  *n_flagged = total;
+  if (maxc > 0) {
+    int64_t* d_all = nullptr;
+    CU(cudaMalloc(&d_all, sizeof(int64_t) * (size_t)maxc * (m->world + 1)));
+    int64_t* d_send = d_all + (size_t)maxc * m->world;
+    if (local_total > 0)
+      CU(cudaMemcpyAsync(d_send, m->idx_dev, sizeof(int64_t) * local_total, cudaMemcpyDeviceToDevice, m->stream));
+    ncclResult_t r = ncclAllGather(d_send, d_all, (size_t)maxc, ncclInt64, m->comm, m->stream);
+    if (r != ncclSuccess) {
+      cudaFree(d_all);
+      m->poisoned = true;
+      return fail(KDE_ENCCL, "karma index allgather: %s", ncclGetErrorString(r));
+    }
+    int64_t pos = 0;
+    for (int rr = 0; rr < m->world && pos < idx_cap; ++rr) {
+      const int64_t k = std::min(counts[rr], idx_cap - pos);
+      if (k > 0)
+        CU(cudaMemcpyAsync(idx_out + pos, d_all + (size_t)rr * maxc, sizeof(int64_t) * k, cudaMemcpyDeviceToHost,
+                           m->stream));
+      pos += k;
+    }
+    CU(cudaStreamSynchronize(m->stream));
+    cudaFree(d_all);
+  }
+  return total > idx_cap ? fail(KDE_ETRUNC, "%lld flagged > idx_cap %lld", (long long)total, (long long)idx_cap) : KDE_OK;
+}
+
+extern "C" kde_status kde_online_update(kde_model* m, const float* lo, const float* hi, double true_sel,
+                                        const kde_online_params* op, int32_t* updated) {
+  CHECK_MODEL(m);
+  kde_status st = validate_bounds(lo, hi, 1, m->d);
+  if (st != KDE_OK) return st;
+  if (!op) return fail(KDE_EINVAL, "NULL online params");
+  if (!(true_sel >= 0.0 && true_sel <= 1.0)) return fail(KDE_EINVAL, "true_sel outside [0, 1]");
+  st = validate_loss(op->loss, op->lambda);
+  if (st != KDE_OK) return st;
+  if (op->minibatch < 1 || !(op->alpha >= 0.0 && op->alpha < 1.0) || !(op->lr_min > 0.0) ||
+      !(op->lr_max >= op->lr_min) || !(op->lr_inc >= 1.0) || !(op->lr_dec > 0.0 && op->lr_dec <= 1.0) ||
+      !(op->lr0 > 0.0))
+    return fail(KDE_EINVAL, "bad online parameters");
+  DeviceGuard g(m->device);
+  if (!m->online_init) {
+    OnlineState s0;
+    memset(&s0, 0, sizeof(s0));
+    for (int j = 0; j < kMaxDim; ++j) s0.lr[j] = op->lr0;
+    CU(cudaMemcpyAsync(m->online, &s0, sizeof(s0), cudaMemcpyHostToDevice, m->stream));
+    CU(cudaStreamSynchronize(m->stream));
+    m->online_init = true;
+  }
+  st = ensure_retained(m, lo, hi, false, true);
+  if (st != KDE_OK) return st;
+  OnlineParamsDev od;
+  od.minibatch = op->minibatch;
+  od.log_bw = op->log_bandwidth;
+  od.loss = op->loss;
+  od.lambda = op->lambda;
+  od.alpha = op->alpha;
+  od.lr_min = op->lr_min;
+  od.lr_max = op->lr_max;
+  od.lr_inc = op->lr_inc;
+  od.lr_dec = op->lr_dec;
+  CUL(launch_online_update(m->ret, true_sel, od, m->d, m->online, m->consts, m->stream));
+  int32_t upd = 0;
+  CU(cudaMemcpyAsync(&upd, &m->online->updated, sizeof(int32_t), cudaMemcpyDeviceToHost, m->stream));
+  CU(cudaStreamSynchronize(m->stream));
+  if (upd) ++m->gen;
+  if (updated) *updated = upd;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_replace_points(kde_model* m, const int64_t* idx, const float* rows, int64_t k,
+                                         double k_init) {
+  CHECK_MODEL(m);
+  if (k < 0) return fail(KDE_EINVAL, "k < 0");
+  if (k == 0) return KDE_OK;
+  if (!idx || !rows) return fail(KDE_EINVAL, "NULL idx / rows");
+  if (!std::isfinite(k_init)) return fail(KDE_EINVAL, "k_init not finite");
+  std::vector<int64_t> sorted(idx, idx + k);
+  std::sort(sorted.begin(), sorted.end());
+  for (int64_t r = 0; r < k; ++r) {
+    if (sorted[r] < 0 || sorted[r] >= m->n_global) return fail(KDE_EINVAL, "index %lld out of range", (long long)sorted[r]);
+    if (r > 0 && sorted[r] == sorted[r - 1]) return fail(KDE_EINVAL, "duplicate index %lld", (long long)sorted[r]);
+  }
+  for (int64_t e = 0; e < k * m->d; ++e)
+    if (!std::isfinite(rows[e])) return fail(KDE_EINVAL, "non-finite value in replacement rows");
+  // rows owned by this shard
+  std::vector<int64_t> li;
+  std::vector<float> lr;
+  for (int64_t r = 0; r < k; ++r) {
+    const int64_t i = idx[r] - m->row_offset;
+    if (i >= 0 && i < m->n) {
+      li.push_back(i);
+      lr.insert(lr.end(), rows + r * m->d, rows + (r + 1) * m->d);
+    }
+  }
+  DeviceGuard g(m->device);
+  const int64_t kl = (int64_t)li.size();
+  if (kl > 0) {
+    const size_t ib = sizeof(int64_t) * kl, rb = sizeof(float) * kl * m->d;
+    kde_status st = ensure_pinned(m, ib + rb);
+    if (st != KDE_OK) return st;
+    void* dbuf = nullptr;
+    CU(cudaMalloc(&dbuf, ib + rb));
+    memcpy(m->pinned, li.data(), ib);
+    memcpy((char*)m->pinned + ib, lr.data(), rb);
+    CU(cudaMemcpyAsync(dbuf, m->pinned, ib + rb, cudaMemcpyHostToDevice, m->stream));
+    CUL(launch_scatter_rows((const int64_t*)dbuf, (const float*)((char*)dbuf + ib), kl, m->d, m->cols, m->ld,
+                           m->karma, k_init, m->stream));
+    CU(cudaStreamSynchronize(m->stream));
+    cudaFree(dbuf);
+  }
+  ++m->gen;
+  return KDE_OK;
+}
+
+// ------------------------------------------------------------------ inspection
+extern "C" kde_status kde_get_karma(kde_model* m, double* karma) {
+  CHECK_MODEL(m);
+  if (!karma) return fail(KDE_EINVAL, "NULL karma");
+  DeviceGuard g(m->device);
+  CU(cudaStreamSynchronize(m->stream));
+  CU(cudaMemcpy(karma, m->karma, sizeof(double) * m->n, cudaMemcpyDeviceToHost));
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_set_karma(kde_model* m, const double* karma) {
+  CHECK_MODEL(m);
+  if (!karma) return fail(KDE_EINVAL, "NULL karma");
+  for (int64_t i = 0; i < m->n; ++i)
+    if (std::isnan(karma[i])) return fail(KDE_EINVAL, "NaN karma");
+  DeviceGuard g(m->device);
+  CU(cudaStreamSynchronize(m->stream));
+  CU(cudaMemcpy(m->karma, karma, sizeof(double) * m->n, cudaMemcpyHostToDevice));
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_get_sample(kde_model* m, float* rows) {
+  CHECK_MODEL(m);
+  if (!rows) return fail(KDE_EINVAL, "NULL rows");
+  DeviceGuard g(m->device);
+  float* d_rows = nullptr;
+  CU(cudaMalloc(&d_rows, sizeof(float) * (size_t)m->n * m->d));
+  CUL(launch_cols_to_rows(m->cols, m->ld, m->n, m->d, d_rows, m->stream));
+  CU(cudaStreamSynchronize(m->stream));
+  CU(cudaMemcpy(rows, d_rows, sizeof(float) * (size_t)m->n * m->d, cudaMemcpyDeviceToHost));
+  cudaFree(d_rows);
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_get_contributions(kde_model* m, float* c) {
+  CHECK_MODEL(m);
+  if (!c) return fail(KDE_EINVAL, "NULL c");
+  if (!m->ret_valid || !m->ret_has_c) return fail(KDE_ESTATE, "no retained contributions");
+  DeviceGuard g(m->device);
+  CU(cudaStreamSynchronize(m->stream));
+  CU(cudaMemcpy(c, m->cret, sizeof(float) * m->n, cudaMemcpyDeviceToHost));
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_get_online_state(kde_model* m, double* acc, double* ms, double* lr, double* gprev,
+                                           int32_t* count) {
+  CHECK_MODEL(m);
+  DeviceGuard g(m->device);
+  OnlineState s;
+  CU(cudaStreamSynchronize(m->stream));
+  CU(cudaMemcpy(&s, m->online, sizeof(s), cudaMemcpyDeviceToHost));
+  const size_t b = sizeof(double) * m->d;
+  if (acc) memcpy(acc, s.acc, b);
+  if (ms) memcpy(ms, s.ms, b);
+  if (lr) memcpy(lr, s.lr, b);
+  if (gprev) memcpy(gprev, s.gprev, b);
+  if (count) *count = s.count;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_set_online_state(kde_model* m, const double* acc, const double* ms, const double* lr,
+                                           const double* gprev, int32_t count) {
+  CHECK_MODEL(m);
+  if (!acc || !ms || !lr || !gprev || count < 0) return fail(KDE_EINVAL, "bad online state");
+  DeviceGuard g(m->device);
+  OnlineState s;
+  memset(&s, 0, sizeof(s));
+  const size_t b = sizeof(double) * m->d;
+  memcpy(s.acc, acc, b);
+  memcpy(s.ms, ms, b);
+  memcpy(s.lr, lr, b);
+  memcpy(s.gprev, gprev, b);
+  s.count = count;
+  CU(cudaStreamSynchronize(m->stream));
+  CU(cudaMemcpy(m->online, &s, sizeof(s), cudaMemcpyHostToDevice));
+  m->online_init = true;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_set_profiling(kde_model* m, int32_t on) {
+  CHECK_MODEL(m);
+  m->prof = on != 0;
+  m->ev_used = 0;
+  m->scan_launches = 0;
+  m->launches = 0;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_get_profile(kde_model* m, double* scan_ms, int64_t* scan_launches, int64_t* launches) {
+  CHECK_MODEL(m);
+  DeviceGuard g(m->device);
+  CU(cudaDeviceSynchronize());
+  double tot = 0.0;
+  for (size_t i = 0; i + 1 < m->ev_used; i += 2) {
+    float ms = 0.f;
+    CU(cudaEventElapsedTime(&ms, m->ev[i], m->ev[i + 1]));
+    tot += ms;
+  }
+  if (scan_ms) *scan_ms = tot;
+  if (scan_launches) *scan_launches = m->scan_launches;
+  if (launches) *launches = m->launches;
+  m->ev_used = 0;
+  m->scan_launches = 0;
+  m->launches = 0;
+  return KDE_OK;
+}
+
+// ------------------------------------------------------------------ harness
+extern "C" kde_status kde_count_in_box_dev(const float* d_rows, int64_t n, int32_t d, const float* d_lo,
+                                           const float* d_hi, int64_t q, int64_t* d_counts, void* stream) {
+  kde_model* m = nullptr;
+  if (d < 1 || d > KDE_MAX_DIM || n < 0 || q < 0) return fail(KDE_EINVAL, "bad count_in_box arguments");
+  if (q == 0) return KDE_OK;
+  if (!d_rows || !d_lo || !d_hi || !d_counts) return fail(KDE_EINVAL, "NULL device pointer");
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaStream_t s = (cudaStream_t)stream;
+  CU(cudaMemsetAsync(d_counts, 0, sizeof(int64_t) * q, s));
+  CUL(launch_count_in_box(d_rows, n, d, d_lo, d_hi, q, (unsigned long long*)d_counts, sms, s));
+  return KDE_OK;
+}

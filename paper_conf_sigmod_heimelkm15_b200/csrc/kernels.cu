@@ -1,0 +1,532 @@
+// kernels.cu -- everything on the path except the scan itself:
+//   sample layout (row-major -> SoA), Scott moments (eq. 3), constant
+//   derivation, split / rank reduction + finalisation, loss epilogue (eq. 5,
+//   14, 18, C.1), karma pass + ordered compaction (eq. 6-8, 19-20),
+//   row replacement, the on-device Listing 1 step (Section 4.1)
+//   and the harness box counter.
+// All reductions use a fixed order, so results are bitwise reproducible.
+#include <cstdint>
+#include <cuda_runtime.h>
+#include <math_constants.h>
+
+#include "common.cuh"
+#include "kernels.cuh"
+
+namespace kde {
+
+// ------------------------------------------------------------ layout
+// rows: device row-major [n][d]; cols: [d][ld].  Flags non-finite values.
+__global__ void rows_to_cols_kernel(const float* __restrict__ rows, int64_t n, int d, float* __restrict__ cols,
+                                    int64_t ld, int* bad) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  for (int j = 0; j < d; ++j) {
+    const float x = rows[i * d + j];
+    if (!isfinite(x)) *bad = 1;
+    cols[(int64_t)j * ld + i] = x;
+  }
+}
+
+// rows[r][j] -> cols[j][idx_local[r]], karma[idx_local[r]] = k_init
+__global__ void scatter_rows_kernel(const int64_t* __restrict__ idx_local, const float* __restrict__ rows, int64_t k,
+                                    int d, float* __restrict__ cols, int64_t ld, double* __restrict__ karma,
+                                    double k_init) {
+  const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= k) return;
+  const int64_t i = idx_local[r];
+  for (int j = 0; j < d; ++j) cols[(int64_t)j * ld + i] = rows[r * d + j];
+  karma[i] = k_init;
+}
+
+__global__ void cols_to_rows_kernel(const float* __restrict__ cols, int64_t ld, int64_t n, int d,
+                                    float* __restrict__ rows) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  for (int j = 0; j < d; ++j) rows[i * d + j] = cols[(int64_t)j * ld + i];
+}
+
+// ------------------------------------------------------------ Scott moments
+// Per (block, column) fp64 Welford over a contiguous chunk, Chan merge in a
+// fixed tree inside the block.  out[(j*nb + b)*3 + {0,1,2}] = (count, mean, M2).
+__device__ __forceinline__ void chan_merge(double& na, double& ma, double& m2a, double nb, double mb, double m2b) {
+  if (nb == 0.0) return;
+  if (na == 0.0) {
+    na = nb; ma = mb; m2a = m2b;
+    return;
+  }
+  const double n = na + nb;
+  const double delta = mb - ma;
+  ma = ma + delta * (nb / n);
+  m2a = m2a + m2b + delta * delta * (na * nb / n);
+  na = n;
+}
+
+__global__ void moments_partial_kernel(const float* __restrict__ cols, int64_t ld, int64_t n, int64_t chunk,
+                                       double* __restrict__ out) {
+  const int j = blockIdx.y, b = blockIdx.x, nb = gridDim.x;
+  const int64_t a0 = (int64_t)b * chunk;
+  const int64_t a1 = min(n, a0 + chunk);
+  double cnt = 0.0, mean = 0.0, m2 = 0.0;
+  for (int64_t i = a0 + threadIdx.x; i < a1; i += blockDim.x) {
+    const double x = (double)cols[(int64_t)j * ld + i];
+    cnt += 1.0;
+    const double delta = x - mean;
+    mean += delta / cnt;
+    m2 += delta * (x - mean);
+  }
+  __shared__ double sc[256], sm[256], s2[256];
+  sc[threadIdx.x] = cnt; sm[threadIdx.x] = mean; s2[threadIdx.x] = m2;
+  __syncthreads();
+  for (int o = blockDim.x / 2; o > 0; o >>= 1) {
+    if (threadIdx.x < o) {
+      double na = sc[threadIdx.x], ma = sm[threadIdx.x], m2a = s2[threadIdx.x];
+      chan_merge(na, ma, m2a, sc[threadIdx.x + o], sm[threadIdx.x + o], s2[threadIdx.x + o]);
+      sc[threadIdx.x] = na; sm[threadIdx.x] = ma; s2[threadIdx.x] = m2a;
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    double* o = out + ((int64_t)j * nb + b) * 3;
+    o[0] = sc[0]; o[1] = sm[0]; o[2] = s2[0];
+  }
+}
+
+// Sequential Chan merge of np partials per column (fixed order) -> mom[j*3..].
+__global__ void moments_merge_kernel(const double* __restrict__ part, int np, int d, double* __restrict__ mom) {
+  const int j = threadIdx.x;
+  if (j >= d) return;
+  double na = 0.0, ma = 0.0, m2a = 0.0;
+  for (int b = 0; b < np; ++b) {
+    const double* p = part + ((int64_t)j * np + b) * 3;
+    chan_merge(na, ma, m2a, p[0], p[1], p[2]);
+  }
+  mom[j * 3 + 0] = na; mom[j * 3 + 1] = ma; mom[j * 3 + 2] = m2a;
+}
+
+// Merge per-rank moments gathered as [rank][d][3] in rank order.
+__global__ void moments_merge_ranks_kernel(const double* __restrict__ g, int world, int d, double* __restrict__ mom) {
+  const int j = threadIdx.x;
+  if (j >= d) return;
+  double na = 0.0, ma = 0.0, m2a = 0.0;
+  for (int r = 0; r < world; ++r) {
+    const double* p = g + ((int64_t)r * d + j) * 3;
+    chan_merge(na, ma, m2a, p[0], p[1], p[2]);
+  }
+  mom[j * 3 + 0] = na; mom[j * 3 + 1] = ma; mom[j * 3 + 2] = m2a;
+}
+
+__device__ void set_consts_dev(DevConsts* c, int j, double h) {
+  const double kSqrtLog2e = 1.2011224087864498;  // sqrt(log2 e)
+  const double kSqrtPi = 1.7724538509055160273;
+  const double kSqrt2 = 1.4142135623730950488;
+  c->h[j] = h;
+  c->ap[j] = (float)(kSqrtLog2e / (kSqrt2 * h));
+  c->gconst[j] = 1.0 / (kSqrtPi * kSqrtLog2e * h);
+}
+
+// eq. (3): h_j = s^(-1/(d+4)) sigma_j, population sigma.
+__global__ void scott_kernel(const double* __restrict__ mom, int d, DevConsts* c, int* bad) {
+  const int j = threadIdx.x;
+  if (j >= d) return;
+  const double n = mom[j * 3 + 0];
+  const double sigma = sqrt(mom[j * 3 + 2] / n);
+  const double h = pow(n, -1.0 / (d + 4.0)) * sigma;
+  if (!(h >= 1e-30 && h <= 1e30)) *bad = 1;  // e.g. a constant column
+  set_consts_dev(c, j, h);
+}
+
+__global__ void set_consts_kernel(HVec hv, int d, DevConsts* c) {
+  const int j = threadIdx.x;
+  if (j < d) set_consts_dev(c, j, hv.v[j]);
+}
+
+// ------------------------------------------------------------ reductions
+// sums[qi][k] = sum_{s in split order} partials[(s*NA + k)*q + qi]; with
+// finalisation (world == 1): est[qi] = S_0/N, dpdh[qi][j] = S_j gconst_j / N.
+__global__ void reduce_splits_kernel(const double* __restrict__ partials, int splits, int64_t q, int na,
+                                     double* __restrict__ sums) {
+  const int64_t qi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (qi >= q) return;
+  for (int k = 0; k < na; ++k) {
+    double t = 0.0;
+    for (int s = 0; s < splits; ++s) t += partials[((int64_t)s * na + k) * q + qi];
+    sums[qi * na + k] = t;
+  }
+}
+
+// gathered[r][q][na] summed in rank order -> sums[q][na]
+__global__ void combine_ranks_kernel(const double* __restrict__ gathered, int world, int64_t q, int na,
+                                     double* __restrict__ sums) {
+  const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (e >= q * na) return;
+  double t = 0.0;
+  for (int r = 0; r < world; ++r) t += gathered[(int64_t)r * q * na + e];
+  sums[e] = t;
+}
+
+__global__ void finalize_kernel(const double* __restrict__ sums, int64_t q, int d, int na, const DevConsts* c,
+                                double n_global, double* __restrict__ est, double* __restrict__ dpdh) {
+  const int64_t qi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (qi >= q) return;
+  est[qi] = sums[qi * na] / n_global;
+  if (dpdh && na > 1)
+    for (int j = 0; j < d; ++j) dpdh[qi * d + j] = sums[qi * na + 1 + j] * c->gconst[j] / n_global;
+}
+
+// ------------------------------------------------------------ losses (Appendix C.1)
+__device__ __forceinline__ double sgn3(double a, double b) { return a < b ? -1.0 : (a > b ? 1.0 : 0.0); }
+
+__device__ void loss_eval(int kind, double lambda, double phat, double p, double* L, double* dL) {
+  switch (kind) {
+    case 0: *L = (phat - p) * (phat - p); *dL = 2.0 * (phat - p); break;
+    case 1: *L = fabs(phat - p); *dL = sgn3(phat, p); break;
+    case 2: *L = fabs(phat - p) / (lambda + p); *dL = sgn3(phat, p) / (lambda + p); break;
+    case 3: {
+      const double r = (phat - p) / (lambda + p);
+      *L = r * r;
+      *dL = 2.0 * r / (lambda + p);  // reading R7: true derivative of the printed loss
+    } break;
+    default: {
+      const double r = log(lambda + phat) - log(lambda + p);
+      *L = r * r;
+      *dL = 2.0 * r / (lambda + phat);
+    }
+  }
+}
+
+// eq. (5): loss = (1/q) sum L_k; eq. (14): grad_j = (1/q) sum L'_k dp_k/dh_j;
+// eq. (18): x h_j in log mode.  One block, fixed strided order + fixed tree.
+__global__ void loss_epilogue_kernel(const double* __restrict__ est, const double* __restrict__ dpdh,
+                                     const double* __restrict__ true_sel, int64_t q, int d, int kind, double lambda,
+                                     int log_bw, const DevConsts* c, double* __restrict__ loss_out,
+                                     double* __restrict__ grad_out) {
+  constexpr int T = 512;
+  __shared__ double red[T / 32][kMaxDim + 1];
+  double acc[kMaxDim + 1];
+  for (int k = 0; k <= d; ++k) acc[k] = 0.0;
+  for (int64_t qi = threadIdx.x; qi < q; qi += T) {
+    double L, dL;
+    loss_eval(kind, lambda, est[qi], true_sel[qi], &L, &dL);
+    acc[0] += L;
+    for (int j = 0; j < d; ++j) acc[1 + j] += dL * dpdh[qi * d + j];
+  }
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  for (int k = 0; k <= d; ++k) {
+    double v = acc[k];
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if (lane == 0) red[warp][k] = v;
+  }
+  __syncthreads();
+  if (threadIdx.x <= d) {
+    double t = 0.0;
+    for (int w = 0; w < T / 32; ++w) t += red[w][threadIdx.x];
+    t /= (double)q;
+    if (threadIdx.x == 0) {
+      *loss_out = t;
+    } else {
+      const int j = threadIdx.x - 1;
+      grad_out[j] = log_bw ? t * c->h[j] : t;
+    }
+  }
+}
+
+// ------------------------------------------------------------ karma
+// Each block owns a contiguous range of kKarmaPts points, visited in ascending
+// order (pass-major, thread-minor), so the flag bitmap words are in index order.
+// eq. (19)-(20) threshold computed per block in fp64 from (lo, hi, h).
+__device__ double thr20_dev(const float* lo, const float* hi, int d, const DevConsts* c) {
+  const double kSqrt2 = 1.4142135623730950488;
+  double pmax = 1.0, best = 0.0;
+  for (int j = 0; j < d; ++j) {
+    const double w = (double)hi[j] - (double)lo[j];
+    if (!(w > 0.0)) return CUDART_INF;  // zero width: shortcut disabled (reading R5)
+    const double half = erf(w / (2.0 * kSqrt2 * c->h[j]));
+    const double full = erf(w / (kSqrt2 * c->h[j]));
+    pmax *= half;
+    const double ratio = isinf(w) ? 1.0 : full / half;
+    best = fmax(best, ratio);
+  }
+  return pmax / 2.0 * best;
+}
+
+__global__ void karma_kernel(const float* __restrict__ cvals, double* __restrict__ karma, int64_t n, double n_global,
+                             const double* __restrict__ phat_ptr, double p, KarmaParamsDev kp, const float* lo,
+                             const float* hi, int d, const DevConsts* c, uint32_t* __restrict__ bitmap,
+                             int32_t* __restrict__ block_counts) {
+  __shared__ double thr_s;
+  __shared__ int32_t wcount[kKarmaThreads / 32];
+  if (threadIdx.x == 0) thr_s = (kp.empty_region && p == 0.0) ? thr20_dev(lo, hi, d, c) : CUDART_INF;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  if (lane == 0) wcount[warp] = 0;
+  __syncthreads();
+  const double phat = *phat_ptr;
+  double L_full, dummy;
+  loss_eval(kp.loss, kp.lambda, phat, p, &L_full, &dummy);
+  const double thr = thr_s;
+  const int64_t base = (int64_t)blockIdx.x * kKarmaPts;
+  int32_t my = 0;
+#pragma unroll 1
+  for (int pass = 0; pass < kKarmaPts / kKarmaThreads; ++pass) {
+    const int64_t i = base + pass * kKarmaThreads + threadIdx.x;
+    bool flag = false;
+    if (i < n) {
+      const double ci = (double)cvals[i];
+      const double p_minus = (phat * n_global - ci) / (n_global - 1.0);  // eq. (6)
+      double L_minus;
+      loss_eval(kp.loss, kp.lambda, p_minus, p, &L_minus, &dummy);
+      const double k = fmin(karma[i] + (L_minus - L_full), kp.k_max);  // eq. (7)-(8)
+      karma[i] = k;
+      flag = (k < kp.threshold) || (ci >= thr);
+    }
+    const uint32_t word = __ballot_sync(0xffffffffu, flag);
+    if (lane == 0) {
+      bitmap[(i - threadIdx.x + warp * 32) / 32] = word;
+      my += __popc(word);
+    }
+  }
+  if (lane == 0) wcount[warp] = my;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int32_t t = 0;
+    for (int w = 0; w < kKarmaThreads / 32; ++w) t += wcount[w];
+    block_counts[blockIdx.x] = t;
+  }
+}
+
+// exclusive scan of block counts (single block, fixed order); offsets[nb] = total
+__global__ void scan_counts_kernel(const int32_t* __restrict__ counts, int nb, int64_t* __restrict__ offsets) {
+  __shared__ int64_t part[1024];
+  const int T = blockDim.x;
+  const int per = (nb + T - 1) / T;
+  const int a0 = threadIdx.x * per, a1 = min(nb, a0 + per);
+  int64_t s = 0;
+  for (int b = a0; b < a1; ++b) s += counts[b];
+  part[threadIdx.x] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int64_t run = 0;
+    for (int t = 0; t < T; ++t) {
+      const int64_t v = part[t];
+      part[t] = run;
+      run += v;
+    }
+    offsets[nb] = run;
+  }
+  __syncthreads();
+  int64_t run = part[threadIdx.x];
+  for (int b = a0; b < a1; ++b) {
+    offsets[b] = run;
+    run += counts[b];
+  }
+}
+
+// write ascending global indices (row_offset + i), at most cap of them
+__global__ void compact_kernel(const uint32_t* __restrict__ bitmap, int64_t n, const int64_t* __restrict__ offsets,
+                               int64_t row_offset, int64_t* __restrict__ idx_out, int64_t cap) {
+  constexpr int W = kKarmaPts / 32;  // bitmap words per block
+  __shared__ int32_t wpre[W];
+  const int64_t wbase = (int64_t)blockIdx.x * W;
+  const int64_t nwords = (n + 31) / 32;
+  if (threadIdx.x == 0) {
+    int32_t run = 0;
+    for (int w = 0; w < W; ++w) {
+      wpre[w] = run;
+      if (wbase + w < nwords) run += __popc(bitmap[wbase + w]);
+    }
+  }
+  __syncthreads();
+  const int64_t off = offsets[blockIdx.x];
+  for (int w = threadIdx.x / 32; w < W; w += blockDim.x / 32) {
+    if (wbase + w >= nwords) break;
+    const uint32_t word = bitmap[wbase + w];
+    const int lane = threadIdx.x & 31;
+    if (word & (1u << lane)) {
+      const int64_t pos = off + wpre[w] + __popc(word & ((1u << lane) - 1u));
+      if (pos < cap) idx_out[pos] = row_offset + (wbase + w) * 32 + lane;
+    }
+  }
+}
+
+// ------------------------------------------------------------ online bandwidth (Listing 1, reconstructed)
+// ret: [1+d] = (p_hat, dp/dh_j) of the retained query.  Adds L' dp/dh (x h in
+// log mode, eq. 18) to the mini-batch; every `minibatch` queries applies the
+// RMSprop / Rprop step of P:L179-183 and re-derives the constants.
+__global__ void online_update_kernel(const double* __restrict__ ret, double p, OnlineParamsDev op, int d,
+                                     OnlineState* st, DevConsts* c) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  double L, dL;
+  loss_eval(op.loss, op.lambda, ret[0], p, &L, &dL);
+  for (int j = 0; j < d; ++j) {
+    double g = dL * ret[1 + j];
+    if (op.log_bw) g *= c->h[j];
+    st->acc[j] += g;
+  }
+  st->count += 1;
+  st->updated = 0;
+  if (st->count < op.minibatch) return;
+  for (int j = 0; j < d; ++j) {
+    const double g = st->acc[j] / (double)op.minibatch;           // line 12
+    st->ms[j] = op.alpha * st->ms[j] + (1.0 - op.alpha) * g * g;   // line 14
+    if (g * st->gprev[j] > 0.0) {                                  // lines 15-16
+      st->lr[j] = fmin(st->lr[j] * op.lr_inc, op.lr_max);
+    } else if (g * st->gprev[j] < 0.0) {
+      st->lr[j] = fmax(st->lr[j] * op.lr_dec, op.lr_min);
+    }
+    double step = st->ms[j] > 0.0 ? st->lr[j] * g / sqrt(st->ms[j]) : 0.0;  // line 17
+    double h = c->h[j];
+    if (op.log_bw) {
+      h = exp(log(h) - step);
+    } else {
+      if (step > h / 2.0) step = h / 2.0;  // positivity safeguard
+      h = h - step;
+    }
+    set_consts_dev(c, j, h);
+    st->gprev[j] = g;
+    st->acc[j] = 0.0;
+  }
+  st->count = 0;
+  st->updated = 1;
+}
+
+// ------------------------------------------------------------ harness: exact box counts
+// counts[k] = |{r : l_kj < R_rj < u_kj for all j}|, open box as in P:L45.
+__global__ void count_in_box_kernel(const float* __restrict__ rows, int64_t n, int d, const float* __restrict__ lo,
+                                    const float* __restrict__ hi, int64_t q, int64_t rows_per_block,
+                                    unsigned long long* __restrict__ counts) {
+  const int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t r0 = (int64_t)blockIdx.y * rows_per_block;
+  const int64_t r1 = min(n, r0 + rows_per_block);
+  __shared__ float tile[256 * kMaxDim];
+  float l[kMaxDim], u[kMaxDim];
+  const int64_t kk = k < q ? k : q - 1;
+  for (int j = 0; j < d; ++j) {
+    l[j] = lo[kk * d + j];
+    u[j] = hi[kk * d + j];
+  }
+  unsigned long long cnt = 0;
+  for (int64_t t0 = r0; t0 < r1; t0 += 256) {
+    const int m = (r1 - t0) < 256 ? (int)(r1 - t0) : 256;
+    __syncthreads();
+    for (int e = threadIdx.x; e < m * d; e += blockDim.x) tile[e] = rows[t0 * d + e];
+    __syncthreads();
+    for (int r = 0; r < m; ++r) {
+      bool in = true;
+      for (int j = 0; j < d; ++j) {
+        const float x = tile[r * d + j];
+        in = in && (x > l[j]) && (x < u[j]);
+      }
+      cnt += in ? 1ull : 0ull;
+    }
+  }
+  if (k < q && cnt) atomicAdd(counts + k, cnt);
+}
+
+// ------------------------------------------------------------ launchers
+#define KDE_LAUNCH_CHECK() return cudaGetLastError()
+
+cudaError_t launch_rows_to_cols(const float* rows, int64_t n, int d, float* cols, int64_t ld, int* bad,
+                                cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  rows_to_cols_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(rows, n, d, cols, ld, bad);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_cols_to_rows(const float* cols, int64_t ld, int64_t n, int d, float* rows, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  cols_to_rows_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(cols, ld, n, d, rows);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_scatter_rows(const int64_t* idx_local, const float* rows, int64_t k, int d, float* cols,
+                                int64_t ld, double* karma, double k_init, cudaStream_t s) {
+  if (k == 0) return cudaSuccess;
+  scatter_rows_kernel<<<(unsigned)((k + 255) / 256), 256, 0, s>>>(idx_local, rows, k, d, cols, ld, karma, k_init);
+  KDE_LAUNCH_CHECK();
+}
+int moments_blocks(int64_t n) {
+  int64_t nb = (n + 65535) / 65536;
+  if (nb < 1) nb = 1;
+  if (nb > 1024) nb = 1024;
+  return (int)nb;
+}
+cudaError_t launch_moments(const float* cols, int64_t ld, int64_t n, int d, double* part, double* mom,
+                           cudaStream_t s) {
+  const int nb = moments_blocks(n);
+  const int64_t chunk = (n + nb - 1) / nb;
+  moments_partial_kernel<<<dim3(nb, d), 256, 0, s>>>(cols, ld, n, chunk, part);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  moments_merge_kernel<<<1, 32, 0, s>>>(part, nb, d, mom);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_moments_merge_ranks(const double* g, int world, int d, double* mom, cudaStream_t s) {
+  moments_merge_ranks_kernel<<<1, 32, 0, s>>>(g, world, d, mom);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_scott(const double* mom, int d, DevConsts* c, int* bad, cudaStream_t s) {
+  scott_kernel<<<1, 32, 0, s>>>(mom, d, c, bad);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_set_consts(const double* h, int d, DevConsts* c, cudaStream_t s) {
+  HVec hv;
+  for (int j = 0; j < d; ++j) hv.v[j] = h[j];
+  set_consts_kernel<<<1, 32, 0, s>>>(hv, d, c);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_reduce_splits(const double* partials, int splits, int64_t q, int na, double* sums,
+                                 cudaStream_t s) {
+  reduce_splits_kernel<<<(unsigned)((q + 255) / 256), 256, 0, s>>>(partials, splits, q, na, sums);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_combine_ranks(const double* gathered, int world, int64_t q, int na, double* sums,
+                                 cudaStream_t s) {
+  const int64_t e = q * na;
+  combine_ranks_kernel<<<(unsigned)((e + 255) / 256), 256, 0, s>>>(gathered, world, q, na, sums);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_finalize(const double* sums, int64_t q, int d, int na, const DevConsts* c, double n_global,
+                            double* est, double* dpdh, cudaStream_t s) {
+  finalize_kernel<<<(unsigned)((q + 255) / 256), 256, 0, s>>>(sums, q, d, na, c, n_global, est, dpdh);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const double* true_sel, int64_t q, int d,
+                                 int kind, double lambda, int log_bw, const DevConsts* c, double* loss_out,
+                                 double* grad_out, cudaStream_t s) {
+  loss_epilogue_kernel<<<1, 512, 0, s>>>(est, dpdh, true_sel, q, d, kind, lambda, log_bw, c, loss_out, grad_out);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, double p,
+                         const KarmaParamsDev& kp, const float* lo, const float* hi, int d, const DevConsts* c,
+                         uint32_t* bitmap, int32_t* block_counts, int64_t* offsets, int64_t row_offset,
+                         int64_t* idx_out, int64_t cap, cudaStream_t s) {
+  const int nb = karma_blocks(n);
+  if (nb == 0) return cudaSuccess;
+  karma_kernel<<<nb, kKarmaThreads, 0, s>>>(cvals, karma, n, n_global, phat, p, kp, lo, hi, d, c, bitmap,
+                                            block_counts);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  scan_counts_kernel<<<1, 1024, 0, s>>>(block_counts, nb, offsets);
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  compact_kernel<<<nb, kKarmaThreads, 0, s>>>(bitmap, n, offsets, row_offset, idx_out, cap);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_online_update(const double* ret, double p, const OnlineParamsDev& op, int d, OnlineState* st,
+                                 DevConsts* c, cudaStream_t s) {
+  online_update_kernel<<<1, 32, 0, s>>>(ret, p, op, d, st, c);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_count_in_box(const float* rows, int64_t n, int d, const float* lo, const float* hi, int64_t q,
+                                unsigned long long* counts, int num_sms, cudaStream_t s) {
+  if (q == 0 || n == 0) return cudaSuccess;
+  const int64_t qb = (q + 255) / 256;
+  int64_t rb = (num_sms * 8 + qb - 1) / qb;
+  const int64_t maxrb = (n + 255) / 256;
+  if (rb > maxrb) rb = maxrb;
+  if (rb < 1) rb = 1;
+  int64_t rows_per_block = (n + rb - 1) / rb;
+  rows_per_block = (rows_per_block + 255) / 256 * 256;
+  rb = (n + rows_per_block - 1) / rows_per_block;
+  count_in_box_kernel<<<dim3((unsigned)qb, (unsigned)rb), 256, 0, s>>>(rows, n, d, lo, hi, q, rows_per_block, counts);
+  KDE_LAUNCH_CHECK();
+}
+
+}  // namespace kde

@@ -1,0 +1,47 @@
+// kernels.cuh -- launchers for the non-scan kernels (kernels.cu).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "common.cuh"
+
+namespace kde {
+
+constexpr int kKarmaThreads = 256;
+constexpr int kKarmaPts = 2048;  // contiguous points per karma block (8 passes)
+inline int karma_blocks(int64_t n) { return (int)((n + kKarmaPts - 1) / kKarmaPts); }
+
+struct HVec {
+  double v[kMaxDim];
+};
+
+cudaError_t launch_rows_to_cols(const float* rows, int64_t n, int d, float* cols, int64_t ld, int* bad,
+                                cudaStream_t s);
+cudaError_t launch_cols_to_rows(const float* cols, int64_t ld, int64_t n, int d, float* rows, cudaStream_t s);
+cudaError_t launch_scatter_rows(const int64_t* idx_local, const float* rows, int64_t k, int d, float* cols,
+                                int64_t ld, double* karma, double k_init, cudaStream_t s);
+int moments_blocks(int64_t n);
+cudaError_t launch_moments(const float* cols, int64_t ld, int64_t n, int d, double* part, double* mom,
+                           cudaStream_t s);
+cudaError_t launch_moments_merge_ranks(const double* g, int world, int d, double* mom, cudaStream_t s);
+cudaError_t launch_scott(const double* mom, int d, DevConsts* c, int* bad, cudaStream_t s);
+cudaError_t launch_set_consts(const double* h, int d, DevConsts* c, cudaStream_t s);
+cudaError_t launch_reduce_splits(const double* partials, int splits, int64_t q, int na, double* sums,
+                                 cudaStream_t s);
+cudaError_t launch_combine_ranks(const double* gathered, int world, int64_t q, int na, double* sums,
+                                 cudaStream_t s);
+cudaError_t launch_finalize(const double* sums, int64_t q, int d, int na, const DevConsts* c, double n_global,
+                            double* est, double* dpdh, cudaStream_t s);
+cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const double* true_sel, int64_t q, int d,
+                                 int kind, double lambda, int log_bw, const DevConsts* c, double* loss_out,
+                                 double* grad_out, cudaStream_t s);
+cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, double p,
+                         const KarmaParamsDev& kp, const float* lo, const float* hi, int d, const DevConsts* c,
+                         uint32_t* bitmap, int32_t* block_counts, int64_t* offsets, int64_t row_offset,
+                         int64_t* idx_out, int64_t cap, cudaStream_t s);
+cudaError_t launch_online_update(const double* ret, double p, const OnlineParamsDev& op, int d, OnlineState* st,
+                                 DevConsts* c, cudaStream_t s);
+cudaError_t launch_count_in_box(const float* rows, int64_t n, int d, const float* lo, const float* hi, int64_t q,
+                                unsigned long long* counts, int num_sms, cudaStream_t s);
+
+}  // namespace kde

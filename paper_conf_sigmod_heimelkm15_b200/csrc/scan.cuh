@@ -1,0 +1,354 @@
+// scan.cuh -- the hot path: one pass over the sample computing, per box,
+//   S_0   = sum_i p^(i)(Omega)                         eq. (2)+(13)
+//   S_j   = sum_i w_ij prod_{k!=j} D_ik                eq. (17), P:L545 (d p^(i)/d h_j = gconst_j S_j-term)
+// and optionally the retained per-point contributions p^(i).
+//
+// scan_single_kernel  (q == 1): HBM-streaming reduction.  Each thread owns
+//   float4 chunks of the SoA columns (coalesced 128-bit loads, streaming cache
+//   hint), fp32 math per point, fp32 sums over 8 points flushed to fp64,
+//   warp-shuffle + block reduction, and a deterministic last-block second pass
+//   (fixed order) that also finalises p_hat and dp_hat/dh.
+// scan_batched_kernel (q > 1): FP32/SFU-bound.  A CTA owns 256*QT boxes (QT per
+//   thread, bounds in registers) and one contiguous split of the sample; sample
+//   tiles of 256 points x d columns are staged into shared memory by TMA bulk
+//   copies (cp.async.bulk + mbarrier, double buffered) and read as broadcasts.
+//   fp32 sums over 32 points are flushed into per-thread fp64 accumulators in
+//   shared memory; per-(split, box) partials go to global memory and are
+//   reduced in fixed split order by reduce_splits_kernel (kernels.cu).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "common.cuh"
+#include "phi.cuh"
+
+namespace kde {
+
+template <int D>
+struct QT_for {
+  static constexpr int value = D <= 3 ? 4 : (D <= 6 ? 2 : 1);
+};
+
+constexpr int kSingleThreads = 256;
+constexpr int kBatchedThreads = 256;
+constexpr int kTilePts = 256;  // points per shared-memory tile
+constexpr int kFlushPts = 32;  // fp32 partial sums are flushed to fp64 every kFlushPts points
+
+__device__ __forceinline__ float f4c(const float4& v, int p) {
+  return p == 0 ? v.x : (p == 1 ? v.y : (p == 2 ? v.z : v.w));
+}
+
+// All d factors of eq. (13) for one point and one box, the product p^(i), and
+// (GRAD) the d gradient terms w_j prod_{k!=j} D_k, added into s[0..D].
+// Returns p^(i).  `valid` masks padding points (contributes exactly 0).
+template <int D, bool GRAD>
+__device__ __forceinline__ float point_box(const float2 (&ul)[D], const float (&t)[D], const float (&ap)[D],
+                                           float* s, bool valid) {
+  float Dv[D], wv[D];
+#pragma unroll
+  for (int j = 0; j < D; ++j) Dv[j] = phi_diff<GRAD>(ul[j], t[j], ap[j], wv[j]);
+  float pre[D + 1];
+  pre[0] = 1.0f;
+#pragma unroll
+  for (int j = 0; j < D; ++j) pre[j + 1] = pre[j] * Dv[j];
+  const float c = valid ? pre[D] : 0.0f;
+  s[0] += c;
+  if (GRAD) {
+    float suf = valid ? 1.0f : 0.0f;
+#pragma unroll
+    for (int j = D - 1; j >= 0; --j) {
+      s[1 + j] = fmaf(wv[j], pre[j] * suf, s[1 + j]);
+      suf *= Dv[j];
+    }
+  }
+  return c;
+}
+
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// ---------------------------------------------------------------- single box
+template <int D, bool GRAD>
+__device__ __forceinline__ void single_group(const float4 (&tv)[D], const float2 (&ul)[D], const float (&ap)[D],
+                                             float* s, float* c_out, int64_t v, int valid) {
+  float cs[4];
+#pragma unroll
+  for (int p = 0; p < 4; ++p) {
+    float t[D];
+#pragma unroll
+    for (int j = 0; j < D; ++j) t[j] = f4c(tv[j], p);
+    cs[p] = point_box<D, GRAD>(ul, t, ap, s, p < valid);
+  }
+  if (c_out) __stcs(reinterpret_cast<float4*>(c_out) + v, make_float4(cs[0], cs[1], cs[2], cs[3]));
+}
+
+template <int D, bool GRAD>
+__global__ void __launch_bounds__(kSingleThreads, (D <= 8 ? 3 : 2)) scan_single_kernel(const ScanSingleArgs a) {
+  constexpr int NA = GRAD ? D + 1 : 1;
+  float2 ul[D];
+  float ap[D];
+#pragma unroll
+  for (int j = 0; j < D; ++j) {
+    ul[j] = make_float2(__ldg(a.hi + j), __ldg(a.lo + j));
+    ap[j] = a.consts->ap[j];
+  }
+  double acc[NA];
+#pragma unroll
+  for (int k = 0; k < NA; ++k) acc[k] = 0.0;
+
+  const float4* col = reinterpret_cast<const float4*>(a.cols);
+  const int64_t ld4 = a.ld >> 2;
+  const int64_t nfull = a.n >> 2;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  int64_t v = gtid;
+  // two float4 groups (8 points) per iteration: 2*d 16-byte loads in flight
+  for (; v + stride < nfull; v += 2 * stride) {
+    float4 t0[D], t1[D];
+#pragma unroll
+    for (int j = 0; j < D; ++j) t0[j] = __ldcs(col + j * ld4 + v);
+#pragma unroll
+    for (int j = 0; j < D; ++j) t1[j] = __ldcs(col + j * ld4 + v + stride);
+    float s[NA];
+#pragma unroll
+    for (int k = 0; k < NA; ++k) s[k] = 0.0f;
+    single_group<D, GRAD>(t0, ul, ap, s, a.c_out, v, 4);
+    single_group<D, GRAD>(t1, ul, ap, s, a.c_out, v + stride, 4);
+#pragma unroll
+    for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
+  }
+  // at most one more full group, then the ragged tail group (n % 4 points)
+  for (; v <= nfull; v += stride) {
+    const int valid = v < nfull ? 4 : (int)(a.n - 4 * nfull);
+    if (valid == 0) break;
+    float4 t0[D];
+#pragma unroll
+    for (int j = 0; j < D; ++j) t0[j] = __ldcs(col + j * ld4 + v);
+    float s[NA];
+#pragma unroll
+    for (int k = 0; k < NA; ++k) s[k] = 0.0f;
+    single_group<D, GRAD>(t0, ul, ap, s, a.c_out, v, valid);
+#pragma unroll
+    for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
+  }
+
+  // block reduction (fixed order)
+  __shared__ double red[kSingleThreads / 32][NA];
+  __shared__ bool am_last;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+#pragma unroll
+  for (int k = 0; k < NA; ++k) {
+    const double r = warp_sum(acc[k]);
+    if (lane == 0) red[warp][k] = r;
+  }
+  __syncthreads();
+  if (threadIdx.x < NA) {
+    double t = 0.0;
+#pragma unroll
+    for (int w = 0; w < kSingleThreads / 32; ++w) t += red[w][threadIdx.x];
+    a.block_partials[(int64_t)blockIdx.x * NA + threadIdx.x] = t;
+    __threadfence();
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) am_last = (atomicAdd(a.counter, 1u) == gridDim.x - 1);
+  __syncthreads();
+  if (!am_last) return;
+  __threadfence();
+  // deterministic second pass over the block partials (fixed strided order + fixed tree)
+  for (int k = 0; k < NA; ++k) {
+    double t = 0.0;
+    for (int b = threadIdx.x; b < (int)gridDim.x; b += kSingleThreads) t += __ldcg(a.block_partials + (int64_t)b * NA + k);
+    t = warp_sum(t);
+    __syncthreads();
+    if (lane == 0) red[warp][0] = t;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      double tot = 0.0;
+#pragma unroll
+      for (int w = 0; w < kSingleThreads / 32; ++w) tot += red[w][0];
+      a.sums_out[k] = tot;
+      if (a.fin_out) a.fin_out[k] = k == 0 ? tot / a.n_global : tot * a.consts->gconst[k - 1] / a.n_global;
+    }
+  }
+  if (threadIdx.x == 0) *a.counter = 0u;
+}
+
+// ---------------------------------------------------------------- many boxes
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "KDE_WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra KDE_WAIT_%=;\n\t}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+template <int D, bool GRAD>
+constexpr size_t batched_smem_bytes() {
+  constexpr int QT = QT_for<D>::value;
+  constexpr int NA = GRAD ? D + 1 : 1;
+  return 2ull * D * kTilePts * sizeof(float) + (size_t)QT * NA * kBatchedThreads * sizeof(double) + 16;
+}
+
+template <int D, bool GRAD>
+__global__ void __launch_bounds__(kBatchedThreads, (D <= 8 ? 2 : 1)) scan_batched_kernel(const ScanBatchedArgs a) {
+  constexpr int QT = QT_for<D>::value;
+  constexpr int NA = GRAD ? D + 1 : 1;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  float* tile = reinterpret_cast<float*>(smem_raw);                                   // [2][D][kTilePts]
+  double* accsh = reinterpret_cast<double*>(smem_raw + 2ull * D * kTilePts * sizeof(float));  // [QT*NA][threads]
+  uint64_t* bar = reinterpret_cast<uint64_t*>(reinterpret_cast<unsigned char*>(accsh) +
+                                              (size_t)QT * NA * kBatchedThreads * sizeof(double));
+  const int tid = threadIdx.x;
+
+  // this CTA's boxes: qi = qbase + qq*256 + tid (consecutive threads -> consecutive boxes)
+  const int64_t qbase = (int64_t)blockIdx.x * kBatchedThreads * QT;
+  float2 ul[QT][D];
+  float ap[D];
+#pragma unroll
+  for (int j = 0; j < D; ++j) ap[j] = a.consts->ap[j];
+#pragma unroll
+  for (int qq = 0; qq < QT; ++qq) {
+    int64_t qi = qbase + qq * kBatchedThreads + tid;
+    if (qi >= a.q) qi = a.q - 1;  // duplicate a valid box; its partial is never written
+#pragma unroll
+    for (int j = 0; j < D; ++j) ul[qq][j] = make_float2(__ldg(a.hi + qi * D + j), __ldg(a.lo + qi * D + j));
+  }
+#pragma unroll
+  for (int k = 0; k < QT * NA; ++k) accsh[k * kBatchedThreads + tid] = 0.0;
+
+  const int64_t s0 = (int64_t)blockIdx.y * a.split_len;
+  const int64_t s1 = min(a.n, s0 + a.split_len);
+  const int ntiles = (int)((s1 - s0 + kTilePts - 1) / kTilePts);
+  if (tid == 0) {
+    mbar_init(&bar[0], 1);
+    mbar_init(&bar[1], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  auto issue = [&](int k) {
+    const int buf = k & 1;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    mbar_arrive_expect_tx(&bar[buf], (uint32_t)(D * kTilePts * sizeof(float)));
+#pragma unroll
+    for (int j = 0; j < D; ++j)
+      bulk_g2s(tile + (buf * D + j) * kTilePts, a.cols + (int64_t)j * a.ld + s0 + (int64_t)k * kTilePts,
+               (uint32_t)(kTilePts * sizeof(float)), &bar[buf]);
+  };
+  if (tid == 0 && ntiles > 0) issue(0);
+
+  for (int k = 0; k < ntiles; ++k) {
+    const int buf = k & 1;
+    if (tid == 0 && k + 1 < ntiles) issue(k + 1);  // buffer buf^1 was released by the barrier ending tile k-1
+    mbar_wait_parity(&bar[buf], (uint32_t)((k >> 1) & 1));
+    const float* tl = tile + buf * D * kTilePts;
+    const int64_t rem = s1 - (s0 + (int64_t)k * kTilePts);
+    const int npts = rem < kTilePts ? (int)rem : kTilePts;
+    for (int p0 = 0; p0 < npts; p0 += kFlushPts) {
+      const int pe = min(p0 + kFlushPts, npts);
+      float s[QT][NA];
+#pragma unroll
+      for (int qq = 0; qq < QT; ++qq)
+#pragma unroll
+        for (int kk = 0; kk < NA; ++kk) s[qq][kk] = 0.0f;
+      for (int p = p0; p < pe; ++p) {
+        float t[D];
+#pragma unroll
+        for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
+#pragma unroll
+        for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD>(ul[qq], t, ap, s[qq], true);
+      }
+#pragma unroll
+      for (int qq = 0; qq < QT; ++qq)
+#pragma unroll
+        for (int kk = 0; kk < NA; ++kk) accsh[(qq * NA + kk) * kBatchedThreads + tid] += (double)s[qq][kk];
+    }
+    __syncthreads();
+  }
+
+  // partials[(split*(NA) + comp) * q + qi]
+#pragma unroll
+  for (int qq = 0; qq < QT; ++qq) {
+    const int64_t qi = qbase + qq * kBatchedThreads + tid;
+    if (qi < a.q) {
+#pragma unroll
+      for (int kk = 0; kk < NA; ++kk)
+        a.partials[((int64_t)blockIdx.y * NA + kk) * a.q + qi] = accsh[(qq * NA + kk) * kBatchedThreads + tid];
+    }
+  }
+}
+
+// ---------------------------------------------------------------- launchers
+template <int D>
+cudaError_t launch_single_t(bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s) {
+  if (grad)
+    scan_single_kernel<D, true><<<grid, kSingleThreads, 0, s>>>(a);
+  else
+    scan_single_kernel<D, false><<<grid, kSingleThreads, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+template <int D, bool GRAD>
+cudaError_t launch_batched_tg(const ScanBatchedArgs& a, dim3 grid, cudaStream_t s) {
+  constexpr size_t smem = batched_smem_bytes<D, GRAD>();
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(scan_batched_kernel<D, GRAD>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)smem);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  scan_batched_kernel<D, GRAD><<<grid, kBatchedThreads, smem, s>>>(a);
+  return cudaGetLastError();
+}
+
+// Grid for the batched scan: query tiles x sample splits, sized to ~8 CTAs
+// per SM (4 waves at 2 resident CTAs/SM); split_len is a tile multiple.
+template <int D>
+cudaError_t launch_batched_t(bool grad, const ScanBatchedArgs& a_in, int num_sms, int* splits_out, cudaStream_t s,
+                             bool dry_run) {
+  constexpr int QT = QT_for<D>::value;
+  ScanBatchedArgs a = a_in;
+  const int64_t qtiles = (a.q + (int64_t)kBatchedThreads * QT - 1) / ((int64_t)kBatchedThreads * QT);
+  const int64_t ntile_pts = (a.n + kTilePts - 1) / kTilePts;
+  const int64_t target = (int64_t)num_sms * 8;
+  int64_t splits = (target + qtiles - 1) / qtiles;
+  if (splits > ntile_pts) splits = ntile_pts;
+  if (splits < 1) splits = 1;
+  int64_t split_len = ((a.n + splits - 1) / splits + kTilePts - 1) / kTilePts * kTilePts;
+  if (split_len < kTilePts) split_len = kTilePts;
+  splits = (a.n + split_len - 1) / split_len;
+  if (splits < 1) splits = 1;
+  if (splits_out) *splits_out = (int)splits;
+  if (dry_run) return cudaSuccess;
+  a.split_len = split_len;
+  dim3 grid((unsigned)qtiles, (unsigned)splits);
+  return grad ? launch_batched_tg<D, true>(a, grid, s) : launch_batched_tg<D, false>(a, grid, s);
+}
+
+}  // namespace kde
+
+#define KDE_INSTANTIATE_SCAN(D)                                                                              \
+  namespace kde {                                                                                            \
+  template cudaError_t launch_single_t<D>(bool, const ScanSingleArgs&, int, cudaStream_t);                   \
+  template cudaError_t launch_batched_t<D>(bool, const ScanBatchedArgs&, int, int*, cudaStream_t, bool);     \
+  }

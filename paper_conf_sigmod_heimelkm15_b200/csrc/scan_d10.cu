@@ -1,0 +1,3 @@
+// Explicit instantiation of the scan kernels for d = 10 (see scan.cuh).
+#include "scan.cuh"
+KDE_INSTANTIATE_SCAN(10)

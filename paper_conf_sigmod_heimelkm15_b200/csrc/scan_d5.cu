@@ -1,0 +1,3 @@
+// Explicit instantiation of the scan kernels for d = 5 (see scan.cuh).
+#include "scan.cuh"
+KDE_INSTANTIATE_SCAN(5)

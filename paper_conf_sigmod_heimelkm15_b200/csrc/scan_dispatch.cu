@@ -1,0 +1,45 @@
+// scan_dispatch.cu -- runtime d -> template D dispatch for the scan kernels.
+#include "scan.cuh"
+
+namespace kde {
+
+#define KDE_DECL(D)                                                                                    \
+  extern template cudaError_t launch_single_t<D>(bool, const ScanSingleArgs&, int, cudaStream_t);      \
+  extern template cudaError_t launch_batched_t<D>(bool, const ScanBatchedArgs&, int, int*, cudaStream_t, bool);
+KDE_DECL(1) KDE_DECL(2) KDE_DECL(3) KDE_DECL(4) KDE_DECL(5) KDE_DECL(6) KDE_DECL(7) KDE_DECL(8)
+KDE_DECL(9) KDE_DECL(10) KDE_DECL(11) KDE_DECL(12) KDE_DECL(13) KDE_DECL(14) KDE_DECL(15) KDE_DECL(16)
+#undef KDE_DECL
+
+#define KDE_CASES(X) X(1) X(2) X(3) X(4) X(5) X(6) X(7) X(8) X(9) X(10) X(11) X(12) X(13) X(14) X(15) X(16)
+
+cudaError_t launch_scan_single(int d, bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s) {
+  switch (d) {
+#define X(D) case D: return launch_single_t<D>(grad, a, grid, s);
+    KDE_CASES(X)
+#undef X
+  }
+  return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int num_sms, int* splits_out,
+                                cudaStream_t s, bool dry_run) {
+  switch (d) {
+#define X(D) case D: return launch_batched_t<D>(grad, a, num_sms, splits_out, s, dry_run);
+    KDE_CASES(X)
+#undef X
+  }
+  return cudaErrorInvalidValue;
+}
+
+// ~3 resident CTAs of 256 threads per SM, never more CTAs than 8-point work items.
+int scan_single_grid(int d, int64_t n, int num_sms) {
+  const int per_sm = d <= 8 ? 3 : 2;
+  int64_t grid = (int64_t)num_sms * per_sm;
+  const int64_t items = (n + 7) / 8;
+  const int64_t need = (items + kSingleThreads - 1) / kSingleThreads;
+  if (grid > need) grid = need;
+  if (grid < 1) grid = 1;
+  return (int)grid;
+}
+
+}  // namespace kde

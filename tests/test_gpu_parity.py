@@ -1,0 +1,388 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle on the
+same seeded inputs.  Tolerances (north star):
+  selectivities  |gpu - oracle| <= 1e-7 + 1e-5 |oracle|
+  gradients      |gpu - oracle| <= 1e-4 |oracle| + 1e-4 m_j,
+                 m_j = eq. (17) with per-point terms in absolute value (oracle)
+  karma / indices  bit-exact flag sets outside a documented guard band.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+
+K = pytest.importorskip("paper_conf_sigmod_heimelkm15_b200")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _need_cuda():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    oracle.set_threads(0)
+
+
+def sel_ok(gpu, ora):
+    gpu, ora = np.asarray(gpu), np.asarray(ora)
+    err = np.abs(gpu - ora)
+    tol = 1e-7 + 1e-5 * np.abs(ora)
+    bad = np.nonzero(err > tol)
+    assert err.shape == ora.shape
+    assert len(bad[0]) == 0, f"{len(bad[0])} selectivities out of tolerance; worst {np.max(err / tol):.3g}x " \
+                             f"(gpu {gpu[bad][:4]}, oracle {ora[bad][:4]})"
+
+
+def grad_ok(gpu, ora, scale):
+    gpu, ora, scale = np.asarray(gpu), np.asarray(ora), np.asarray(scale)
+    err = np.abs(gpu - ora)
+    tol = 1e-4 * np.abs(ora) + 1e-4 * scale
+    bad = np.nonzero(err > tol)
+    assert len(bad[0]) == 0, f"{len(bad[0])} gradients out of tolerance; worst {np.max(err / np.maximum(tol, 1e-300)):.3g}x"
+
+
+def model(S, h=None):
+    return K.KDEModel.create(S, h)
+
+
+def boxes_mix(S, q, seed):
+    lo1, hi1 = synth.random_boxes(S, q, seed)
+    lo2, hi2 = synth.special_boxes(S, seed)
+    return np.concatenate([lo1, lo2]), np.concatenate([hi1, hi2])
+
+
+# ------------------------------------------------------------------ C1
+def test_c1_scott_estimates_gradients_both_paths():
+    """configs[0]: d=2, N=1024 G-A sample, 100 random boxes, Scott h (eq. 3)."""
+    S = synth.make_data("gauss", 1024, 2, seed=1)
+    lo, hi = synth.random_boxes(S, 100, seed=2)
+    m = model(S)
+    h_gpu = m.bandwidth
+    h_ora = oracle.scott(S)
+    assert np.allclose(h_gpu, h_ora, rtol=1e-12, atol=0)
+    est_o, g_o = oracle.estimate_grad(S, h_gpu, lo, hi)
+    mabs = oracle.grad_abs_scale(S, h_gpu, lo, hi)
+    est_b, g_b = m.estimate(lo, hi, grad=True)          # batched kernel
+    sel_ok(est_b, est_o)
+    grad_ok(g_b, g_o, mabs)
+    est_only = m.estimate(lo, hi)                        # estimate-only variant
+    sel_ok(est_only, est_o)
+    for k in range(0, 100, 7):                           # single-box streaming kernel
+        e1, g1 = m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+        sel_ok(e1, est_o[k:k + 1])
+        grad_ok(g1, g_o[k:k + 1], mabs[k:k + 1])
+
+
+# ------------------------------------------------------------------ shapes
+@pytest.mark.parametrize("d", [1, 2, 3, 4, 5, 7, 8, 10, 13, 16])
+@pytest.mark.parametrize("n", [2, 5, 1027, 70001])
+def test_dims_and_ragged_sizes(d, n):
+    """Every template width, tail groups (n % 4), partial tiles, multi-split grids."""
+    S = synth.make_data("gauss", n, d, seed=10 + d)
+    g = synth.rng(d, n)
+    h = oracle.scott(S) * g.uniform(0.5, 2.0, d) if n > 2 else np.full(d, 3.0)
+    lo, hi = boxes_mix(S, 24, seed=d * 100 + n % 97)
+    m = model(S, h)
+    est_o, g_o = oracle.estimate_grad(S, h, lo, hi)
+    mabs = oracle.grad_abs_scale(S, h, lo, hi)
+    est, gr = m.estimate(lo, hi, grad=True)
+    sel_ok(est, est_o)
+    grad_ok(gr, g_o, mabs)
+    for k in (0, 3, 5, len(lo) - 1):
+        e1, g1 = m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+        sel_ok(e1, est_o[k:k + 1])
+        grad_ok(g1, g_o[k:k + 1], mabs[k:k + 1])
+        e0 = m.estimate(lo[k:k + 1], hi[k:k + 1])
+        sel_ok(e0, est_o[k:k + 1])
+
+
+@pytest.mark.parametrize("kind", ["rect", "skew"])
+def test_other_data_shapes(kind):
+    """G-B rectangles with uniform interiors; G-C heavy tails, ties, 1e4 offset."""
+    S = synth.make_data(kind, 20000, 5, seed=3)
+    h = oracle.scott(S)
+    lo, hi = synth.mixed_workload(S, 64, seed=4)
+    m = model(S)
+    assert np.allclose(m.bandwidth, h, rtol=1e-11)
+    est_o, g_o = oracle.estimate_grad(S, h, lo, hi)
+    mabs = oracle.grad_abs_scale(S, h, lo, hi)
+    est, gr = m.estimate(lo, hi, grad=True)
+    sel_ok(est, est_o)
+    grad_ok(gr, g_o, mabs)
+
+
+# ------------------------------------------------------------------ special cases
+def test_unbounded_box_is_exactly_one_and_empty_interval_zero():
+    S = synth.make_data("gauss", 5003, 6, seed=5)
+    m = model(S)
+    inf = np.float32(np.inf)
+    lo = np.array([[-inf] * 6, S[0]], np.float32)
+    hi = np.array([[inf] * 6, S[0]], np.float32)
+    est, g = m.estimate(lo, hi, grad=True)
+    assert est[0] == 1.0 and np.all(g[0] == 0.0)
+    assert est[1] == 0.0 and np.all(g[1] == 0.0)
+    e1, g1 = m.estimate(lo[:1], hi[:1], grad=True)
+    assert e1[0] == 1.0 and np.all(g1 == 0.0)
+
+
+def test_small_bandwidth_degrades_to_exact_count():
+    """h -> 0 counts points in the box (exact in fp32 when every point is >= 10h from the faces)."""
+    g = synth.rng(6)
+    S = g.integers(-50, 50, size=(30000, 3)).astype(np.float32)
+    h = np.full(3, 0.01)
+    lo = np.array([[-20.5, -10.5, -30.5], [0.5, 0.5, 0.5]], np.float32)
+    hi = np.array([[15.5, 30.5, 5.5], [10.5, 40.5, 20.5]], np.float32)
+    m = model(S, h)
+    est = m.estimate(lo, hi)
+    cnt = [np.all((S > lo[k]) & (S < hi[k]), axis=1).sum() for k in range(2)]
+    assert est[0] == cnt[0] / len(S) and est[1] == cnt[1] / len(S)
+    assert m.estimate(lo[:1], hi[:1])[0] == cnt[0] / len(S)
+
+
+def test_large_offset_data():
+    """Subtract-then-scale argument formation keeps accuracy for data offset by 1e4."""
+    S = (synth.make_data("gauss", 40000, 3, seed=7) + np.float32(1e4)).astype(np.float32)
+    lo, hi = synth.mixed_workload(S, 32, seed=8)
+    m = model(S)
+    h = m.bandwidth
+    sel_ok(m.estimate(lo, hi), oracle.estimate(S, h, lo, hi))
+
+
+# ------------------------------------------------------------------ losses
+@pytest.mark.parametrize("kind", range(5))
+@pytest.mark.parametrize("log_bw", [False, True])
+def test_loss_and_grad_all_losses(kind, log_bw):
+    S = synth.make_data("gauss", 30000, 4, seed=9)
+    lo, hi = synth.mixed_workload(S, 96, seed=10)
+    R = synth.make_data("gauss", 60000, 4, seed=9)
+    p = synth.true_selectivity_cpu(R, lo, hi)
+    lam = 1e-3
+    m = model(S)
+    h = m.bandwidth
+    L_o, g_o, est_o = oracle.loss_and_grad(S, h, lo, hi, p, kind, lam, log_bw)
+    L_g, g_g, est_g = m.loss_and_grad(lo, hi, p, kind, lam, log_bw, return_est=True)
+    sel_ok(est_g, est_o)
+    dL = np.array([abs(oracle.loss(kind, lam, e, pp)[1]) for e, pp in zip(est_o, p)])
+    mabs = oracle.grad_abs_scale(S, h, lo, hi)
+    scale = (dL[:, None] * mabs).mean(axis=0) * (h if log_bw else 1.0)
+    grad_ok(g_g, g_o, scale)
+    # loss tolerance propagated from the selectivity tolerance
+    Ltol = np.mean(dL * (1e-7 + 1e-5 * np.abs(est_o))) * 2 + 1e-12
+    assert abs(L_g - L_o) <= Ltol + 1e-9 * abs(L_o)
+    # single-box path of the same entry point
+    L1, g1 = m.loss_and_grad(lo[:1], hi[:1], p[:1], kind, lam, log_bw)
+    L1o, g1o, _ = oracle.loss_and_grad(S, h, lo[:1], hi[:1], p[:1], kind, lam, log_bw)
+    grad_ok(g1, g1o, dL[0] * mabs[0] * (h if log_bw else 1.0))
+
+
+# ------------------------------------------------------------------ karma
+def _karma_guard(K_ora, tau, c_ora, thr, n):
+    amb = np.abs(K_ora - tau) < 1e-6 / (n - 1) + 1e-9 * np.abs(tau)
+    if np.isfinite(thr):
+        amb |= np.abs(c_ora - thr) < 1e-6 * thr
+    return amb
+
+
+@pytest.mark.parametrize("loss", [K.LOSS_ABSOLUTE, K.LOSS_SQUARED, K.LOSS_RELATIVE])
+def test_karma_update_lockstep(loss):
+    """eq. (6)-(8) + P:L250 flags over a sequence of queries, compared in lockstep."""
+    n, d = 5000, 3
+    S = synth.make_data("gauss", n, d, seed=11)
+    R = synth.make_data("gauss", 50000, d, seed=12)
+    lo, hi = synth.mixed_workload(S, 12, seed=13)
+    lo = np.concatenate([lo, [[200, 200, 200]]]).astype(np.float32)  # an empty region
+    hi = np.concatenate([hi, [[300, 300, 300]]]).astype(np.float32)
+    p = synth.true_selectivity_cpu(R, lo, hi)
+    p[3] = 0.0  # true selectivity 0 on a populated box: exercises eq. (20)
+    lam = 1e-3
+    tau = -1.0 / (n - 1) if loss != K.LOSS_RELATIVE else -0.5
+    m = model(S)
+    m.set_retain(True)
+    h = m.bandwidth
+    kp = K.karma_params(loss=loss, lam=lam, k_max=4.0, threshold=tau, empty_region=True)
+    Kora = np.zeros(n)
+    total_amb = 0
+    for k in range(len(lo)):
+        m.karma = Kora  # lockstep: same pre-step state
+        est = m.estimate(lo[k:k + 1], hi[k:k + 1])
+        idx, nf, trunc = m.karma_update(lo[k], hi[k], p[k], kp)
+        assert not trunc and nf == len(idx)
+        assert np.all(np.diff(idx) > 0)
+        c_o = oracle.contributions(S, h, lo[k], hi[k])
+        thr, _ = oracle.empty_region_threshold(h, lo[k], hi[k]) if p[k] == 0 else (np.inf, 0)
+        Kora_new = Kora.copy()
+        idx_o = oracle.karma_update(c_o, c_o.mean(), p[k], loss, lam, 4.0, tau, thr, Kora_new)
+        Kg = m.karma
+        # karma values: difference driven by the fp32 contributions only
+        dK_scale = np.abs(Kora_new - Kora) + 1.0 / (n - 1)
+        assert np.all(np.abs(Kg - Kora_new) <= 1e-4 * dK_scale + 1e-12)
+        amb = _karma_guard(Kora_new, tau, c_o, thr, n)
+        total_amb += amb.sum()
+        fg = np.zeros(n, bool); fg[idx] = True
+        fo = np.zeros(n, bool); fo[idx_o] = True
+        assert np.array_equal(fg[~amb], fo[~amb]), f"query {k}: flag sets differ"
+        Kora = Kora_new
+    assert total_amb < 5
+
+
+def test_karma_truncation_and_retained_vs_rescan():
+    n, d = 4000, 2
+    S = synth.make_data("gauss", n, d, seed=14)
+    m = model(S)
+    lo = np.array([-1e6, -1e6], np.float32)
+    hi = np.array([1e6, 1e6], np.float32)
+    kp = K.karma_params(loss=K.LOSS_ABSOLUTE, threshold=1.0)  # everyone below 1 -> all flagged
+    idx, nf, trunc = m.karma_update(lo, hi, 0.5, kp, cap=100)
+    assert trunc and nf == n and np.array_equal(idx, np.arange(100))
+    # retained (estimate with retain) and rescanned paths give identical karma
+    m2 = model(S)
+    m2.set_retain(True)
+    m2.estimate(lo[None], hi[None])
+    m3 = model(S)
+    a = m2.karma_update(lo, hi, 0.3, kp)[0]
+    b = m3.karma_update(lo, hi, 0.3, kp)[0]
+    assert np.array_equal(a, b) and np.array_equal(m2.karma, m3.karma)
+
+
+# ------------------------------------------------------------------ replace / reservoir
+def test_replace_points_then_estimate():
+    n, d = 3000, 4
+    S = synth.make_data("gauss", n, d, seed=15)
+    m = model(S)
+    h = m.bandwidth
+    m.karma = np.full(n, 2.5)
+    idx = np.array([5, 0, 2999, 1234], np.int64)
+    rows = synth.make_data("gauss", 4, d, seed=16)
+    m.replace_points(idx, rows, k_init=0.0)
+    S2 = S.copy()
+    S2[idx] = rows
+    assert np.array_equal(m.sample, S2)
+    kk = m.karma
+    assert np.all(kk[idx] == 0.0) and np.sum(kk == 2.5) == n - 4
+    lo, hi = synth.mixed_workload(S2, 16, seed=17)
+    sel_ok(m.estimate(lo, hi), oracle.estimate(S2, h, lo, hi))
+    with pytest.raises(K.KDEError):
+        m.replace_points(np.array([1, 1]), rows[:2])
+    with pytest.raises(K.KDEError):
+        m.replace_points(np.array([n]), rows[:1])
+    assert np.array_equal(m.sample, S2)  # state unchanged after EINVAL
+
+
+# ------------------------------------------------------------------ online bandwidth (Listing 1)
+def test_online_update_lockstep():
+    """Reconstructed Listing 1 (PARITY UNPINNED by the paper): GPU step == oracle step from the same state."""
+    n, d = 8000, 3
+    S = synth.make_data("gauss", n, d, seed=18)
+    R = synth.make_data("gauss", 40000, d, seed=19)
+    lo, hi = synth.mixed_workload(S, 40, seed=20)
+    p = synth.true_selectivity_cpu(R, lo, hi)
+    m = model(S)
+    op = K.online_params(minibatch=5, log_bandwidth=True, loss=K.LOSS_SQUARED)
+    st = oracle.OnlineState(d, lr0=op.lr0)
+    for k in range(len(lo)):
+        h = m.bandwidth
+        # lockstep: oracle starts from the GPU's state
+        gs = m.online_state()
+        st.acc, st.ms, st.lr, st.gprev, st.count = gs["acc"].copy(), gs["ms"].copy(), gs["lr"].copy(), \
+            gs["gprev"].copy(), gs["count"]
+        _, g_o, _ = oracle.loss_and_grad(S, h, lo[k:k + 1], hi[k:k + 1], p[k:k + 1], 0, 0.0, True)
+        h_o = h.copy()
+        upd_o = oracle.online_step(st, h_o, g_o, batch=5, log_bw=True)
+        upd = m.online_update(lo[k], hi[k], p[k], op)
+        assert upd == upd_o
+        assert np.allclose(m.bandwidth, h_o, rtol=1e-4, atol=0)
+
+
+# ------------------------------------------------------------------ determinism, errors
+def test_bitwise_determinism():
+    S = synth.make_data("gauss", 200000, 5, seed=21)
+    lo, hi = synth.mixed_workload(S, 700, seed=22)
+    m = model(S)
+    a = m.estimate(lo, hi, grad=True)
+    b = m.estimate(lo, hi, grad=True)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+    s1 = m.estimate(lo[:1], hi[:1], grad=True)
+    s2 = m.estimate(lo[:1], hi[:1], grad=True)
+    assert np.array_equal(s1[0], s2[0]) and np.array_equal(s1[1], s2[1])
+
+
+def test_invalid_arguments_leave_state_unchanged():
+    S = synth.make_data("gauss", 1000, 2, seed=23)
+    m = model(S)
+    h0 = m.bandwidth
+    bad = [
+        lambda: m.estimate(np.array([[1, 0]], np.float32), np.array([[0, 1]], np.float32)),   # lo > hi
+        lambda: m.estimate(np.array([[np.nan, 0]], np.float32), np.array([[1, 1]], np.float32)),
+        lambda: K.kde_set_bandwidth(m.handle, [1.0, -1.0]),
+        lambda: m.loss_and_grad(np.zeros((1, 2)), np.ones((1, 2)), [1.5]),                      # p > 1
+        lambda: m.loss_and_grad(np.zeros((1, 2)), np.ones((1, 2)), [0.5], loss=K.LOSS_RELATIVE, lam=0.0),
+        lambda: K.kde_create(np.array([[0, np.inf], [1, 1]], np.float32)),
+    ]
+    for f in bad:
+        with pytest.raises(K.KDEError) as e:
+            f()
+        assert e.value.status == K.KDE_EINVAL
+    assert np.array_equal(m.bandwidth, h0)
+    lo, hi = synth.random_boxes(S, 5, seed=24)
+    sel_ok(m.estimate(lo, hi), oracle.estimate(S, h0, lo, hi))
+
+
+def test_virtual_shards_combine_to_full_estimate():
+    """Shard arithmetic on one GPU: G world-1 shard models over row blocks with
+    n_global = N give partial estimates whose sum is the full estimate."""
+    from paper_conf_sigmod_heimelkm15_b200.dist import shard_range
+    n, d, G = 50001, 4, 3
+    S = synth.make_data("gauss", n, d, seed=25)
+    h = oracle.scott(S)
+    lo, hi = synth.mixed_workload(S, 40, seed=26)
+    tot = np.zeros(len(lo))
+    for r in range(G):
+        off, k = shard_range(n, r, G)
+        hd = K.kde_create_sharded(S[off:off + k], off, n, h, None, 0, 1)
+        try:
+            tot += K.kde_estimate_batch(hd, lo, hi, d)
+        finally:
+            K.kde_destroy(hd)
+    sel_ok(tot, oracle.estimate(S, h, lo, hi))
+
+
+# ------------------------------------------------------------------ full-size sampled parity
+def test_c3_full_size_single_and_batched_sampled():
+    """configs[2]: d=5, N=2^24 G-A; single DT queries and a 4096-box batch
+    (DT/DV/UT/UV mix) in the bench launch configuration, sampled against the oracle."""
+    n, d = 1 << 24, 5
+    S = synth.make_data("gauss", n, d, seed=27)
+    m = model(S)
+    h = m.bandwidth
+    lo, hi = synth.mixed_workload(S, 4096, seed=28)
+    est, g = m.estimate(lo, hi, grad=True)
+    pick = np.array([0, 1, 1000, 4095])
+    est_o, g_o = oracle.estimate_grad(S, h, lo[pick], hi[pick])
+    mabs = oracle.grad_abs_scale(S, h, lo[pick], hi[pick])
+    sel_ok(est[pick], est_o)
+    grad_ok(g[pick], g_o, mabs)
+    for k in pick[:2]:
+        e1, g1 = m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+        assert abs(e1[0] - est[k]) <= 1e-12 + 1e-9 * est[k]
+    assert np.all(est >= 0) and np.all(est <= 1.0 + 1e-12)
+
+
+def test_c2_full_size_loss_grad_sampled():
+    """configs[1]: d=3, N=2^20, 10k boxes: loss/grad consistent with the per-box
+    estimates; a 64-box subset matches the oracle's loss and gradient."""
+    n, d = 1 << 20, 3
+    S = synth.make_data("gauss", n, d, seed=29)
+    lo, hi = synth.mixed_workload(S, 10000, seed=30)
+    p = synth.rng(31).uniform(0, 0.05, size=10000)
+    m = model(S)
+    h = m.bandwidth
+    L, g, est = m.loss_and_grad(lo, hi, p, K.LOSS_SQUARED, 0.0, False, return_est=True)
+    assert abs(L - np.mean((est - p) ** 2)) <= 1e-12 * max(L, 1e-30) + 1e-18
+    sub = np.arange(0, 10000, 157)[:64]
+    L_o, g_o, est_o = oracle.loss_and_grad(S, h, lo[sub], hi[sub], p[sub], 0, 0.0, False)
+    sel_ok(est[sub], est_o)
+    Ls, gs = m.loss_and_grad(lo[sub], hi[sub], p[sub], K.LOSS_SQUARED, 0.0, False)
+    dL = 2 * np.abs(est_o - p[sub])
+    mabs = oracle.grad_abs_scale(S, h, lo[sub], hi[sub])
+    grad_ok(gs, g_o, (dL[:, None] * mabs).mean(axis=0))
