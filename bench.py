@@ -50,8 +50,13 @@ CONFIGS = {
                desc="configs[1]: d=3, N=2^20/GPU, 10k-box batch, estimate + L2 loss + bandwidth gradient"),
     "c3": dict(d=5, n=1 << 24, q=4096, path="loss_grad", data="gauss",
                desc="configs[2] batched: d=5, N=2^24/GPU, 4096-box DT/DV/UT/UV batch, estimate + gradient"),
-    "c3s": dict(d=5, n=1 << 24, q=1, path="single", data="gauss",
-                desc="configs[2] single box: d=5, N=2^24/GPU, one DT box per step (HBM-streaming scan)"),
+    "c3s": dict(d=5, n=1 << 24, q=1, path="single", grad=False, retain=False, data="gauss",
+                desc="configs[2] single box: d=5, N=2^24/GPU, one DT box per step, estimate (HBM-streaming scan)"),
+    "c3sg": dict(d=5, n=1 << 24, q=1, path="single", grad=True, retain=False, data="gauss",
+                 desc="configs[2] single box: d=5, N=2^24/GPU, one DT box per step, estimate + bandwidth gradient"),
+    "c5s": dict(d=10, n=1 << 22, q=1, path="single", grad=True, retain=True, data="gauss",
+                desc="configs[4] estimate step: d=10, N=2^22/GPU, one DT box, estimate + gradient + retained "
+                     "contributions (Adaptive, P:L240)"),
     "c4": dict(d=8, n=1 << 25, q=4096, path="loss_grad", data="gauss",
                desc="configs[3] per-GPU shard: d=8, 2^25 rows/GPU (2^28 at 8 GPUs), 4096 boxes, estimate + gradient + NCCL"),
 }
@@ -253,10 +258,14 @@ def run_cuda(args, cfg, rank, world, local_rank):
     flush_l2 = cfg["n"] * d * 4 < 2 * l2  # sample smaller than ~2x L2 -> flush between timed steps
     nbox = len(lo)
 
+    if cfg.get("retain"):
+        m.set_retain(True)
+
     def step(i):
         if cfg["path"] == "single":
             k = i % nbox
-            K.kde_estimate_batch_dev(m.handle, d_lo[k:k + 1], d_hi[k:k + 1], d_est[:1], d_dpdh[:1], stream=stream)
+            K.kde_estimate_batch_dev(m.handle, d_lo[k:k + 1], d_hi[k:k + 1], d_est[:1],
+                                     d_dpdh[:1] if cfg.get("grad") else None, stream=stream)
         else:
             K.kde_loss_and_grad_dev(m.handle, d_lo, d_hi, d_true, d_loss, d_grad, K.LOSS_SQUARED, 0.0, False,
                                     stream=stream)
@@ -304,7 +313,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
     for i in range(e2e_steps):
         if cfg["path"] == "single":
             k = i % nbox
-            m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+            m.estimate(lo[k:k + 1], hi[k:k + 1], grad=bool(cfg.get("grad")))
         else:
             m.loss_and_grad(lo, hi, p, K.LOSS_SQUARED, 0.0, False)
     torch.cuda.synchronize()
@@ -314,7 +323,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     e2e_s = float(t.item())
     if cfg["path"] == "single":
-        h2d, d2h = 2 * d * 4, 8 * (1 + d)
+        h2d, d2h = 2 * d * 4, 8 * (1 + (d if cfg.get("grad") else 0))
     else:
         h2d, d2h = 2 * q * d * 4 + q * 8, 8 * (1 + d)
 
@@ -325,12 +334,12 @@ def run_cuda(args, cfg, rank, world, local_rank):
     avg_scan_ms = scan_ms / max(scan_launches, 1)
     sms = torch.cuda.get_device_properties(dev).multi_processor_count
     if cfg["path"] == "single":
-        alg_bytes = n * d * 4  # 4d bytes per point read once (SoA fp32)
+        alg_bytes = n * d * 4 + (n * 4 if cfg.get("retain") else 0)  # 4d B/point read (+4 B/point retained c)
         achieved = alg_bytes / (avg_scan_ms * 1e-3) / 1e9
         peak = _measured_hbm()
         roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": _traffic(args.config), "kernel": f"scan_single_kernel<{d}>",
-                "algorithmic": f"4*d bytes/point x {n} points per launch",
+                "traffic": _traffic(args.config), "kernel": f"scan_single_kernel<{d},{'grad' if cfg.get('grad') else 'est'}>",
+                "algorithmic": f"4*d bytes/point{' + 4 B/point retained' if cfg.get('retain') else ''} x {n} points per launch",
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
     else:
         achieved = n * q / (avg_scan_ms * 1e-3) / 1e9

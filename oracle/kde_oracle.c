@@ -126,9 +126,13 @@ void oracle_estimate_grad(const float *sample, int64_t n, int32_t d, const doubl
     }
 }
 
-/* Gradient magnitude scale used by the parity tolerance (test infrastructure):
- *   m_ij = sqrt2 / (sqrtpi h_i^2 2^d s) * sum_j | [bracket of eq. 17] * prod_{k != i} [...] |
- * i.e. eq. (17) with every per-point term taken in absolute value. */
+/* Gradient magnitude scale used by the parity tolerance (test infrastructure,
+ * not a paper quantity):
+ *   m_ij = sqrt2 / (sqrtpi h_i^2 2^d s) * sum_j ( |(l_i - t_i) e^{..}| + |(u_i - t_i) e^{..}| )
+ *                                             * | prod_{k != i} [...] |
+ * i.e. eq. (17) with both terms of the bracket and every per-point term taken
+ * in absolute value -- the condition-number scale of evaluating eq. (17) in
+ * finite precision (the bracket cancels when both bounds give equal terms). */
 void oracle_grad_abs_scale(const float *sample, int64_t n, int32_t d, const double *h,
                            const float *lo, const float *hi, int64_t q, double *mabs)
 {
@@ -142,14 +146,14 @@ void oracle_grad_abs_scale(const float *sample, int64_t n, int32_t d, const doub
             for (int32_t i = 0; i < d; ++i) {
                 double li = (double)l[i] - (double)t[i];
                 double ui = (double)u[i] - (double)t[i];
-                double bracket = xexp(li, h[i]) - xexp(ui, h[i]);
+                double bracket = fabs(xexp(li, h[i])) + fabs(xexp(ui, h[i]));
                 double prod = 1.0;
                 for (int32_t k = 0; k < d; ++k) {
                     if (k == i) continue;
                     prod *= erf(((double)u[k] - (double)t[k]) / (OR_SQRT2 * h[k]))
                           - erf(((double)l[k] - (double)t[k]) / (OR_SQRT2 * h[k]));
                 }
-                gsum[i] += fabs(bracket * prod);
+                gsum[i] += bracket * fabs(prod);
             }
         }
         for (int32_t i = 0; i < d; ++i)

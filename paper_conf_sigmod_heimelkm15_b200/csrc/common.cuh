@@ -78,6 +78,6 @@ struct ScanBatchedArgs {
 cudaError_t launch_scan_single(int d, bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s);
 cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int num_sms, int* splits_out,
                                 cudaStream_t s, bool dry_run);
-int scan_single_grid(int d, int64_t n, int num_sms);
+int scan_single_grid(int d, bool grad, int64_t n, int num_sms);
 
 }  // namespace kde

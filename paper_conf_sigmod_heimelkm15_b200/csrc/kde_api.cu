@@ -237,7 +237,7 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     a.sums_out = d_sums;
     a.fin_out = nullptr;
     a.n_global = (double)m->n_global;
-    const int grid = scan_single_grid(d, m->n, m->num_sms);
+    const int grid = scan_single_grid(d, grad, m->n, m->num_sms);
     cudaEvent_t e1 = nullptr, e2 = nullptr;
     kde_status pst = prof_begin(m, s, &e1, &e2);
     if (pst != KDE_OK) return pst;
@@ -975,6 +975,6 @@ extern "C" kde_status kde_count_in_box_dev(const float* d_rows, int64_t n, int32
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   cudaStream_t s = (cudaStream_t)stream;
   CU(cudaMemsetAsync(d_counts, 0, sizeof(int64_t) * q, s));
-  CUL(launch_count_in_box(d_rows, n, d, d_lo, d_hi, q, (unsigned long long*)d_counts, sms, s));
+  CU(launch_count_in_box(d_rows, n, d, d_lo, d_hi, q, (unsigned long long*)d_counts, sms, s));
   return KDE_OK;
 }

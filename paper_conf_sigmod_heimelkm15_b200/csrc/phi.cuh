@@ -39,16 +39,42 @@ __device__ __forceinline__ float rcp_approx(float x) {
 }
 __device__ __forceinline__ float2 f2(float a) { return make_float2(a, a); }
 
-// One dimension for one point and one box.
-//   ul = (u_j, l_j), t = t_ij, ap = sqrt(log2 e)/(sqrt2 h_j)
-// returns D_j; if GRAD, w = y'_l E_l - y'_u E_u  (so dD_j/dh_j = gconst_j * w).
+// ---------------------------------------------------------------------------
+// Per (box, dimension) evaluation setup, computed once per box.
+//   normal: b = (u, l), hd = 0           y = (b - t) * ap
+//   narrow: b = (l, l), hd = delta'/2    y = (l - t) * ap + hd (1 +- 1/sqrt3)
+// A dimension is "narrow" when its width in erf units dz = (u - l)/(sqrt2 h)
+// is below kNarrowZ: there the difference of two erf values (and of the two
+// gradient terms) cancels catastrophically in fp32, so the interval integral
+// of eq. (12) and the gradient integral are taken with 2-point Gauss-Legendre
+// on the same two exponentials (relative error < dz^4 / 360 (1 + z^4)).
+constexpr float kNarrowZ = 0.05f;
+constexpr float kNarrowY = kNarrowZ * kSqrtLog2e;          // threshold in y' units
+constexpr float kGaussC = 0.57735026918962576f;            // 1/sqrt(3)
+constexpr float kInvSqrtPiLog2e = 0.46971863934982566f;    // 1/(sqrt(pi) sqrt(log2 e))
+constexpr float kTwoLn2 = 1.3862943611198906f;
+
+struct BoxDim {
+  float2 b;   // (b1, b2) evaluation bounds
+  float hd;   // half-width in y' units for narrow dims, 0 otherwise
+};
+
+__device__ __forceinline__ BoxDim make_boxdim(float l, float u, float ap) {
+  BoxDim r;
+  const float dy = (u - l) * ap;  // inf for unbounded, NaN for (inf, inf): both normal
+  if (dy > 0.0f && dy < kNarrowY) {
+    r.b = make_float2(l, l);
+    r.hd = 0.5f * dy;
+  } else {
+    r.b = make_float2(u, l);
+    r.hd = 0.0f;
+  }
+  return r;
+}
+
+// erf-difference path: D = 1/2 [erf(z_u) - erf(z_l)], w = y'_l E_l - y'_u E_u
 template <bool GRAD>
-__device__ __forceinline__ float phi_diff(float2 ul, float t, float ap, float& w) {
-  float2 y = __fmul2_rn(__fadd2_rn(ul, f2(-t)), f2(ap));
-  y.x = fminf(fmaxf(y.x, -kYClamp), kYClamp);
-  y.y = fminf(fmaxf(y.y, -kYClamp), kYClamp);
-  const float2 yy = __fmul2_rn(y, y);
-  const float2 E = make_float2(ex2_approx(-yy.x), ex2_approx(-yy.y));
+__device__ __forceinline__ float phi_normal(const float2 y, const float2 E, float& w) {
   const float2 den = __ffma2_rn(make_float2(fabsf(y.x), fabsf(y.y)), f2(kPprime), f2(1.0f));
   const float2 t2 = make_float2(rcp_approx(den.x), rcp_approx(den.y));
   // Horner for Q(t)/2 (the 1/2 of eq. 13 folded into the coefficients)
@@ -56,12 +82,46 @@ __device__ __forceinline__ float phi_diff(float2 ul, float t, float ap, float& w
 #pragma unroll
   for (int k = KDE_PHI_DEG - 1; k >= 0; --k) q = __ffma2_rn(q, t2, f2(0.5f * kde_phi_q(k)));
   const float2 ch = __fmul2_rn(__fmul2_rn(q, t2), E);          // 1/2 erfc(|z|)
-  const float2 g = __ffma2_rn(ch, f2(-1.0f), f2(0.5f));        // 1/2 erf(|z|)
   if (GRAD) {
     const float2 yE = __fmul2_rn(y, E);
     w = yE.y - yE.x;
   }
-  return copysignf(g.x, y.x) - copysignf(g.y, y.y);
+  // 1/2 erf(z) = sgn(z) (1/2 - ch).  D = [1/2 sgn(z_u) - 1/2 sgn(z_l)] + [sgn(z_l) ch_l - sgn(z_u) ch_u]:
+  // the first bracket is exactly 0 or 1, so a box seen from one side keeps the
+  // full relative accuracy of the erfc tails (no 1/2 - ch rounding).
+  const float hs = copysignf(0.5f, y.x) - copysignf(0.5f, y.y);
+  const float cs = copysignf(ch.y, y.y) - copysignf(ch.x, y.x);
+  return hs + cs;
+}
+
+// narrow path: 2-point Gauss-Legendre on [y_l, y_u] (nodes y.x, y.y, weights hd)
+template <bool GRAD>
+__device__ __forceinline__ float phi_narrow(const float2 y, const float2 E, float hd, float& w) {
+  const float s = E.x + E.y;
+  if (GRAD) {
+    const float2 yy = __fmul2_rn(y, y);
+    w = -hd * (s - kTwoLn2 * fmaf(E.x, yy.x, E.y * yy.y));
+  }
+  return hd * kInvSqrtPiLog2e * s;
+}
+
+// One dimension of eq. (13) for one point and one box; GENERAL handles narrow
+// dimensions (a per-box uniform property), the fast variant assumes none.
+template <bool GRAD, bool GENERAL>
+__device__ __forceinline__ float phi_diff(const BoxDim& bd, float t, float ap, float& w) {
+  float2 y;
+  if (GENERAL) {
+    const float2 o = __fmul2_rn(f2(bd.hd), make_float2(1.0f + kGaussC, 1.0f - kGaussC));
+    y = __ffma2_rn(__fadd2_rn(bd.b, f2(-t)), f2(ap), o);
+  } else {
+    y = __fmul2_rn(__fadd2_rn(bd.b, f2(-t)), f2(ap));
+  }
+  y.x = fminf(fmaxf(y.x, -kYClamp), kYClamp);
+  y.y = fminf(fmaxf(y.y, -kYClamp), kYClamp);
+  const float2 yy = __fmul2_rn(y, y);
+  const float2 E = make_float2(ex2_approx(-yy.x), ex2_approx(-yy.y));
+  if (GENERAL && bd.hd > 0.0f) return phi_narrow<GRAD>(y, E, bd.hd, w);
+  return phi_normal<GRAD>(y, E, w);
 }
 
 }  // namespace kde

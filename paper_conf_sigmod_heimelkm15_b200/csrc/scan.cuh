@@ -33,6 +33,12 @@ constexpr int kSingleThreads = 256;
 constexpr int kBatchedThreads = 256;
 constexpr int kTilePts = 256;  // points per shared-memory tile
 constexpr int kFlushPts = 32;  // fp32 partial sums are flushed to fp64 every kFlushPts points
+constexpr int kSingleFlushPts = 16;  // single-box scan: fp32 partials flushed every 16 points
+
+// resident 256-thread CTAs per SM for the single-box scan (register budget)
+__host__ __device__ constexpr int single_occ(int d, bool grad) {
+  return grad ? (d <= 3 ? 4 : (d <= 6 ? 3 : (d <= 8 ? 2 : 1))) : (d <= 8 ? 4 : (d <= 14 ? 2 : 1));
+}
 
 __device__ __forceinline__ float f4c(const float4& v, int p) {
   return p == 0 ? v.x : (p == 1 ? v.y : (p == 2 ? v.z : v.w));
@@ -41,12 +47,12 @@ __device__ __forceinline__ float f4c(const float4& v, int p) {
 // All d factors of eq. (13) for one point and one box, the product p^(i), and
 // (GRAD) the d gradient terms w_j prod_{k!=j} D_k, added into s[0..D].
 // Returns p^(i).  `valid` masks padding points (contributes exactly 0).
-template <int D, bool GRAD>
-__device__ __forceinline__ float point_box(const float2 (&ul)[D], const float (&t)[D], const float (&ap)[D],
+template <int D, bool GRAD, bool GENERAL>
+__device__ __forceinline__ float point_box(const BoxDim (&bd)[D], const float (&t)[D], const float (&ap)[D],
                                            float* s, bool valid) {
   float Dv[D], wv[D];
 #pragma unroll
-  for (int j = 0; j < D; ++j) Dv[j] = phi_diff<GRAD>(ul[j], t[j], ap[j], wv[j]);
+  for (int j = 0; j < D; ++j) Dv[j] = phi_diff<GRAD, GENERAL>(bd[j], t[j], ap[j], wv[j]);
   float pre[D + 1];
   pre[0] = 1.0f;
 #pragma unroll
@@ -71,66 +77,117 @@ __device__ __forceinline__ double warp_sum(double v) {
 }
 
 // ---------------------------------------------------------------- single box
+// The box is uniform over the CTA: its per-dimension setup (b1, b2, hd, ap)
+// lives in shared memory and is re-read (broadcast LDS.128) per point group.
+// Each thread processes VW consecutive points per column load (VW-wide
+// vector loads, coalesced across the warp).
 template <int D, bool GRAD>
-__device__ __forceinline__ void single_group(const float4 (&tv)[D], const float2 (&ul)[D], const float (&ap)[D],
+struct SingleVW {
+  static constexpr int value = 2;
+};
+
+template <int VW>
+struct VecT;
+template <>
+struct VecT<2> {
+  using type = float2;
+};
+template <>
+struct VecT<4> {
+  using type = float4;
+};
+
+__device__ __forceinline__ float vcomp(const float2& v, int p) { return p == 0 ? v.x : v.y; }
+__device__ __forceinline__ float vcomp(const float4& v, int p) { return f4c(v, p); }
+__device__ __forceinline__ float2 ldcs_v(const float2* p) { return __ldcs(p); }
+__device__ __forceinline__ float4 ldcs_v(const float4* p) { return __ldcs(p); }
+__device__ __forceinline__ void stcs_v(float2* p, const float* c) { __stcs(p, make_float2(c[0], c[1])); }
+__device__ __forceinline__ void stcs_v(float4* p, const float* c) { __stcs(p, make_float4(c[0], c[1], c[2], c[3])); }
+
+template <int D, bool GRAD, bool GENERAL, int VW>
+__device__ __forceinline__ void single_group(const typename VecT<VW>::type (&tv)[D], const float4* __restrict__ smc,
                                              float* s, float* c_out, int64_t v, int valid) {
-  float cs[4];
+  float cs[VW];
 #pragma unroll
-  for (int p = 0; p < 4; ++p) {
-    float t[D];
+  for (int p = 0; p < VW; ++p) {
+    BoxDim bd[D];
+    float ap[D], t[D];
 #pragma unroll
-    for (int j = 0; j < D; ++j) t[j] = f4c(tv[j], p);
-    cs[p] = point_box<D, GRAD>(ul, t, ap, s, p < valid);
+    for (int j = 0; j < D; ++j) {
+      const float4 c = smc[j];
+      bd[j].b = make_float2(c.x, c.y);
+      bd[j].hd = c.z;
+      ap[j] = c.w;
+      t[j] = vcomp(tv[j], p);
+    }
+    cs[p] = point_box<D, GRAD, GENERAL>(bd, t, ap, s, p < valid);
   }
-  if (c_out) __stcs(reinterpret_cast<float4*>(c_out) + v, make_float4(cs[0], cs[1], cs[2], cs[3]));
+  if (c_out) stcs_v(reinterpret_cast<typename VecT<VW>::type*>(c_out) + v, cs);
 }
 
+template <int D, bool GRAD, bool GENERAL>
+__device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const float4* smc);
+
 template <int D, bool GRAD>
-__global__ void __launch_bounds__(kSingleThreads, (D <= 8 ? 3 : 2)) scan_single_kernel(const ScanSingleArgs a) {
-  constexpr int NA = GRAD ? D + 1 : 1;
-  float2 ul[D];
-  float ap[D];
-#pragma unroll
-  for (int j = 0; j < D; ++j) {
-    ul[j] = make_float2(__ldg(a.hi + j), __ldg(a.lo + j));
-    ap[j] = a.consts->ap[j];
+__global__ void __launch_bounds__(kSingleThreads, single_occ(D, GRAD)) scan_single_kernel(const ScanSingleArgs a) {
+  __shared__ float4 smc[D];
+  __shared__ int narrow_s;
+  if (threadIdx.x == 0) narrow_s = 0;
+  __syncthreads();
+  if (threadIdx.x < D) {
+    const int j = threadIdx.x;
+    const float ap = a.consts->ap[j];
+    const BoxDim bd = make_boxdim(__ldg(a.lo + j), __ldg(a.hi + j), ap);
+    smc[j] = make_float4(bd.b.x, bd.b.y, bd.hd, ap);
+    if (bd.hd > 0.0f) atomicOr(&narrow_s, 1);
   }
+  __syncthreads();
+  if (narrow_s)
+    scan_single_body<D, GRAD, true>(a, smc);
+  else
+    scan_single_body<D, GRAD, false>(a, smc);
+}
+
+template <int D, bool GRAD, bool GENERAL>
+__device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const float4* smc) {
+  constexpr int NA = GRAD ? D + 1 : 1;
+  constexpr int VW = SingleVW<D, GRAD>::value;
+  using V = typename VecT<VW>::type;
   double acc[NA];
 #pragma unroll
   for (int k = 0; k < NA; ++k) acc[k] = 0.0;
 
-  const float4* col = reinterpret_cast<const float4*>(a.cols);
-  const int64_t ld4 = a.ld >> 2;
-  const int64_t nfull = a.n >> 2;
+  const V* col = reinterpret_cast<const V*>(a.cols);
+  const int64_t ldv = a.ld / VW;
+  const int64_t nfull = a.n / VW;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  int64_t v = gtid;
-  // two float4 groups (8 points) per iteration: 2*d 16-byte loads in flight
-  for (; v + stride < nfull; v += 2 * stride) {
-    float4 t0[D], t1[D];
-#pragma unroll
-    for (int j = 0; j < D; ++j) t0[j] = __ldcs(col + j * ld4 + v);
-#pragma unroll
-    for (int j = 0; j < D; ++j) t1[j] = __ldcs(col + j * ld4 + v + stride);
+  int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  // fp32 partial sums over up to kSingleFlushPts points, then flushed into fp64
+  constexpr int kGroups = kSingleFlushPts / VW;
+  while (v < nfull) {
     float s[NA];
 #pragma unroll
     for (int k = 0; k < NA; ++k) s[k] = 0.0f;
-    single_group<D, GRAD>(t0, ul, ap, s, a.c_out, v, 4);
-    single_group<D, GRAD>(t1, ul, ap, s, a.c_out, v + stride, 4);
+#pragma unroll 1
+    for (int u = 0; u < kGroups && v < nfull; ++u, v += stride) {
+      V t0[D];
+#pragma unroll
+      for (int j = 0; j < D; ++j) t0[j] = ldcs_v(col + j * ldv + v);
+      single_group<D, GRAD, GENERAL, VW>(t0, smc, s, a.c_out, v, VW);
+    }
 #pragma unroll
     for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
   }
-  // at most one more full group, then the ragged tail group (n % 4 points)
-  for (; v <= nfull; v += stride) {
-    const int valid = v < nfull ? 4 : (int)(a.n - 4 * nfull);
-    if (valid == 0) break;
-    float4 t0[D];
+  // the ragged tail group (n % VW points) belongs to the thread that reaches v == nfull
+  if (v == nfull && a.n > (int64_t)VW * nfull) {
+    const int valid = (int)(a.n - (int64_t)VW * nfull);
+    V t0[D];
 #pragma unroll
-    for (int j = 0; j < D; ++j) t0[j] = __ldcs(col + j * ld4 + v);
+    for (int j = 0; j < D; ++j) t0[j] = ldcs_v(col + j * ldv + v);
     float s[NA];
 #pragma unroll
     for (int k = 0; k < NA; ++k) s[k] = 0.0f;
-    single_group<D, GRAD>(t0, ul, ap, s, a.c_out, v, valid);
+    single_group<D, GRAD, GENERAL, VW>(t0, smc, s, a.c_out, v, valid);
 #pragma unroll
     for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
   }
@@ -202,6 +259,47 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       : "memory");
 }
 
+// The tile loop of the batched scan: wait for tile k (TMA bulk copies
+// completing on bar[k&1]), prefetch tile k+1, accumulate every point of the
+// tile against the thread's QT boxes.
+template <int D, bool GRAD, bool GENERAL, typename Issue>
+__device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const float* tile, uint64_t* bar,
+                                              double* accsh, const BoxDim (&bd)[QT_for<D>::value][D],
+                                              const float (&ap)[D], int64_t s0, int64_t s1, int ntiles,
+                                              Issue& issue) {
+  constexpr int QT = QT_for<D>::value;
+  constexpr int NA = GRAD ? D + 1 : 1;
+  const int tid = threadIdx.x;
+  for (int k = 0; k < ntiles; ++k) {
+    const int buf = k & 1;
+    if (tid == 0 && k + 1 < ntiles) issue(k + 1);  // buffer buf^1 was released by the barrier ending tile k-1
+    mbar_wait_parity(&bar[buf], (uint32_t)((k >> 1) & 1));
+    const float* tl = tile + buf * D * kTilePts;
+    const int64_t rem = s1 - (s0 + (int64_t)k * kTilePts);
+    const int npts = rem < kTilePts ? (int)rem : kTilePts;
+    for (int p0 = 0; p0 < npts; p0 += kFlushPts) {
+      const int pe = min(p0 + kFlushPts, npts);
+      float s[QT][NA];
+#pragma unroll
+      for (int qq = 0; qq < QT; ++qq)
+#pragma unroll
+        for (int kk = 0; kk < NA; ++kk) s[qq][kk] = 0.0f;
+      for (int p = p0; p < pe; ++p) {
+        float t[D];
+#pragma unroll
+        for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
+#pragma unroll
+        for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, GENERAL>(bd[qq], t, ap, s[qq], true);
+      }
+#pragma unroll
+      for (int qq = 0; qq < QT; ++qq)
+#pragma unroll
+        for (int kk = 0; kk < NA; ++kk) accsh[(qq * NA + kk) * kBatchedThreads + tid] += (double)s[qq][kk];
+    }
+    __syncthreads();
+  }
+}
+
 template <int D, bool GRAD>
 constexpr size_t batched_smem_bytes() {
   constexpr int QT = QT_for<D>::value;
@@ -222,7 +320,8 @@ __global__ void __launch_bounds__(kBatchedThreads, (D <= 8 ? 2 : 1)) scan_batche
 
   // this CTA's boxes: qi = qbase + qq*256 + tid (consecutive threads -> consecutive boxes)
   const int64_t qbase = (int64_t)blockIdx.x * kBatchedThreads * QT;
-  float2 ul[QT][D];
+  BoxDim bd[QT][D];
+  bool narrow[QT];
   float ap[D];
 #pragma unroll
   for (int j = 0; j < D; ++j) ap[j] = a.consts->ap[j];
@@ -230,8 +329,12 @@ __global__ void __launch_bounds__(kBatchedThreads, (D <= 8 ? 2 : 1)) scan_batche
   for (int qq = 0; qq < QT; ++qq) {
     int64_t qi = qbase + qq * kBatchedThreads + tid;
     if (qi >= a.q) qi = a.q - 1;  // duplicate a valid box; its partial is never written
+    narrow[qq] = false;
 #pragma unroll
-    for (int j = 0; j < D; ++j) ul[qq][j] = make_float2(__ldg(a.hi + qi * D + j), __ldg(a.lo + qi * D + j));
+    for (int j = 0; j < D; ++j) {
+      bd[qq][j] = make_boxdim(__ldg(a.lo + qi * D + j), __ldg(a.hi + qi * D + j), ap[j]);
+      narrow[qq] |= bd[qq][j].hd > 0.0f;
+    }
   }
 #pragma unroll
   for (int k = 0; k < QT * NA; ++k) accsh[k * kBatchedThreads + tid] = 0.0;
@@ -256,34 +359,16 @@ __global__ void __launch_bounds__(kBatchedThreads, (D <= 8 ? 2 : 1)) scan_batche
   };
   if (tid == 0 && ntiles > 0) issue(0);
 
-  for (int k = 0; k < ntiles; ++k) {
-    const int buf = k & 1;
-    if (tid == 0 && k + 1 < ntiles) issue(k + 1);  // buffer buf^1 was released by the barrier ending tile k-1
-    mbar_wait_parity(&bar[buf], (uint32_t)((k >> 1) & 1));
-    const float* tl = tile + buf * D * kTilePts;
-    const int64_t rem = s1 - (s0 + (int64_t)k * kTilePts);
-    const int npts = rem < kTilePts ? (int)rem : kTilePts;
-    for (int p0 = 0; p0 < npts; p0 += kFlushPts) {
-      const int pe = min(p0 + kFlushPts, npts);
-      float s[QT][NA];
+  // One warp-uniform variant for the whole split: boxes with a narrow
+  // dimension (rare) switch the warp to the general per-dimension path, so
+  // the common path stays branch-free and the QT boxes interleave for ILP.
+  bool my_narrow = false;
 #pragma unroll
-      for (int qq = 0; qq < QT; ++qq)
-#pragma unroll
-        for (int kk = 0; kk < NA; ++kk) s[qq][kk] = 0.0f;
-      for (int p = p0; p < pe; ++p) {
-        float t[D];
-#pragma unroll
-        for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
-#pragma unroll
-        for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD>(ul[qq], t, ap, s[qq], true);
-      }
-#pragma unroll
-      for (int qq = 0; qq < QT; ++qq)
-#pragma unroll
-        for (int kk = 0; kk < NA; ++kk) accsh[(qq * NA + kk) * kBatchedThreads + tid] += (double)s[qq][kk];
-    }
-    __syncthreads();
-  }
+  for (int qq = 0; qq < QT; ++qq) my_narrow |= narrow[qq];
+  if (__any_sync(0xffffffffu, my_narrow))
+    batched_tiles<D, GRAD, true>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
+  else
+    batched_tiles<D, GRAD, false>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
 
   // partials[(split*(NA) + comp) * q + qi]
 #pragma unroll

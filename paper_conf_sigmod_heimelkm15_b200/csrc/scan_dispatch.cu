@@ -32,10 +32,10 @@ cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int 
 }
 
 // ~3 resident CTAs of 256 threads per SM, never more CTAs than 8-point work items.
-int scan_single_grid(int d, int64_t n, int num_sms) {
-  const int per_sm = d <= 8 ? 3 : 2;
+int scan_single_grid(int d, bool grad, int64_t n, int num_sms) {
+  const int per_sm = single_occ(d, grad);
   int64_t grid = (int64_t)num_sms * per_sm;
-  const int64_t items = (n + 7) / 8;
+  const int64_t items = (n + 15) / 16;
   const int64_t need = (items + kSingleThreads - 1) / kSingleThreads;
   if (grid > need) grid = need;
   if (grid < 1) grid = 1;

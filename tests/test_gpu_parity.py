@@ -34,10 +34,14 @@ def sel_ok(gpu, ora):
                              f"(gpu {gpu[bad][:4]}, oracle {ora[bad][:4]})"
 
 
-def grad_ok(gpu, ora, scale):
+def grad_ok(gpu, ora, scale, h=None):
+    """1e-4 relative + 1e-4 of the absolute-term scale + an underflow floor:
+    the kernel's e^{-z^2} flushes to zero below 2^-126, so gradient
+    components under 1e-15/h_j are not representable."""
     gpu, ora, scale = np.asarray(gpu), np.asarray(ora), np.asarray(scale)
     err = np.abs(gpu - ora)
-    tol = 1e-4 * np.abs(ora) + 1e-4 * scale
+    floor = 1e-15 / (np.asarray(h) if h is not None else 1e-3)
+    tol = 1e-4 * np.abs(ora) + 1e-4 * scale + floor
     bad = np.nonzero(err > tol)
     assert len(bad[0]) == 0, f"{len(bad[0])} gradients out of tolerance; worst {np.max(err / np.maximum(tol, 1e-300)):.3g}x"
 
@@ -364,7 +368,7 @@ def test_c3_full_size_single_and_batched_sampled():
     grad_ok(g[pick], g_o, mabs)
     for k in pick[:2]:
         e1, g1 = m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
-        assert abs(e1[0] - est[k]) <= 1e-12 + 1e-9 * est[k]
+        assert abs(e1[0] - est[k]) <= 1e-12 + 1e-7 * est[k]  # two kernels, two summation orders
     assert np.all(est >= 0) and np.all(est <= 1.0 + 1e-12)
 
 
