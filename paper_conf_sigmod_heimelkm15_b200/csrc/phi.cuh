@@ -15,8 +15,10 @@
 // Scaling: the kernels carry y' = z sqrt(log2 e) = (b - t) * ap, so that
 // E = e^{-z^2} = 2^{-y'^2} is a bare ex2.approx; x = |z| = |y'| / sqrt(log2 e)
 // is folded into the constant P' = P / sqrt(log2 e).
-// Infinite bounds: y' is clamped to +-13 (2^-169 flushes to 0), giving
-// E = 0, erfc = 0, 1/2 erf = +-1/2 exactly and a zero gradient term.
+// Infinite bounds: without the gradient y' = +-inf flows through exactly
+// (E = 2^-inf = 0, t = 1/inf = 0, erfc = 0, 1/2 erf = +-1/2).  With the
+// gradient y' is clamped to +-13 (2^-169 flushes to 0) so that y' E = 0
+// instead of inf * 0.
 #pragma once
 #include <cuda_runtime.h>
 #include "phi_coeffs.h"
@@ -116,8 +118,10 @@ __device__ __forceinline__ float phi_diff(const BoxDim& bd, float t, float ap, f
   } else {
     y = __fmul2_rn(__fadd2_rn(bd.b, f2(-t)), f2(ap));
   }
-  y.x = fminf(fmaxf(y.x, -kYClamp), kYClamp);
-  y.y = fminf(fmaxf(y.y, -kYClamp), kYClamp);
+  if (GRAD) {  // y * E would be inf * 0 for an infinite bound; without GRAD inf flows through exactly
+    y.x = fminf(fmaxf(y.x, -kYClamp), kYClamp);
+    y.y = fminf(fmaxf(y.y, -kYClamp), kYClamp);
+  }
   const float2 yy = __fmul2_rn(y, y);
   const float2 E = make_float2(ex2_approx(-yy.x), ex2_approx(-yy.y));
   if (GENERAL && bd.hd > 0.0f) return phi_narrow<GRAD>(y, E, bd.hd, w);

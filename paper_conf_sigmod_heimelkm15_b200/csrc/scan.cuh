@@ -24,9 +24,15 @@
 
 namespace kde {
 
+// boxes per thread (QT) and resident CTAs per SM (MINB) of the batched scan
+// (measured on B200 by tools/tune_batched.cu, gpurun_out/tune1.jsonl)
 template <int D>
 struct QT_for {
-  static constexpr int value = D <= 3 ? 4 : (D <= 6 ? 2 : 1);
+  static constexpr int value = D <= 3 ? 2 : 1;
+};
+template <int D>
+struct MINB_for {
+  static constexpr int value = D <= 6 ? 4 : (D <= 8 ? 3 : (D <= 12 ? 2 : 1));
 };
 
 constexpr int kSingleThreads = 256;
@@ -36,8 +42,9 @@ constexpr int kFlushPts = 32;  // fp32 partial sums are flushed to fp64 every kF
 constexpr int kSingleFlushPts = 16;  // single-box scan: fp32 partials flushed every 16 points
 
 // resident 256-thread CTAs per SM for the single-box scan (register budget)
+// (measured on B200 by tools/tune_single.cu, gpurun_out/tune_single1.jsonl)
 __host__ __device__ constexpr int single_occ(int d, bool grad) {
-  return grad ? (d <= 3 ? 4 : (d <= 6 ? 3 : (d <= 8 ? 2 : 1))) : (d <= 8 ? 4 : (d <= 14 ? 2 : 1));
+  return grad ? (d <= 3 ? 4 : (d <= 10 ? 3 : 1)) : (d <= 10 ? 4 : (d <= 14 ? 2 : 1));
 }
 
 __device__ __forceinline__ float f4c(const float4& v, int p) {
@@ -85,9 +92,17 @@ template <int D, bool GRAD>
 struct SingleVW {
   static constexpr int value = 2;
 };
+template <int D, bool GRAD>
+struct SinglePF {  // register double-buffered prefetch: spills, measured slower (tools/tune_single.cu)
+  static constexpr bool value = false;
+};
 
 template <int VW>
 struct VecT;
+template <>
+struct VecT<1> {
+  using type = float;
+};
 template <>
 struct VecT<2> {
   using type = float2;
@@ -97,7 +112,10 @@ struct VecT<4> {
   using type = float4;
 };
 
+__device__ __forceinline__ float vcomp(const float& v, int) { return v; }
 __device__ __forceinline__ float vcomp(const float2& v, int p) { return p == 0 ? v.x : v.y; }
+__device__ __forceinline__ float ldcs_v(const float* p) { return __ldcs(p); }
+__device__ __forceinline__ void stcs_v(float* p, const float* c) { __stcs(p, c[0]); }
 __device__ __forceinline__ float vcomp(const float4& v, int p) { return f4c(v, p); }
 __device__ __forceinline__ float2 ldcs_v(const float2* p) { return __ldcs(p); }
 __device__ __forceinline__ float4 ldcs_v(const float4* p) { return __ldcs(p); }
@@ -125,11 +143,12 @@ __device__ __forceinline__ void single_group(const typename VecT<VW>::type (&tv)
   if (c_out) stcs_v(reinterpret_cast<typename VecT<VW>::type*>(c_out) + v, cs);
 }
 
-template <int D, bool GRAD, bool GENERAL>
+template <int D, bool GRAD, bool GENERAL, int VW, bool PF>
 __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const float4* smc);
 
-template <int D, bool GRAD>
-__global__ void __launch_bounds__(kSingleThreads, single_occ(D, GRAD)) scan_single_kernel(const ScanSingleArgs a) {
+template <int D, bool GRAD, int VW = SingleVW<D, GRAD>::value, int OCC = single_occ(D, GRAD),
+          bool PF = SinglePF<D, GRAD>::value>
+__global__ void __launch_bounds__(kSingleThreads, OCC) scan_single_kernel(const ScanSingleArgs a) {
   __shared__ float4 smc[D];
   __shared__ int narrow_s;
   if (threadIdx.x == 0) narrow_s = 0;
@@ -143,15 +162,14 @@ __global__ void __launch_bounds__(kSingleThreads, single_occ(D, GRAD)) scan_sing
   }
   __syncthreads();
   if (narrow_s)
-    scan_single_body<D, GRAD, true>(a, smc);
+    scan_single_body<D, GRAD, true, VW, PF>(a, smc);
   else
-    scan_single_body<D, GRAD, false>(a, smc);
+    scan_single_body<D, GRAD, false, VW, PF>(a, smc);
 }
 
-template <int D, bool GRAD, bool GENERAL>
+template <int D, bool GRAD, bool GENERAL, int VW, bool PF>
 __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const float4* smc) {
   constexpr int NA = GRAD ? D + 1 : 1;
-  constexpr int VW = SingleVW<D, GRAD>::value;
   using V = typename VecT<VW>::type;
   double acc[NA];
 #pragma unroll
@@ -162,21 +180,56 @@ __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const 
   const int64_t nfull = a.n / VW;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  // fp32 partial sums over up to kSingleFlushPts points, then flushed into fp64
+  // fp32 partial sums over up to kSingleFlushPts points, then flushed into
+  // fp64.  The next group's column loads are issued before the current group
+  // is computed (register double buffer), so each warp keeps d loads in flight.
   constexpr int kGroups = kSingleFlushPts / VW;
-  while (v < nfull) {
-    float s[NA];
+  if (PF) {
+    V cur[D], nxt[D];
+    if (v < nfull) {
 #pragma unroll
-    for (int k = 0; k < NA; ++k) s[k] = 0.0f;
-#pragma unroll 1
-    for (int u = 0; u < kGroups && v < nfull; ++u, v += stride) {
-      V t0[D];
-#pragma unroll
-      for (int j = 0; j < D; ++j) t0[j] = ldcs_v(col + j * ldv + v);
-      single_group<D, GRAD, GENERAL, VW>(t0, smc, s, a.c_out, v, VW);
+      for (int j = 0; j < D; ++j) cur[j] = ldcs_v(col + j * ldv + v);
     }
+    while (v < nfull) {
+      float s[NA];
 #pragma unroll
-    for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
+      for (int k = 0; k < NA; ++k) s[k] = 0.0f;
+#pragma unroll 1
+      for (int u = 0; u < kGroups && v < nfull; u += 2) {
+        int64_t vn = v + stride;
+        if (vn < nfull) {
+#pragma unroll
+          for (int j = 0; j < D; ++j) nxt[j] = ldcs_v(col + j * ldv + vn);
+        }
+        single_group<D, GRAD, GENERAL, VW>(cur, smc, s, a.c_out, v, VW);
+        v = vn;
+        if (v >= nfull) break;
+        vn = v + stride;
+        if (vn < nfull) {
+#pragma unroll
+          for (int j = 0; j < D; ++j) cur[j] = ldcs_v(col + j * ldv + vn);
+        }
+        single_group<D, GRAD, GENERAL, VW>(nxt, smc, s, a.c_out, v, VW);
+        v = vn;
+      }
+#pragma unroll
+      for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
+    }
+  } else {
+    while (v < nfull) {
+      float s[NA];
+#pragma unroll
+      for (int k = 0; k < NA; ++k) s[k] = 0.0f;
+#pragma unroll 1
+      for (int u = 0; u < kGroups && v < nfull; ++u, v += stride) {
+        V t0[D];
+#pragma unroll
+        for (int j = 0; j < D; ++j) t0[j] = ldcs_v(col + j * ldv + v);
+        single_group<D, GRAD, GENERAL, VW>(t0, smc, s, a.c_out, v, VW);
+      }
+#pragma unroll
+      for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
+    }
   }
   // the ragged tail group (n % VW points) belongs to the thread that reaches v == nfull
   if (v == nfull && a.n > (int64_t)VW * nfull) {
@@ -262,12 +315,11 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 // The tile loop of the batched scan: wait for tile k (TMA bulk copies
 // completing on bar[k&1]), prefetch tile k+1, accumulate every point of the
 // tile against the thread's QT boxes.
-template <int D, bool GRAD, bool GENERAL, typename Issue>
+template <int D, bool GRAD, bool GENERAL, int QT, typename Issue>
 __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const float* tile, uint64_t* bar,
-                                              double* accsh, const BoxDim (&bd)[QT_for<D>::value][D],
+                                              double* accsh, const BoxDim (&bd)[QT][D],
                                               const float (&ap)[D], int64_t s0, int64_t s1, int ntiles,
                                               Issue& issue) {
-  constexpr int QT = QT_for<D>::value;
   constexpr int NA = GRAD ? D + 1 : 1;
   const int tid = threadIdx.x;
   for (int k = 0; k < ntiles; ++k) {
@@ -300,16 +352,14 @@ __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const fl
   }
 }
 
-template <int D, bool GRAD>
+template <int D, bool GRAD, int QT = QT_for<D>::value>
 constexpr size_t batched_smem_bytes() {
-  constexpr int QT = QT_for<D>::value;
   constexpr int NA = GRAD ? D + 1 : 1;
   return 2ull * D * kTilePts * sizeof(float) + (size_t)QT * NA * kBatchedThreads * sizeof(double) + 16;
 }
 
-template <int D, bool GRAD>
-__global__ void __launch_bounds__(kBatchedThreads, (D <= 8 ? 2 : 1)) scan_batched_kernel(const ScanBatchedArgs a) {
-  constexpr int QT = QT_for<D>::value;
+template <int D, bool GRAD, int QT = QT_for<D>::value, int MINB = MINB_for<D>::value>
+__global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(const ScanBatchedArgs a) {
   constexpr int NA = GRAD ? D + 1 : 1;
   extern __shared__ __align__(16) unsigned char smem_raw[];
   float* tile = reinterpret_cast<float*>(smem_raw);                                   // [2][D][kTilePts]
@@ -366,9 +416,9 @@ __global__ void __launch_bounds__(kBatchedThreads, (D <= 8 ? 2 : 1)) scan_batche
 #pragma unroll
   for (int qq = 0; qq < QT; ++qq) my_narrow |= narrow[qq];
   if (__any_sync(0xffffffffu, my_narrow))
-    batched_tiles<D, GRAD, true>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
+    batched_tiles<D, GRAD, true, QT>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
   else
-    batched_tiles<D, GRAD, false>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
+    batched_tiles<D, GRAD, false, QT>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
 
   // partials[(split*(NA) + comp) * q + qi]
 #pragma unroll
@@ -392,37 +442,53 @@ cudaError_t launch_single_t(bool grad, const ScanSingleArgs& a, int grid, cudaSt
   return cudaGetLastError();
 }
 
-template <int D, bool GRAD>
-cudaError_t launch_batched_tg(const ScanBatchedArgs& a, dim3 grid, cudaStream_t s) {
-  constexpr size_t smem = batched_smem_bytes<D, GRAD>();
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(scan_batched_kernel<D, GRAD>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)smem);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
-  scan_batched_kernel<D, GRAD><<<grid, kBatchedThreads, smem, s>>>(a);
+// tuning entry point (tools/tune_single.cu)
+template <int D, bool GRAD, int VW, int OCC, bool PF>
+cudaError_t launch_single_variant(const ScanSingleArgs& a, int grid, cudaStream_t s) {
+  scan_single_kernel<D, GRAD, VW, OCC, PF><<<grid, kSingleThreads, 0, s>>>(a);
   return cudaGetLastError();
 }
 
-// Grid for the batched scan: query tiles x sample splits, sized to ~8 CTAs
-// per SM (4 waves at 2 resident CTAs/SM); split_len is a tile multiple.
+template <int D, bool GRAD, int QT = QT_for<D>::value, int MINB = MINB_for<D>::value>
+cudaError_t launch_batched_tg(const ScanBatchedArgs& a, dim3 grid, cudaStream_t s) {
+  constexpr size_t smem = batched_smem_bytes<D, GRAD, QT>();
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(scan_batched_kernel<D, GRAD, QT, MINB>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  scan_batched_kernel<D, GRAD, QT, MINB><<<grid, kBatchedThreads, smem, s>>>(a);
+  return cudaGetLastError();
+}
+
+// Grid for the batched scan: query tiles (256*QT boxes) x sample splits,
+// about `waves` x MINB CTAs per SM; split_len is a tile multiple.
+inline void batched_grid(int64_t q, int64_t n, int qt, int minb, int num_sms, int waves, int64_t* qtiles,
+                         int64_t* splits, int64_t* split_len) {
+  *qtiles = (q + (int64_t)kBatchedThreads * qt - 1) / ((int64_t)kBatchedThreads * qt);
+  const int64_t ntile_pts = (n + kTilePts - 1) / kTilePts;
+  const int64_t target = (int64_t)num_sms * minb * waves;
+  int64_t sp = (target + *qtiles - 1) / *qtiles;
+  if (sp > ntile_pts) sp = ntile_pts;
+  if (sp < 1) sp = 1;
+  int64_t len = ((n + sp - 1) / sp + kTilePts - 1) / kTilePts * kTilePts;
+  if (len < kTilePts) len = kTilePts;
+  sp = (n + len - 1) / len;
+  if (sp < 1) sp = 1;
+  *splits = sp;
+  *split_len = len;
+}
+
 template <int D>
 cudaError_t launch_batched_t(bool grad, const ScanBatchedArgs& a_in, int num_sms, int* splits_out, cudaStream_t s,
                              bool dry_run) {
   constexpr int QT = QT_for<D>::value;
+  constexpr int MINB = MINB_for<D>::value;
   ScanBatchedArgs a = a_in;
-  const int64_t qtiles = (a.q + (int64_t)kBatchedThreads * QT - 1) / ((int64_t)kBatchedThreads * QT);
-  const int64_t ntile_pts = (a.n + kTilePts - 1) / kTilePts;
-  const int64_t target = (int64_t)num_sms * 8;
-  int64_t splits = (target + qtiles - 1) / qtiles;
-  if (splits > ntile_pts) splits = ntile_pts;
-  if (splits < 1) splits = 1;
-  int64_t split_len = ((a.n + splits - 1) / splits + kTilePts - 1) / kTilePts * kTilePts;
-  if (split_len < kTilePts) split_len = kTilePts;
-  splits = (a.n + split_len - 1) / split_len;
-  if (splits < 1) splits = 1;
+  int64_t qtiles, splits, split_len;
+  batched_grid(a.q, a.n, QT, MINB, num_sms, 4, &qtiles, &splits, &split_len);
   if (splits_out) *splits_out = (int)splits;
   if (dry_run) return cudaSuccess;
   a.split_len = split_len;
