@@ -57,6 +57,10 @@ CONFIGS = {
     "c5s": dict(d=10, n=1 << 22, q=1, path="single", grad=True, retain=True, data="gauss",
                 desc="configs[4] estimate step: d=10, N=2^22/GPU, one DT box, estimate + gradient + retained "
                      "contributions (Adaptive, P:L240)"),
+    "c5": dict(d=10, n=1 << 22, q=1, path="stream", grad=True, retain=True, data="gauss",
+               desc="configs[4] streaming step: d=10, N=2^22, one DT box per step: estimate + gradient + retained "
+                    "contributions, karma pass + compaction, Listing 1 bandwidth step, replacement of flagged points "
+                    "(device-resident, single GPU)"),
     "c4": dict(d=8, n=1 << 25, q=4096, path="loss_grad", data="gauss",
                desc="configs[3] per-GPU shard: d=8, 2^25 rows/GPU (2^28 at 8 GPUs), 4096 boxes, estimate + gradient + NCCL"),
 }
@@ -162,7 +166,7 @@ def cpu_oracle_rate(S, h, lo, hi, p, path, budget_s=12.0, per_step=False):
     n = len(S)
     oracle.set_threads(1)
     t0 = time.perf_counter()
-    if path == "single":
+    if path in ("single", "stream"):
         oracle.estimate_grad(S, h, lo[:1], hi[:1])
     else:
         oracle.loss_and_grad(S, h, lo[:1], hi[:1], p[:1], 0, 0.0, False)
@@ -172,7 +176,7 @@ def cpu_oracle_rate(S, h, lo, hi, p, path, budget_s=12.0, per_step=False):
     use = min(cores, k)
     oracle.set_threads(use)
     t0 = time.perf_counter()
-    if path == "single":
+    if path in ("single", "stream"):
         oracle.estimate_grad(S, h, lo[:k], hi[:k])
     else:
         oracle.loss_and_grad(S, h, lo[:k], hi[:k], p[:k], 0, 0.0, False)
@@ -194,7 +198,7 @@ def run_reference(args, cfg, rank, world):
     times = []
     for i in range(args.warmup + args.steps):
         t0 = time.perf_counter()
-        if cfg["path"] == "single":
+        if cfg["path"] in ("single", "stream"):
             oracle.estimate_grad(S, h, lo[:k], hi[:k])
         else:
             oracle.loss_and_grad(S, h, lo[:k], hi[:k], p[:k], 0, 0.0, False)
@@ -236,6 +240,8 @@ def run_cuda(args, cfg, rank, world, local_rank):
     d, n, q = cfg["d"], cfg["n"], cfg["q"]
     R, S, lo, hi = make_inputs(cfg, rank)
     p = true_selectivities(R, lo, hi) if cfg["path"] != "single" else None
+    if cfg["path"] == "stream" and world > 1:
+        raise SystemExit("c5 (device-resident streaming) is single-GPU")
 
     n_global = n * world
     if world > 1:
@@ -260,8 +266,25 @@ def run_cuda(args, cfg, rank, world, local_rank):
 
     if cfg.get("retain"):
         m.set_retain(True)
+    if cfg["path"] == "stream":
+        cap = 1 << 16
+        kp = K.karma_params(loss=K.LOSS_ABSOLUTE, threshold=-1.0 / (n_global - 1), k_max=4.0)
+        op = K.online_params(minibatch=10, loss=K.LOSS_ABSOLUTE, log_bandwidth=True)
+        d_pool = torch.from_numpy(R).to(dev)  # replacement rows drawn from the database R
+        d_idx = torch.zeros(cap, dtype=torch.int64, device=dev)
+        d_cnt = torch.zeros(1, dtype=torch.int64, device=dev)
+        npool = len(R) - cap
+        flagged = []
 
     def step(i):
+        if cfg["path"] == "stream":
+            k = i % nbox
+            K.kde_estimate_batch_dev(m.handle, d_lo[k:k + 1], d_hi[k:k + 1], d_est[:1], d_dpdh[:1], stream=stream)
+            K.kde_karma_update_dev(m.handle, d_lo[k], d_hi[k], d_true[k:k + 1], kp, d_idx, d_cnt, stream=stream)
+            K.kde_online_update_dev(m.handle, d_true[k:k + 1], op, stream=stream)
+            off = (i * 977) % npool
+            K.kde_replace_points_dev(m.handle, d_idx, d_pool[off:off + cap], d_cnt, stream=stream)
+            return
         if cfg["path"] == "single":
             k = i % nbox
             K.kde_estimate_batch_dev(m.handle, d_lo[k:k + 1], d_hi[k:k + 1], d_est[:1],
@@ -281,6 +304,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
         dist.barrier()
     torch.cuda.synchronize()
     with ClockSampler(local_rank) as clk:
+        t_start = time.perf_counter()
         with torch.cuda.stream(stream):
             for i in range(args.steps):
                 if flush_l2:
@@ -289,10 +313,24 @@ def run_cuda(args, cfg, rank, world, local_rank):
                 step(i)
                 evs[i][1].record(stream)
         torch.cuda.synchronize()
+        # short timed regions (< 1 s) are followed by an identical untimed soak so
+        # that nvidia-smi (100 ms period) samples the clocks under this load
+        soak = 0
+        while time.perf_counter() - t_start < 1.0 and soak < 100000:
+            with torch.cuda.stream(stream):
+                for _ in range(8):
+                    step(args.steps + soak)
+                    soak += 1
+            torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     scan_ms, scan_launches, launches = K.kde_get_profile(m.handle)
+    # the soak steps launched the same kernels: keep the timed steps' share
+    per_step = launches / max(args.steps + soak, 1)
+    launches = int(round(per_step * args.steps))
+    scan_ms *= args.steps / max(args.steps + soak, 1)
+    scan_launches = int(round(scan_launches * args.steps / max(args.steps + soak, 1)))
     K.kde_set_profiling(m.handle, False)
     step_ms = [a.elapsed_time(b) for a, b in evs]
     tot_ms = sum(step_ms)
@@ -311,7 +349,15 @@ def run_cuda(args, cfg, rank, world, local_rank):
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     for i in range(e2e_steps):
-        if cfg["path"] == "single":
+        if cfg["path"] == "stream":
+            k = i % nbox
+            m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+            idx, nf, _ = m.karma_update(lo[k], hi[k], p[k], kp, cap=cap)
+            m.online_update(lo[k], hi[k], p[k], op)
+            off = (i * 977) % npool
+            m.replace_points(idx, R[off:off + len(idx)])
+            flagged.append(nf)
+        elif cfg["path"] == "single":
             k = i % nbox
             m.estimate(lo[k:k + 1], hi[k:k + 1], grad=bool(cfg.get("grad")))
         else:
@@ -322,7 +368,11 @@ def run_cuda(args, cfg, rank, world, local_rank):
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     e2e_s = float(t.item())
-    if cfg["path"] == "single":
+    if cfg["path"] == "stream":
+        mean_flag = float(np.mean(flagged)) if flagged else 0.0
+        h2d = 2 * d * 4 * 3 + 8 * 2 + int(mean_flag * (8 + 4 * d))  # bounds (3 calls), true sel (2), replacement idx+rows
+        d2h = 8 * (1 + d) + int(mean_flag * 8) + 8 + 4  # estimate+gradient, flagged indices, count, update flag
+    elif cfg["path"] == "single":
         h2d, d2h = 2 * d * 4, 8 * (1 + (d if cfg.get("grad") else 0))
     else:
         h2d, d2h = 2 * q * d * 4 + q * 8, 8 * (1 + d)
@@ -333,7 +383,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
     clocks = clk.summary()
     avg_scan_ms = scan_ms / max(scan_launches, 1)
     sms = torch.cuda.get_device_properties(dev).multi_processor_count
-    if cfg["path"] == "single":
+    if cfg["path"] in ("single", "stream"):
         alg_bytes = n * d * 4 + (n * 4 if cfg.get("retain") else 0)  # 4d B/point read (+4 B/point retained c)
         achieved = alg_bytes / (avg_scan_ms * 1e-3) / 1e9
         peak = _measured_hbm()
@@ -366,8 +416,12 @@ def run_cuda(args, cfg, rank, world, local_rank):
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": cfg["desc"], "d": d, "n_per_gpu": n, "n_global": n_global, "q": q,
                    "l2": "flushed between timed steps" if flush_l2 else "sample larger than L2",
+                   "clock_sampling": "nvidia-smi every 100 ms over the timed steps"
+                                     + (f" + {soak} identical untimed soak steps (timed region < 1 s)" if soak else ""),
                    "accumulation": "fp32 per <=32 points, fp64 above"},
         "estimates_per_s": q / (ms_per_step * 1e-3),
+        **({"stream": {"queries_per_s": 1e3 / ms_per_step, "mean_flagged_per_query_e2e": float(np.mean(flagged))}}
+           if cfg["path"] == "stream" else {}),
         "e2e": {"value": units_per_step * e2e_steps / e2e_s, "unit": "point·query evals/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": e2e_steps},
         "gpu_launches": launches, "scan_launches": scan_launches,

@@ -209,6 +209,30 @@ kde_status kde_online_update(kde_model *m, const float *lo, const float *hi, dou
 kde_status kde_replace_points(kde_model *m, const int64_t *idx, const float *rows, int64_t k,
                               double k_init);
 
+/* ---------------------------------------------------------------- device-resident feedback loop
+ * Single-GPU (world == 1) device-pointer variants of the feedback calls, so a
+ * whole streaming step (estimate -> karma -> bandwidth -> replacement) runs
+ * without a host round trip (the paper ships the bitmap to the
+ * host).  They enqueue on `stream` (NULL = the model's stream) and use
+ * the retained state of the preceding kde_estimate_batch_dev(q == 1) on the
+ * same stream: p_hat and dp_hat/dh always, the contributions p^(i) only when
+ * retain is on (kde_set_retain).  Arguments are NOT validated on the device:
+ * the caller guarantees a valid box, 0 <= p <= 1, and (replace) unique
+ * in-range indices -- the karma output satisfies this by construction. */
+/* karma pass: d_true_sel 1 fp64; ascending GLOBAL flagged indices -> d_idx_out
+ * (first idx_cap), total count -> *d_n_flagged (device int64). */
+kde_status kde_karma_update_dev(kde_model *m, const float *d_lo, const float *d_hi, const double *d_true_sel,
+                                const kde_karma_params *kp, int64_t *d_idx_out, int64_t idx_cap,
+                                int64_t *d_n_flagged, void *stream);
+/* Listing 1 step from the retained (p_hat, dp_hat/dh); requires the preceding
+ * single-box estimate to have computed the gradient. */
+kde_status kde_online_update_dev(kde_model *m, const double *d_true_sel, const kde_online_params *op, void *stream);
+/* the first min(*d_k, cap) GLOBAL indices d_idx[] receive rows d_rows[] (device,
+ * row-major, at least cap x d), karma reset to k_init; the column ranges used
+ * for bound clamping are widened on the device. */
+kde_status kde_replace_points_dev(kde_model *m, const int64_t *d_idx, const float *d_rows, const int64_t *d_k,
+                                  int64_t cap, double k_init, void *stream);
+
 /* ---------------------------------------------------------------- inspection */
 kde_status kde_get_karma(kde_model *m, double *karma);   /* local n fp64          */
 kde_status kde_set_karma(kde_model *m, const double *karma); /* local n fp64      */

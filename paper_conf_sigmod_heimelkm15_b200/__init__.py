@@ -34,6 +34,7 @@ ABI_SYMBOLS = (
     "kde_loss_and_grad_dev", "kde_karma_update", "kde_online_update", "kde_replace_points",
     "kde_get_karma", "kde_set_karma", "kde_get_sample", "kde_get_contributions", "kde_get_online_state",
     "kde_set_online_state", "kde_synchronize", "kde_count_in_box_dev", "kde_set_profiling", "kde_get_profile",
+    "kde_karma_update_dev", "kde_online_update_dev", "kde_replace_points_dev",
 )
 
 
@@ -114,6 +115,9 @@ def lib() -> ctypes.CDLL:
         "kde_count_in_box_dev": (ctypes.c_int, [P, i64, i32, P, P, i64, P, P]),
         "kde_set_profiling": (ctypes.c_int, [P, i32]),
         "kde_get_profile": (ctypes.c_int, [P, P, P, P]),
+        "kde_karma_update_dev": (ctypes.c_int, [P, P, P, P, ctypes.POINTER(KarmaParams), P, i64, P, P]),
+        "kde_online_update_dev": (ctypes.c_int, [P, P, ctypes.POINTER(OnlineParams), P]),
+        "kde_replace_points_dev": (ctypes.c_int, [P, P, P, P, i64, f64, P]),
     }
     for name, (res, args) in sigs.items():
         fn = getattr(L, name)
@@ -265,6 +269,22 @@ def kde_online_update(m, lo, hi, true_sel: float, params: OnlineParams) -> bool:
     upd = ctypes.c_int32()
     _check(lib().kde_online_update(m, _p(lo), _p(hi), float(true_sel), ctypes.byref(params), ctypes.byref(upd)))
     return bool(upd.value)
+
+
+def kde_karma_update_dev(m, d_lo, d_hi, d_true, params: KarmaParams, d_idx, d_count, stream=None):
+    """Device-resident karma pass (single GPU): enqueue only."""
+    _check(lib().kde_karma_update_dev(m, _tp(d_lo), _tp(d_hi), _tp(d_true), ctypes.byref(params), _tp(d_idx),
+                                      d_idx.numel(), _tp(d_count), _stream_ptr(stream)))
+
+
+def kde_online_update_dev(m, d_true, params: OnlineParams, stream=None):
+    _check(lib().kde_online_update_dev(m, _tp(d_true), ctypes.byref(params), _stream_ptr(stream)))
+
+
+def kde_replace_points_dev(m, d_idx, d_rows, d_count, k_init=0.0, stream=None):
+    """Rows d_rows[r] -> global index d_idx[r] for r < min(d_count, len(d_idx))."""
+    _check(lib().kde_replace_points_dev(m, _tp(d_idx), _tp(d_rows), _tp(d_count), d_idx.numel(), float(k_init),
+                                        _stream_ptr(stream)))
 
 
 def kde_replace_points(m, idx, rows, k_init=0.0):

@@ -19,10 +19,16 @@ constexpr int kColAlign = 1024;  // columns padded to a multiple of this many po
 //                                                  z = (b - t)/(sqrt2 h) is the erf argument of eq. (13)
 //   gconst[j] = 1 / (sqrt(pi) sqrt(log2 e) h_j)   so that d p^(i)/d h_j = gconst[j] * w_j * prod_{k!=j} D_k,
 //                                                  w_j = y'_l E_l - y'_u E_u (eq. 17 rewritten in z)
+//   tmin/tmax = per-column range of the (local) sample: query bounds are
+//   clamped to [tmin - 14/ap, tmax + 14/ap] at box setup, which leaves every
+//   fp32 result unchanged (|y'| >= 14 gives E = 0, erf = +-1 exactly) and
+//   keeps y' finite, so the gradient term y' E never meets inf * 0.
 struct DevConsts {
   double h[kMaxDim];
   double gconst[kMaxDim];
   float ap[kMaxDim];
+  float tmin[kMaxDim];
+  float tmax[kMaxDim];
 };
 
 // Listing 1 state (reconstruction, R6), device resident.
@@ -57,7 +63,9 @@ struct ScanSingleArgs {
   double* block_partials; // [gridDim.x][1+d]
   unsigned* counter;      // zero on entry; the last block resets it to zero
   double* sums_out;       // [1+d] raw sums S_0 = sum_i p^(i), S_j = sum_i w_j prod_{k!=j} D_k
-  double* fin_out;        // nullable: [1+d] finalised (p_hat, dp_hat/dh_j) for world == 1
+  double* fin_out;        // nullable: [1+d] finalised (p_hat, dp_hat/dh_j) for world == 1 (retained copy)
+  double* est_out;        // nullable: p_hat (caller's buffer), world == 1
+  double* dpdh_out;       // nullable: d x dp_hat/dh_j (caller's buffer), world == 1, GRAD only
   double n_global;        // s (results are divided by s, so s ones give exactly 1)
 };
 

@@ -71,6 +71,8 @@ struct kde_model {
   int64_t* idx_dev = nullptr;
   int64_t idx_cap = 0;
   int32_t* bad = nullptr;            // device flag
+  unsigned* range_enc = nullptr;     // [d][2] encoded column min/max (kernels.cu)
+  double* scal = nullptr;            // [8] device scalars (true selectivity staging)
   void* pinned = nullptr;            // pinned host staging
   size_t pinned_cap = 0;
 
@@ -220,7 +222,7 @@ static kde_status prof_begin(kde_model* m, cudaStream_t s, cudaEvent_t* e1, cuda
 // Raw sums for q boxes (device bounds) -> sums[q][na] combined over ranks.
 // For q == 1 also retains c (if c_out) and writes the finalised values to fin.
 static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, int64_t q, bool grad, float* c_out,
-                            double* d_sums, cudaStream_t s) {
+                            double* d_sums, cudaStream_t s, double* d_est = nullptr, double* d_dpdh = nullptr) {
   const int d = m->d;
   const int na = grad ? d + 1 : 1;
   if (q == 1) {
@@ -235,7 +237,10 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     a.block_partials = m->block_partials;
     a.counter = m->counter;
     a.sums_out = d_sums;
-    a.fin_out = nullptr;
+    // world == 1: the last block finalises straight into the retained copy and the caller's buffers
+    a.fin_out = m->world == 1 ? m->ret : nullptr;
+    a.est_out = m->world == 1 ? d_est : nullptr;
+    a.dpdh_out = m->world == 1 ? d_dpdh : nullptr;
     a.n_global = (double)m->n_global;
     const int grid = scan_single_grid(d, grad, m->n, m->num_sms);
     cudaEvent_t e1 = nullptr, e2 = nullptr;
@@ -276,7 +281,8 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
   return KDE_OK;
 }
 
-// est/dpdh (device) for q boxes with device bounds.
+// est/dpdh (device) for q boxes with device bounds.  A single box also leaves
+// (p_hat, dp_hat/dh) in m->ret for the feedback calls (karma / online update).
 static kde_status estimate_dev(kde_model* m, const float* d_lo, const float* d_hi, int64_t q, double* d_est,
                                double* d_dpdh, cudaStream_t s, bool retain_c) {
   const bool grad = d_dpdh != nullptr;
@@ -284,8 +290,16 @@ static kde_status estimate_dev(kde_model* m, const float* d_lo, const float* d_h
   kde_status st = ensure_q(m, q);
   if (st != KDE_OK) return st;
   double* sums = o_sums(m);
-  st = scan_sums(m, d_lo, d_hi, q, grad, (q == 1 && retain_c) ? m->cret : nullptr, sums, s);
+  st = scan_sums(m, d_lo, d_hi, q, grad, (q == 1 && retain_c) ? m->cret : nullptr, sums, s, d_est, d_dpdh);
   if (st != KDE_OK) return st;
+  if (q == 1 && m->world == 1) return KDE_OK;  // finalised by the scan's last block
+  if (q == 1) {
+    CUL(launch_finalize(sums, 1, m->d, na, m->consts, (double)m->n_global, m->ret, grad ? m->ret + 1 : nullptr, s));
+    if (d_est != m->ret) CU(cudaMemcpyAsync(d_est, m->ret, sizeof(double), cudaMemcpyDeviceToDevice, s));
+    if (grad && d_dpdh != m->ret + 1)
+      CU(cudaMemcpyAsync(d_dpdh, m->ret + 1, sizeof(double) * m->d, cudaMemcpyDeviceToDevice, s));
+    return KDE_OK;
+  }
   CUL(launch_finalize(sums, q, m->d, na, m->consts, (double)m->n_global, d_est, d_dpdh, s));
   return KDE_OK;
 }
@@ -337,6 +351,8 @@ static void free_model(kde_model* m) {
   cudaFree(m->offsets);
   cudaFree(m->idx_dev);
   cudaFree(m->bad);
+  cudaFree(m->range_enc);
+  cudaFree(m->scal);
   if (m->pinned) cudaFreeHost(m->pinned);
   for (cudaEvent_t e : m->ev) cudaEventDestroy(e);
   if (m->comm) ncclCommDestroy(m->comm);
@@ -396,6 +412,8 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
   CUB(cudaMalloc(&m->ret, sizeof(double) * (kMaxDim + 1)));
   CUB(cudaMalloc(&m->single_sums, sizeof(double) * (kMaxDim + 1)));
   CUB(cudaMalloc(&m->bad, sizeof(int32_t)));
+  CUB(cudaMalloc(&m->range_enc, sizeof(unsigned) * 2 * kMaxDim));
+  CUB(cudaMalloc(&m->scal, sizeof(double) * 8));
   const int nkb = karma_blocks(n_local);
   CUB(cudaMalloc(&m->bitmap, sizeof(uint32_t) * (size_t)nkb * (kKarmaPts / 32)));
   CUB(cudaMalloc(&m->block_counts, sizeof(int32_t) * (size_t)nkb));
@@ -442,6 +460,18 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
     int32_t bad = 0;
     CUB(cudaMemcpy(&bad, m->bad, sizeof(int32_t), cudaMemcpyDeviceToHost));
     if (bad) return bail(fail(KDE_EINVAL, "non-finite value in sample"));
+  }
+
+  // column ranges (bound clamping, see DevConsts)
+  {
+    std::vector<unsigned> init(2 * kMaxDim);
+    for (int j = 0; j < kMaxDim; ++j) {
+      init[2 * j] = 0xFFFFFFFFu;
+      init[2 * j + 1] = 0u;
+    }
+    CUB(cudaMemcpy(m->range_enc, init.data(), sizeof(unsigned) * 2 * kMaxDim, cudaMemcpyHostToDevice));
+    ++m->launches;
+    CUB(launch_col_range(m->cols, m->ld, n_local, d, m->range_enc, m->consts, s));
   }
 
   // bandwidth: caller's h, or Scott's rule (eq. 3) over the global sample
@@ -652,6 +682,48 @@ extern "C" kde_status kde_loss_and_grad_dev(kde_model* m, const float* d_lo, con
   return loss_grad_dev_impl(m, d_lo, d_hi, d_true_sel, q, loss, lambda, log_bandwidth, d_loss, d_grad, d_est, s);
 }
 
+// ------------------------------------------------------------------ feedback parameter checks
+static kde_status karma_params_dev(const kde_karma_params* kp, KarmaParamsDev* kd) {
+  if (!kp) return fail(KDE_EINVAL, "NULL karma params");
+  kde_status st = validate_loss(kp->loss, kp->lambda);
+  if (st != KDE_OK) return st;
+  if (std::isnan(kp->k_max) || std::isnan(kp->threshold)) return fail(KDE_EINVAL, "NaN k_max / threshold");
+  kd->loss = kp->loss;
+  kd->empty_region = kp->empty_region;
+  kd->lambda = kp->lambda;
+  kd->k_max = kp->k_max;
+  kd->threshold = kp->threshold;
+  return KDE_OK;
+}
+
+static kde_status online_params_dev(kde_model* m, const kde_online_params* op, OnlineParamsDev* od, cudaStream_t s) {
+  if (!op) return fail(KDE_EINVAL, "NULL online params");
+  kde_status st = validate_loss(op->loss, op->lambda);
+  if (st != KDE_OK) return st;
+  if (op->minibatch < 1 || !(op->alpha >= 0.0 && op->alpha < 1.0) || !(op->lr_min > 0.0) ||
+      !(op->lr_max >= op->lr_min) || !(op->lr_inc >= 1.0) || !(op->lr_dec > 0.0 && op->lr_dec <= 1.0) ||
+      !(op->lr0 > 0.0))
+    return fail(KDE_EINVAL, "bad online parameters");
+  if (!m->online_init) {
+    OnlineState s0;
+    memset(&s0, 0, sizeof(s0));
+    for (int j = 0; j < kMaxDim; ++j) s0.lr[j] = op->lr0;
+    CU(cudaMemcpyAsync(m->online, &s0, sizeof(s0), cudaMemcpyHostToDevice, s));
+    CU(cudaStreamSynchronize(s));
+    m->online_init = true;
+  }
+  od->minibatch = op->minibatch;
+  od->log_bw = op->log_bandwidth;
+  od->loss = op->loss;
+  od->lambda = op->lambda;
+  od->alpha = op->alpha;
+  od->lr_min = op->lr_min;
+  od->lr_max = op->lr_max;
+  od->lr_inc = op->lr_inc;
+  od->lr_dec = op->lr_dec;
+  return KDE_OK;
+}
+
 // ------------------------------------------------------------------ ABI: feedback
 static bool retained_matches(kde_model* m, const float* lo, const float* hi, bool need_c, bool need_grad) {
   if (!m->ret_valid || m->ret_gen != m->gen) return false;
@@ -706,8 +778,9 @@ extern "C" kde_status kde_karma_update(kde_model* m, const float* lo, const floa
   kd.k_max = kp->k_max;
   kd.threshold = kp->threshold;
   const int nkb = karma_blocks(m->n);
+  CU(cudaMemcpyAsync(m->scal, &true_sel, sizeof(double), cudaMemcpyHostToDevice, m->stream));
   m->launches += 2;  // karma + scan_counts + compact
-  CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, true_sel, kd, m->qbuf, m->qbuf + m->d, m->d,
+  CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, m->scal, kd, m->qbuf, m->qbuf + m->d, m->d,
                   m->consts, m->bitmap, m->block_counts, m->offsets, m->row_offset, m->idx_dev, local_cap,
                   m->stream));
   int64_t local_total = 0;
@@ -773,36 +846,15 @@ extern "C" kde_status kde_online_update(kde_model* m, const float* lo, const flo
   CHECK_MODEL(m);
   kde_status st = validate_bounds(lo, hi, 1, m->d);
   if (st != KDE_OK) return st;
-  if (!op) return fail(KDE_EINVAL, "NULL online params");
   if (!(true_sel >= 0.0 && true_sel <= 1.0)) return fail(KDE_EINVAL, "true_sel outside [0, 1]");
-  st = validate_loss(op->loss, op->lambda);
-  if (st != KDE_OK) return st;
-  if (op->minibatch < 1 || !(op->alpha >= 0.0 && op->alpha < 1.0) || !(op->lr_min > 0.0) ||
-      !(op->lr_max >= op->lr_min) || !(op->lr_inc >= 1.0) || !(op->lr_dec > 0.0 && op->lr_dec <= 1.0) ||
-      !(op->lr0 > 0.0))
-    return fail(KDE_EINVAL, "bad online parameters");
   DeviceGuard g(m->device);
-  if (!m->online_init) {
-    OnlineState s0;
-    memset(&s0, 0, sizeof(s0));
-    for (int j = 0; j < kMaxDim; ++j) s0.lr[j] = op->lr0;
-    CU(cudaMemcpyAsync(m->online, &s0, sizeof(s0), cudaMemcpyHostToDevice, m->stream));
-    CU(cudaStreamSynchronize(m->stream));
-    m->online_init = true;
-  }
+  OnlineParamsDev od;
+  st = online_params_dev(m, op, &od, m->stream);
+  if (st != KDE_OK) return st;
   st = ensure_retained(m, lo, hi, false, true);
   if (st != KDE_OK) return st;
-  OnlineParamsDev od;
-  od.minibatch = op->minibatch;
-  od.log_bw = op->log_bandwidth;
-  od.loss = op->loss;
-  od.lambda = op->lambda;
-  od.alpha = op->alpha;
-  od.lr_min = op->lr_min;
-  od.lr_max = op->lr_max;
-  od.lr_inc = op->lr_inc;
-  od.lr_dec = op->lr_dec;
-  CUL(launch_online_update(m->ret, true_sel, od, m->d, m->online, m->consts, m->stream));
+  CU(cudaMemcpyAsync(m->scal + 1, &true_sel, sizeof(double), cudaMemcpyHostToDevice, m->stream));
+  CUL(launch_online_update(m->ret, m->scal + 1, od, m->d, m->online, m->consts, m->stream));
   int32_t upd = 0;
   CU(cudaMemcpyAsync(&upd, &m->online->updated, sizeof(int32_t), cudaMemcpyDeviceToHost, m->stream));
   CU(cudaStreamSynchronize(m->stream));
@@ -847,11 +899,60 @@ extern "C" kde_status kde_replace_points(kde_model* m, const int64_t* idx, const
     memcpy(m->pinned, li.data(), ib);
     memcpy((char*)m->pinned + ib, lr.data(), rb);
     CU(cudaMemcpyAsync(dbuf, m->pinned, ib + rb, cudaMemcpyHostToDevice, m->stream));
+    CUL(launch_row_range((const float*)((char*)dbuf + ib), kl, m->d, m->range_enc, m->consts, m->stream));
     CUL(launch_scatter_rows((const int64_t*)dbuf, (const float*)((char*)dbuf + ib), kl, m->d, m->cols, m->ld,
                            m->karma, k_init, m->stream));
     CU(cudaStreamSynchronize(m->stream));
     cudaFree(dbuf);
   }
+  ++m->gen;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_karma_update_dev(kde_model* m, const float* d_lo, const float* d_hi,
+                                           const double* d_true_sel, const kde_karma_params* kp, int64_t* d_idx_out,
+                                           int64_t idx_cap, int64_t* d_n_flagged, void* stream) {
+  CHECK_MODEL(m);
+  if (m->world != 1) return fail(KDE_EINVAL, "device-resident feedback calls are single-GPU (world == 1)");
+  if (!d_lo || !d_hi || !d_true_sel || !d_n_flagged || idx_cap < 0 || (idx_cap > 0 && !d_idx_out))
+    return fail(KDE_EINVAL, "NULL device pointer / bad idx_cap");
+  KarmaParamsDev kd;
+  kde_status st = karma_params_dev(kp, &kd);
+  if (st != KDE_OK) return st;
+  DeviceGuard g(m->device);
+  cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
+  const int nkb = karma_blocks(m->n);
+  m->launches += 2;
+  CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, d_true_sel, kd, d_lo, d_hi, m->d,
+                   m->consts, m->bitmap, m->block_counts, m->offsets, m->row_offset, d_idx_out, idx_cap, s));
+  CU(cudaMemcpyAsync(d_n_flagged, m->offsets + nkb, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_online_update_dev(kde_model* m, const double* d_true_sel, const kde_online_params* op,
+                                            void* stream) {
+  CHECK_MODEL(m);
+  if (!d_true_sel) return fail(KDE_EINVAL, "NULL device pointer");
+  DeviceGuard g(m->device);
+  cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
+  OnlineParamsDev od;
+  kde_status st = online_params_dev(m, op, &od, s);
+  if (st != KDE_OK) return st;
+  CUL(launch_online_update(m->ret, d_true_sel, od, m->d, m->online, m->consts, s));
+  ++m->gen;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_replace_points_dev(kde_model* m, const int64_t* d_idx, const float* d_rows,
+                                             const int64_t* d_k, int64_t cap, double k_init, void* stream) {
+  CHECK_MODEL(m);
+  if (cap < 0 || (cap > 0 && (!d_idx || !d_rows || !d_k))) return fail(KDE_EINVAL, "NULL device pointer / cap");
+  if (!std::isfinite(k_init)) return fail(KDE_EINVAL, "k_init not finite");
+  DeviceGuard g(m->device);
+  cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
+  ++m->launches;
+  CUL(launch_scatter_rows_dev(d_idx, d_rows, d_k, cap, m->d, m->cols, m->ld, m->n, m->row_offset, m->karma, k_init,
+                              m->range_enc, m->consts, s));
   ++m->gen;
   return KDE_OK;
 }

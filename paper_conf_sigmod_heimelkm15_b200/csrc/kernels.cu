@@ -45,6 +45,72 @@ __global__ void cols_to_rows_kernel(const float* __restrict__ cols, int64_t ld, 
   for (int j = 0; j < d; ++j) rows[i * d + j] = cols[(int64_t)j * ld + i];
 }
 
+// ------------------------------------------------------------ column ranges
+// order-preserving float <-> uint encoding for atomicMin/atomicMax
+__device__ __forceinline__ unsigned fenc(float f) {
+  const unsigned u = __float_as_uint(f);
+  return (u & 0x80000000u) ? ~u : (u | 0x80000000u);
+}
+__device__ __forceinline__ float fdec(unsigned e) {
+  return __uint_as_float((e & 0x80000000u) ? (e & 0x7fffffffu) : ~e);
+}
+
+// enc[2j] = min, enc[2j+1] = max of column j over points [0, n) (accumulating)
+__global__ void col_range_kernel(const float* __restrict__ cols, int64_t ld, int64_t n, unsigned* enc) {
+  const int j = blockIdx.y;
+  float lo = CUDART_INF_F, hi = -CUDART_INF_F;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const float x = cols[(int64_t)j * ld + i];
+    lo = fminf(lo, x);
+    hi = fmaxf(hi, x);
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    lo = fminf(lo, __shfl_xor_sync(0xffffffffu, lo, o));
+    hi = fmaxf(hi, __shfl_xor_sync(0xffffffffu, hi, o));
+  }
+  if ((threadIdx.x & 31) == 0) {
+    atomicMin(enc + 2 * j, fenc(lo));
+    atomicMax(enc + 2 * j + 1, fenc(hi));
+  }
+}
+
+// widen the ranges by k host-supplied rows (row-major, device)
+__global__ void row_range_kernel(const float* __restrict__ rows, int64_t k, int d, unsigned* enc) {
+  const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (e >= k * d) return;
+  const int j = (int)(e % d);
+  atomicMin(enc + 2 * j, fenc(rows[e]));
+  atomicMax(enc + 2 * j + 1, fenc(rows[e]));
+}
+
+__global__ void range_finalize_kernel(const unsigned* __restrict__ enc, int d, DevConsts* c) {
+  const int j = threadIdx.x;
+  if (j >= d) return;
+  c->tmin[j] = fdec(enc[2 * j]);
+  c->tmax[j] = fdec(enc[2 * j + 1]);
+}
+
+// device-resident replacement: the first min(*d_k, cap) GLOBAL indices of
+// idx_global (e.g. the karma compaction output) receive rows[0..], karma reset.
+// Indices outside this shard [row_offset, row_offset + n) are skipped.
+__global__ void scatter_rows_dev_kernel(const int64_t* __restrict__ idx_global, const float* __restrict__ rows,
+                                        const int64_t* __restrict__ d_k, int64_t cap, int d, float* __restrict__ cols,
+                                        int64_t ld, int64_t n, int64_t row_offset, double* __restrict__ karma,
+                                        double k_init, unsigned* __restrict__ enc) {
+  const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t k = min(*d_k, cap);
+  if (r >= k) return;
+  const int64_t i = idx_global[r] - row_offset;
+  if (i < 0 || i >= n) return;
+  for (int j = 0; j < d; ++j) {
+    const float x = rows[r * d + j];
+    cols[(int64_t)j * ld + i] = x;
+    atomicMin(enc + 2 * j, fenc(x));
+    atomicMax(enc + 2 * j + 1, fenc(x));
+  }
+  karma[i] = k_init;
+}
+
 // ------------------------------------------------------------ Scott moments
 // Per (block, column) fp64 Welford over a contiguous chunk, Chan merge in a
 // fixed tree inside the block.  out[(j*nb + b)*3 + {0,1,2}] = (count, mean, M2).
@@ -250,11 +316,13 @@ __device__ double thr20_dev(const float* lo, const float* hi, int d, const DevCo
 }
 
 __global__ void karma_kernel(const float* __restrict__ cvals, double* __restrict__ karma, int64_t n, double n_global,
-                             const double* __restrict__ phat_ptr, double p, KarmaParamsDev kp, const float* lo,
+                             const double* __restrict__ phat_ptr, const double* __restrict__ p_ptr, KarmaParamsDev kp,
+                             const float* lo,
                              const float* hi, int d, const DevConsts* c, uint32_t* __restrict__ bitmap,
                              int32_t* __restrict__ block_counts) {
   __shared__ double thr_s;
   __shared__ int32_t wcount[kKarmaThreads / 32];
+  const double p = *p_ptr;
   if (threadIdx.x == 0) thr_s = (kp.empty_region && p == 0.0) ? thr20_dev(lo, hi, d, c) : CUDART_INF;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   if (lane == 0) wcount[warp] = 0;
@@ -351,9 +419,10 @@ __global__ void compact_kernel(const uint32_t* __restrict__ bitmap, int64_t n, c
 // ret: [1+d] = (p_hat, dp/dh_j) of the retained query.  Adds L' dp/dh (x h in
 // log mode, eq. 18) to the mini-batch; every `minibatch` queries applies the
 // RMSprop / Rprop step of P:L179-183 and re-derives the constants.
-__global__ void online_update_kernel(const double* __restrict__ ret, double p, OnlineParamsDev op, int d,
-                                     OnlineState* st, DevConsts* c) {
+__global__ void online_update_kernel(const double* __restrict__ ret, const double* __restrict__ p_ptr,
+                                     OnlineParamsDev op, int d, OnlineState* st, DevConsts* c) {
   if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  const double p = *p_ptr;
   double L, dL;
   loss_eval(op.loss, op.lambda, ret[0], p, &L, &dL);
   for (int j = 0; j < d; ++j) {
@@ -435,6 +504,36 @@ cudaError_t launch_cols_to_rows(const float* cols, int64_t ld, int64_t n, int d,
   cols_to_rows_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(cols, ld, n, d, rows);
   KDE_LAUNCH_CHECK();
 }
+cudaError_t launch_col_range(const float* cols, int64_t ld, int64_t n, int d, unsigned* enc, DevConsts* c,
+                             cudaStream_t s) {
+  int64_t nb = (n + 255) / 256;
+  if (nb > 1024) nb = 1024;
+  if (nb < 1) nb = 1;
+  col_range_kernel<<<dim3((unsigned)nb, d), 256, 0, s>>>(cols, ld, n, enc);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  range_finalize_kernel<<<1, 32, 0, s>>>(enc, d, c);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_row_range(const float* rows, int64_t k, int d, unsigned* enc, DevConsts* c, cudaStream_t s) {
+  if (k == 0) return cudaSuccess;
+  row_range_kernel<<<(unsigned)((k * d + 255) / 256), 256, 0, s>>>(rows, k, d, enc);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  range_finalize_kernel<<<1, 32, 0, s>>>(enc, d, c);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_scatter_rows_dev(const int64_t* idx_global, const float* rows, const int64_t* d_k, int64_t cap, int d,
+                                    float* cols, int64_t ld, int64_t n, int64_t row_offset, double* karma, double k_init,
+                                    unsigned* enc, DevConsts* c, cudaStream_t s) {
+  if (cap == 0) return cudaSuccess;
+  scatter_rows_dev_kernel<<<(unsigned)((cap + 255) / 256), 256, 0, s>>>(idx_global, rows, d_k, cap, d, cols, ld, n,
+                                                                         row_offset, karma, k_init, enc);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  range_finalize_kernel<<<1, 32, 0, s>>>(enc, d, c);
+  KDE_LAUNCH_CHECK();
+}
 cudaError_t launch_scatter_rows(const int64_t* idx_local, const float* rows, int64_t k, int d, float* cols,
                                 int64_t ld, double* karma, double k_init, cudaStream_t s) {
   if (k == 0) return cudaSuccess;
@@ -493,7 +592,7 @@ cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const do
   loss_epilogue_kernel<<<1, 512, 0, s>>>(est, dpdh, true_sel, q, d, kind, lambda, log_bw, c, loss_out, grad_out);
   KDE_LAUNCH_CHECK();
 }
-cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, double p,
+cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, const double* p,
                          const KarmaParamsDev& kp, const float* lo, const float* hi, int d, const DevConsts* c,
                          uint32_t* bitmap, int32_t* block_counts, int64_t* offsets, int64_t row_offset,
                          int64_t* idx_out, int64_t cap, cudaStream_t s) {
@@ -509,7 +608,7 @@ cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_
   compact_kernel<<<nb, kKarmaThreads, 0, s>>>(bitmap, n, offsets, row_offset, idx_out, cap);
   KDE_LAUNCH_CHECK();
 }
-cudaError_t launch_online_update(const double* ret, double p, const OnlineParamsDev& op, int d, OnlineState* st,
+cudaError_t launch_online_update(const double* ret, const double* p, const OnlineParamsDev& op, int d, OnlineState* st,
                                  DevConsts* c, cudaStream_t s) {
   online_update_kernel<<<1, 32, 0, s>>>(ret, p, op, d, st, c);
   KDE_LAUNCH_CHECK();

@@ -18,6 +18,13 @@ struct HVec {
 cudaError_t launch_rows_to_cols(const float* rows, int64_t n, int d, float* cols, int64_t ld, int* bad,
                                 cudaStream_t s);
 cudaError_t launch_cols_to_rows(const float* cols, int64_t ld, int64_t n, int d, float* rows, cudaStream_t s);
+// per-column [min, max] of the local sample into DevConsts (enc: device [d][2] uint, init 0xFFFFFFFF / 0)
+cudaError_t launch_col_range(const float* cols, int64_t ld, int64_t n, int d, unsigned* enc, DevConsts* c,
+                             cudaStream_t s);
+cudaError_t launch_row_range(const float* rows, int64_t k, int d, unsigned* enc, DevConsts* c, cudaStream_t s);
+cudaError_t launch_scatter_rows_dev(const int64_t* idx_global, const float* rows, const int64_t* d_k, int64_t cap, int d,
+                                    float* cols, int64_t ld, int64_t n, int64_t row_offset, double* karma, double k_init,
+                                    unsigned* enc, DevConsts* c, cudaStream_t s);
 cudaError_t launch_scatter_rows(const int64_t* idx_local, const float* rows, int64_t k, int d, float* cols,
                                 int64_t ld, double* karma, double k_init, cudaStream_t s);
 int moments_blocks(int64_t n);
@@ -35,11 +42,11 @@ cudaError_t launch_finalize(const double* sums, int64_t q, int d, int na, const 
 cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const double* true_sel, int64_t q, int d,
                                  int kind, double lambda, int log_bw, const DevConsts* c, double* loss_out,
                                  double* grad_out, cudaStream_t s);
-cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, double p,
+cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, const double* p,
                          const KarmaParamsDev& kp, const float* lo, const float* hi, int d, const DevConsts* c,
                          uint32_t* bitmap, int32_t* block_counts, int64_t* offsets, int64_t row_offset,
                          int64_t* idx_out, int64_t cap, cudaStream_t s);
-cudaError_t launch_online_update(const double* ret, double p, const OnlineParamsDev& op, int d, OnlineState* st,
+cudaError_t launch_online_update(const double* ret, const double* p, const OnlineParamsDev& op, int d, OnlineState* st,
                                  DevConsts* c, cudaStream_t s);
 cudaError_t launch_count_in_box(const float* rows, int64_t n, int d, const float* lo, const float* hi, int64_t q,
                                 unsigned long long* counts, int num_sms, cudaStream_t s);

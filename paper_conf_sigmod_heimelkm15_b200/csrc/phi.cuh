@@ -15,10 +15,9 @@
 // Scaling: the kernels carry y' = z sqrt(log2 e) = (b - t) * ap, so that
 // E = e^{-z^2} = 2^{-y'^2} is a bare ex2.approx; x = |z| = |y'| / sqrt(log2 e)
 // is folded into the constant P' = P / sqrt(log2 e).
-// Infinite bounds: without the gradient y' = +-inf flows through exactly
-// (E = 2^-inf = 0, t = 1/inf = 0, erfc = 0, 1/2 erf = +-1/2).  With the
-// gradient y' is clamped to +-13 (2^-169 flushes to 0) so that y' E = 0
-// instead of inf * 0.
+// Infinite / far bounds: make_boxdim clamps every bound to the sample's
+// column range widened by 14/ap, so y' stays finite (no inf * 0 in y' E) while
+// |y'| >= 14 still gives E = 0 and erf = +-1 exactly: results are unchanged.
 #pragma once
 #include <cuda_runtime.h>
 #include "phi_coeffs.h"
@@ -61,9 +60,14 @@ struct BoxDim {
   float hd;   // half-width in y' units for narrow dims, 0 otherwise
 };
 
-__device__ __forceinline__ BoxDim make_boxdim(float l, float u, float ap) {
+constexpr float kBoundMargin = 14.0f;  // |y'| >= 14: 2^-196 flushes to 0, erf(z) == +-1 in fp32
+
+__device__ __forceinline__ BoxDim make_boxdim(float l, float u, float ap, float tmin, float tmax) {
   BoxDim r;
   const float dy = (u - l) * ap;  // inf for unbounded, NaN for (inf, inf): both normal
+  const float m = kBoundMargin / ap;
+  l = fminf(fmaxf(l, tmin - m), tmax + m);
+  u = fminf(fmaxf(u, tmin - m), tmax + m);
   if (dy > 0.0f && dy < kNarrowY) {
     r.b = make_float2(l, l);
     r.hd = 0.5f * dy;
@@ -117,10 +121,6 @@ __device__ __forceinline__ float phi_diff(const BoxDim& bd, float t, float ap, f
     y = __ffma2_rn(__fadd2_rn(bd.b, f2(-t)), f2(ap), o);
   } else {
     y = __fmul2_rn(__fadd2_rn(bd.b, f2(-t)), f2(ap));
-  }
-  if (GRAD) {  // y * E would be inf * 0 for an infinite bound; without GRAD inf flows through exactly
-    y.x = fminf(fmaxf(y.x, -kYClamp), kYClamp);
-    y.y = fminf(fmaxf(y.y, -kYClamp), kYClamp);
   }
   const float2 yy = __fmul2_rn(y, y);
   const float2 E = make_float2(ex2_approx(-yy.x), ex2_approx(-yy.y));

@@ -156,7 +156,7 @@ __global__ void __launch_bounds__(kSingleThreads, OCC) scan_single_kernel(const 
   if (threadIdx.x < D) {
     const int j = threadIdx.x;
     const float ap = a.consts->ap[j];
-    const BoxDim bd = make_boxdim(__ldg(a.lo + j), __ldg(a.hi + j), ap);
+    const BoxDim bd = make_boxdim(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->tmin[j], a.consts->tmax[j]);
     smc[j] = make_float4(bd.b.x, bd.b.y, bd.hd, ap);
     if (bd.hd > 0.0f) atomicOr(&narrow_s, 1);
   }
@@ -280,7 +280,10 @@ __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const 
 #pragma unroll
       for (int w = 0; w < kSingleThreads / 32; ++w) tot += red[w][0];
       a.sums_out[k] = tot;
-      if (a.fin_out) a.fin_out[k] = k == 0 ? tot / a.n_global : tot * a.consts->gconst[k - 1] / a.n_global;
+      const double fin = k == 0 ? tot / a.n_global : tot * a.consts->gconst[k - 1] / a.n_global;
+      if (a.fin_out) a.fin_out[k] = fin;
+      if (k == 0 && a.est_out) *a.est_out = fin;
+      if (k > 0 && a.dpdh_out) a.dpdh_out[k - 1] = fin;
     }
   }
   if (threadIdx.x == 0) *a.counter = 0u;
@@ -382,7 +385,8 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
     narrow[qq] = false;
 #pragma unroll
     for (int j = 0; j < D; ++j) {
-      bd[qq][j] = make_boxdim(__ldg(a.lo + qi * D + j), __ldg(a.hi + qi * D + j), ap[j]);
+      bd[qq][j] = make_boxdim(__ldg(a.lo + qi * D + j), __ldg(a.hi + qi * D + j), ap[j], a.consts->tmin[j],
+                               a.consts->tmax[j]);
       narrow[qq] |= bd[qq][j].hd > 0.0f;
     }
   }

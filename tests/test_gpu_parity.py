@@ -390,3 +390,58 @@ def test_c2_full_size_loss_grad_sampled():
     dL = 2 * np.abs(est_o - p[sub])
     mabs = oracle.grad_abs_scale(S, h, lo[sub], hi[sub])
     grad_ok(gs, g_o, (dL[:, None] * mabs).mean(axis=0))
+
+
+# ------------------------------------------------------------------ device-resident streaming step
+def test_device_resident_stream_matches_host_path_and_oracle():
+    """NEXT-2 loop (estimate -> karma -> Listing 1 -> replacement) with device
+    pointers only, bit-identical to the host-pointer calls step by step; the
+    first step's flags also match the oracle."""
+    import torch
+    n, d, steps, cap = 20000, 4, 24, 4096
+    S = synth.make_data("gauss", n, d, seed=40)
+    R = synth.make_data("gauss", 80000, d, seed=40)
+    lo, hi = synth.workload(S, steps, seed=41, kind="DT")
+    p = synth.true_selectivity_cpu(R, lo, hi)
+    p[5] = 0.0
+    pool = synth.replacement_rows(R, steps * cap, seed=42, step=0)
+    kp = K.karma_params(loss=K.LOSS_ABSOLUTE, threshold=-1.0 / (n - 1), k_max=4.0)
+    op = K.online_params(minibatch=5, loss=K.LOSS_ABSOLUTE, log_bandwidth=True)
+    mh, md = model(S), model(S)
+    mh.set_retain(True)
+    md.set_retain(True)
+    dev = torch.device("cuda")
+    dlo, dhi = torch.from_numpy(lo).to(dev), torch.from_numpy(hi).to(dev)
+    dp = torch.from_numpy(p).to(dev)
+    dpool = torch.from_numpy(pool).to(dev)
+    dest = torch.zeros(1, dtype=torch.float64, device=dev)
+    ddpdh = torch.zeros((1, d), dtype=torch.float64, device=dev)
+    didx = torch.zeros(cap, dtype=torch.int64, device=dev)
+    dcnt = torch.zeros(1, dtype=torch.int64, device=dev)
+    s = torch.cuda.current_stream()
+    for k in range(steps):
+        h0 = mh.bandwidth
+        e_h, g_h = mh.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+        idx, nf, trunc = mh.karma_update(lo[k], hi[k], p[k], kp)
+        assert nf <= cap and not trunc
+        if k == 0:
+            c_o = oracle.contributions(S, h0, lo[0], hi[0])
+            Ko = np.zeros(n)
+            idx_o = oracle.karma_update(c_o, c_o.mean(), p[0], K.LOSS_ABSOLUTE, 0.0, 4.0, -1.0 / (n - 1), np.inf, Ko)
+            amb = _karma_guard(Ko, -1.0 / (n - 1), c_o, np.inf, n)
+            fo = np.zeros(n, bool); fo[idx_o] = True
+            fg = np.zeros(n, bool); fg[idx] = True
+            assert np.array_equal(fo[~amb], fg[~amb])
+        mh.online_update(lo[k], hi[k], p[k], op)
+        mh.replace_points(idx, pool[k * cap:k * cap + len(idx)])
+
+        K.kde_estimate_batch_dev(md.handle, dlo[k:k + 1], dhi[k:k + 1], dest, ddpdh, stream=s)
+        K.kde_karma_update_dev(md.handle, dlo[k], dhi[k], dp[k:k + 1], kp, didx, dcnt, stream=s)
+        K.kde_online_update_dev(md.handle, dp[k:k + 1], op, stream=s)
+        K.kde_replace_points_dev(md.handle, didx, dpool[k * cap:(k + 1) * cap], dcnt, stream=s)
+        torch.cuda.synchronize()
+        assert dest.item() == e_h[0] and np.array_equal(ddpdh.cpu().numpy(), g_h)
+        assert int(dcnt.item()) == nf and np.array_equal(didx[:nf].cpu().numpy(), idx)
+        assert np.array_equal(md.bandwidth, mh.bandwidth)
+    assert np.array_equal(md.karma, mh.karma)
+    assert np.array_equal(md.sample, mh.sample)
