@@ -2,6 +2,7 @@
 // Citations "P:L<n>" refer to lines of the paper text.
 #pragma once
 #include <cstdint>
+#include <cstring>
 #include <cuda_runtime.h>
 
 #ifndef KDE_MAX_DIM
@@ -27,9 +28,21 @@ struct DevConsts {
   double h[kMaxDim];
   double gconst[kMaxDim];
   float ap[kMaxDim];
-  float tmin[kMaxDim];
-  float tmax[kMaxDim];
+  unsigned renc[2 * kMaxDim];  // (min, max) per column, order-preserving uint encoding (atomicMin/Max)
 };
+
+// order-preserving float <-> uint encoding used for the column ranges
+__host__ __device__ __forceinline__ unsigned fenc_range(float f) {
+  unsigned u;
+  memcpy(&u, &f, sizeof(u));
+  return (u & 0x80000000u) ? ~u : (u | 0x80000000u);
+}
+__host__ __device__ __forceinline__ float fdec_range(unsigned e) {
+  const unsigned u = (e & 0x80000000u) ? (e & 0x7fffffffu) : ~e;
+  float f;
+  memcpy(&f, &u, sizeof(f));
+  return f;
+}
 
 // Listing 1 state (reconstruction, R6), device resident.
 struct OnlineState {

@@ -6,6 +6,7 @@
 // Every numeric step runs in the kernels of scan.cuh / kernels.cu; this file
 // only moves arguments, validates them and orders launches on one stream.
 #include <algorithm>
+#include <cstddef>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -71,7 +72,7 @@ struct kde_model {
   int64_t* idx_dev = nullptr;
   int64_t idx_cap = 0;
   int32_t* bad = nullptr;            // device flag
-  unsigned* range_enc = nullptr;     // [d][2] encoded column min/max (kernels.cu)
+  unsigned* range_enc = nullptr;     // = consts->renc: [d][2] encoded column min/max (kernels.cu)
   double* scal = nullptr;            // [8] device scalars (true selectivity staging)
   void* pinned = nullptr;            // pinned host staging
   size_t pinned_cap = 0;
@@ -351,7 +352,6 @@ static void free_model(kde_model* m) {
   cudaFree(m->offsets);
   cudaFree(m->idx_dev);
   cudaFree(m->bad);
-  cudaFree(m->range_enc);
   cudaFree(m->scal);
   if (m->pinned) cudaFreeHost(m->pinned);
   for (cudaEvent_t e : m->ev) cudaEventDestroy(e);
@@ -412,7 +412,6 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
   CUB(cudaMalloc(&m->ret, sizeof(double) * (kMaxDim + 1)));
   CUB(cudaMalloc(&m->single_sums, sizeof(double) * (kMaxDim + 1)));
   CUB(cudaMalloc(&m->bad, sizeof(int32_t)));
-  CUB(cudaMalloc(&m->range_enc, sizeof(unsigned) * 2 * kMaxDim));
   CUB(cudaMalloc(&m->scal, sizeof(double) * 8));
   const int nkb = karma_blocks(n_local);
   CUB(cudaMalloc(&m->bitmap, sizeof(uint32_t) * (size_t)nkb * (kKarmaPts / 32)));
@@ -469,7 +468,9 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
       init[2 * j] = 0xFFFFFFFFu;
       init[2 * j + 1] = 0u;
     }
-    CUB(cudaMemcpy(m->range_enc, init.data(), sizeof(unsigned) * 2 * kMaxDim, cudaMemcpyHostToDevice));
+    m->range_enc = reinterpret_cast<unsigned*>(reinterpret_cast<char*>(m->consts) + offsetof(DevConsts, renc));
+    CUB(cudaMemcpyAsync(m->range_enc, init.data(), sizeof(unsigned) * 2 * kMaxDim, cudaMemcpyHostToDevice, s));
+    CUB(cudaStreamSynchronize(s));
     ++m->launches;
     CUB(launch_col_range(m->cols, m->ld, n_local, d, m->range_enc, m->consts, s));
   }
@@ -782,7 +783,7 @@ extern "C" kde_status kde_karma_update(kde_model* m, const float* lo, const floa
   m->launches += 2;  // karma + scan_counts + compact
   CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, m->scal, kd, m->qbuf, m->qbuf + m->d, m->d,
                   m->consts, m->bitmap, m->block_counts, m->offsets, m->row_offset, m->idx_dev, local_cap,
-                  m->stream));
+                  nullptr, m->stream));
   int64_t local_total = 0;
   CU(cudaMemcpyAsync(&local_total, m->offsets + nkb, sizeof(int64_t), cudaMemcpyDeviceToHost, m->stream));
   CU(cudaStreamSynchronize(m->stream));
@@ -921,11 +922,10 @@ extern "C" kde_status kde_karma_update_dev(kde_model* m, const float* d_lo, cons
   if (st != KDE_OK) return st;
   DeviceGuard g(m->device);
   cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
-  const int nkb = karma_blocks(m->n);
   m->launches += 2;
   CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, d_true_sel, kd, d_lo, d_hi, m->d,
-                   m->consts, m->bitmap, m->block_counts, m->offsets, m->row_offset, d_idx_out, idx_cap, s));
-  CU(cudaMemcpyAsync(d_n_flagged, m->offsets + nkb, sizeof(int64_t), cudaMemcpyDeviceToDevice, s));
+                   m->consts, m->bitmap, m->block_counts, m->offsets, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
+                   s));
   return KDE_OK;
 }
 

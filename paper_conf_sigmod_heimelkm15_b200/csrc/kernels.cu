@@ -46,14 +46,8 @@ __global__ void cols_to_rows_kernel(const float* __restrict__ cols, int64_t ld, 
 }
 
 // ------------------------------------------------------------ column ranges
-// order-preserving float <-> uint encoding for atomicMin/atomicMax
-__device__ __forceinline__ unsigned fenc(float f) {
-  const unsigned u = __float_as_uint(f);
-  return (u & 0x80000000u) ? ~u : (u | 0x80000000u);
-}
-__device__ __forceinline__ float fdec(unsigned e) {
-  return __uint_as_float((e & 0x80000000u) ? (e & 0x7fffffffu) : ~e);
-}
+#define fenc fenc_range
+#define fdec fdec_range
 
 // enc[2j] = min, enc[2j+1] = max of column j over points [0, n) (accumulating)
 __global__ void col_range_kernel(const float* __restrict__ cols, int64_t ld, int64_t n, unsigned* enc) {
@@ -83,12 +77,6 @@ __global__ void row_range_kernel(const float* __restrict__ rows, int64_t k, int 
   atomicMax(enc + 2 * j + 1, fenc(rows[e]));
 }
 
-__global__ void range_finalize_kernel(const unsigned* __restrict__ enc, int d, DevConsts* c) {
-  const int j = threadIdx.x;
-  if (j >= d) return;
-  c->tmin[j] = fdec(enc[2 * j]);
-  c->tmax[j] = fdec(enc[2 * j + 1]);
-}
 
 // device-resident replacement: the first min(*d_k, cap) GLOBAL indices of
 // idx_global (e.g. the karma compaction output) receive rows[0..], karma reset.
@@ -332,24 +320,38 @@ __global__ void karma_kernel(const float* __restrict__ cvals, double* __restrict
   loss_eval(kp.loss, kp.lambda, phat, p, &L_full, &dummy);
   const double thr = thr_s;
   const int64_t base = (int64_t)blockIdx.x * kKarmaPts;
+  constexpr int P = kKarmaPts / kKarmaThreads;
+  constexpr int PB = 8;  // points per load batch (PB loads of c and K in flight per thread)
+  const double inv_nm1 = 1.0 / (n_global - 1.0);
   int32_t my = 0;
 #pragma unroll 1
-  for (int pass = 0; pass < kKarmaPts / kKarmaThreads; ++pass) {
-    const int64_t i = base + pass * kKarmaThreads + threadIdx.x;
-    bool flag = false;
-    if (i < n) {
-      const double ci = (double)cvals[i];
-      const double p_minus = (phat * n_global - ci) / (n_global - 1.0);  // eq. (6)
-      double L_minus;
-      loss_eval(kp.loss, kp.lambda, p_minus, p, &L_minus, &dummy);
-      const double k = fmin(karma[i] + (L_minus - L_full), kp.k_max);  // eq. (7)-(8)
-      karma[i] = k;
-      flag = (k < kp.threshold) || (ci >= thr);
+  for (int r0 = 0; r0 < P; r0 += PB) {
+    float cv[PB];
+    double kv[PB];
+#pragma unroll
+    for (int r = 0; r < PB; ++r) {
+      const int64_t i = base + (r0 + r) * kKarmaThreads + threadIdx.x;
+      cv[r] = i < n ? cvals[i] : 0.0f;
+      kv[r] = i < n ? karma[i] : 0.0;
     }
-    const uint32_t word = __ballot_sync(0xffffffffu, flag);
-    if (lane == 0) {
-      bitmap[(i - threadIdx.x + warp * 32) / 32] = word;
-      my += __popc(word);
+#pragma unroll
+    for (int r = 0; r < PB; ++r) {
+      const int64_t i = base + (r0 + r) * kKarmaThreads + threadIdx.x;
+      bool flag = false;
+      if (i < n) {
+        const double ci = (double)cv[r];
+        const double p_minus = (phat * n_global - ci) * inv_nm1;  // eq. (6)
+        double L_minus;
+        loss_eval(kp.loss, kp.lambda, p_minus, p, &L_minus, &dummy);
+        const double k = fmin(kv[r] + (L_minus - L_full), kp.k_max);  // eq. (7)-(8)
+        karma[i] = k;
+        flag = (k < kp.threshold) || (ci >= thr);
+      }
+      const uint32_t word = __ballot_sync(0xffffffffu, flag);
+      if (lane == 0) {
+        bitmap[(base + (r0 + r) * kKarmaThreads + warp * 32) / 32] = word;
+        my += __popc(word);
+      }
     }
   }
   if (lane == 0) wcount[warp] = my;
@@ -361,27 +363,41 @@ __global__ void karma_kernel(const float* __restrict__ cvals, double* __restrict
   }
 }
 
-// exclusive scan of block counts (single block, fixed order); offsets[nb] = total
-__global__ void scan_counts_kernel(const int32_t* __restrict__ counts, int nb, int64_t* __restrict__ offsets) {
-  __shared__ int64_t part[1024];
+// exclusive scan of block counts (one block of 1024 threads: per-thread serial
+// sums of a contiguous range, warp shuffles, warp totals); offsets[nb] = total
+__global__ void scan_counts_kernel(const int32_t* __restrict__ counts, int nb, int64_t* __restrict__ offsets,
+                                   int64_t* __restrict__ total_out) {
+  __shared__ int64_t wsum[32];
   const int T = blockDim.x;
   const int per = (nb + T - 1) / T;
   const int a0 = threadIdx.x * per, a1 = min(nb, a0 + per);
   int64_t s = 0;
   for (int b = a0; b < a1; ++b) s += counts[b];
-  part[threadIdx.x] = s;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  int64_t incl = s;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int64_t v = __shfl_up_sync(0xffffffffu, incl, o);
+    if (lane >= o) incl += v;
+  }
+  if (lane == 31) wsum[warp] = incl;
   __syncthreads();
-  if (threadIdx.x == 0) {
-    int64_t run = 0;
-    for (int t = 0; t < T; ++t) {
-      const int64_t v = part[t];
-      part[t] = run;
-      run += v;
+  if (warp == 0) {
+    int64_t w = lane < T / 32 ? wsum[lane] : 0;
+    int64_t wi = w;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int64_t v = __shfl_up_sync(0xffffffffu, wi, o);
+      if (lane >= o) wi += v;
     }
-    offsets[nb] = run;
+    if (lane < T / 32) wsum[lane] = wi - w;  // exclusive warp offsets
+    if (lane == T / 32 - 1) {
+      offsets[nb] = wi;
+      if (total_out) *total_out = wi;
+    }
   }
   __syncthreads();
-  int64_t run = part[threadIdx.x];
+  int64_t run = wsum[warp] + incl - s;
   for (int b = a0; b < a1; ++b) {
     offsets[b] = run;
     run += counts[b];
@@ -395,11 +411,27 @@ __global__ void compact_kernel(const uint32_t* __restrict__ bitmap, int64_t n, c
   __shared__ int32_t wpre[W];
   const int64_t wbase = (int64_t)blockIdx.x * W;
   const int64_t nwords = (n + 31) / 32;
-  if (threadIdx.x == 0) {
-    int32_t run = 0;
-    for (int w = 0; w < W; ++w) {
-      wpre[w] = run;
-      if (wbase + w < nwords) run += __popc(bitmap[wbase + w]);
+  constexpr int WPL = W / 32;  // bitmap words per lane in the prefix
+  if (threadIdx.x < 32) {  // exclusive prefix of the block's word popcounts
+    const int lane = threadIdx.x;
+    int c[WPL], tot = 0;
+#pragma unroll
+    for (int k = 0; k < WPL; ++k) {
+      const int64_t w = wbase + WPL * lane + k;
+      c[k] = w < nwords ? __popc(bitmap[w]) : 0;
+      tot += c[k];
+    }
+    int incl = tot;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int v = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += v;
+    }
+    int run = incl - tot;
+#pragma unroll
+    for (int k = 0; k < WPL; ++k) {
+      wpre[WPL * lane + k] = run;
+      run += c[k];
     }
   }
   __syncthreads();
@@ -421,40 +453,45 @@ __global__ void compact_kernel(const uint32_t* __restrict__ bitmap, int64_t n, c
 // RMSprop / Rprop step of P:L179-183 and re-derives the constants.
 __global__ void online_update_kernel(const double* __restrict__ ret, const double* __restrict__ p_ptr,
                                      OnlineParamsDev op, int d, OnlineState* st, DevConsts* c) {
-  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  // one thread per dimension (the Listing 1 update is element-wise in j)
+  const int j = threadIdx.x;
   const double p = *p_ptr;
   double L, dL;
   loss_eval(op.loss, op.lambda, ret[0], p, &L, &dL);
-  for (int j = 0; j < d; ++j) {
+  const int count = st->count + 1;
+  const bool apply = count >= op.minibatch;
+  if (j < d) {
     double g = dL * ret[1 + j];
     if (op.log_bw) g *= c->h[j];
-    st->acc[j] += g;
-  }
-  st->count += 1;
-  st->updated = 0;
-  if (st->count < op.minibatch) return;
-  for (int j = 0; j < d; ++j) {
-    const double g = st->acc[j] / (double)op.minibatch;           // line 12
-    st->ms[j] = op.alpha * st->ms[j] + (1.0 - op.alpha) * g * g;   // line 14
-    if (g * st->gprev[j] > 0.0) {                                  // lines 15-16
-      st->lr[j] = fmin(st->lr[j] * op.lr_inc, op.lr_max);
-    } else if (g * st->gprev[j] < 0.0) {
-      st->lr[j] = fmax(st->lr[j] * op.lr_dec, op.lr_min);
-    }
-    double step = st->ms[j] > 0.0 ? st->lr[j] * g / sqrt(st->ms[j]) : 0.0;  // line 17
-    double h = c->h[j];
-    if (op.log_bw) {
-      h = exp(log(h) - step);
+    const double acc = st->acc[j] + g;
+    if (!apply) {
+      st->acc[j] = acc;
     } else {
-      if (step > h / 2.0) step = h / 2.0;  // positivity safeguard
-      h = h - step;
+      const double gm = acc / (double)op.minibatch;                  // line 12
+      const double ms = op.alpha * st->ms[j] + (1.0 - op.alpha) * gm * gm;  // line 14
+      double lr = st->lr[j];
+      if (gm * st->gprev[j] > 0.0) lr = fmin(lr * op.lr_inc, op.lr_max);   // lines 15-16
+      else if (gm * st->gprev[j] < 0.0) lr = fmax(lr * op.lr_dec, op.lr_min);
+      double step = ms > 0.0 ? lr * gm / sqrt(ms) : 0.0;             // line 17
+      double h = c->h[j];
+      if (op.log_bw) {
+        h = exp(log(h) - step);
+      } else {
+        if (step > h / 2.0) step = h / 2.0;  // positivity safeguard
+        h = h - step;
+      }
+      set_consts_dev(c, j, h);
+      st->ms[j] = ms;
+      st->lr[j] = lr;
+      st->gprev[j] = gm;
+      st->acc[j] = 0.0;
     }
-    set_consts_dev(c, j, h);
-    st->gprev[j] = g;
-    st->acc[j] = 0.0;
   }
-  st->count = 0;
-  st->updated = 1;
+  __syncthreads();
+  if (j == 0) {
+    st->count = apply ? 0 : count;
+    st->updated = apply ? 1 : 0;
+  }
 }
 
 // ------------------------------------------------------------ harness: exact box counts
@@ -510,17 +547,11 @@ cudaError_t launch_col_range(const float* cols, int64_t ld, int64_t n, int d, un
   if (nb > 1024) nb = 1024;
   if (nb < 1) nb = 1;
   col_range_kernel<<<dim3((unsigned)nb, d), 256, 0, s>>>(cols, ld, n, enc);
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess) return e;
-  range_finalize_kernel<<<1, 32, 0, s>>>(enc, d, c);
   KDE_LAUNCH_CHECK();
 }
 cudaError_t launch_row_range(const float* rows, int64_t k, int d, unsigned* enc, DevConsts* c, cudaStream_t s) {
   if (k == 0) return cudaSuccess;
   row_range_kernel<<<(unsigned)((k * d + 255) / 256), 256, 0, s>>>(rows, k, d, enc);
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess) return e;
-  range_finalize_kernel<<<1, 32, 0, s>>>(enc, d, c);
   KDE_LAUNCH_CHECK();
 }
 cudaError_t launch_scatter_rows_dev(const int64_t* idx_global, const float* rows, const int64_t* d_k, int64_t cap, int d,
@@ -529,9 +560,6 @@ cudaError_t launch_scatter_rows_dev(const int64_t* idx_global, const float* rows
   if (cap == 0) return cudaSuccess;
   scatter_rows_dev_kernel<<<(unsigned)((cap + 255) / 256), 256, 0, s>>>(idx_global, rows, d_k, cap, d, cols, ld, n,
                                                                          row_offset, karma, k_init, enc);
-  cudaError_t e = cudaGetLastError();
-  if (e != cudaSuccess) return e;
-  range_finalize_kernel<<<1, 32, 0, s>>>(enc, d, c);
   KDE_LAUNCH_CHECK();
 }
 cudaError_t launch_scatter_rows(const int64_t* idx_local, const float* rows, int64_t k, int d, float* cols,
@@ -595,14 +623,14 @@ cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const do
 cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, const double* p,
                          const KarmaParamsDev& kp, const float* lo, const float* hi, int d, const DevConsts* c,
                          uint32_t* bitmap, int32_t* block_counts, int64_t* offsets, int64_t row_offset,
-                         int64_t* idx_out, int64_t cap, cudaStream_t s) {
+                         int64_t* idx_out, int64_t cap, int64_t* total_out, cudaStream_t s) {
   const int nb = karma_blocks(n);
   if (nb == 0) return cudaSuccess;
   karma_kernel<<<nb, kKarmaThreads, 0, s>>>(cvals, karma, n, n_global, phat, p, kp, lo, hi, d, c, bitmap,
                                             block_counts);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  scan_counts_kernel<<<1, 1024, 0, s>>>(block_counts, nb, offsets);
+  scan_counts_kernel<<<1, 1024, 0, s>>>(block_counts, nb, offsets, total_out);
   e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   compact_kernel<<<nb, kKarmaThreads, 0, s>>>(bitmap, n, offsets, row_offset, idx_out, cap);

@@ -8,7 +8,7 @@
 namespace kde {
 
 constexpr int kKarmaThreads = 256;
-constexpr int kKarmaPts = 2048;  // contiguous points per karma block (8 passes)
+constexpr int kKarmaPts = 4096;  // contiguous points per karma block (16 passes, 2 load batches)
 inline int karma_blocks(int64_t n) { return (int)((n + kKarmaPts - 1) / kKarmaPts); }
 
 struct HVec {
@@ -45,7 +45,7 @@ cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const do
 cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, const double* p,
                          const KarmaParamsDev& kp, const float* lo, const float* hi, int d, const DevConsts* c,
                          uint32_t* bitmap, int32_t* block_counts, int64_t* offsets, int64_t row_offset,
-                         int64_t* idx_out, int64_t cap, cudaStream_t s);
+                         int64_t* idx_out, int64_t cap, int64_t* total_out, cudaStream_t s);
 cudaError_t launch_online_update(const double* ret, const double* p, const OnlineParamsDev& op, int d, OnlineState* st,
                                  DevConsts* c, cudaStream_t s);
 cudaError_t launch_count_in_box(const float* rows, int64_t n, int d, const float* lo, const float* hi, int64_t q,

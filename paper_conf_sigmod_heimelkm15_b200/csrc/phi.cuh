@@ -20,6 +20,7 @@
 // |y'| >= 14 still gives E = 0 and erf = +-1 exactly: results are unchanged.
 #pragma once
 #include <cuda_runtime.h>
+#include "common.cuh"
 #include "phi_coeffs.h"
 
 namespace kde {
@@ -62,8 +63,9 @@ struct BoxDim {
 
 constexpr float kBoundMargin = 14.0f;  // |y'| >= 14: 2^-196 flushes to 0, erf(z) == +-1 in fp32
 
-__device__ __forceinline__ BoxDim make_boxdim(float l, float u, float ap, float tmin, float tmax) {
+__device__ __forceinline__ BoxDim make_boxdim(float l, float u, float ap, unsigned rmin_enc, unsigned rmax_enc) {
   BoxDim r;
+  const float tmin = fdec_range(rmin_enc), tmax = fdec_range(rmax_enc);
   const float dy = (u - l) * ap;  // inf for unbounded, NaN for (inf, inf): both normal
   const float m = kBoundMargin / ap;
   l = fminf(fmaxf(l, tmin - m), tmax + m);

@@ -42,7 +42,8 @@ constexpr int kFlushPts = 32;  // fp32 partial sums are flushed to fp64 every kF
 constexpr int kSingleFlushPts = 16;  // single-box scan: fp32 partials flushed every 16 points
 
 // resident 256-thread CTAs per SM for the single-box scan (register budget)
-// (measured on B200 by tools/tune_single.cu, gpurun_out/tune_single1.jsonl)
+// (measured on B200 by tools/tune_single.cu, profiles/r01_tune_single*.jsonl)
+__host__ __device__ constexpr bool single_uses_tma(int d) { return d <= 8; }
 __host__ __device__ constexpr int single_occ(int d, bool grad) {
   return grad ? (d <= 3 ? 4 : (d <= 10 ? 3 : 1)) : (d <= 10 ? 4 : (d <= 14 ? 2 : 1));
 }
@@ -81,6 +82,54 @@ __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
   return v;
+}
+
+// Block reduction of the per-thread fp64 sums (fixed order), one fp64 partial
+// per block, and a deterministic second pass by the last block to finish
+// (fixed strided order + fixed tree) that also finalises p_hat, dp_hat/dh.
+template <int NA>
+__device__ __forceinline__ void single_reduce_finalize(const ScanSingleArgs& a, const double (&acc)[NA]) {
+  __shared__ double red[kSingleThreads / 32][NA];
+  __shared__ bool am_last;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+#pragma unroll
+  for (int k = 0; k < NA; ++k) {
+    const double r = warp_sum(acc[k]);
+    if (lane == 0) red[warp][k] = r;
+  }
+  __syncthreads();
+  if (threadIdx.x < NA) {
+    double t = 0.0;
+#pragma unroll
+    for (int w = 0; w < kSingleThreads / 32; ++w) t += red[w][threadIdx.x];
+    a.block_partials[(int64_t)blockIdx.x * NA + threadIdx.x] = t;
+    __threadfence();
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) am_last = (atomicAdd(a.counter, 1u) == gridDim.x - 1);
+  __syncthreads();
+  if (!am_last) return;
+  __threadfence();
+  // deterministic second pass over the block partials (fixed strided order + fixed tree)
+  for (int k = 0; k < NA; ++k) {
+    double t = 0.0;
+    for (int b = threadIdx.x; b < (int)gridDim.x; b += kSingleThreads) t += __ldcg(a.block_partials + (int64_t)b * NA + k);
+    t = warp_sum(t);
+    __syncthreads();
+    if (lane == 0) red[warp][0] = t;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      double tot = 0.0;
+#pragma unroll
+      for (int w = 0; w < kSingleThreads / 32; ++w) tot += red[w][0];
+      a.sums_out[k] = tot;
+      const double fin = k == 0 ? tot / a.n_global : tot * a.consts->gconst[k - 1] / a.n_global;
+      if (a.fin_out) a.fin_out[k] = fin;
+      if (k == 0 && a.est_out) *a.est_out = fin;
+      if (k > 0 && a.dpdh_out) a.dpdh_out[k - 1] = fin;
+    }
+  }
+  if (threadIdx.x == 0) *a.counter = 0u;
 }
 
 // ---------------------------------------------------------------- single box
@@ -156,7 +205,7 @@ __global__ void __launch_bounds__(kSingleThreads, OCC) scan_single_kernel(const 
   if (threadIdx.x < D) {
     const int j = threadIdx.x;
     const float ap = a.consts->ap[j];
-    const BoxDim bd = make_boxdim(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->tmin[j], a.consts->tmax[j]);
+    const BoxDim bd = make_boxdim(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
     smc[j] = make_float4(bd.b.x, bd.b.y, bd.hd, ap);
     if (bd.hd > 0.0f) atomicOr(&narrow_s, 1);
   }
@@ -245,48 +294,7 @@ __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const 
     for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
   }
 
-  // block reduction (fixed order)
-  __shared__ double red[kSingleThreads / 32][NA];
-  __shared__ bool am_last;
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-#pragma unroll
-  for (int k = 0; k < NA; ++k) {
-    const double r = warp_sum(acc[k]);
-    if (lane == 0) red[warp][k] = r;
-  }
-  __syncthreads();
-  if (threadIdx.x < NA) {
-    double t = 0.0;
-#pragma unroll
-    for (int w = 0; w < kSingleThreads / 32; ++w) t += red[w][threadIdx.x];
-    a.block_partials[(int64_t)blockIdx.x * NA + threadIdx.x] = t;
-    __threadfence();
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) am_last = (atomicAdd(a.counter, 1u) == gridDim.x - 1);
-  __syncthreads();
-  if (!am_last) return;
-  __threadfence();
-  // deterministic second pass over the block partials (fixed strided order + fixed tree)
-  for (int k = 0; k < NA; ++k) {
-    double t = 0.0;
-    for (int b = threadIdx.x; b < (int)gridDim.x; b += kSingleThreads) t += __ldcg(a.block_partials + (int64_t)b * NA + k);
-    t = warp_sum(t);
-    __syncthreads();
-    if (lane == 0) red[warp][0] = t;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      double tot = 0.0;
-#pragma unroll
-      for (int w = 0; w < kSingleThreads / 32; ++w) tot += red[w][0];
-      a.sums_out[k] = tot;
-      const double fin = k == 0 ? tot / a.n_global : tot * a.consts->gconst[k - 1] / a.n_global;
-      if (a.fin_out) a.fin_out[k] = fin;
-      if (k == 0 && a.est_out) *a.est_out = fin;
-      if (k > 0 && a.dpdh_out) a.dpdh_out[k - 1] = fin;
-    }
-  }
-  if (threadIdx.x == 0) *a.counter = 0u;
+  single_reduce_finalize<NA>(a, acc);
 }
 
 // ---------------------------------------------------------------- many boxes
@@ -371,22 +379,70 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
                                               (size_t)QT * NA * kBatchedThreads * sizeof(double));
   const int tid = threadIdx.x;
 
-  // this CTA's boxes: qi = qbase + qq*256 + tid (consecutive threads -> consecutive boxes)
+  // This CTA's 256*QT boxes (slots), qbase + slot.  Boxes with a narrow
+  // dimension need the general Phi path; a CTA-local stable partition puts
+  // them into the last slots so at most one warp mixes both kinds and every
+  // other warp runs the branch-free path.
   const int64_t qbase = (int64_t)blockIdx.x * kBatchedThreads * QT;
-  BoxDim bd[QT][D];
-  bool narrow[QT];
+  __shared__ int perm_s[kBatchedThreads * QT];
+  __shared__ int base_s[2 * QT * (kBatchedThreads / 32) + 1];
+  const int lane = tid & 31, warp = tid >> 5;
   float ap[D];
 #pragma unroll
   for (int j = 0; j < D; ++j) ap[j] = a.consts->ap[j];
+  unsigned nmask[QT];
 #pragma unroll
   for (int qq = 0; qq < QT; ++qq) {
     int64_t qi = qbase + qq * kBatchedThreads + tid;
     if (qi >= a.q) qi = a.q - 1;  // duplicate a valid box; its partial is never written
+    bool nar = false;
+#pragma unroll
+    for (int j = 0; j < D; ++j) {
+      const float l = __ldg(a.lo + qi * D + j), u = __ldg(a.hi + qi * D + j);
+      const float dy = (u - l) * ap[j];
+      nar |= dy > 0.0f && dy < kNarrowY;
+    }
+    nmask[qq] = __ballot_sync(0xffffffffu, nar);
+    if (lane == 0) {
+      base_s[2 * (qq * (kBatchedThreads / 32) + warp)] = 32 - __popc(nmask[qq]);  // normal count
+      base_s[2 * (qq * (kBatchedThreads / 32) + warp) + 1] = __popc(nmask[qq]);  // narrow count
+    }
+  }
+  __syncthreads();
+  if (tid == 0) {  // exclusive prefixes in slot order: normals first, then narrows
+    constexpr int G = QT * (kBatchedThreads / 32);
+    int tn = 0;
+    for (int g = 0; g < G; ++g) tn += base_s[2 * g];
+    int rn = 0, rw = tn;
+    for (int g = 0; g < G; ++g) {
+      const int cn = base_s[2 * g], cw = base_s[2 * g + 1];
+      base_s[2 * g] = rn;
+      base_s[2 * g + 1] = rw;
+      rn += cn;
+      rw += cw;
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int qq = 0; qq < QT; ++qq) {
+    const int g = qq * (kBatchedThreads / 32) + warp;
+    const bool nar = (nmask[qq] >> lane) & 1u;
+    const unsigned lt = (1u << lane) - 1u;
+    const int pos = nar ? base_s[2 * g + 1] + __popc(nmask[qq] & lt) : base_s[2 * g] + __popc(~nmask[qq] & lt);
+    perm_s[pos] = qq * kBatchedThreads + tid;
+  }
+  __syncthreads();
+  BoxDim bd[QT][D];
+  bool narrow[QT];
+#pragma unroll
+  for (int qq = 0; qq < QT; ++qq) {
+    int64_t qi = qbase + perm_s[qq * kBatchedThreads + tid];
+    if (qi >= a.q) qi = a.q - 1;
     narrow[qq] = false;
 #pragma unroll
     for (int j = 0; j < D; ++j) {
-      bd[qq][j] = make_boxdim(__ldg(a.lo + qi * D + j), __ldg(a.hi + qi * D + j), ap[j], a.consts->tmin[j],
-                               a.consts->tmax[j]);
+      bd[qq][j] = make_boxdim(__ldg(a.lo + qi * D + j), __ldg(a.hi + qi * D + j), ap[j], a.consts->renc[2 * j],
+                               a.consts->renc[2 * j + 1]);
       narrow[qq] |= bd[qq][j].hd > 0.0f;
     }
   }
@@ -427,7 +483,7 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
   // partials[(split*(NA) + comp) * q + qi]
 #pragma unroll
   for (int qq = 0; qq < QT; ++qq) {
-    const int64_t qi = qbase + qq * kBatchedThreads + tid;
+    const int64_t qi = qbase + perm_s[qq * kBatchedThreads + tid];
     if (qi < a.q) {
 #pragma unroll
       for (int kk = 0; kk < NA; ++kk)
@@ -437,8 +493,18 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
 }
 
 // ---------------------------------------------------------------- launchers
+// forward declaration (scan_single_tma.cuh, included below)
+template <int D, bool GRAD, int TILE, int STAGES, int OCC>
+cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStream_t s);
+
+// d <= 8: TMA-pipelined variant (1024-point tiles, 3 stages, 2 CTAs/SM);
+// d > 8: register-streaming variant (measured faster or equal there).
 template <int D>
 cudaError_t launch_single_t(bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s) {
+  if (single_uses_tma(D)) {
+    return grad ? launch_single_tma_variant<D, true, 1024, 3, 2>(a, grid, s)
+                : launch_single_tma_variant<D, false, 1024, 3, 2>(a, grid, s);
+  }
   if (grad)
     scan_single_kernel<D, true><<<grid, kSingleThreads, 0, s>>>(a);
   else
@@ -501,6 +567,8 @@ cudaError_t launch_batched_t(bool grad, const ScanBatchedArgs& a_in, int num_sms
 }
 
 }  // namespace kde
+
+#include "scan_single_tma.cuh"
 
 #define KDE_INSTANTIATE_SCAN(D)                                                                              \
   namespace kde {                                                                                            \

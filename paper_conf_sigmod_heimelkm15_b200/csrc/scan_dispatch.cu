@@ -33,6 +33,12 @@ cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int 
 
 // ~3 resident CTAs of 256 threads per SM, never more CTAs than 8-point work items.
 int scan_single_grid(int d, bool grad, int64_t n, int num_sms) {
+  if (single_uses_tma(d)) {  // one contiguous chunk of >= 1 tile per CTA
+    int64_t grid = (int64_t)num_sms * 2;
+    const int64_t ntiles = (n + 1023) / 1024;
+    if (grid > ntiles) grid = ntiles;
+    return (int)(grid < 1 ? 1 : grid);
+  }
   const int per_sm = single_occ(d, grad);
   int64_t grid = (int64_t)num_sms * per_sm;
   const int64_t items = (n + 15) / 16;

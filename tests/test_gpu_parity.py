@@ -445,3 +445,25 @@ def test_device_resident_stream_matches_host_path_and_oracle():
         assert np.array_equal(md.bandwidth, mh.bandwidth)
     assert np.array_equal(md.karma, mh.karma)
     assert np.array_equal(md.sample, mh.sample)
+
+
+def test_batched_mixed_narrow_and_normal_boxes():
+    """Every third box has a dimension narrower than the Gauss-path threshold;
+    the CTA-local partition must return each box's result at its own index."""
+    n, d, q = 30000, 3, 700
+    S = synth.make_data("gauss", n, d, seed=50)
+    m = model(S)
+    h = m.bandwidth
+    lo, hi = synth.mixed_workload(S, q, seed=51)
+    g = synth.rng(52)
+    for k in range(0, q, 3):
+        j = k % d
+        mid = 0.5 * (float(lo[k, j]) + float(hi[k, j]))
+        w = float(h[j]) * g.uniform(1e-4, 0.05)
+        lo[k, j], hi[k, j] = np.float32(mid - w / 2), np.float32(mid + w / 2)
+    est_o, g_o = oracle.estimate_grad(S, h, lo, hi)
+    mabs = oracle.grad_abs_scale(S, h, lo, hi)
+    est, gr = m.estimate(lo, hi, grad=True)
+    sel_ok(est, est_o)
+    grad_ok(gr, g_o, mabs)
+    sel_ok(m.estimate(lo, hi), est_o)

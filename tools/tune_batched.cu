@@ -49,7 +49,7 @@ void setup_and_sweep(int64_t n, int64_t q, int sms) {
   DevConsts hc{};
   const double h = 100.0 * pow((double)n, -1.0 / (D + 4)) * 0.29;
   for (int j = 0; j < D; ++j) {
-    hc.h[j] = h; hc.ap[j] = (float)(1.2011224087864498 / (1.4142135623730951 * h)); hc.tmin[j] = 0.f; hc.tmax[j] = 100.f;
+    hc.h[j] = h; hc.ap[j] = (float)(1.2011224087864498 / (1.4142135623730951 * h)); hc.renc[2 * j] = fenc_range(0.f); hc.renc[2 * j + 1] = fenc_range(100.f);
     hc.gconst[j] = 1.0 / (1.7724538509055160 * 1.2011224087864498 * h);
   }
   float *cols, *lo, *hi; DevConsts* c; double* part;
