@@ -28,11 +28,15 @@ namespace kde {
 // (measured on B200 by tools/tune_batched.cu, gpurun_out/tune1.jsonl)
 template <int D>
 struct QT_for {
-  static constexpr int value = D <= 3 ? 2 : 1;
+  static constexpr int value = 1;
+};
+template <int D>
+struct PU_for {  // points per inner iteration
+  static constexpr int value = (D <= 3 || (D >= 7 && D <= 8)) ? 2 : 1;
 };
 template <int D>
 struct MINB_for {
-  static constexpr int value = D <= 6 ? 4 : (D <= 8 ? 3 : (D <= 12 ? 2 : 1));
+  static constexpr int value = D <= 6 ? 4 : (D <= 12 ? 2 : 1);
 };
 
 constexpr int kSingleThreads = 256;
@@ -326,7 +330,7 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 // The tile loop of the batched scan: wait for tile k (TMA bulk copies
 // completing on bar[k&1]), prefetch tile k+1, accumulate every point of the
 // tile against the thread's QT boxes.
-template <int D, bool GRAD, bool GENERAL, int QT, typename Issue>
+template <int D, bool GRAD, bool GENERAL, int QT, int PU, typename Issue>
 __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const float* tile, uint64_t* bar,
                                               double* accsh, const BoxDim (&bd)[QT][D],
                                               const float (&ap)[D], int64_t s0, int64_t s1, int ntiles,
@@ -347,7 +351,18 @@ __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const fl
       for (int qq = 0; qq < QT; ++qq)
 #pragma unroll
         for (int kk = 0; kk < NA; ++kk) s[qq][kk] = 0.0f;
-      for (int p = p0; p < pe; ++p) {
+      int p = p0;
+      for (; p + PU <= pe; p += PU) {  // PU points per iteration: more independent chains per warp
+#pragma unroll
+        for (int u = 0; u < PU; ++u) {
+          float t[D];
+#pragma unroll
+          for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p + u];
+#pragma unroll
+          for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, GENERAL>(bd[qq], t, ap, s[qq], true);
+        }
+      }
+      for (; p < pe; ++p) {
         float t[D];
 #pragma unroll
         for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
@@ -369,7 +384,7 @@ constexpr size_t batched_smem_bytes() {
   return 2ull * D * kTilePts * sizeof(float) + (size_t)QT * NA * kBatchedThreads * sizeof(double) + 16;
 }
 
-template <int D, bool GRAD, int QT = QT_for<D>::value, int MINB = MINB_for<D>::value>
+template <int D, bool GRAD, int QT = QT_for<D>::value, int MINB = MINB_for<D>::value, int PU = PU_for<D>::value>
 __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(const ScanBatchedArgs a) {
   constexpr int NA = GRAD ? D + 1 : 1;
   extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -476,9 +491,9 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
 #pragma unroll
   for (int qq = 0; qq < QT; ++qq) my_narrow |= narrow[qq];
   if (__any_sync(0xffffffffu, my_narrow))
-    batched_tiles<D, GRAD, true, QT>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
+    batched_tiles<D, GRAD, true, QT, PU>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
   else
-    batched_tiles<D, GRAD, false, QT>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
+    batched_tiles<D, GRAD, false, QT, PU>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
 
   // partials[(split*(NA) + comp) * q + qi]
 #pragma unroll
@@ -519,17 +534,17 @@ cudaError_t launch_single_variant(const ScanSingleArgs& a, int grid, cudaStream_
   return cudaGetLastError();
 }
 
-template <int D, bool GRAD, int QT = QT_for<D>::value, int MINB = MINB_for<D>::value>
+template <int D, bool GRAD, int QT = QT_for<D>::value, int MINB = MINB_for<D>::value, int PU = PU_for<D>::value>
 cudaError_t launch_batched_tg(const ScanBatchedArgs& a, dim3 grid, cudaStream_t s) {
   constexpr size_t smem = batched_smem_bytes<D, GRAD, QT>();
   static bool attr_set = false;
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(scan_batched_kernel<D, GRAD, QT, MINB>,
+    cudaError_t e = cudaFuncSetAttribute(scan_batched_kernel<D, GRAD, QT, MINB, PU>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  scan_batched_kernel<D, GRAD, QT, MINB><<<grid, kBatchedThreads, smem, s>>>(a);
+  scan_batched_kernel<D, GRAD, QT, MINB, PU><<<grid, kBatchedThreads, smem, s>>>(a);
   return cudaGetLastError();
 }
 

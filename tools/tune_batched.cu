@@ -10,7 +10,7 @@
 
 using namespace kde;
 
-template <int D, int QT, int MINB>
+template <int D, int QT, int MINB, int PU = 1>
 void run(int64_t n, int64_t q, int waves, const float* cols, int64_t ld, const float* lo, const float* hi,
          const DevConsts* consts, double* partials, int sms) {
   ScanBatchedArgs a{};
@@ -23,7 +23,7 @@ void run(int64_t n, int64_t q, int waves, const float* cols, int64_t ld, const f
   std::vector<float> ts;
   for (int r = 0; r < 7; ++r) {
     cudaEventRecord(e0);
-    cudaError_t err = launch_batched_tg<D, true, QT, MINB>(a, grid, 0);
+    cudaError_t err = launch_batched_tg<D, true, QT, MINB, PU>(a, grid, 0);
     cudaEventRecord(e1);
     cudaEventSynchronize(e1);
     if (err != cudaSuccess) { printf("err %s\n", cudaGetErrorString(err)); return; }
@@ -32,7 +32,7 @@ void run(int64_t n, int64_t q, int waves, const float* cols, int64_t ld, const f
   }
   std::sort(ts.begin(), ts.end());
   const double ms = ts[ts.size() / 2];
-  printf("{\"D\":%d,\"QT\":%d,\"MINB\":%d,\"waves\":%d,\"grid\":[%lld,%lld],\"ms\":%.3f,\"Gptq_s\":%.1f}\n", D, QT, MINB,
+  printf("{\"D\":%d,\"PU\":%d,\"QT\":%d,\"MINB\":%d,\"waves\":%d,\"grid\":[%lld,%lld],\"ms\":%.3f,\"Gptq_s\":%.1f}\n", D, PU, QT, MINB,
          waves, (long long)qtiles, (long long)splits, ms, n * (double)q / (ms * 1e-3) / 1e9);
 }
 
@@ -43,7 +43,7 @@ void setup_and_sweep(int64_t n, int64_t q, int sms) {
   srand(1);
   for (auto& x : h_cols) x = 100.0f * rand() / RAND_MAX;
   for (int64_t k = 0; k < q * D; ++k) {
-    float c = 100.0f * rand() / RAND_MAX, w = 30.0f * rand() / RAND_MAX;
+    float c = 100.0f * rand() / RAND_MAX, w = 5.0f + 30.0f * rand() / RAND_MAX;
     h_lo[k] = c - w / 2; h_hi[k] = c + w / 2;
   }
   DevConsts hc{};
@@ -60,12 +60,13 @@ void setup_and_sweep(int64_t n, int64_t q, int sms) {
   cudaMemcpy(hi, h_hi.data(), q * D * 4, cudaMemcpyHostToDevice);
   cudaMemcpy(c, &hc, sizeof(hc), cudaMemcpyHostToDevice);
 #define R(QT, MINB, W) run<D, QT, MINB>(n, q, W, cols, ld, lo, hi, c, part, sms);
+#define RU(QT, MINB, W, PU) run<D, QT, MINB, PU>(n, q, W, cols, ld, lo, hi, c, part, sms);
   if constexpr (D <= 3) {
-    R(4, 2, 4) R(4, 2, 8) R(4, 1, 8) R(2, 2, 4) R(2, 3, 4) R(2, 4, 4) R(1, 4, 4) R(1, 3, 4) R(2, 3, 8) R(4, 2, 16)
+    R(2, 4, 4) RU(2, 4, 4, 2) RU(2, 3, 4, 2) RU(1, 4, 4, 2) RU(1, 4, 4, 4) RU(2, 2, 4, 2) RU(4, 2, 4, 2)
   } else if constexpr (D <= 6) {
-    R(2, 2, 4) R(2, 2, 8) R(2, 3, 4) R(1, 2, 4) R(1, 3, 4) R(1, 4, 4) R(2, 1, 4) R(1, 4, 8)
+    R(1, 4, 4) RU(1, 4, 4, 2) RU(1, 3, 4, 2) RU(2, 3, 4, 2) RU(2, 2, 4, 2)
   } else {
-    R(1, 2, 4) R(1, 1, 4) R(1, 3, 4) R(2, 1, 4) R(1, 2, 8)
+    R(1, 3, 4) RU(1, 3, 4, 2) RU(1, 2, 4, 2)
   }
   cudaFree(cols); cudaFree(lo); cudaFree(hi); cudaFree(c); cudaFree(part);
 }
