@@ -327,15 +327,54 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
       : "memory");
 }
 
-// The tile loop of the batched scan: wait for tile k (TMA bulk copies
-// completing on bar[k&1]), prefetch tile k+1, accumulate every point of the
-// tile against the thread's QT boxes.
-template <int D, bool GRAD, bool GENERAL, int QT, int PU, typename Issue>
-__device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const float* tile, uint64_t* bar,
-                                              double* accsh, const BoxDim (&bd)[QT][D],
-                                              const float (&ap)[D], int64_t s0, int64_t s1, int ntiles,
-                                              Issue& issue) {
+// Accumulate every point of one shared-memory tile against the thread's QT
+// boxes.  No barriers inside, so the GENERAL (narrow-dimension) and fast
+// variants can be chosen per warp.
+template <int D, bool GRAD, bool GENERAL, int QT, int PU>
+__device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, double* accsh,
+                                                     const BoxDim (&bd)[QT][D], const float (&ap)[D]) {
   constexpr int NA = GRAD ? D + 1 : 1;
+  const int tid = threadIdx.x;
+  for (int p0 = 0; p0 < npts; p0 += kFlushPts) {
+    const int pe = min(p0 + kFlushPts, npts);
+    float s[QT][NA];
+#pragma unroll
+    for (int qq = 0; qq < QT; ++qq)
+#pragma unroll
+      for (int kk = 0; kk < NA; ++kk) s[qq][kk] = 0.0f;
+    int p = p0;
+    for (; p + PU <= pe; p += PU) {  // PU points per iteration: more independent chains per warp
+#pragma unroll
+      for (int u = 0; u < PU; ++u) {
+        float t[D];
+#pragma unroll
+        for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p + u];
+#pragma unroll
+        for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, GENERAL>(bd[qq], t, ap, s[qq], true);
+      }
+    }
+    for (; p < pe; ++p) {
+      float t[D];
+#pragma unroll
+      for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
+#pragma unroll
+      for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, GENERAL>(bd[qq], t, ap, s[qq], true);
+    }
+#pragma unroll
+    for (int qq = 0; qq < QT; ++qq)
+#pragma unroll
+      for (int kk = 0; kk < NA; ++kk) accsh[(qq * NA + kk) * kBatchedThreads + tid] += (double)s[qq][kk];
+  }
+}
+
+// The tile loop of the batched scan: wait for tile k (TMA bulk copies
+// completing on bar[k&1]), prefetch tile k+1, compute (warp-uniform variant),
+// then the CTA barrier that releases the buffer -- barriers stay outside the
+// warp-divergent part.
+template <int D, bool GRAD, int QT, int PU, typename Issue>
+__device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const float* tile, uint64_t* bar,
+                                              double* accsh, const BoxDim (&bd)[QT][D], const float (&ap)[D],
+                                              int64_t s0, int64_t s1, int ntiles, bool warp_general, Issue& issue) {
   const int tid = threadIdx.x;
   for (int k = 0; k < ntiles; ++k) {
     const int buf = k & 1;
@@ -344,36 +383,10 @@ __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const fl
     const float* tl = tile + buf * D * kTilePts;
     const int64_t rem = s1 - (s0 + (int64_t)k * kTilePts);
     const int npts = rem < kTilePts ? (int)rem : kTilePts;
-    for (int p0 = 0; p0 < npts; p0 += kFlushPts) {
-      const int pe = min(p0 + kFlushPts, npts);
-      float s[QT][NA];
-#pragma unroll
-      for (int qq = 0; qq < QT; ++qq)
-#pragma unroll
-        for (int kk = 0; kk < NA; ++kk) s[qq][kk] = 0.0f;
-      int p = p0;
-      for (; p + PU <= pe; p += PU) {  // PU points per iteration: more independent chains per warp
-#pragma unroll
-        for (int u = 0; u < PU; ++u) {
-          float t[D];
-#pragma unroll
-          for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p + u];
-#pragma unroll
-          for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, GENERAL>(bd[qq], t, ap, s[qq], true);
-        }
-      }
-      for (; p < pe; ++p) {
-        float t[D];
-#pragma unroll
-        for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
-#pragma unroll
-        for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, GENERAL>(bd[qq], t, ap, s[qq], true);
-      }
-#pragma unroll
-      for (int qq = 0; qq < QT; ++qq)
-#pragma unroll
-        for (int kk = 0; kk < NA; ++kk) accsh[(qq * NA + kk) * kBatchedThreads + tid] += (double)s[qq][kk];
-    }
+    if (warp_general)
+      batched_tile_compute<D, GRAD, true, QT, PU>(tl, npts, accsh, bd, ap);
+    else
+      batched_tile_compute<D, GRAD, false, QT, PU>(tl, npts, accsh, bd, ap);
     __syncthreads();
   }
 }
@@ -490,10 +503,8 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
   bool my_narrow = false;
 #pragma unroll
   for (int qq = 0; qq < QT; ++qq) my_narrow |= narrow[qq];
-  if (__any_sync(0xffffffffu, my_narrow))
-    batched_tiles<D, GRAD, true, QT, PU>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
-  else
-    batched_tiles<D, GRAD, false, QT, PU>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, issue);
+  const bool warp_general = __any_sync(0xffffffffu, my_narrow);
+  batched_tiles<D, GRAD, QT, PU>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, warp_general, issue);
 
   // partials[(split*(NA) + comp) * q + qi]
 #pragma unroll

@@ -1,0 +1,62 @@
+"""Small run through every libkde entry point, for compute-sanitizer
+(memcheck / racecheck / synccheck / initcheck) on the GPU box:
+
+  compute-sanitizer --tool memcheck python tools/sanitize_run.py
+"""
+import os
+import sys
+
+import numpy as np
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+import paper_conf_sigmod_heimelkm15_b200 as K  # noqa: E402
+import synth  # noqa: E402
+
+
+def run(d, n, q):
+    S = synth.make_data("gauss", n, d, seed=d)
+    lo, hi = synth.mixed_workload(S, q, seed=d + 1)
+    lo2, hi2 = synth.special_boxes(S, seed=d + 2)
+    lo, hi = np.concatenate([lo, lo2]), np.concatenate([hi, hi2])
+    p = synth.true_selectivity_cpu(S, lo, hi)
+    m = K.KDEModel.create(S)
+    m.set_retain(True)
+    m.estimate(lo, hi, grad=True)
+    m.estimate(lo, hi)
+    for k in (0, 3, len(lo) - 1):
+        m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+        m.estimate(lo[k:k + 1], hi[k:k + 1])
+    m.loss_and_grad(lo, hi, p, K.LOSS_RELATIVE, 1e-3, True)
+    m.loss_and_grad(lo[:1], hi[:1], p[:1], K.LOSS_SQUARED_Q, 1e-3, False)
+    kp = K.karma_params(threshold=-1.0 / (n - 1))
+    idx, nf, _ = m.karma_update(lo[0], hi[0], 0.0, kp)
+    m.online_update(lo[1], hi[1], p[1], K.online_params(minibatch=1))
+    if nf:
+        m.replace_points(idx, S[:nf][::-1].copy())
+    dev = torch.device("cuda")
+    dlo, dhi = torch.from_numpy(lo).to(dev), torch.from_numpy(hi).to(dev)
+    dp = torch.from_numpy(p).to(dev)
+    est = torch.zeros(len(lo), dtype=torch.float64, device=dev)
+    g = torch.zeros((len(lo), d), dtype=torch.float64, device=dev)
+    K.kde_estimate_batch_dev(m.handle, dlo[:1], dhi[:1], est[:1], g[:1])
+    didx = torch.zeros(256, dtype=torch.int64, device=dev)
+    dcnt = torch.zeros(1, dtype=torch.int64, device=dev)
+    K.kde_karma_update_dev(m.handle, dlo[0], dhi[0], dp[:1], kp, didx, dcnt)
+    K.kde_online_update_dev(m.handle, dp[:1], K.online_params(minibatch=1))
+    rows = torch.from_numpy(S[:256].copy()).to(dev)
+    K.kde_replace_points_dev(m.handle, didx, rows, dcnt)
+    loss = torch.zeros(1, dtype=torch.float64, device=dev)
+    K.kde_loss_and_grad_dev(m.handle, dlo, dhi, dp, loss, g[0], K.LOSS_ABSOLUTE, 0.0, False)
+    torch.cuda.synchronize()
+    cnt = torch.zeros(len(lo), dtype=torch.int64, device=dev)
+    K.kde_count_in_box_dev(torch.from_numpy(S).to(dev), dlo, dhi, cnt)
+    torch.cuda.synchronize()
+    m.close()
+
+
+if __name__ == "__main__":
+    for d, n, q in [(3, 5003, 40), (10, 3001, 17), (13, 2053, 9)]:
+        run(d, n, q)
+    print("sanitize run ok")
