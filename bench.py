@@ -60,7 +60,7 @@ CONFIGS = {
     "c5": dict(d=10, n=1 << 22, q=1, path="stream", grad=True, retain=True, data="gauss",
                desc="configs[4] streaming step: d=10, N=2^22, one DT box per step: estimate + gradient + retained "
                     "contributions, karma pass + compaction, Listing 1 bandwidth step, replacement of flagged points "
-                    "(device-resident, single GPU)"),
+                    "(device-resident kde_stream_step_dev: 3 kernels, single GPU)"),
     "c4": dict(d=8, n=1 << 25, q=4096, path="loss_grad", data="gauss",
                desc="configs[3] per-GPU shard: d=8, 2^25 rows/GPU (2^28 at 8 GPUs), 4096 boxes, estimate + gradient + NCCL"),
 }
@@ -279,11 +279,9 @@ def run_cuda(args, cfg, rank, world, local_rank):
     def step(i):
         if cfg["path"] == "stream":
             k = i % nbox
-            K.kde_estimate_batch_dev(m.handle, d_lo[k:k + 1], d_hi[k:k + 1], d_est[:1], d_dpdh[:1], stream=stream)
-            K.kde_karma_update_dev(m.handle, d_lo[k], d_hi[k], d_true[k:k + 1], kp, d_idx, d_cnt, stream=stream)
-            K.kde_online_update_dev(m.handle, d_true[k:k + 1], op, stream=stream)
             off = (i * 977) % npool
-            K.kde_replace_points_dev(m.handle, d_idx, d_pool[off:off + cap], d_cnt, stream=stream)
+            K.kde_stream_step_dev(m.handle, d_lo[k:k + 1], d_hi[k:k + 1], d_true[k:k + 1], kp, op, d_idx, d_cnt,
+                                  d_pool[off:off + cap], d_est[:1], d_dpdh[0], stream=stream)
             return
         if cfg["path"] == "single":
             k = i % nbox

@@ -233,6 +233,21 @@ kde_status kde_online_update_dev(kde_model *m, const double *d_true_sel, const k
 kde_status kde_replace_points_dev(kde_model *m, const int64_t *d_idx, const float *d_rows, const int64_t *d_k,
                                   int64_t cap, double k_init, void *stream);
 
+/* One whole streaming step in three kernels (device pointers, single GPU):
+ * single-box estimate (eq. 2/13) -> d_est[1]; gradient (eq. 17) -> d_dpdh[d]
+ * when op != NULL; karma pass (eq. 6-8, 20) with retained contributions;
+ * ordered compaction of the flagged GLOBAL indices -> d_idx_out (first
+ * idx_cap), count -> *d_n_flagged; then, in the compaction's last block, the
+ * Listing 1 step (op != NULL) and the replacement of the first
+ * min(count, idx_cap) flagged points by d_rows (row-major, idx_cap x d;
+ * NULL = no replacement), karma reset to k_init.  Equivalent to
+ * kde_estimate_batch_dev + kde_karma_update_dev + kde_online_update_dev +
+ * kde_replace_points_dev with the same arguments (retain is implied). */
+kde_status kde_stream_step_dev(kde_model *m, const float *d_lo, const float *d_hi, const double *d_true_sel,
+                               const kde_karma_params *kp, const kde_online_params *op, int64_t *d_idx_out,
+                               int64_t idx_cap, int64_t *d_n_flagged, const float *d_rows, double k_init,
+                               double *d_est, double *d_dpdh, void *stream);
+
 /* ---------------------------------------------------------------- inspection */
 kde_status kde_get_karma(kde_model *m, double *karma);   /* local n fp64          */
 kde_status kde_set_karma(kde_model *m, const double *karma); /* local n fp64      */

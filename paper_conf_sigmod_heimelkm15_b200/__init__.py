@@ -34,7 +34,7 @@ ABI_SYMBOLS = (
     "kde_loss_and_grad_dev", "kde_karma_update", "kde_online_update", "kde_replace_points",
     "kde_get_karma", "kde_set_karma", "kde_get_sample", "kde_get_contributions", "kde_get_online_state",
     "kde_set_online_state", "kde_synchronize", "kde_count_in_box_dev", "kde_set_profiling", "kde_get_profile",
-    "kde_karma_update_dev", "kde_online_update_dev", "kde_replace_points_dev",
+    "kde_karma_update_dev", "kde_online_update_dev", "kde_replace_points_dev", "kde_stream_step_dev",
 )
 
 
@@ -118,6 +118,8 @@ def lib() -> ctypes.CDLL:
         "kde_karma_update_dev": (ctypes.c_int, [P, P, P, P, ctypes.POINTER(KarmaParams), P, i64, P, P]),
         "kde_online_update_dev": (ctypes.c_int, [P, P, ctypes.POINTER(OnlineParams), P]),
         "kde_replace_points_dev": (ctypes.c_int, [P, P, P, P, i64, f64, P]),
+        "kde_stream_step_dev": (ctypes.c_int, [P, P, P, P, ctypes.POINTER(KarmaParams), ctypes.POINTER(OnlineParams),
+                                               P, i64, P, P, f64, P, P, P]),
     }
     for name, (res, args) in sigs.items():
         fn = getattr(L, name)
@@ -285,6 +287,16 @@ def kde_replace_points_dev(m, d_idx, d_rows, d_count, k_init=0.0, stream=None):
     """Rows d_rows[r] -> global index d_idx[r] for r < min(d_count, len(d_idx))."""
     _check(lib().kde_replace_points_dev(m, _tp(d_idx), _tp(d_rows), _tp(d_count), d_idx.numel(), float(k_init),
                                         _stream_ptr(stream)))
+
+
+def kde_stream_step_dev(m, d_lo, d_hi, d_true, kparams: KarmaParams, oparams, d_idx, d_count, d_rows, d_est,
+                        d_dpdh, k_init=0.0, stream=None):
+    """One device-resident streaming step (estimate + gradient + karma +
+    Listing 1 + replacement) in three kernels; enqueue only."""
+    _check(lib().kde_stream_step_dev(m, _tp(d_lo), _tp(d_hi), _tp(d_true), ctypes.byref(kparams),
+                                     None if oparams is None else ctypes.byref(oparams), _tp(d_idx), d_idx.numel(),
+                                     _tp(d_count), _tp(d_rows), float(k_init), _tp(d_est), _tp(d_dpdh),
+                                     _stream_ptr(stream)))
 
 
 def kde_replace_points(m, idx, rows, k_init=0.0):

@@ -68,7 +68,8 @@ struct kde_model {
   size_t gather_cap = 0;
   uint32_t* bitmap = nullptr;
   int32_t* block_counts = nullptr;
-  int64_t* offsets = nullptr;
+  int64_t* offsets = nullptr;        // [0] = total flagged (karma compaction)
+  unsigned* done = nullptr;          // compaction last-block counter (self-resetting)
   int64_t* idx_dev = nullptr;
   int64_t idx_cap = 0;
   int32_t* bad = nullptr;            // device flag
@@ -350,6 +351,7 @@ static void free_model(kde_model* m) {
   cudaFree(m->bitmap);
   cudaFree(m->block_counts);
   cudaFree(m->offsets);
+  cudaFree(m->done);
   cudaFree(m->idx_dev);
   cudaFree(m->bad);
   cudaFree(m->scal);
@@ -416,7 +418,8 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
   const int nkb = karma_blocks(n_local);
   CUB(cudaMalloc(&m->bitmap, sizeof(uint32_t) * (size_t)nkb * (kKarmaPts / 32)));
   CUB(cudaMalloc(&m->block_counts, sizeof(int32_t) * (size_t)nkb));
-  CUB(cudaMalloc(&m->offsets, sizeof(int64_t) * (size_t)(nkb + 1)));
+  CUB(cudaMalloc(&m->offsets, sizeof(int64_t) * 2));
+  CUB(cudaMalloc(&m->done, sizeof(unsigned)));
   cudaStream_t s = m->stream;
   CUB(cudaMemsetAsync(m->cols, 0, sizeof(float) * (size_t)d * m->ld, s));
   CUB(cudaMemsetAsync(m->karma, 0, sizeof(double) * (size_t)n_local, s));
@@ -424,6 +427,7 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
   CUB(cudaMemsetAsync(m->consts, 0, sizeof(DevConsts), s));
   CUB(cudaMemsetAsync(m->online, 0, sizeof(OnlineState), s));
   CUB(cudaMemsetAsync(m->counter, 0, sizeof(unsigned), s));
+  CUB(cudaMemsetAsync(m->done, 0, sizeof(unsigned), s));
   CUB(cudaMemsetAsync(m->bad, 0, sizeof(int32_t), s));
 
   if (world > 1) {
@@ -778,14 +782,13 @@ extern "C" kde_status kde_karma_update(kde_model* m, const float* lo, const floa
   kd.lambda = kp->lambda;
   kd.k_max = kp->k_max;
   kd.threshold = kp->threshold;
-  const int nkb = karma_blocks(m->n);
   CU(cudaMemcpyAsync(m->scal, &true_sel, sizeof(double), cudaMemcpyHostToDevice, m->stream));
-  m->launches += 2;  // karma + scan_counts + compact
+  m->launches += 1;  // karma + fused compaction
   CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, m->scal, kd, m->qbuf, m->qbuf + m->d, m->d,
-                  m->consts, m->bitmap, m->block_counts, m->offsets, m->row_offset, m->idx_dev, local_cap,
-                  nullptr, m->stream));
+                  m->consts, m->bitmap, m->block_counts, m->done, m->row_offset, m->idx_dev, local_cap, m->offsets,
+                  StreamTail{}, m->stream));
   int64_t local_total = 0;
-  CU(cudaMemcpyAsync(&local_total, m->offsets + nkb, sizeof(int64_t), cudaMemcpyDeviceToHost, m->stream));
+  CU(cudaMemcpyAsync(&local_total, m->offsets, sizeof(int64_t), cudaMemcpyDeviceToHost, m->stream));
   CU(cudaStreamSynchronize(m->stream));
   if (m->world == 1) {
     const int64_t ncopy = std::min(local_total, idx_cap);
@@ -922,10 +925,10 @@ extern "C" kde_status kde_karma_update_dev(kde_model* m, const float* d_lo, cons
   if (st != KDE_OK) return st;
   DeviceGuard g(m->device);
   cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
-  m->launches += 2;
+  m->launches += 1;
   CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, d_true_sel, kd, d_lo, d_hi, m->d,
-                   m->consts, m->bitmap, m->block_counts, m->offsets, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
-                   s));
+                   m->consts, m->bitmap, m->block_counts, m->done, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
+                   StreamTail{}, s));
   return KDE_OK;
 }
 
@@ -953,6 +956,55 @@ extern "C" kde_status kde_replace_points_dev(kde_model* m, const int64_t* d_idx,
   ++m->launches;
   CUL(launch_scatter_rows_dev(d_idx, d_rows, d_k, cap, m->d, m->cols, m->ld, m->n, m->row_offset, m->karma, k_init,
                               m->range_enc, m->consts, s));
+  ++m->gen;
+  return KDE_OK;
+}
+
+// One device-resident streaming step in three kernels: the
+// single-box scan (estimate, gradient when op != NULL, retained p^(i)), the
+// karma pass, and the fused compaction whose last block also runs the
+// Listing 1 step and replaces the flagged points by d_rows.
+extern "C" kde_status kde_stream_step_dev(kde_model* m, const float* d_lo, const float* d_hi,
+                                          const double* d_true_sel, const kde_karma_params* kp,
+                                          const kde_online_params* op, int64_t* d_idx_out, int64_t idx_cap,
+                                          int64_t* d_n_flagged, const float* d_rows, double k_init, double* d_est,
+                                          double* d_dpdh, void* stream) {
+  CHECK_MODEL(m);
+  if (m->world != 1) return fail(KDE_EINVAL, "device-resident streaming step is single-GPU (world == 1)");
+  if (!d_lo || !d_hi || !d_true_sel || !d_n_flagged || !d_est || idx_cap < 0 || (idx_cap > 0 && !d_idx_out))
+    return fail(KDE_EINVAL, "NULL device pointer / bad idx_cap");
+  if (op && !d_dpdh) return fail(KDE_EINVAL, "the online update needs d_dpdh (gradient of the estimate)");
+  if (!std::isfinite(k_init)) return fail(KDE_EINVAL, "k_init not finite");
+  KarmaParamsDev kd;
+  kde_status st = karma_params_dev(kp, &kd);
+  if (st != KDE_OK) return st;
+  DeviceGuard g(m->device);
+  cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
+  StreamTail tail;
+  if (op) {
+    st = online_params_dev(m, op, &tail.op, s);
+    if (st != KDE_OK) return st;
+    tail.online = 1;
+    tail.ret = m->ret;
+    tail.p = d_true_sel;
+    tail.st = m->online;
+  }
+  tail.c = m->consts;
+  tail.d = m->d;
+  if (d_rows && idx_cap > 0) {
+    tail.rows = d_rows;
+    tail.cols = m->cols;
+    tail.ld = m->ld;
+    tail.karma = m->karma;
+    tail.k_init = k_init;
+  }
+  m->ret_valid = false;
+  st = estimate_dev(m, d_lo, d_hi, 1, d_est, op ? d_dpdh : nullptr, s, true);
+  if (st != KDE_OK) return st;
+  m->launches += 1;
+  CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, d_true_sel, kd, d_lo, d_hi, m->d,
+                   m->consts, m->bitmap, m->block_counts, m->done, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
+                   tail, s));
   ++m->gen;
   return KDE_OK;
 }

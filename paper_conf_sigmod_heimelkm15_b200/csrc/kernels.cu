@@ -363,57 +363,33 @@ __global__ void karma_kernel(const float* __restrict__ cvals, double* __restrict
   }
 }
 
-// exclusive scan of block counts (one block of 1024 threads: per-thread serial
-// sums of a contiguous range, warp shuffles, warp totals); offsets[nb] = total
-__global__ void scan_counts_kernel(const int32_t* __restrict__ counts, int nb, int64_t* __restrict__ offsets,
-                                   int64_t* __restrict__ total_out) {
-  __shared__ int64_t wsum[32];
-  const int T = blockDim.x;
-  const int per = (nb + T - 1) / T;
-  const int a0 = threadIdx.x * per, a1 = min(nb, a0 + per);
-  int64_t s = 0;
-  for (int b = a0; b < a1; ++b) s += counts[b];
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  int64_t incl = s;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const int64_t v = __shfl_up_sync(0xffffffffu, incl, o);
-    if (lane >= o) incl += v;
-  }
-  if (lane == 31) wsum[warp] = incl;
-  __syncthreads();
-  if (warp == 0) {
-    int64_t w = lane < T / 32 ? wsum[lane] : 0;
-    int64_t wi = w;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const int64_t v = __shfl_up_sync(0xffffffffu, wi, o);
-      if (lane >= o) wi += v;
-    }
-    if (lane < T / 32) wsum[lane] = wi - w;  // exclusive warp offsets
-    if (lane == T / 32 - 1) {
-      offsets[nb] = wi;
-      if (total_out) *total_out = wi;
-    }
-  }
-  __syncthreads();
-  int64_t run = wsum[warp] + incl - s;
-  for (int b = a0; b < a1; ++b) {
-    offsets[b] = run;
-    run += counts[b];
-  }
-}
+__device__ void online_update_body(const double* __restrict__ ret, const double* __restrict__ p_ptr,
+                                   const OnlineParamsDev& op, int d, OnlineState* st, DevConsts* c);
 
-// write ascending global indices (row_offset + i), at most cap of them
-__global__ void compact_kernel(const uint32_t* __restrict__ bitmap, int64_t n, const int64_t* __restrict__ offsets,
-                               int64_t row_offset, int64_t* __restrict__ idx_out, int64_t cap) {
+// Ordered compaction of the karma flags: block b writes the ascending GLOBAL
+// indices of its flagged points at offset sum_{b' < b} count[b'] (computed by
+// the block itself -- no separate scan pass); at most cap are written.  The
+// last block to finish writes the total and runs the optional tail of a
+// device-resident streaming step: the Listing 1 bandwidth update and the
+// replacement of the first min(total, cap) flagged points by tail.rows.
+__global__ void compact_fused_kernel(const uint32_t* __restrict__ bitmap, int64_t n, const int32_t* __restrict__ counts,
+                                     int nb, int64_t row_offset, int64_t* __restrict__ idx_out, int64_t cap,
+                                     int64_t* __restrict__ total_out, unsigned* __restrict__ done, StreamTail tail) {
   constexpr int W = kKarmaPts / 32;  // bitmap words per block
+  constexpr int WPL = W / 32;
   __shared__ int32_t wpre[W];
+  __shared__ int64_t red[kKarmaThreads / 32];
+  __shared__ int64_t off_s;
+  __shared__ bool last_s;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  // block offset: fixed-order integer sum of the preceding block counts
+  int64_t o = 0;
+  for (int b = tid; b < (int)blockIdx.x; b += kKarmaThreads) o += counts[b];
+  for (int k = 16; k > 0; k >>= 1) o += __shfl_xor_sync(0xffffffffu, o, k);
+  if (lane == 0) red[warp] = o;
   const int64_t wbase = (int64_t)blockIdx.x * W;
   const int64_t nwords = (n + 31) / 32;
-  constexpr int WPL = W / 32;  // bitmap words per lane in the prefix
-  if (threadIdx.x < 32) {  // exclusive prefix of the block's word popcounts
-    const int lane = threadIdx.x;
+  if (tid < 32) {  // exclusive prefix of the block's word popcounts
     int c[WPL], tot = 0;
 #pragma unroll
     for (int k = 0; k < WPL; ++k) {
@@ -423,9 +399,9 @@ __global__ void compact_kernel(const uint32_t* __restrict__ bitmap, int64_t n, c
     }
     int incl = tot;
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const int v = __shfl_up_sync(0xffffffffu, incl, o);
-      if (lane >= o) incl += v;
+    for (int k = 1; k < 32; k <<= 1) {
+      const int v = __shfl_up_sync(0xffffffffu, incl, k);
+      if (lane >= k) incl += v;
     }
     int run = incl - tot;
 #pragma unroll
@@ -435,14 +411,65 @@ __global__ void compact_kernel(const uint32_t* __restrict__ bitmap, int64_t n, c
     }
   }
   __syncthreads();
-  const int64_t off = offsets[blockIdx.x];
-  for (int w = threadIdx.x / 32; w < W; w += blockDim.x / 32) {
+  if (tid == 0) {
+    int64_t t = 0;
+    for (int w = 0; w < kKarmaThreads / 32; ++w) t += red[w];
+    off_s = t;
+  }
+  __syncthreads();
+  const int64_t off = off_s;
+  for (int w = warp; w < W; w += kKarmaThreads / 32) {
     if (wbase + w >= nwords) break;
     const uint32_t word = bitmap[wbase + w];
-    const int lane = threadIdx.x & 31;
     if (word & (1u << lane)) {
       const int64_t pos = off + wpre[w] + __popc(word & ((1u << lane) - 1u));
       if (pos < cap) idx_out[pos] = row_offset + (wbase + w) * 32 + lane;
+    }
+  }
+  // last block: total + optional streaming tail
+  __threadfence();
+  __syncthreads();
+  if (tid == 0) last_s = atomicAdd(done, 1u) == (unsigned)nb - 1;
+  __syncthreads();
+  if (!last_s) return;
+  __threadfence();
+  int64_t t = 0;
+  for (int b = tid; b < nb; b += kKarmaThreads) t += __ldcg(counts + b);
+  for (int k = 16; k > 0; k >>= 1) t += __shfl_xor_sync(0xffffffffu, t, k);
+  __syncthreads();
+  if (lane == 0) red[warp] = t;
+  __syncthreads();
+  if (tid == 0) {
+    int64_t tot = 0;
+    for (int w = 0; w < kKarmaThreads / 32; ++w) tot += red[w];
+    off_s = tot;
+    if (total_out) *total_out = tot;
+    *done = 0u;
+  }
+  __syncthreads();
+  if (tail.online) online_update_body(tail.ret, tail.p, tail.op, tail.d, tail.st, tail.c);
+  if (tail.rows) {
+    __shared__ unsigned rmin[kMaxDim], rmax[kMaxDim];
+    if (tid < kMaxDim) {
+      rmin[tid] = 0xFFFFFFFFu;
+      rmax[tid] = 0u;
+    }
+    __syncthreads();
+    const int64_t k = min(off_s, cap);
+    for (int64_t e = tid; e < k * tail.d; e += kKarmaThreads) {
+      const int64_t r = e / tail.d;
+      const int j = (int)(e - r * tail.d);
+      const int64_t i = __ldcg(idx_out + r) - row_offset;
+      const float x = tail.rows[e];
+      tail.cols[(int64_t)j * tail.ld + i] = x;
+      atomicMin(rmin + j, fenc(x));  // shared-memory range of the new rows
+      atomicMax(rmax + j, fenc(x));
+      if (j == 0) tail.karma[i] = tail.k_init;
+    }
+    __syncthreads();
+    if (tid < tail.d && k > 0) {
+      atomicMin(tail.c->renc + 2 * tid, rmin[tid]);
+      atomicMax(tail.c->renc + 2 * tid + 1, rmax[tid]);
     }
   }
 }
@@ -451,15 +478,16 @@ __global__ void compact_kernel(const uint32_t* __restrict__ bitmap, int64_t n, c
 // ret: [1+d] = (p_hat, dp/dh_j) of the retained query.  Adds L' dp/dh (x h in
 // log mode, eq. 18) to the mini-batch; every `minibatch` queries applies the
 // RMSprop / Rprop step of P:L179-183 and re-derives the constants.
-__global__ void online_update_kernel(const double* __restrict__ ret, const double* __restrict__ p_ptr,
-                                     OnlineParamsDev op, int d, OnlineState* st, DevConsts* c) {
-  // one thread per dimension (the Listing 1 update is element-wise in j)
+// One Listing 1 step, executed by one whole block (thread j < d owns dimension j).
+__device__ void online_update_body(const double* __restrict__ ret, const double* __restrict__ p_ptr,
+                                   const OnlineParamsDev& op, int d, OnlineState* st, DevConsts* c) {
   const int j = threadIdx.x;
   const double p = *p_ptr;
   double L, dL;
   loss_eval(op.loss, op.lambda, ret[0], p, &L, &dL);
   const int count = st->count + 1;
   const bool apply = count >= op.minibatch;
+  __syncthreads();  // every thread has read st->count
   if (j < d) {
     double g = dL * ret[1 + j];
     if (op.log_bw) g *= c->h[j];
@@ -467,12 +495,12 @@ __global__ void online_update_kernel(const double* __restrict__ ret, const doubl
     if (!apply) {
       st->acc[j] = acc;
     } else {
-      const double gm = acc / (double)op.minibatch;                  // line 12
+      const double gm = acc / (double)op.minibatch;                        // line 12
       const double ms = op.alpha * st->ms[j] + (1.0 - op.alpha) * gm * gm;  // line 14
       double lr = st->lr[j];
-      if (gm * st->gprev[j] > 0.0) lr = fmin(lr * op.lr_inc, op.lr_max);   // lines 15-16
+      if (gm * st->gprev[j] > 0.0) lr = fmin(lr * op.lr_inc, op.lr_max);  // lines 15-16
       else if (gm * st->gprev[j] < 0.0) lr = fmax(lr * op.lr_dec, op.lr_min);
-      double step = ms > 0.0 ? lr * gm / sqrt(ms) : 0.0;             // line 17
+      double step = ms > 0.0 ? lr * gm / sqrt(ms) : 0.0;  // line 17
       double h = c->h[j];
       if (op.log_bw) {
         h = exp(log(h) - step);
@@ -487,11 +515,16 @@ __global__ void online_update_kernel(const double* __restrict__ ret, const doubl
       st->acc[j] = 0.0;
     }
   }
-  __syncthreads();
   if (j == 0) {
     st->count = apply ? 0 : count;
     st->updated = apply ? 1 : 0;
   }
+  __syncthreads();
+}
+
+__global__ void online_update_kernel(const double* __restrict__ ret, const double* __restrict__ p_ptr,
+                                     OnlineParamsDev op, int d, OnlineState* st, DevConsts* c) {
+  online_update_body(ret, p_ptr, op, d, st, c);
 }
 
 // ------------------------------------------------------------ harness: exact box counts
@@ -622,18 +655,16 @@ cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const do
 }
 cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, const double* p,
                          const KarmaParamsDev& kp, const float* lo, const float* hi, int d, const DevConsts* c,
-                         uint32_t* bitmap, int32_t* block_counts, int64_t* offsets, int64_t row_offset,
-                         int64_t* idx_out, int64_t cap, int64_t* total_out, cudaStream_t s) {
+                         uint32_t* bitmap, int32_t* block_counts, unsigned* done, int64_t row_offset, int64_t* idx_out,
+                         int64_t cap, int64_t* total_out, const StreamTail& tail, cudaStream_t s) {
   const int nb = karma_blocks(n);
   if (nb == 0) return cudaSuccess;
   karma_kernel<<<nb, kKarmaThreads, 0, s>>>(cvals, karma, n, n_global, phat, p, kp, lo, hi, d, c, bitmap,
                                             block_counts);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  scan_counts_kernel<<<1, 1024, 0, s>>>(block_counts, nb, offsets, total_out);
-  e = cudaGetLastError();
-  if (e != cudaSuccess) return e;
-  compact_kernel<<<nb, kKarmaThreads, 0, s>>>(bitmap, n, offsets, row_offset, idx_out, cap);
+  compact_fused_kernel<<<nb, kKarmaThreads, 0, s>>>(bitmap, n, block_counts, nb, row_offset, idx_out, cap, total_out,
+                                                    done, tail);
   KDE_LAUNCH_CHECK();
 }
 cudaError_t launch_online_update(const double* ret, const double* p, const OnlineParamsDev& op, int d, OnlineState* st,

@@ -15,6 +15,22 @@ struct HVec {
   double v[kMaxDim];
 };
 
+// optional work done by the last block of the karma compaction (device-resident streaming step)
+struct StreamTail {
+  int online = 0;  // run the Listing 1 step
+  const double* ret = nullptr;
+  const double* p = nullptr;
+  OnlineParamsDev op{};
+  OnlineState* st = nullptr;
+  DevConsts* c = nullptr;
+  int d = 0;
+  const float* rows = nullptr;  // non-null: replace the flagged points by rows[0..]
+  float* cols = nullptr;
+  int64_t ld = 0;
+  double* karma = nullptr;
+  double k_init = 0.0;
+};
+
 cudaError_t launch_rows_to_cols(const float* rows, int64_t n, int d, float* cols, int64_t ld, int* bad,
                                 cudaStream_t s);
 cudaError_t launch_cols_to_rows(const float* cols, int64_t ld, int64_t n, int d, float* rows, cudaStream_t s);
@@ -44,8 +60,8 @@ cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const do
                                  double* grad_out, cudaStream_t s);
 cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, const double* p,
                          const KarmaParamsDev& kp, const float* lo, const float* hi, int d, const DevConsts* c,
-                         uint32_t* bitmap, int32_t* block_counts, int64_t* offsets, int64_t row_offset,
-                         int64_t* idx_out, int64_t cap, int64_t* total_out, cudaStream_t s);
+                         uint32_t* bitmap, int32_t* block_counts, unsigned* done, int64_t row_offset, int64_t* idx_out,
+                         int64_t cap, int64_t* total_out, const StreamTail& tail, cudaStream_t s);
 cudaError_t launch_online_update(const double* ret, const double* p, const OnlineParamsDev& op, int d, OnlineState* st,
                                  DevConsts* c, cudaStream_t s);
 cudaError_t launch_count_in_box(const float* rows, int64_t n, int d, const float* lo, const float* hi, int64_t q,

@@ -407,7 +407,7 @@ def test_device_resident_stream_matches_host_path_and_oracle():
     pool = synth.replacement_rows(R, steps * cap, seed=42, step=0)
     kp = K.karma_params(loss=K.LOSS_ABSOLUTE, threshold=-1.0 / (n - 1), k_max=4.0)
     op = K.online_params(minibatch=5, loss=K.LOSS_ABSOLUTE, log_bandwidth=True)
-    mh, md = model(S), model(S)
+    mh, md, mf = model(S), model(S), model(S)
     mh.set_retain(True)
     md.set_retain(True)
     dev = torch.device("cuda")
@@ -418,6 +418,10 @@ def test_device_resident_stream_matches_host_path_and_oracle():
     ddpdh = torch.zeros((1, d), dtype=torch.float64, device=dev)
     didx = torch.zeros(cap, dtype=torch.int64, device=dev)
     dcnt = torch.zeros(1, dtype=torch.int64, device=dev)
+    fidx = torch.zeros(cap, dtype=torch.int64, device=dev)
+    fcnt = torch.zeros(1, dtype=torch.int64, device=dev)
+    fest = torch.zeros(1, dtype=torch.float64, device=dev)
+    fdpdh = torch.zeros(d, dtype=torch.float64, device=dev)
     s = torch.cuda.current_stream()
     for k in range(steps):
         h0 = mh.bandwidth
@@ -439,12 +443,18 @@ def test_device_resident_stream_matches_host_path_and_oracle():
         K.kde_karma_update_dev(md.handle, dlo[k], dhi[k], dp[k:k + 1], kp, didx, dcnt, stream=s)
         K.kde_online_update_dev(md.handle, dp[k:k + 1], op, stream=s)
         K.kde_replace_points_dev(md.handle, didx, dpool[k * cap:(k + 1) * cap], dcnt, stream=s)
+        # the same step fused into three kernels
+        K.kde_stream_step_dev(mf.handle, dlo[k:k + 1], dhi[k:k + 1], dp[k:k + 1], kp, op, fidx, fcnt,
+                              dpool[k * cap:(k + 1) * cap], fest, fdpdh, stream=s)
         torch.cuda.synchronize()
+        assert fest.item() == e_h[0] and np.array_equal(fdpdh.cpu().numpy(), g_h[0])
+        assert int(fcnt.item()) == nf and np.array_equal(fidx[:nf].cpu().numpy(), idx)
+        assert np.array_equal(mf.bandwidth, mh.bandwidth)
         assert dest.item() == e_h[0] and np.array_equal(ddpdh.cpu().numpy(), g_h)
         assert int(dcnt.item()) == nf and np.array_equal(didx[:nf].cpu().numpy(), idx)
         assert np.array_equal(md.bandwidth, mh.bandwidth)
-    assert np.array_equal(md.karma, mh.karma)
-    assert np.array_equal(md.sample, mh.sample)
+    assert np.array_equal(md.karma, mh.karma) and np.array_equal(mf.karma, mh.karma)
+    assert np.array_equal(md.sample, mh.sample) and np.array_equal(mf.sample, mh.sample)
 
 
 def test_batched_mixed_narrow_and_normal_boxes():
