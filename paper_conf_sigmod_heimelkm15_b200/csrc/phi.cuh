@@ -29,6 +29,10 @@ constexpr float kSqrtLog2e = 1.2011224087864498f;  // sqrt(log2(e))
 constexpr float kYClamp = 13.0f;
 constexpr float kPprime = KDE_PHI_P / kSqrtLog2e;
 
+#ifndef KDE_SHARED_RCP
+#define KDE_SHARED_RCP 0  // 1: one MUFU.RCP per (u, l) pair (+2 FP32 ops); see tools/tune_batched.cu
+#endif
+
 __device__ __forceinline__ float ex2_approx(float x) {
   float y;
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
@@ -84,7 +88,13 @@ __device__ __forceinline__ BoxDim make_boxdim(float l, float u, float ap, unsign
 template <bool GRAD>
 __device__ __forceinline__ float phi_normal(const float2 y, const float2 E, float& w) {
   const float2 den = __ffma2_rn(make_float2(fabsf(y.x), fabsf(y.y)), f2(kPprime), f2(1.0f));
+#if KDE_SHARED_RCP
+  // one MUFU.RCP for the pair: t_u = den_l / (den_u den_l), t_l = den_u / (den_u den_l)
+  const float r = rcp_approx(den.x * den.y);
+  const float2 t2 = __fmul2_rn(make_float2(den.y, den.x), f2(r));
+#else
   const float2 t2 = make_float2(rcp_approx(den.x), rcp_approx(den.y));
+#endif
   // Horner for Q(t)/2 (the 1/2 of eq. 13 folded into the coefficients)
   float2 q = f2(0.5f * kde_phi_q(KDE_PHI_DEG));
 #pragma unroll
