@@ -100,14 +100,14 @@ __device__ __forceinline__ float phi_normal(const float2 y, const float2 E, floa
 #pragma unroll
   for (int k = KDE_PHI_DEG - 1; k >= 0; --k) q = __ffma2_rn(q, t2, f2(0.5f * kde_phi_q(k)));
   const float2 ch = __fmul2_rn(__fmul2_rn(q, t2), E);          // 1/2 erfc(|z|)
-  if (GRAD) {
-    const float2 yE = __fmul2_rn(y, E);
-    w = yE.y - yE.x;
-  }
+  if (GRAD) w = fmaf(y.y, E.y, -(y.x * E.x));                  // FMUL + FFMA: 2 FMA-pipe cycles
   // 1/2 erf(z) = sgn(z) (1/2 - ch).  D = [1/2 sgn(z_u) - 1/2 sgn(z_l)] + [sgn(z_l) ch_l - sgn(z_u) ch_u]:
   // the first bracket is exactly 0 or 1, so a box seen from one side keeps the
-  // full relative accuracy of the erfc tails (no 1/2 - ch rounding).
-  const float hs = copysignf(0.5f, y.x) - copysignf(0.5f, y.y);
+  // full relative accuracy of the erfc tails (no 1/2 - ch rounding).  It is 1
+  // iff z_l < 0 <= z_u (z_u >= z_l always) and is built from the sign bits on
+  // the integer (ALU) pipe, leaving the FMA pipe -- the binding one -- alone.
+  const unsigned lneg_upos = __float_as_uint(y.y) & ~__float_as_uint(y.x);
+  const float hs = __uint_as_float((unsigned)((int)lneg_upos >> 31) & 0x3f800000u);
   const float cs = copysignf(ch.y, y.y) - copysignf(ch.x, y.x);
   return hs + cs;
 }
