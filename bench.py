@@ -266,6 +266,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
 
     if cfg.get("retain"):
         m.set_retain(True)
+    use_graph = cfg["path"] == "stream" and not args.no_graph
     if cfg["path"] == "stream":
         cap = 1 << 16
         kp = K.karma_params(loss=K.LOSS_ABSOLUTE, threshold=-1.0 / (n_global - 1), k_max=4.0)
@@ -279,7 +280,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
     def step(i):
         if cfg["path"] == "stream":
             k = i % nbox
-            off = (i * 977) % npool
+            off = (k * 977) % npool
             K.kde_stream_step_dev(m.handle, d_lo[k:k + 1], d_hi[k:k + 1], d_true[k:k + 1], kp, op, d_idx, d_cnt,
                                   d_pool[off:off + cap], d_est[:1], d_dpdh[0], stream=stream)
             return
@@ -295,6 +296,31 @@ def run_cuda(args, cfg, rank, world, local_rank):
         for i in range(args.warmup):
             step(i)
     torch.cuda.synchronize()
+
+    graphs = None
+    prof_pre = None
+    if use_graph:
+        # launch-bound multi-kernel steps: one CUDA graph per box (the step's
+        # arguments depend only on the box index), replayed per step.  The scan
+        # kernel's own duration for the roofline is taken from profiled eager
+        # steps first (kernel events cannot be read back from a replayed graph).
+        K.kde_set_profiling(m.handle, True)
+        with torch.cuda.stream(stream):
+            for i in range(args.warmup, args.warmup + max(args.steps, 8)):
+                step(i)
+        torch.cuda.synchronize()
+        prof_pre = K.kde_get_profile(m.handle)
+        K.kde_set_profiling(m.handle, False)
+        graphs = []
+        for k in range(nbox):
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=stream):
+                step(k)
+            graphs.append(g)
+        torch.cuda.synchronize()
+
+        def step(i):  # noqa: F811
+            graphs[i % nbox].replay()
 
     K.kde_set_profiling(m.handle, True)
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
@@ -329,6 +355,12 @@ def run_cuda(args, cfg, rank, world, local_rank):
     launches = int(round(per_step * args.steps))
     scan_ms *= args.steps / max(args.steps + soak, 1)
     scan_launches = int(round(scan_launches * args.steps / max(args.steps + soak, 1)))
+    if graphs is not None:  # graph replays bypass libkde's host-side counters
+        ms_pre, sl_pre, l_pre = prof_pre
+        n_pre = max(args.steps, 8)
+        launches = int(round(l_pre / n_pre * args.steps))
+        scan_launches = int(round(sl_pre / n_pre * args.steps))
+        scan_ms = ms_pre / n_pre * args.steps
     K.kde_set_profiling(m.handle, False)
     step_ms = [a.elapsed_time(b) for a, b in evs]
     tot_ms = sum(step_ms)
@@ -414,6 +446,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": cfg["desc"], "d": d, "n_per_gpu": n, "n_global": n_global, "q": q,
                    "l2": "flushed between timed steps" if flush_l2 else "sample larger than L2",
+                   "cuda_graph": bool(graphs is not None),
                    "clock_sampling": "nvidia-smi every 100 ms over the timed steps"
                                      + (f" + {soak} identical untimed soak steps (timed region < 1 s)" if soak else ""),
                    "accumulation": "fp32 per <=32 points, fp64 above"},
@@ -453,6 +486,7 @@ def main():
     ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="cuda", choices=["cuda", "reference"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-graph", action="store_true", help="stream configs: launch eagerly instead of CUDA graphs")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of all-core oracle work")
     args = ap.parse_args()
     if args.warmup < 3:

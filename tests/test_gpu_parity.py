@@ -477,3 +477,31 @@ def test_batched_mixed_narrow_and_normal_boxes():
     sel_ok(est, est_o)
     grad_ok(gr, g_o, mabs)
     sel_ok(m.estimate(lo, hi), est_o)
+
+
+def test_sharded_create_world1_through_torch_distributed():
+    """dist.create_sharded under a one-rank NCCL process group (the bench's
+    N = 1 torchrun path): identical results to kde_create."""
+    import os
+    import socket
+
+    import torch.distributed as dist
+    from paper_conf_sigmod_heimelkm15_b200.dist import create_sharded
+    sck = socket.socket()
+    sck.bind(("127.0.0.1", 0))
+    port = sck.getsockname()[1]
+    sck.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("nccl", rank=0, world_size=1)
+    try:
+        S = synth.make_data("gauss", 9001, 4, seed=70)
+        lo, hi = synth.mixed_workload(S, 50, seed=71)
+        a = create_sharded(S, 0, len(S))
+        b = model(S)
+        assert np.array_equal(a.bandwidth, b.bandwidth)
+        ea, ga = a.estimate(lo, hi, grad=True)
+        eb, gb = b.estimate(lo, hi, grad=True)
+        assert np.array_equal(ea, eb) and np.array_equal(ga, gb)
+        a.close()
+    finally:
+        dist.destroy_process_group()

@@ -347,3 +347,48 @@ def test_online_update_reduces_training_loss():
             oracle.online_step(st, h, g, log_bw=True)
     L1, _, _ = oracle.loss_and_grad(S, h, lo, hi, p, 0, 0.0, True)
     assert L1 < L0
+
+
+# --- property-based pins (hypothesis) ---------------------------------------------
+from hypothesis import given, settings, strategies as st  # noqa: E402
+
+
+@settings(max_examples=60, deadline=None)
+@given(seed=st.integers(0, 2**31 - 1), d=st.integers(1, 4), n=st.integers(1, 30))
+def test_property_mass_is_a_probability_and_additive(seed, d, n):
+    """For any sample, bandwidth and box: 0 <= p_hat <= 1 (eq. 2 averages
+    probabilities, eq. 13), splitting the box along a random axis adds up
+    (eq. 12 integral), and widening the box never decreases p_hat."""
+    g = np.random.default_rng(seed)
+    S = g.normal(size=(n, d)).astype(np.float32)
+    h = g.uniform(0.05, 3.0, d)
+    lo = g.uniform(-2, 0, d).astype(np.float32)
+    hi = (lo + g.uniform(0.01, 3, d)).astype(np.float32)
+    p = oracle.estimate(S, h, lo[None], hi[None])[0]
+    assert -1e-15 <= p <= 1 + 1e-15
+    j = int(g.integers(0, d))
+    c = np.float32(g.uniform(lo[j], hi[j]))
+    h1, l2 = hi.copy(), lo.copy()
+    h1[j] = c
+    l2[j] = c
+    parts = oracle.estimate(S, h, lo[None], h1[None])[0] + oracle.estimate(S, h, l2[None], hi[None])[0]
+    assert parts == pytest.approx(p, rel=1e-12, abs=1e-15)
+    wide = oracle.estimate(S, h, (lo - 1)[None], (hi + 1)[None])[0]
+    assert wide >= p - 1e-15
+
+
+@settings(max_examples=40, deadline=None)
+@given(seed=st.integers(0, 2**31 - 1), d=st.integers(1, 3))
+def test_property_gradient_along_h_matches_scaling_derivative(seed, d):
+    """Scaling every h_j by (1+e) changes p_hat by sum_j h_j dp/dh_j * e to
+    first order (eq. 17 contracted with the direction h)."""
+    g = np.random.default_rng(seed)
+    S = g.normal(size=(20, d)).astype(np.float32)
+    h = g.uniform(0.2, 2.0, d)
+    lo = g.uniform(-1.5, 0, d).astype(np.float32)
+    hi = (lo + g.uniform(0.2, 2, d)).astype(np.float32)
+    _, gr = oracle.estimate_grad(S, h, lo[None], hi[None])
+    e = 1e-6
+    fd = (oracle.estimate(S, h * (1 + e), lo[None], hi[None])[0]
+          - oracle.estimate(S, h * (1 - e), lo[None], hi[None])[0]) / (2 * e)
+    assert float(np.dot(h, gr[0])) == pytest.approx(fd, rel=1e-6, abs=1e-13)

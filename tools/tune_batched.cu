@@ -62,7 +62,7 @@ void setup_and_sweep(int64_t n, int64_t q, int sms) {
 #define R(QT, MINB, W) run<D, QT, MINB>(n, q, W, cols, ld, lo, hi, c, part, sms);
 #define RU(QT, MINB, W, PU) run<D, QT, MINB, PU>(n, q, W, cols, ld, lo, hi, c, part, sms);
   if constexpr (D <= 3) {
-    R(2, 4, 4) RU(2, 4, 4, 2) RU(2, 3, 4, 2) RU(1, 4, 4, 2) RU(1, 4, 4, 4) RU(2, 2, 4, 2) RU(4, 2, 4, 2)
+    RU(1, 4, 4, 2) R(2, 4, 4) RU(2, 4, 4, 2) RU(2, 3, 4, 2) RU(1, 4, 4, 2) RU(1, 4, 4, 4) RU(2, 2, 4, 2) RU(4, 2, 4, 2)
   } else if constexpr (D <= 6) {
     R(1, 4, 4) RU(1, 4, 4, 2) RU(1, 3, 4, 2) RU(2, 3, 4, 2) RU(2, 2, 4, 2)
   } else {
