@@ -92,6 +92,7 @@ struct ScanBatchedArgs {
   int64_t q;
   const DevConsts* consts;
   int64_t split_len;      // points per split (multiple of the tile size)
+  int qb;                 // boxes per CTA (power of two <= 256; 256/qb threads share a box)
   double* partials;       // [splits][1+d][q]
 };
 

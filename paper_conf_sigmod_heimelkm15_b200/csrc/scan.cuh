@@ -8,8 +8,9 @@
 //   hint), fp32 math per point, fp32 sums over 8 points flushed to fp64,
 //   warp-shuffle + block reduction, and a deterministic last-block second pass
 //   (fixed order) that also finalises p_hat and dp_hat/dh.
-// scan_batched_kernel (q > 1): FP32/SFU-bound.  A CTA owns 256*QT boxes (QT per
-//   thread, bounds in registers) and one contiguous split of the sample; sample
+// scan_batched_kernel (q > 1): FP32/SFU-bound.  A CTA owns QB <= 256 boxes
+//   (bounds in registers; 256/QB threads share a box and split its points)
+//   and one contiguous split of the sample; sample
 //   tiles of 256 points x d columns are staged into shared memory by TMA bulk
 //   copies (cp.async.bulk + mbarrier, double buffered) and read as broadcasts.
 //   fp32 sums over 32 points are flushed into per-thread fp64 accumulators in
@@ -331,29 +332,33 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 // boxes.  No barriers inside, so the GENERAL (narrow-dimension) and fast
 // variants can be chosen per warp.
 template <int D, bool GRAD, bool GENERAL, int QT, int PU>
-__device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, double* accsh,
+__device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, int phase, int R, double* accsh,
                                                      const BoxDim (&bd)[QT][D], const float (&ap)[D]) {
   constexpr int NA = GRAD ? D + 1 : 1;
   const int tid = threadIdx.x;
-  for (int p0 = 0; p0 < npts; p0 += kFlushPts) {
-    const int pe = min(p0 + kFlushPts, npts);
+  // this thread's points of the tile: phase, phase + R, phase + 2R, ...
+  const int mine = npts > phase ? (npts - phase + R - 1) / R : 0;
+  for (int m0 = 0; m0 < mine; m0 += kFlushPts) {
+    const int me = min(m0 + kFlushPts, mine);
     float s[QT][NA];
 #pragma unroll
     for (int qq = 0; qq < QT; ++qq)
 #pragma unroll
       for (int kk = 0; kk < NA; ++kk) s[qq][kk] = 0.0f;
-    int p = p0;
-    for (; p + PU <= pe; p += PU) {  // PU points per iteration: more independent chains per warp
+    int m = m0;
+    for (; m + PU <= me; m += PU) {  // PU points per iteration: more independent chains per warp
 #pragma unroll
       for (int u = 0; u < PU; ++u) {
+        const int p = phase + (m + u) * R;
         float t[D];
 #pragma unroll
-        for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p + u];
+        for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
 #pragma unroll
         for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, GENERAL>(bd[qq], t, ap, s[qq], true);
       }
     }
-    for (; p < pe; ++p) {
+    for (; m < me; ++m) {
+      const int p = phase + m * R;
       float t[D];
 #pragma unroll
       for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
@@ -374,7 +379,8 @@ __device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, 
 template <int D, bool GRAD, int QT, int PU, typename Issue>
 __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const float* tile, uint64_t* bar,
                                               double* accsh, const BoxDim (&bd)[QT][D], const float (&ap)[D],
-                                              int64_t s0, int64_t s1, int ntiles, bool warp_general, Issue& issue) {
+                                              int64_t s0, int64_t s1, int ntiles, bool warp_general, int phase, int R,
+                                              Issue& issue) {
   const int tid = threadIdx.x;
   for (int k = 0; k < ntiles; ++k) {
     const int buf = k & 1;
@@ -384,9 +390,9 @@ __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const fl
     const int64_t rem = s1 - (s0 + (int64_t)k * kTilePts);
     const int npts = rem < kTilePts ? (int)rem : kTilePts;
     if (warp_general)
-      batched_tile_compute<D, GRAD, true, QT, PU>(tl, npts, accsh, bd, ap);
+      batched_tile_compute<D, GRAD, true, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
     else
-      batched_tile_compute<D, GRAD, false, QT, PU>(tl, npts, accsh, bd, ap);
+      batched_tile_compute<D, GRAD, false, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
     __syncthreads();
   }
 }
@@ -407,38 +413,43 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
                                               (size_t)QT * NA * kBatchedThreads * sizeof(double));
   const int tid = threadIdx.x;
 
-  // This CTA's 256*QT boxes (slots), qbase + slot.  Boxes with a narrow
-  // dimension need the general Phi path; a CTA-local stable partition puts
-  // them into the last slots so at most one warp mixes both kinds and every
-  // other warp runs the branch-free path.
-  const int64_t qbase = (int64_t)blockIdx.x * kBatchedThreads * QT;
-  __shared__ int perm_s[kBatchedThreads * QT];
-  __shared__ int base_s[2 * QT * (kBatchedThreads / 32) + 1];
+  // This CTA's QB boxes (slots 0..QB-1, box qbase + slot).  With QB < 256 each
+  // box is handled by R = 256/QB threads ("phases") that split the points of
+  // every tile, so small batches (e.g. the ~100-box training sets of batch
+  // optimisation) still keep all threads busy.  Boxes with a
+  // narrow dimension need the general Phi path; a CTA-local stable partition
+  // puts them into the last slots so at most one warp mixes both kinds.
+  static_assert(QT == 1, "the phase mapping assumes one box per thread");
+  const int QB = a.qb;
+  const int R = kBatchedThreads / QB;
+  const int slot = tid % QB, phase = tid / QB;
+  const int64_t qbase = (int64_t)blockIdx.x * QB;
+  __shared__ int perm_s[kBatchedThreads];
+  __shared__ int base_s[2 * (kBatchedThreads / 32) + 1];
   const int lane = tid & 31, warp = tid >> 5;
   float ap[D];
 #pragma unroll
   for (int j = 0; j < D; ++j) ap[j] = a.consts->ap[j];
-  unsigned nmask[QT];
-#pragma unroll
-  for (int qq = 0; qq < QT; ++qq) {
-    int64_t qi = qbase + qq * kBatchedThreads + tid;
+  bool nar = false;
+  if (tid < QB) {
+    int64_t qi = qbase + tid;
     if (qi >= a.q) qi = a.q - 1;  // duplicate a valid box; its partial is never written
-    bool nar = false;
 #pragma unroll
     for (int j = 0; j < D; ++j) {
       const float l = __ldg(a.lo + qi * D + j), u = __ldg(a.hi + qi * D + j);
       const float dy = (u - l) * ap[j];
       nar |= dy > 0.0f && dy < kNarrowY;
     }
-    nmask[qq] = __ballot_sync(0xffffffffu, nar);
-    if (lane == 0) {
-      base_s[2 * (qq * (kBatchedThreads / 32) + warp)] = 32 - __popc(nmask[qq]);  // normal count
-      base_s[2 * (qq * (kBatchedThreads / 32) + warp) + 1] = __popc(nmask[qq]);  // narrow count
-    }
+  }
+  const unsigned live = __ballot_sync(0xffffffffu, tid < QB);
+  const unsigned nmask = __ballot_sync(0xffffffffu, nar);
+  if (lane == 0) {
+    base_s[2 * warp] = __popc(live & ~nmask);  // normal count
+    base_s[2 * warp + 1] = __popc(nmask);      // narrow count
   }
   __syncthreads();
   if (tid == 0) {  // exclusive prefixes in slot order: normals first, then narrows
-    constexpr int G = QT * (kBatchedThreads / 32);
+    constexpr int G = kBatchedThreads / 32;
     int tn = 0;
     for (int g = 0; g < G; ++g) tn += base_s[2 * g];
     int rn = 0, rw = tn;
@@ -451,27 +462,23 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
     }
   }
   __syncthreads();
-#pragma unroll
-  for (int qq = 0; qq < QT; ++qq) {
-    const int g = qq * (kBatchedThreads / 32) + warp;
-    const bool nar = (nmask[qq] >> lane) & 1u;
+  if (tid < QB) {
     const unsigned lt = (1u << lane) - 1u;
-    const int pos = nar ? base_s[2 * g + 1] + __popc(nmask[qq] & lt) : base_s[2 * g] + __popc(~nmask[qq] & lt);
-    perm_s[pos] = qq * kBatchedThreads + tid;
+    const int pos = nar ? base_s[2 * warp + 1] + __popc(nmask & lt) : base_s[2 * warp] + __popc(live & ~nmask & lt);
+    perm_s[pos] = tid;
   }
   __syncthreads();
   BoxDim bd[QT][D];
   bool narrow[QT];
-#pragma unroll
-  for (int qq = 0; qq < QT; ++qq) {
-    int64_t qi = qbase + perm_s[qq * kBatchedThreads + tid];
+  {
+    int64_t qi = qbase + perm_s[slot];
     if (qi >= a.q) qi = a.q - 1;
-    narrow[qq] = false;
+    narrow[0] = false;
 #pragma unroll
     for (int j = 0; j < D; ++j) {
-      bd[qq][j] = make_boxdim(__ldg(a.lo + qi * D + j), __ldg(a.hi + qi * D + j), ap[j], a.consts->renc[2 * j],
-                               a.consts->renc[2 * j + 1]);
-      narrow[qq] |= bd[qq][j].hd > 0.0f;
+      bd[0][j] = make_boxdim(__ldg(a.lo + qi * D + j), __ldg(a.hi + qi * D + j), ap[j], a.consts->renc[2 * j],
+                              a.consts->renc[2 * j + 1]);
+      narrow[0] |= bd[0][j].hd > 0.0f;
     }
   }
 #pragma unroll
@@ -504,16 +511,20 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
 #pragma unroll
   for (int qq = 0; qq < QT; ++qq) my_narrow |= narrow[qq];
   const bool warp_general = __any_sync(0xffffffffu, my_narrow);
-  batched_tiles<D, GRAD, QT, PU>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, warp_general, issue);
+  batched_tiles<D, GRAD, QT, PU>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, warp_general, phase, R, issue);
 
+  // combine the R phases of each box in phase order, then
   // partials[(split*(NA) + comp) * q + qi]
-#pragma unroll
-  for (int qq = 0; qq < QT; ++qq) {
-    const int64_t qi = qbase + perm_s[qq * kBatchedThreads + tid];
+  if (R > 1) __syncthreads();
+  if (tid < QB) {
+    const int64_t qi = qbase + perm_s[tid];
     if (qi < a.q) {
 #pragma unroll
-      for (int kk = 0; kk < NA; ++kk)
-        a.partials[((int64_t)blockIdx.y * NA + kk) * a.q + qi] = accsh[(qq * NA + kk) * kBatchedThreads + tid];
+      for (int kk = 0; kk < NA; ++kk) {
+        double t = 0.0;
+        for (int ph = 0; ph < R; ++ph) t += accsh[kk * kBatchedThreads + ph * QB + tid];
+        a.partials[((int64_t)blockIdx.y * NA + kk) * a.q + qi] = t;
+      }
     }
   }
 }
@@ -561,9 +572,26 @@ cudaError_t launch_batched_tg(const ScanBatchedArgs& a, dim3 grid, cudaStream_t 
 
 // Grid for the batched scan: query tiles (256*QT boxes) x sample splits,
 // about `waves` x MINB CTAs per SM; split_len is a tile multiple.
-inline void batched_grid(int64_t q, int64_t n, int qt, int minb, int num_sms, int waves, int64_t* qtiles,
+// boxes per CTA: the power of two QB in [16, 256] minimising the padded
+// work ceil(q/QB)*QB, with a 3% penalty per halving (smaller QB re-reads the
+// sample tiles for fewer boxes); 256 for large batches.
+inline int batched_qb(int64_t q) {
+  int best = kBatchedThreads;
+  double best_cost = -1.0;
+  double pen = 1.0;
+  for (int qb = kBatchedThreads; qb >= 16; qb >>= 1, pen *= 1.03) {
+    const double cost = (double)((q + qb - 1) / qb * qb) * pen;
+    if (best_cost < 0.0 || cost < best_cost) {
+      best = qb;
+      best_cost = cost;
+    }
+  }
+  return best;
+}
+
+inline void batched_grid(int64_t q, int64_t n, int qb, int minb, int num_sms, int waves, int64_t* qtiles,
                          int64_t* splits, int64_t* split_len) {
-  *qtiles = (q + (int64_t)kBatchedThreads * qt - 1) / ((int64_t)kBatchedThreads * qt);
+  *qtiles = (q + qb - 1) / qb;
   const int64_t ntile_pts = (n + kTilePts - 1) / kTilePts;
   const int64_t target = (int64_t)num_sms * minb * waves;
   int64_t sp = (target + *qtiles - 1) / *qtiles;
@@ -584,7 +612,8 @@ cudaError_t launch_batched_t(bool grad, const ScanBatchedArgs& a_in, int num_sms
   constexpr int MINB = MINB_for<D>::value;
   ScanBatchedArgs a = a_in;
   int64_t qtiles, splits, split_len;
-  batched_grid(a.q, a.n, QT, MINB, num_sms, 4, &qtiles, &splits, &split_len);
+  a.qb = batched_qb(a.q) * QT;
+  batched_grid(a.q, a.n, a.qb, MINB, num_sms, 4, &qtiles, &splits, &split_len);
   if (splits_out) *splits_out = (int)splits;
   if (dry_run) return cudaSuccess;
   a.split_len = split_len;

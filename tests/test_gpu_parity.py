@@ -505,3 +505,18 @@ def test_sharded_create_world1_through_torch_distributed():
         a.close()
     finally:
         dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("q", [2, 3, 17, 100, 300])
+def test_small_batches_phase_mapping(q):
+    """Batches smaller than a CTA's 256 boxes: 256/QB threads share a box and
+    split the points of each tile; results must not depend on the mapping."""
+    S = synth.make_data("gauss", 20011, 3, seed=80 + q)
+    m = model(S)
+    h = m.bandwidth
+    lo, hi = synth.mixed_workload(S, q, seed=81)
+    est_o, g_o = oracle.estimate_grad(S, h, lo, hi)
+    mabs = oracle.grad_abs_scale(S, h, lo, hi)
+    est, g = m.estimate(lo, hi, grad=True)
+    sel_ok(est, est_o)
+    grad_ok(g, g_o, mabs)

@@ -16,7 +16,8 @@ void run(int64_t n, int64_t q, int waves, const float* cols, int64_t ld, const f
   ScanBatchedArgs a{};
   a.cols = cols; a.ld = ld; a.n = n; a.lo = lo; a.hi = hi; a.q = q; a.consts = consts; a.partials = partials;
   int64_t qtiles, splits, len;
-  batched_grid(q, n, QT, MINB, sms, waves, &qtiles, &splits, &len);
+  a.qb = batched_qb(q);
+  batched_grid(q, n, a.qb, MINB, sms, waves, &qtiles, &splits, &len);
   a.split_len = len;
   dim3 grid((unsigned)qtiles, (unsigned)splits);
   cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
@@ -62,9 +63,9 @@ void setup_and_sweep(int64_t n, int64_t q, int sms) {
 #define R(QT, MINB, W) run<D, QT, MINB>(n, q, W, cols, ld, lo, hi, c, part, sms);
 #define RU(QT, MINB, W, PU) run<D, QT, MINB, PU>(n, q, W, cols, ld, lo, hi, c, part, sms);
   if constexpr (D <= 3) {
-    RU(1, 4, 4, 2) R(2, 4, 4) RU(2, 4, 4, 2) RU(2, 3, 4, 2) RU(1, 4, 4, 2) RU(1, 4, 4, 4) RU(2, 2, 4, 2) RU(4, 2, 4, 2)
+    RU(1, 4, 4, 2) R(1, 4, 4) RU(1, 4, 4, 4) RU(1, 3, 4, 2) RU(1, 4, 8, 2)
   } else if constexpr (D <= 6) {
-    R(1, 4, 4) RU(1, 4, 4, 2) RU(1, 3, 4, 2) RU(2, 3, 4, 2) RU(2, 2, 4, 2)
+    R(1, 4, 4) RU(1, 4, 4, 2) RU(1, 3, 4, 2)
   } else {
     R(1, 3, 4) RU(1, 3, 4, 2) RU(1, 2, 4, 2)
   }
@@ -74,6 +75,8 @@ void setup_and_sweep(int64_t n, int64_t q, int sms) {
 int main() {
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
+  setup_and_sweep<3>(1 << 20, 100, sms);   // batch-optimisation training set size
+  setup_and_sweep<3>(1 << 20, 300, sms);
   setup_and_sweep<3>(1 << 20, 10000, sms);
   setup_and_sweep<5>(1 << 22, 4096, sms);
   setup_and_sweep<8>(1 << 22, 4096, sms);
