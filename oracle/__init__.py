@@ -17,6 +17,8 @@ Parity status:
   empty_region_threshold                     pinned (eq. 19 centre point, boundary max)
   karma_update                               pinned (brute-force leave-one-out)
   online_apply (Listing 1 reconstruction)    PARITY UNPINNED (listing missing from PAPER.md)
+  epan_* (Epanechnikov product kernel)       pinned (quadrature of the density, FD, closed forms);
+                                             the kernel's bandwidth convention is reading R14
 """
 from __future__ import annotations
 
@@ -55,6 +57,11 @@ def _L():
             "oracle_estimate": (None, [P, i64, i32, P, P, P, i64, P]),
             "oracle_estimate_grad": (None, [P, i64, i32, P, P, P, i64, P, P]),
             "oracle_grad_abs_scale": (None, [P, i64, i32, P, P, P, i64, P]),
+            "oracle_epan_point_mass": (f64, [P, i32, P, P, P]),
+            "oracle_epan_contributions": (None, [P, i64, i32, P, P, P, P]),
+            "oracle_epan_estimate_grad": (None, [P, i64, i32, P, P, P, i64, P, P]),
+            "oracle_epan_grad_abs_scale": (None, [P, i64, i32, P, P, P, i64, P]),
+            "oracle_epan_empty_region_threshold": (f64, [i32, P, P, P, P]),
             "oracle_loss": (None, [i32, f64, f64, f64, P, P]),
             "oracle_loss_and_grad": (None, [P, i64, i32, P, P, P, P, i64, i32, f64, i32, P, P, P]),
             "oracle_scott": (None, [P, i64, i32, P]),
@@ -225,3 +232,62 @@ def online_step(state: OnlineState, h: np.ndarray, grad, batch=10, alpha=0.9, lr
                              _p(h), _p(state.acc), _p(state.ms), _p(state.lr), _p(state.gprev))
     state.count = 0
     return True
+
+
+# ---------------------------------------------------------------- Epanechnikov (NEXT-4, reading R14)
+def epan_point_mass(t, h, lo, hi) -> float:
+    t, lo, hi, h = _f32(t), _f32(lo), _f32(hi), _f64(h)
+    return _L().oracle_epan_point_mass(_p(t), len(h), _p(h), _p(lo), _p(hi))
+
+
+def epan_contributions(sample, h, lo, hi) -> np.ndarray:
+    sample, h, lo, hi = _f32(sample), _f64(h), _f32(lo).ravel(), _f32(hi).ravel()
+    n, d = sample.shape
+    out = np.empty(n, dtype=np.float64)
+    _L().oracle_epan_contributions(_p(sample), n, d, _p(h), _p(lo), _p(hi), _p(out))
+    return out
+
+
+def epan_estimate_grad(sample, h, lo, hi):
+    """(p_hat[q], dp_hat/dh[q, d]) for the Epanechnikov product kernel."""
+    sample, h = _f32(sample), _f64(h)
+    lo, hi = _f32(np.atleast_2d(lo)), _f32(np.atleast_2d(hi))
+    n, d = sample.shape
+    q = lo.shape[0]
+    est = np.empty(q, dtype=np.float64)
+    g = np.empty((q, d), dtype=np.float64)
+    _L().oracle_epan_estimate_grad(_p(sample), n, d, _p(h), _p(lo), _p(hi), q, _p(est), _p(g))
+    return est, g
+
+
+def epan_estimate(sample, h, lo, hi):
+    return epan_estimate_grad(sample, h, lo, hi)[0]
+
+
+def epan_grad_abs_scale(sample, h, lo, hi):
+    sample, h = _f32(sample), _f64(h)
+    lo, hi = _f32(np.atleast_2d(lo)), _f32(np.atleast_2d(hi))
+    n, d = sample.shape
+    q = lo.shape[0]
+    g = np.empty((q, d), dtype=np.float64)
+    _L().oracle_epan_grad_abs_scale(_p(sample), n, d, _p(h), _p(lo), _p(hi), q, _p(g))
+    return g
+
+
+def epan_empty_region_threshold(h, lo, hi):
+    h, lo, hi = _f64(h), _f32(lo).ravel(), _f32(hi).ravel()
+    pmax = ctypes.c_double()
+    thr = _L().oracle_epan_empty_region_threshold(len(h), _p(h), _p(lo), _p(hi), ctypes.byref(pmax))
+    return thr, pmax.value
+
+
+def epan_loss_and_grad(sample, h, lo, hi, true_sel, kind: int, lam: float, log_bw: bool):
+    """eq. (5)/(14)/(18) with the Epanechnikov estimate and gradient."""
+    est, g = epan_estimate_grad(sample, h, lo, hi)
+    ts = _f64(true_sel)
+    Ls, dLs = zip(*[loss(kind, lam, e, p) for e, p in zip(est, ts)])
+    L = float(np.mean(Ls))
+    grad = np.mean(np.asarray(dLs)[:, None] * g, axis=0)
+    if log_bw:
+        grad = grad * _f64(h)
+    return L, grad, est

@@ -339,3 +339,132 @@ void oracle_online_apply(int32_t d, int32_t batch, double alpha, double lr_min, 
         acc[j] = 0.0;
     }
 }
+
+/* =====================================================================
+ * Epanechnikov product kernel.  The paper names it as the
+ * cheaper alternative ("a truncated second-degree
+ * polynomial") but derives nothing for it.  Reading R14: the
+ * 1-D kernel with bandwidth h is the density
+ *     K_h(x) = 3 / (4 h) * (1 - (x/h)^2)   for |x| <= h,  0 otherwise,
+ * i.e. h is the support half-width, and the d-dim kernel is the product over
+ * dimensions (the product-kernel argument of P:L472).  Everything below is
+ * the plain integral / derivative of that density: the 1-D box mass is
+ * F((u-t)/h) - F((l-t)/h) with the CDF F(v) = (2 + 3v - v^3) / 4 on
+ * [-1, 1] (0 below, 1 above), and d/dh of it is
+ *     F'(v_u) (-v_u / h) - F'(v_l) (-v_l / h),   F'(v) = 3/4 (1 - v^2) on |v| < 1.
+ * ===================================================================== */
+static double epan_cdf(double v)
+{
+    if (v <= -1.0) return 0.0;
+    if (v >= 1.0) return 1.0;
+    return (2.0 + 3.0 * v - v * v * v) / 4.0;
+}
+
+static double epan_pdf01(double v) /* F'(v) */
+{
+    if (v <= -1.0 || v >= 1.0) return 0.0;
+    return 0.75 * (1.0 - v * v);
+}
+
+/* 1-D mass of (l, u) for a point t; +-inf bounds give v = +-inf. */
+static double epan_mass1(double t, double h, double l, double u)
+{
+    return epan_cdf((u - t) / h) - epan_cdf((l - t) / h);
+}
+
+static double epan_dmass1_dh(double t, double h, double l, double u)
+{
+    double vu = (u - t) / h, vl = (l - t) / h;
+    double du = isinf(vu) ? 0.0 : epan_pdf01(vu) * (-vu / h);
+    double dl = isinf(vl) ? 0.0 : epan_pdf01(vl) * (-vl / h);
+    return du - dl;
+}
+
+/* p^(i)(Omega) for the Epanechnikov product kernel (eq. 10-11 with K_h). */
+double oracle_epan_point_mass(const float *t, int32_t d, const double *h, const float *lo, const float *hi)
+{
+    double prod = 1.0;
+    for (int32_t j = 0; j < d; ++j) prod *= epan_mass1((double)t[j], h[j], (double)lo[j], (double)hi[j]);
+    return prod;
+}
+
+void oracle_epan_contributions(const float *sample, int64_t n, int32_t d, const double *h,
+                               const float *lo, const float *hi, double *c_out)
+{
+    for (int64_t i = 0; i < n; ++i) c_out[i] = oracle_epan_point_mass(sample + i * d, d, h, lo, hi);
+}
+
+/* eq. (2) estimate and its h-gradient (product rule as in eq. 16) for q boxes. */
+void oracle_epan_estimate_grad(const float *sample, int64_t n, int32_t d, const double *h,
+                               const float *lo, const float *hi, int64_t q, double *est, double *dpdh)
+{
+    #pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t qq = 0; qq < q; ++qq) {
+        const float *l = lo + qq * d, *u = hi + qq * d;
+        double sum = 0.0, gsum[64];
+        for (int32_t i = 0; i < d; ++i) gsum[i] = 0.0;
+        for (int64_t j = 0; j < n; ++j) {
+            const float *t = sample + j * d;
+            sum += oracle_epan_point_mass(t, d, h, l, u);
+            for (int32_t i = 0; i < d; ++i) {
+                double prod = 1.0;
+                for (int32_t k = 0; k < d; ++k) {
+                    if (k == i) continue;
+                    prod *= epan_mass1((double)t[k], h[k], (double)l[k], (double)u[k]);
+                }
+                gsum[i] += epan_dmass1_dh((double)t[i], h[i], (double)l[i], (double)u[i]) * prod;
+            }
+        }
+        est[qq] = sum / (double)n;
+        if (dpdh)
+            for (int32_t i = 0; i < d; ++i) dpdh[qq * d + i] = gsum[i] / (double)n;
+    }
+}
+
+/* tolerance scale: the derivative terms (both bounds) in absolute value */
+void oracle_epan_grad_abs_scale(const float *sample, int64_t n, int32_t d, const double *h,
+                                const float *lo, const float *hi, int64_t q, double *mabs)
+{
+    #pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t qq = 0; qq < q; ++qq) {
+        const float *l = lo + qq * d, *u = hi + qq * d;
+        double gsum[64];
+        for (int32_t i = 0; i < d; ++i) gsum[i] = 0.0;
+        for (int64_t j = 0; j < n; ++j) {
+            const float *t = sample + j * d;
+            for (int32_t i = 0; i < d; ++i) {
+                double prod = 1.0;
+                for (int32_t k = 0; k < d; ++k) {
+                    if (k == i) continue;
+                    prod *= epan_mass1((double)t[k], h[k], (double)l[k], (double)u[k]);
+                }
+                double vu = ((double)u[i] - (double)t[i]) / h[i], vl = ((double)l[i] - (double)t[i]) / h[i];
+                double a = isinf(vu) ? 0.0 : fabs(epan_pdf01(vu) * vu / h[i]);
+                double b = isinf(vl) ? 0.0 : fabs(epan_pdf01(vl) * vl / h[i]);
+                gsum[i] += (a + b) * fabs(prod);
+            }
+        }
+        for (int32_t i = 0; i < d; ++i) mabs[qq * d + i] = gsum[i] / (double)n;
+    }
+}
+
+/* eq. (19)-(20) derivation for the Epanechnikov product kernel:
+ * p_max = prod_j M_j(centre), thr = max_j p_max / M_j(centre) * M_j(face). */
+double oracle_epan_empty_region_threshold(int32_t d, const double *h, const float *lo, const float *hi,
+                                          double *pmax_out)
+{
+    double pmax = 1.0, best = 0.0;
+    int disabled = 0;
+    for (int32_t j = 0; j < d; ++j) {
+        double w = (double)hi[j] - (double)lo[j];
+        if (!(w > 0.0)) { disabled = 1; continue; }
+        double centre = isinf(w) ? 1.0 : epan_cdf(w / (2.0 * h[j])) - epan_cdf(-w / (2.0 * h[j]));
+        double face = isinf(w) ? 0.5 : epan_cdf(w / h[j]) - epan_cdf(0.0);
+        pmax *= centre;
+        double ratio = face / centre;
+        if (ratio > best) best = ratio;
+    }
+    if (pmax_out) *pmax_out = disabled ? 0.0 : pmax;
+    if (disabled || !(pmax > 0.0)) return INFINITY;
+    return pmax * best;
+}

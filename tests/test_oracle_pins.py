@@ -392,3 +392,75 @@ def test_property_gradient_along_h_matches_scaling_derivative(seed, d):
     fd = (oracle.estimate(S, h * (1 + e), lo[None], hi[None])[0]
           - oracle.estimate(S, h * (1 - e), lo[None], hi[None])[0]) / (2 * e)
     assert float(np.dot(h, gr[0])) == pytest.approx(fd, rel=1e-6, abs=1e-13)
+
+
+# --- Epanechnikov product kernel (NEXT-4, reading R14) ----------------------------
+def _epan_quad_mass(t, h, lo, hi):
+    """Independent pin: numerical quadrature of the density 3/(4h)(1-(x/h)^2) on |x|<=h."""
+    mp.mp.dps = 30
+    m = mp.mpf(1)
+    for tj, hj, lj, uj in zip(t, h, lo, hi):
+        a = max(float(lj), float(tj) - hj)
+        b = min(float(uj), float(tj) + hj)
+        if b <= a:
+            return 0.0
+        m *= mp.quad(lambda x: mp.mpf(3) / (4 * hj) * (1 - ((x - float(tj)) / hj) ** 2), [a, b])
+    return float(m)
+
+
+def test_epan_point_mass_matches_quadrature():
+    g = np.random.default_rng(20)
+    for _ in range(25):
+        d = int(g.integers(1, 4))
+        t = g.normal(size=d).astype(np.float32)
+        h = g.uniform(0.2, 2.0, d)
+        lo = g.uniform(-2, 0.5, d).astype(np.float32)
+        hi = (lo + g.uniform(0.05, 3, d)).astype(np.float32)
+        assert oracle.epan_point_mass(t, h, lo, hi) == pytest.approx(_epan_quad_mass(t, h, lo, hi), rel=1e-12,
+                                                                     abs=1e-15)
+
+
+def test_epan_unbounded_is_one_and_far_is_zero():
+    S = np.random.default_rng(21).normal(size=(50, 3)).astype(np.float32)
+    h = np.array([0.5, 1.0, 2.0])
+    est, g = oracle.epan_estimate_grad(S, h, np.full((1, 3), -np.inf, np.float32), np.full((1, 3), np.inf, np.float32))
+    assert est[0] == 1.0 and np.all(g == 0.0)
+    far = oracle.epan_estimate(S, h, np.full((1, 3), 100, np.float32), np.full((1, 3), 200, np.float32))
+    assert far[0] == 0.0  # compact support: exactly zero
+
+
+@pytest.mark.parametrize("log_bw", [False, True])
+def test_epan_gradient_matches_central_differences(log_bw):
+    g = np.random.default_rng(22)
+    S = g.normal(size=(60, 3)).astype(np.float32)
+    h = np.array([0.7, 1.1, 1.6])
+    lo = np.array([[-0.5, -1.0, -np.inf]], np.float32)
+    hi = np.array([[0.8, 0.4, 0.9]], np.float32)
+    _, gr = oracle.epan_estimate_grad(S, h, lo, hi)
+    for j in range(3):
+        e = 1e-6
+        hp, hm = h.copy(), h.copy()
+        hp[j] *= (1 + e)
+        hm[j] *= (1 - e)
+        fd = (oracle.epan_estimate(S, hp, lo, hi)[0] - oracle.epan_estimate(S, hm, lo, hi)[0]) / (2 * e * h[j])
+        assert gr[0, j] == pytest.approx(fd, rel=1e-6, abs=1e-12)
+
+
+def test_epan_threshold_is_boundary_maximum_and_sound():
+    """eq. (19)-(20) derivation for the Epanechnikov kernel: the threshold is the
+    largest mass of the centre moved to a face, and no outside point reaches it."""
+    h = np.array([0.6, 1.4])
+    lo = np.array([-1.0, 0.0], np.float32)
+    hi = np.array([0.5, 2.0], np.float32)
+    centre = ((lo.astype(np.float64) + hi) / 2).astype(np.float32)
+    thr, pmax = oracle.epan_empty_region_threshold(h, lo, hi)
+    assert oracle.epan_point_mass(centre, h, lo, hi) == pytest.approx(pmax, rel=1e-14)
+    faces = []
+    for j in range(2):
+        t = centre.copy(); t[j] = lo[j]
+        faces.append(oracle.epan_point_mass(t, h, lo, hi))
+    assert thr == pytest.approx(max(faces), rel=1e-13)
+    S = np.random.default_rng(23).uniform(-3, 3, size=(20000, 2)).astype(np.float32)
+    c = oracle.epan_contributions(S, h, lo, hi)
+    outside = ~np.all((S >= lo) & (S <= hi), axis=1)
+    assert np.all(c[outside] < thr * (1 + 1e-12))
