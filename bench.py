@@ -61,6 +61,11 @@ CONFIGS = {
                desc="configs[4] streaming step: d=10, N=2^22, one DT box per step: estimate + gradient + retained "
                     "contributions, karma pass + compaction, Listing 1 bandwidth step, replacement of flagged points "
                     "(device-resident kde_stream_step_dev: 3 kernels, single GPU)"),
+    "c2e": dict(d=3, n=1 << 20, q=10000, path="loss_grad", data="gauss", kernel="epan",
+                desc="configs[1] with the Epanechnikov product kernel (NEXT-4, reading R14): d=3, N=2^20/GPU, "
+                     "10k-box batch, estimate + L2 loss + bandwidth gradient"),
+    "c3se": dict(d=5, n=1 << 24, q=1, path="single", grad=False, retain=False, data="gauss", kernel="epan",
+                 desc="configs[2] single box with the Epanechnikov product kernel: d=5, N=2^24/GPU, estimate"),
     "c4": dict(d=8, n=1 << 25, q=4096, path="loss_grad", data="gauss",
                desc="configs[3] per-GPU shard: d=8, 2^25 rows/GPU (2^28 at 8 GPUs), 4096 boxes, estimate + gradient + NCCL"),
 }
@@ -249,6 +254,9 @@ def run_cuda(args, cfg, rank, world, local_rank):
         m = K.KDEModel.create_sharded(S, rank * n, n_global, None, nid, rank, world)
     else:
         m = K.KDEModel.create(S)
+    if cfg.get("kernel") == "epan":
+        m.set_kernel("epan")
+        m.bandwidth = m.bandwidth * np.sqrt(5.0)  # variance-matched to Scott's Gaussian bandwidth
     h = m.bandwidth
 
     stream = torch.cuda.Stream(device=dev)
@@ -421,6 +429,15 @@ def run_cuda(args, cfg, rank, world, local_rank):
                 "traffic": _traffic(args.config), "kernel": f"scan_single_kernel<{d},{'grad' if cfg.get('grad') else 'est'}>",
                 "algorithmic": f"4*d bytes/point{' + 4 B/point retained' if cfg.get('retain') else ''} x {n} points per launch",
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
+    elif cfg.get("kernel") == "epan":
+        # no transcendental: the algorithmic minimum is the FP32 work, 6 FP32 ops per dimension
+        # (2 subtract-scale, 2 products of the S = a^2 + ab + b^2 form, 2 for D) -> FP32 ceiling
+        achieved = n * q / (avg_scan_ms * 1e-3) / 1e9
+        peak = sms * 128 * SM_MAX_MHZ * 1e6 / (6 * d) / 1e9
+        roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gpt·q/s", "frac": achieved / peak,
+                "traffic": _traffic(args.config), "kernel": f"scan_batched_kernel<{d},grad> (Epanechnikov)",
+                "algorithmic": f"{n} points x {q} boxes per launch; 6d FP32 ops per point*box",
+                "peak_source": f"FP32 ceiling {sms} SMs x 128 lanes x {SM_MAX_MHZ:.0f} MHz / (6d)"}
     else:
         achieved = n * q / (avg_scan_ms * 1e-3) / 1e9
         peak = sms * MUFU_PER_SM_CLK * SM_MAX_MHZ * 1e6 / (2 * d) / 1e9

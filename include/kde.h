@@ -68,6 +68,18 @@ typedef enum {
     KDE_LOSS_SQUARED_Q = 4
 } kde_loss;
 
+/* Kernel function.  GAUSSIAN is the paper's kernel (eq. 9) and the
+ * default.  EPANECHNIKOV ("a truncated second-degree polynomial"; the
+ * paper derives nothing for it): the 1-D density 3/(4h) (1 - (x/h)^2) on
+ * |x| <= h, i.e. h is the support half-width (reading R14); box
+ * masses, gradients and the eq. (20) threshold are its exact counterparts.
+ * Its variance is h^2/5, so h_epan = sqrt(5) h_gauss matches a Gaussian
+ * bandwidth. */
+typedef enum {
+    KDE_KERNEL_GAUSSIAN = 0,
+    KDE_KERNEL_EPANECHNIKOV = 1
+} kde_kernel;
+
 /* Karma-based sample maintenance, Section 4.2 and P:L250.
  *   loss, lambda : the loss L of eq. (7)
  *   k_max        : saturation constant of eq. (8); the paper uses 4
@@ -145,6 +157,12 @@ kde_status kde_get_info(const kde_model *m, int64_t *n_local, int64_t *n_global,
  * every h_j finite in [1e-30, 1e30]; it invalidates retained contributions. */
 kde_status kde_get_bandwidth(kde_model *m, double *h);
 kde_status kde_set_bandwidth(kde_model *m, const double *h);
+
+/* kde_set_kernel / kde_get_kernel -- select the kernel function (kde_kernel);
+ * h is kept, the per-dimension constants are re-derived on the device.
+ * Invalidates retained contributions.  Errors: KDE_EINVAL (unknown kernel). */
+kde_status kde_set_kernel(kde_model *m, int32_t kernel);
+kde_status kde_get_kernel(const kde_model *m, int32_t *kernel);
 
 /* kde_set_retain -- on != 0: single-query scans (q == 1) also store the
  * per-point contributions p^(i) (fp32, 4 B/point) for a following

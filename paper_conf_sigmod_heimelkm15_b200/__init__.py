@@ -23,6 +23,7 @@ LIB_PATH = os.path.join(_HERE, "libkde.so")
 
 KDE_OK, KDE_EINVAL, KDE_ENOMEM, KDE_ECUDA, KDE_ENCCL, KDE_ESTATE, KDE_ETRUNC = range(7)
 LOSS_SQUARED, LOSS_ABSOLUTE, LOSS_RELATIVE, LOSS_SQUARED_RELATIVE, LOSS_SQUARED_Q = range(5)
+KERNEL_GAUSSIAN, KERNEL_EPANECHNIKOV = 0, 1
 KDE_MAX_DIM = 16
 KDE_NCCL_ID_BYTES = 128
 
@@ -35,6 +36,7 @@ ABI_SYMBOLS = (
     "kde_get_karma", "kde_set_karma", "kde_get_sample", "kde_get_contributions", "kde_get_online_state",
     "kde_set_online_state", "kde_synchronize", "kde_count_in_box_dev", "kde_set_profiling", "kde_get_profile",
     "kde_karma_update_dev", "kde_online_update_dev", "kde_replace_points_dev", "kde_stream_step_dev",
+    "kde_set_kernel", "kde_get_kernel",
 )
 
 
@@ -98,6 +100,8 @@ def lib() -> ctypes.CDLL:
         "kde_get_bandwidth": (ctypes.c_int, [P, P]),
         "kde_set_bandwidth": (ctypes.c_int, [P, P]),
         "kde_set_retain": (ctypes.c_int, [P, i32]),
+        "kde_set_kernel": (ctypes.c_int, [P, i32]),
+        "kde_get_kernel": (ctypes.c_int, [P, P]),
         "kde_estimate_batch": (ctypes.c_int, [P, P, P, i64, P, P]),
         "kde_estimate_batch_dev": (ctypes.c_int, [P, P, P, i64, P, P, P]),
         "kde_loss_and_grad": (ctypes.c_int, [P, P, P, P, i64, i32, f64, i32, P, P, P]),
@@ -209,6 +213,16 @@ def kde_get_bandwidth(m, d):
 def kde_set_bandwidth(m, h):
     h = _f64(h)
     _check(lib().kde_set_bandwidth(m, _p(h)))
+
+
+def kde_set_kernel(m, kernel: int):
+    _check(lib().kde_set_kernel(m, int(kernel)))
+
+
+def kde_get_kernel(m) -> int:
+    k = ctypes.c_int32()
+    _check(lib().kde_get_kernel(m, ctypes.byref(k)))
+    return k.value
 
 
 def kde_set_retain(m, on: bool):
@@ -405,6 +419,16 @@ class KDEModel:
     @bandwidth.setter
     def bandwidth(self, h):
         kde_set_bandwidth(self.handle, h)
+
+    def set_kernel(self, kernel):
+        """KERNEL_GAUSSIAN (paper, default) or KERNEL_EPANECHNIKOV (or 'gauss' / 'epan')."""
+        if isinstance(kernel, str):
+            kernel = {"gauss": KERNEL_GAUSSIAN, "epan": KERNEL_EPANECHNIKOV}[kernel]
+        kde_set_kernel(self.handle, kernel)
+
+    @property
+    def kernel(self):
+        return kde_get_kernel(self.handle)
 
     def set_retain(self, on=True):
         kde_set_retain(self.handle, on)

@@ -20,11 +20,16 @@ constexpr int kColAlign = 1024;  // columns padded to a multiple of this many po
 //                                                  z = (b - t)/(sqrt2 h) is the erf argument of eq. (13)
 //   gconst[j] = 1 / (sqrt(pi) sqrt(log2 e) h_j)   so that d p^(i)/d h_j = gconst[j] * w_j * prod_{k!=j} D_k,
 //                                                  w_j = y'_l E_l - y'_u E_u (eq. 17 rewritten in z)
+// Epanechnikov product kernel (reading R14): ap[j] = 1/h_j (v = (b - t)/h),
+//   gconst[j] = -3 / (4 h_j), w_j = Delta (1 - S) (see phi.cuh).
 //   tmin/tmax = per-column range of the (local) sample: query bounds are
 //   clamped to [tmin - 14/ap, tmax + 14/ap] at box setup, which leaves every
 //   fp32 result unchanged (|y'| >= 14 gives E = 0, erf = +-1 exactly) and
 //   keeps y' finite, so the gradient term y' E never meets inf * 0.
+enum KernelType : int { kGaussian = 0, kEpanechnikov = 1 };
+
 struct DevConsts {
+  int kernel;  // KernelType: selects the per-dimension constants below
   double h[kMaxDim];
   double gconst[kMaxDim];
   float ap[kMaxDim];

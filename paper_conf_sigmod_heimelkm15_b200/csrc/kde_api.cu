@@ -85,6 +85,7 @@ struct kde_model {
   uint64_t gen = 1;      // bumped whenever h or the sample changes
   uint64_t ret_gen = 0;
   bool online_init = false;
+  int32_t kernel = 0;  // KDE_KERNEL_GAUSSIAN
 
   // profiling (kde_set_profiling): CUDA events around every scan launch on its
   // own stream, and a count of every kernel this model launched
@@ -552,6 +553,24 @@ extern "C" kde_status kde_set_bandwidth(kde_model* m, const double* h) {
   CUL(launch_set_consts(h, m->d, m->consts, m->stream));
   CU(cudaStreamSynchronize(m->stream));
   ++m->gen;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_set_kernel(kde_model* m, int32_t kernel) {
+  CHECK_MODEL(m);
+  if (kernel != KDE_KERNEL_GAUSSIAN && kernel != KDE_KERNEL_EPANECHNIKOV)
+    return fail(KDE_EINVAL, "unknown kernel %d", kernel);
+  DeviceGuard g(m->device);
+  CUL(launch_set_kernel_type(kernel, m->d, m->consts, m->stream));
+  CU(cudaStreamSynchronize(m->stream));
+  m->kernel = kernel;
+  ++m->gen;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_get_kernel(const kde_model* m, int32_t* kernel) {
+  if (!m || !kernel) return fail(KDE_EINVAL, "NULL argument");
+  *kernel = m->kernel;
   return KDE_OK;
 }
 

@@ -174,8 +174,20 @@ __device__ void set_consts_dev(DevConsts* c, int j, double h) {
   const double kSqrtPi = 1.7724538509055160273;
   const double kSqrt2 = 1.4142135623730950488;
   c->h[j] = h;
-  c->ap[j] = (float)(kSqrtLog2e / (kSqrt2 * h));
-  c->gconst[j] = 1.0 / (kSqrtPi * kSqrtLog2e * h);
+  if (c->kernel == kEpanechnikov) {  // reading R14: v = (b - t)/h, dD/dh = -(3/(4h)) Delta (1 - S)
+    c->ap[j] = (float)(1.0 / h);
+    c->gconst[j] = -0.75 / h;
+  } else {
+    c->ap[j] = (float)(kSqrtLog2e / (kSqrt2 * h));
+    c->gconst[j] = 1.0 / (kSqrtPi * kSqrtLog2e * h);
+  }
+}
+
+__global__ void set_kernel_type_kernel(int kernel, int d, DevConsts* c) {
+  if (threadIdx.x == 0) c->kernel = kernel;
+  __syncthreads();
+  const int j = threadIdx.x;
+  if (j < d) set_consts_dev(c, j, c->h[j]);
 }
 
 // eq. (3): h_j = s^(-1/(d+4)) sigma_j, population sigma.
@@ -288,19 +300,34 @@ __global__ void loss_epilogue_kernel(const double* __restrict__ est, const doubl
 // Each block owns a contiguous range of kKarmaPts points, visited in ascending
 // order (pass-major, thread-minor), so the flag bitmap words are in index order.
 // eq. (19)-(20) threshold computed per block in fp64 from (lo, hi, h).
+__device__ double epan_cdf_dev(double v) {
+  if (v <= -1.0) return 0.0;
+  if (v >= 1.0) return 1.0;
+  return (2.0 + 3.0 * v - v * v * v) / 4.0;
+}
+
+// eq. (19)-(20): p_max = prod_j M_j(centre), thr = max_j p_max M_j(face) / M_j(centre)
+// (Gaussian: M(centre) = erf(w / (2 sqrt2 h)), M(face) = erf(w / (sqrt2 h)) / 2;
+//  Epanechnikov: the same derivation with its CDF).
 __device__ double thr20_dev(const float* lo, const float* hi, int d, const DevConsts* c) {
   const double kSqrt2 = 1.4142135623730950488;
   double pmax = 1.0, best = 0.0;
   for (int j = 0; j < d; ++j) {
     const double w = (double)hi[j] - (double)lo[j];
     if (!(w > 0.0)) return CUDART_INF;  // zero width: shortcut disabled (reading R5)
-    const double half = erf(w / (2.0 * kSqrt2 * c->h[j]));
-    const double full = erf(w / (kSqrt2 * c->h[j]));
-    pmax *= half;
-    const double ratio = isinf(w) ? 1.0 : full / half;
-    best = fmax(best, ratio);
+    double centre, face;
+    if (c->kernel == kEpanechnikov) {
+      centre = isinf(w) ? 1.0 : epan_cdf_dev(w / (2.0 * c->h[j])) - epan_cdf_dev(-w / (2.0 * c->h[j]));
+      face = isinf(w) ? 0.5 : epan_cdf_dev(w / c->h[j]) - 0.5;
+    } else {
+      centre = erf(w / (2.0 * kSqrt2 * c->h[j]));
+      face = isinf(w) ? 0.5 : 0.5 * erf(w / (kSqrt2 * c->h[j]));
+    }
+    pmax *= centre;
+    best = fmax(best, face / centre);
   }
-  return pmax / 2.0 * best;
+  if (!(pmax > 0.0)) return CUDART_INF;
+  return pmax * best;
 }
 
 __global__ void karma_kernel(const float* __restrict__ cvals, double* __restrict__ karma, int64_t n, double n_global,
@@ -623,6 +650,10 @@ cudaError_t launch_moments_merge_ranks(const double* g, int world, int d, double
 }
 cudaError_t launch_scott(const double* mom, int d, DevConsts* c, int* bad, cudaStream_t s) {
   scott_kernel<<<1, 32, 0, s>>>(mom, d, c, bad);
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_set_kernel_type(int kernel, int d, DevConsts* c, cudaStream_t s) {
+  set_kernel_type_kernel<<<1, 32, 0, s>>>(kernel, d, c);
   KDE_LAUNCH_CHECK();
 }
 cudaError_t launch_set_consts(const double* h, int d, DevConsts* c, cudaStream_t s) {

@@ -49,6 +49,7 @@ cudaError_t launch_moments(const float* cols, int64_t ld, int64_t n, int d, doub
 cudaError_t launch_moments_merge_ranks(const double* g, int world, int d, double* mom, cudaStream_t s);
 cudaError_t launch_scott(const double* mom, int d, DevConsts* c, int* bad, cudaStream_t s);
 cudaError_t launch_set_consts(const double* h, int d, DevConsts* c, cudaStream_t s);
+cudaError_t launch_set_kernel_type(int kernel, int d, DevConsts* c, cudaStream_t s);
 cudaError_t launch_reduce_splits(const double* partials, int splits, int64_t q, int na, double* sums,
                                  cudaStream_t s);
 cudaError_t launch_combine_ranks(const double* gathered, int world, int64_t q, int na, double* sums,

@@ -67,9 +67,18 @@ struct BoxDim {
 
 constexpr float kBoundMargin = 14.0f;  // |y'| >= 14: 2^-196 flushes to 0, erf(z) == +-1 in fp32
 
+template <int KT = kGaussian>
 __device__ __forceinline__ BoxDim make_boxdim(float l, float u, float ap, unsigned rmin_enc, unsigned rmax_enc) {
   BoxDim r;
   const float tmin = fdec_range(rmin_enc), tmax = fdec_range(rmax_enc);
+  if (KT == kEpanechnikov) {  // v = (b - t)/h; support |v| < 1: clamp the bounds to the range widened by 2h
+    const float m = 2.0f / ap;
+    l = fminf(fmaxf(l, tmin - m), tmax + m);
+    u = fminf(fmaxf(u, tmin - m), tmax + m);
+    r.b = make_float2(u, l);
+    r.hd = (u - l) * ap;  // Delta of the unclamped case, formed without cancellation
+    return r;
+  }
   const float dy = (u - l) * ap;  // inf for unbounded, NaN for (inf, inf): both normal
   const float m = kBoundMargin / ap;
   l = fminf(fmaxf(l, tmin - m), tmax + m);
@@ -121,6 +130,25 @@ __device__ __forceinline__ float phi_narrow(const float2 y, const float2 E, floa
     w = -hd * (s - kTwoLn2 * fmaf(E.x, yy.x, E.y * yy.y));
   }
   return hd * kInvSqrtPiLog2e * s;
+}
+
+// Epanechnikov product kernel (reading R14), one dimension for one point:
+//   v = (b - t)/h clamped to [-1, 1] (a = v_u, b = v_l),  Delta = a - b,
+//   S = a^2 + a b + b^2,  D = F(a) - F(b) = Delta (3 - S) / 4,
+//   d D / d h = -(3 / (4h)) [g(a) - g(b)],  g(v) = v (1 - v^2),  g(a) - g(b) = Delta (1 - S),
+// so both come from Delta and S without the cancellation of F(a) - F(b) for
+// narrow boxes (Delta = (u - l)/h when neither bound is clamped).
+template <bool GRAD>
+__device__ __forceinline__ float phi_epan(const BoxDim& bd, float t, float ih, float& w) {
+  const float2 v = __fmul2_rn(__fadd2_rn(bd.b, f2(-t)), f2(ih));
+  const float a = fminf(fmaxf(v.x, -1.0f), 1.0f);
+  const float b = fminf(fmaxf(v.y, -1.0f), 1.0f);
+  // both bounds inside the support: the cancellation-free (u - l)/h; otherwise
+  // a clamped value is involved and a - b is exact enough (0 when both clamp alike)
+  const float dl = (v.x == a && v.y == b) ? bd.hd : a - b;
+  const float S = fmaf(a, a + b, b * b);
+  if (GRAD) w = fmaf(-S, dl, dl);
+  return fmaf(S, -0.25f, 0.75f) * dl;
 }
 
 // One dimension of eq. (13) for one point and one box; GENERAL handles narrow

@@ -60,12 +60,15 @@ __device__ __forceinline__ float f4c(const float4& v, int p) {
 // All d factors of eq. (13) for one point and one box, the product p^(i), and
 // (GRAD) the d gradient terms w_j prod_{k!=j} D_k, added into s[0..D].
 // Returns p^(i).  `valid` masks padding points (contributes exactly 0).
-template <int D, bool GRAD, bool GENERAL>
+// MODE: 0 = Gaussian, no narrow dimension; 1 = Gaussian, general (narrow
+// dimensions on the Gauss-Legendre path); 2 = Epanechnikov product kernel.
+template <int D, bool GRAD, int MODE>
 __device__ __forceinline__ float point_box(const BoxDim (&bd)[D], const float (&t)[D], const float (&ap)[D],
                                            float* s, bool valid) {
   float Dv[D], wv[D];
 #pragma unroll
-  for (int j = 0; j < D; ++j) Dv[j] = phi_diff<GRAD, GENERAL>(bd[j], t[j], ap[j], wv[j]);
+  for (int j = 0; j < D; ++j)
+    Dv[j] = MODE == 2 ? phi_epan<GRAD>(bd[j], t[j], ap[j], wv[j]) : phi_diff<GRAD, MODE == 1>(bd[j], t[j], ap[j], wv[j]);
   float pre[D + 1];
   pre[0] = 1.0f;
 #pragma unroll
@@ -176,7 +179,7 @@ __device__ __forceinline__ float4 ldcs_v(const float4* p) { return __ldcs(p); }
 __device__ __forceinline__ void stcs_v(float2* p, const float* c) { __stcs(p, make_float2(c[0], c[1])); }
 __device__ __forceinline__ void stcs_v(float4* p, const float* c) { __stcs(p, make_float4(c[0], c[1], c[2], c[3])); }
 
-template <int D, bool GRAD, bool GENERAL, int VW>
+template <int D, bool GRAD, int MODE, int VW>
 __device__ __forceinline__ void single_group(const typename VecT<VW>::type (&tv)[D], const float4* __restrict__ smc,
                                              float* s, float* c_out, int64_t v, int valid) {
   float cs[VW];
@@ -192,12 +195,12 @@ __device__ __forceinline__ void single_group(const typename VecT<VW>::type (&tv)
       ap[j] = c.w;
       t[j] = vcomp(tv[j], p);
     }
-    cs[p] = point_box<D, GRAD, GENERAL>(bd, t, ap, s, p < valid);
+    cs[p] = point_box<D, GRAD, MODE>(bd, t, ap, s, p < valid);
   }
   if (c_out) stcs_v(reinterpret_cast<typename VecT<VW>::type*>(c_out) + v, cs);
 }
 
-template <int D, bool GRAD, bool GENERAL, int VW, bool PF>
+template <int D, bool GRAD, int MODE, int VW, bool PF>
 __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const float4* smc);
 
 template <int D, bool GRAD, int VW = SingleVW<D, GRAD>::value, int OCC = single_occ(D, GRAD),
@@ -210,18 +213,24 @@ __global__ void __launch_bounds__(kSingleThreads, OCC) scan_single_kernel(const 
   if (threadIdx.x < D) {
     const int j = threadIdx.x;
     const float ap = a.consts->ap[j];
-    const BoxDim bd = make_boxdim(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
+    const bool epan = a.consts->kernel == kEpanechnikov;
+    const BoxDim bd = epan ? make_boxdim<kEpanechnikov>(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->renc[2 * j],
+                                                         a.consts->renc[2 * j + 1])
+                           : make_boxdim(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->renc[2 * j],
+                                         a.consts->renc[2 * j + 1]);
     smc[j] = make_float4(bd.b.x, bd.b.y, bd.hd, ap);
-    if (bd.hd > 0.0f) atomicOr(&narrow_s, 1);
+    if (!epan && bd.hd > 0.0f) atomicOr(&narrow_s, 1);
   }
   __syncthreads();
-  if (narrow_s)
-    scan_single_body<D, GRAD, true, VW, PF>(a, smc);
+  if (a.consts->kernel == kEpanechnikov)
+    scan_single_body<D, GRAD, 2, VW, PF>(a, smc);
+  else if (narrow_s)
+    scan_single_body<D, GRAD, 1, VW, PF>(a, smc);
   else
-    scan_single_body<D, GRAD, false, VW, PF>(a, smc);
+    scan_single_body<D, GRAD, 0, VW, PF>(a, smc);
 }
 
-template <int D, bool GRAD, bool GENERAL, int VW, bool PF>
+template <int D, bool GRAD, int MODE, int VW, bool PF>
 __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const float4* smc) {
   constexpr int NA = GRAD ? D + 1 : 1;
   using V = typename VecT<VW>::type;
@@ -255,7 +264,7 @@ __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const 
 #pragma unroll
           for (int j = 0; j < D; ++j) nxt[j] = ldcs_v(col + j * ldv + vn);
         }
-        single_group<D, GRAD, GENERAL, VW>(cur, smc, s, a.c_out, v, VW);
+        single_group<D, GRAD, MODE, VW>(cur, smc, s, a.c_out, v, VW);
         v = vn;
         if (v >= nfull) break;
         vn = v + stride;
@@ -263,7 +272,7 @@ __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const 
 #pragma unroll
           for (int j = 0; j < D; ++j) cur[j] = ldcs_v(col + j * ldv + vn);
         }
-        single_group<D, GRAD, GENERAL, VW>(nxt, smc, s, a.c_out, v, VW);
+        single_group<D, GRAD, MODE, VW>(nxt, smc, s, a.c_out, v, VW);
         v = vn;
       }
 #pragma unroll
@@ -279,7 +288,7 @@ __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const 
         V t0[D];
 #pragma unroll
         for (int j = 0; j < D; ++j) t0[j] = ldcs_v(col + j * ldv + v);
-        single_group<D, GRAD, GENERAL, VW>(t0, smc, s, a.c_out, v, VW);
+        single_group<D, GRAD, MODE, VW>(t0, smc, s, a.c_out, v, VW);
       }
 #pragma unroll
       for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
@@ -294,7 +303,7 @@ __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const 
     float s[NA];
 #pragma unroll
     for (int k = 0; k < NA; ++k) s[k] = 0.0f;
-    single_group<D, GRAD, GENERAL, VW>(t0, smc, s, a.c_out, v, valid);
+    single_group<D, GRAD, MODE, VW>(t0, smc, s, a.c_out, v, valid);
 #pragma unroll
     for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
   }
@@ -331,7 +340,7 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 // Accumulate every point of one shared-memory tile against the thread's QT
 // boxes.  No barriers inside, so the GENERAL (narrow-dimension) and fast
 // variants can be chosen per warp.
-template <int D, bool GRAD, bool GENERAL, int QT, int PU>
+template <int D, bool GRAD, int MODE, int QT, int PU>
 __device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, int phase, int R, double* accsh,
                                                      const BoxDim (&bd)[QT][D], const float (&ap)[D]) {
   constexpr int NA = GRAD ? D + 1 : 1;
@@ -354,7 +363,7 @@ __device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, 
 #pragma unroll
         for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
 #pragma unroll
-        for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, GENERAL>(bd[qq], t, ap, s[qq], true);
+        for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, MODE>(bd[qq], t, ap, s[qq], true);
       }
     }
     for (; m < me; ++m) {
@@ -363,7 +372,7 @@ __device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, 
 #pragma unroll
       for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
 #pragma unroll
-      for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, GENERAL>(bd[qq], t, ap, s[qq], true);
+      for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, MODE>(bd[qq], t, ap, s[qq], true);
     }
 #pragma unroll
     for (int qq = 0; qq < QT; ++qq)
@@ -379,7 +388,7 @@ __device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, 
 template <int D, bool GRAD, int QT, int PU, typename Issue>
 __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const float* tile, uint64_t* bar,
                                               double* accsh, const BoxDim (&bd)[QT][D], const float (&ap)[D],
-                                              int64_t s0, int64_t s1, int ntiles, bool warp_general, int phase, int R,
+                                              int64_t s0, int64_t s1, int ntiles, int mode, int phase, int R,
                                               Issue& issue) {
   const int tid = threadIdx.x;
   for (int k = 0; k < ntiles; ++k) {
@@ -389,10 +398,12 @@ __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const fl
     const float* tl = tile + buf * D * kTilePts;
     const int64_t rem = s1 - (s0 + (int64_t)k * kTilePts);
     const int npts = rem < kTilePts ? (int)rem : kTilePts;
-    if (warp_general)
-      batched_tile_compute<D, GRAD, true, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
+    if (mode == 2)
+      batched_tile_compute<D, GRAD, 2, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
+    else if (mode == 1)
+      batched_tile_compute<D, GRAD, 1, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
     else
-      batched_tile_compute<D, GRAD, false, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
+      batched_tile_compute<D, GRAD, 0, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
     __syncthreads();
   }
 }
@@ -430,8 +441,9 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
   float ap[D];
 #pragma unroll
   for (int j = 0; j < D; ++j) ap[j] = a.consts->ap[j];
+  const bool epan = a.consts->kernel == kEpanechnikov;
   bool nar = false;
-  if (tid < QB) {
+  if (tid < QB && !epan) {
     int64_t qi = qbase + tid;
     if (qi >= a.q) qi = a.q - 1;  // duplicate a valid box; its partial is never written
 #pragma unroll
@@ -476,9 +488,14 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
     narrow[0] = false;
 #pragma unroll
     for (int j = 0; j < D; ++j) {
-      bd[0][j] = make_boxdim(__ldg(a.lo + qi * D + j), __ldg(a.hi + qi * D + j), ap[j], a.consts->renc[2 * j],
-                              a.consts->renc[2 * j + 1]);
-      narrow[0] |= bd[0][j].hd > 0.0f;
+      if (epan) {
+        bd[0][j] = make_boxdim<kEpanechnikov>(__ldg(a.lo + qi * D + j), __ldg(a.hi + qi * D + j), ap[j],
+                                              a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
+      } else {
+        bd[0][j] = make_boxdim(__ldg(a.lo + qi * D + j), __ldg(a.hi + qi * D + j), ap[j], a.consts->renc[2 * j],
+                               a.consts->renc[2 * j + 1]);
+        narrow[0] |= bd[0][j].hd > 0.0f;
+      }
     }
   }
 #pragma unroll
@@ -510,8 +527,8 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
   bool my_narrow = false;
 #pragma unroll
   for (int qq = 0; qq < QT; ++qq) my_narrow |= narrow[qq];
-  const bool warp_general = __any_sync(0xffffffffu, my_narrow);
-  batched_tiles<D, GRAD, QT, PU>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, warp_general, phase, R, issue);
+  const int mode = epan ? 2 : (__any_sync(0xffffffffu, my_narrow) ? 1 : 0);
+  batched_tiles<D, GRAD, QT, PU>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, mode, phase, R, issue);
 
   // combine the R phases of each box in phase order, then
   // partials[(split*(NA) + comp) * q + qi]

@@ -17,7 +17,7 @@ constexpr size_t single_tma_smem_bytes() {
   return (size_t)STAGES * D * TILE * sizeof(float) + STAGES * sizeof(uint64_t);
 }
 
-template <int D, bool GRAD, bool GENERAL, int TILE, int STAGES>
+template <int D, bool GRAD, int MODE, int TILE, int STAGES>
 __device__ __forceinline__ void scan_single_tma_body(const ScanSingleArgs& a, const float4* smc, float* tiles,
                                                      uint64_t* full, int64_t c0, int64_t c1, int ntiles) {
   constexpr int NA = GRAD ? D + 1 : 1;
@@ -52,7 +52,7 @@ __device__ __forceinline__ void scan_single_tma_body(const ScanSingleArgs& a, co
       float t[D];
 #pragma unroll
       for (int j = 0; j < D; ++j) t[j] = tl[j * TILE + p];
-      const float c = point_box<D, GRAD, GENERAL>(bd, t, ap, s, valid);
+      const float c = point_box<D, GRAD, MODE>(bd, t, ap, s, valid);
       if (a.c_out && valid) __stcs(a.c_out + base + p, c);
     }
 #pragma unroll
@@ -104,15 +104,21 @@ __global__ void __launch_bounds__(kSingleThreads, OCC) scan_single_tma_kernel(co
   if (tid < D) {
     const int j = tid;
     const float ap = a.consts->ap[j];
-    const BoxDim bd = make_boxdim(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
+    const bool epan = a.consts->kernel == kEpanechnikov;
+    const BoxDim bd = epan ? make_boxdim<kEpanechnikov>(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->renc[2 * j],
+                                                         a.consts->renc[2 * j + 1])
+                           : make_boxdim(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->renc[2 * j],
+                                         a.consts->renc[2 * j + 1]);
     smc[j] = make_float4(bd.b.x, bd.b.y, bd.hd, ap);
-    if (bd.hd > 0.0f) atomicOr(&narrow_s, 1);
+    if (!epan && bd.hd > 0.0f) atomicOr(&narrow_s, 1);
   }
   __syncthreads();
-  if (narrow_s)
-    scan_single_tma_body<D, GRAD, true, TILE, STAGES>(a, smc, tiles, full, c0, c1, ntiles);
+  if (a.consts->kernel == kEpanechnikov)
+    scan_single_tma_body<D, GRAD, 2, TILE, STAGES>(a, smc, tiles, full, c0, c1, ntiles);
+  else if (narrow_s)
+    scan_single_tma_body<D, GRAD, 1, TILE, STAGES>(a, smc, tiles, full, c0, c1, ntiles);
   else
-    scan_single_tma_body<D, GRAD, false, TILE, STAGES>(a, smc, tiles, full, c0, c1, ntiles);
+    scan_single_tma_body<D, GRAD, 0, TILE, STAGES>(a, smc, tiles, full, c0, c1, ntiles);
 }
 
 template <int D, bool GRAD, int TILE, int STAGES, int OCC>

@@ -520,3 +520,61 @@ def test_small_batches_phase_mapping(q):
     est, g = m.estimate(lo, hi, grad=True)
     sel_ok(est, est_o)
     grad_ok(g, g_o, mabs)
+
+
+# ------------------------------------------------------------------ Epanechnikov kernel (NEXT-4)
+@pytest.mark.parametrize("d,n", [(1, 5), (3, 20011), (5, 70001), (10, 9001)])
+def test_epanechnikov_estimates_and_gradients(d, n):
+    """Reading R14 kernel: single-box (TMA / register) and batched scans vs the oracle."""
+    S = synth.make_data("gauss", n, d, seed=90 + d)
+    m = model(S)
+    m.set_kernel("epan")
+    assert m.kernel == K.KERNEL_EPANECHNIKOV
+    h = m.bandwidth * np.sqrt(5.0)  # variance-matched to Scott's Gaussian bandwidth
+    m.bandwidth = h
+    lo, hi = boxes_mix(S, 40, seed=91 + d)
+    est_o, g_o = oracle.epan_estimate_grad(S, h, lo, hi)
+    mabs = oracle.epan_grad_abs_scale(S, h, lo, hi)
+    est, g = m.estimate(lo, hi, grad=True)
+    sel_ok(est, est_o)
+    grad_ok(g, g_o, mabs, h)
+    sel_ok(m.estimate(lo, hi), est_o)
+    for k in (0, 1, 5, len(lo) - 1):
+        e1, g1 = m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+        sel_ok(e1, est_o[k:k + 1])
+        grad_ok(g1, g_o[k:k + 1], mabs[k:k + 1], h)
+
+
+def test_epanechnikov_loss_karma_and_switch_back():
+    n, d = 6000, 3
+    S = synth.make_data("gauss", n, d, seed=95)
+    R = synth.make_data("gauss", 40000, d, seed=95)
+    lo, hi = synth.mixed_workload(S, 30, seed=96)
+    p = synth.true_selectivity_cpu(R, lo, hi)
+    m = model(S)
+    h_g = m.bandwidth
+    m.set_kernel("epan")
+    h = h_g * np.sqrt(5.0)
+    m.bandwidth = h
+    L, g = m.loss_and_grad(lo, hi, p, K.LOSS_SQUARED, 0.0, True)
+    L_o, g_o, est_o = oracle.epan_loss_and_grad(S, h, lo, hi, p, 0, 0.0, True)
+    assert abs(L - L_o) <= 1e-6 * abs(L_o) + 1e-12
+    mabs = oracle.epan_grad_abs_scale(S, h, lo, hi)
+    dL = 2 * np.abs(est_o - p)
+    grad_ok(g, g_o, (dL[:, None] * mabs).mean(axis=0) * h, h)
+    # karma with the empty-region rule (true selectivity 0 on a populated box)
+    m.set_retain(True)
+    m.estimate(lo[:1], hi[:1])
+    kp = K.karma_params(loss=K.LOSS_ABSOLUTE, threshold=-1e9, empty_region=True)
+    idx, nf, _ = m.karma_update(lo[0], hi[0], 0.0, kp)
+    c_o = oracle.epan_contributions(S, h, lo[0], hi[0])
+    thr, _ = oracle.epan_empty_region_threshold(h, lo[0], hi[0])
+    expect = np.nonzero(c_o >= thr)[0]
+    amb = np.abs(c_o - thr) < 1e-6 * thr
+    got = np.zeros(n, bool); got[idx] = True
+    exp_ = np.zeros(n, bool); exp_[expect] = True
+    assert np.array_equal(got[~amb], exp_[~amb])
+    # back to the Gaussian kernel: the constants are re-derived from the same h
+    m.set_kernel("gauss")
+    m.bandwidth = h_g
+    sel_ok(m.estimate(lo, hi), oracle.estimate(S, h_g, lo, hi))
