@@ -426,7 +426,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
         achieved = alg_bytes / (avg_scan_ms * 1e-3) / 1e9
         peak = _measured_hbm()
         roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": _traffic(args.config), "kernel": f"scan_single_kernel<{d},{'grad' if cfg.get('grad') else 'est'}>",
+                "traffic": _traffic(args.config), "kernel": f"{'scan_single_tma_kernel' if d <= 8 else 'scan_single_kernel'}<{d},{'grad' if cfg.get('grad') else 'est'}>",
                 "algorithmic": f"4*d bytes/point{' + 4 B/point retained' if cfg.get('retain') else ''} x {n} points per launch",
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
     elif cfg.get("kernel") == "epan":

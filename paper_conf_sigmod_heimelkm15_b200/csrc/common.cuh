@@ -12,7 +12,7 @@
 namespace kde {
 
 constexpr int kMaxDim = KDE_MAX_DIM;
-constexpr int kColAlign = 1024;  // columns padded to a multiple of this many points
+constexpr int kColAlign = 2048;  // columns padded to a multiple of this many points (>= the single-scan TMA tile)
 
 // Per-dimension constants derived from the fp64 bandwidth h (device resident
 // so that an on-device bandwidth update needs no host round trip).

@@ -410,7 +410,8 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
   CUB(cudaMalloc(&m->cret, sizeof(float) * (size_t)m->ld));
   CUB(cudaMalloc(&m->consts, sizeof(DevConsts)));
   CUB(cudaMalloc(&m->online, sizeof(OnlineState)));
-  CUB(cudaMalloc(&m->block_partials, sizeof(double) * (size_t)m->num_sms * 4 * (kMaxDim + 1)));
+  // single-scan grids are at most 8 CTAs per SM (scan_single_grid)
+  CUB(cudaMalloc(&m->block_partials, sizeof(double) * (size_t)m->num_sms * 8 * (kMaxDim + 1)));
   CUB(cudaMalloc(&m->counter, sizeof(unsigned)));
   CUB(cudaMalloc(&m->ret, sizeof(double) * (kMaxDim + 1)));
   CUB(cudaMalloc(&m->single_sums, sizeof(double) * (kMaxDim + 1)));

@@ -5,12 +5,14 @@
 // eq. (17):  d D_j / d h_j = (z_l e^{-z_l^2} - z_u e^{-z_u^2}) / (sqrt(pi) h_j)
 //
 // erf is evaluated through erfc with the exponential factored out,
-//     1/2 erf(|z|) = 1/2 - 1/2 erfc(|z|),   erfc(x) ~= e^{-x^2} t Q(t),  t = 1/(1 + P x),
-// with Q fitted by tools/fit_phi.py (phi_coeffs.h, relative error < 6e-7 in
-// fp32 over [0, inf)).  e^{-z^2} is ONE MUFU.EX2 per bound and is shared with
-// the gradient, so a bound costs 2 MUFU (EX2, RCP) plus ~8 packed FFMA2.
-// The (u, l) pair of a dimension is processed as one float2 with the
-// sm_100 packed FP32 instructions (FADD2/FMUL2/FFMA2), halving issue slots.
+//     1/2 erf(|z|) = 1/2 - 1/2 erfc(|z|),   erfc(x) ~= e^{-x^2} Q(t),  t = 1/(1 + P x),
+// with Q a degree-6 polynomial fitted by tools/fit_phi.py (phi_coeffs.h: relative
+// error < 7.7e-7 in fp32 on [0, 4.5], absolute error < 1e-15 beyond).
+// e^{-z^2} is ONE MUFU.EX2 per bound and is shared with the gradient; the two
+// reciprocals of a dimension share ONE MUFU.RCP, so a dimension costs 3 MUFU
+// plus ~12 packed FP32 instructions.  The (u, l) pair of a dimension is
+// processed as one float2 with the sm_100 packed FP32 instructions
+// (FADD2/FMUL2/FFMA2), halving issue slots.
 //
 // Scaling: the kernels carry y' = z sqrt(log2 e) = (b - t) * ap, so that
 // E = e^{-z^2} = 2^{-y'^2} is a bare ex2.approx; x = |z| = |y'| / sqrt(log2 e)
@@ -26,12 +28,8 @@
 namespace kde {
 
 constexpr float kSqrtLog2e = 1.2011224087864498f;  // sqrt(log2(e))
-constexpr float kYClamp = 13.0f;
 constexpr float kPprime = KDE_PHI_P / kSqrtLog2e;
 
-#ifndef KDE_SHARED_RCP
-#define KDE_SHARED_RCP 0  // 1: one MUFU.RCP per (u, l) pair (+2 FP32 ops); see tools/tune_batched.cu
-#endif
 
 __device__ __forceinline__ float ex2_approx(float x) {
   float y;
@@ -86,6 +84,12 @@ __device__ __forceinline__ BoxDim make_boxdim(float l, float u, float ap, unsign
   if (dy > 0.0f && dy < kNarrowY) {
     r.b = make_float2(l, l);
     r.hd = 0.5f * dy;
+  } else if (!(dy > 0.0f)) {
+    // l == u (or an empty (inf, inf) / (-inf, -inf) box): D = 0 and dD/dh = 0 exactly.  Both bounds
+    // go above the range so y' >= 14 for every point (E = 0, same signs), instead of relying on
+    // the fused bracket cancelling two equal rounded products.
+    r.b = make_float2(tmax + m, tmax + m);
+    r.hd = 0.0f;
   } else {
     r.b = make_float2(u, l);
     r.hd = 0.0f;
@@ -93,32 +97,28 @@ __device__ __forceinline__ BoxDim make_boxdim(float l, float u, float ap, unsign
   return r;
 }
 
-// erf-difference path: D = 1/2 [erf(z_u) - erf(z_l)], w = y'_l E_l - y'_u E_u
+// erf-difference path: D = 1/2 [erf(z_u) - erf(z_l)], w = y'_l E_l - y'_u E_u.
+// One MUFU.RCP serves the pair: t_u = den_l / (den_u den_l), t_l = den_u / (den_u den_l)
+// (den = 1 + P'|y'| with |y'| bounded by the clamped bounds: the product stays finite for any
+// sample whose column range is below ~1e18 bandwidths).
 template <bool GRAD>
 __device__ __forceinline__ float phi_normal(const float2 y, const float2 E, float& w) {
-  const float2 den = __ffma2_rn(make_float2(fabsf(y.x), fabsf(y.y)), f2(kPprime), f2(1.0f));
-#if KDE_SHARED_RCP
-  // one MUFU.RCP for the pair: t_u = den_l / (den_u den_l), t_l = den_u / (den_u den_l)
+  const float2 den = __ffma2_rn(make_float2(fabsf(y.x), fabsf(y.y)), f2(kPprime), f2(1.0f));  // |.| is an operand modifier
   const float r = rcp_approx(den.x * den.y);
   const float2 t2 = __fmul2_rn(make_float2(den.y, den.x), f2(r));
-#else
-  const float2 t2 = make_float2(rcp_approx(den.x), rcp_approx(den.y));
-#endif
   // Horner for Q(t)/2 (the 1/2 of eq. 13 folded into the coefficients)
   float2 q = f2(0.5f * kde_phi_q(KDE_PHI_DEG));
 #pragma unroll
   for (int k = KDE_PHI_DEG - 1; k >= 0; --k) q = __ffma2_rn(q, t2, f2(0.5f * kde_phi_q(k)));
-  const float2 ch = __fmul2_rn(__fmul2_rn(q, t2), E);          // 1/2 erfc(|z|)
-  if (GRAD) w = fmaf(y.y, E.y, -(y.x * E.x));                  // FMUL + FFMA: 2 FMA-pipe cycles
-  // 1/2 erf(z) = sgn(z) (1/2 - ch).  D = [1/2 sgn(z_u) - 1/2 sgn(z_l)] + [sgn(z_l) ch_l - sgn(z_u) ch_u]:
-  // the first bracket is exactly 0 or 1, so a box seen from one side keeps the
-  // full relative accuracy of the erfc tails (no 1/2 - ch rounding).  It is 1
-  // iff z_l < 0 <= z_u (z_u >= z_l always) and is built from the sign bits on
-  // the integer (ALU) pipe, leaving the FMA pipe -- the binding one -- alone.
+  if (GRAD) w = fmaf(y.y, E.y, -(y.x * E.x));  // FMUL + FFMA
+  // 1/2 erf(z) = sgn(z) (1/2 - ch), ch = 1/2 erfc(|z|) = E q.  D = [1/2 sgn(z_u) - 1/2 sgn(z_l)] +
+  // [sgn(z_l) ch_l - sgn(z_u) ch_u]: the first bracket is exactly 0 or 1, so a box seen from one side
+  // keeps the full relative accuracy of the erfc tails.  It is 1 iff z_l < 0 <= z_u (z_u >= z_l
+  // always) and is built from the sign bits on the integer (ALU) pipe; the signs of the second
+  // bracket ride on E (copysign, ALU) and the bracket is two FFMAs with the first as addend.
   const unsigned lneg_upos = __float_as_uint(y.y) & ~__float_as_uint(y.x);
   const float hs = __uint_as_float((unsigned)((int)lneg_upos >> 31) & 0x3f800000u);
-  const float cs = copysignf(ch.y, y.y) - copysignf(ch.x, y.x);
-  return hs + cs;
+  return fmaf(q.y, copysignf(E.y, y.y), fmaf(-q.x, copysignf(E.x, y.x), hs));
 }
 
 // narrow path: 2-point Gauss-Legendre on [y_l, y_u] (nodes y.x, y.y, weights hd)
@@ -166,6 +166,78 @@ __device__ __forceinline__ float phi_diff(const BoxDim& bd, float t, float ap, f
   const float2 E = make_float2(ex2_approx(-yy.x), ex2_approx(-yy.y));
   if (GENERAL && bd.hd > 0.0f) return phi_narrow<GRAD>(y, E, bd.hd, w);
   return phi_normal<GRAD>(y, E, w);
+}
+
+// ---------------------------------------------------------------------------
+// Two points (p0, p1) against one box dimension, the float2 lanes being the
+// two POINTS: every FP32 step of phi_normal -- including the ones that are
+// scalar per point there (the pair reciprocal's product, the bracket FFMAs,
+// the gradient term, the product over dimensions) -- is one packed
+// FADD2/FMUL2/FFMA2 for both points.  The kernels carry the negated
+// coordinate  yn = (t - b) ap = -y'  (t first: FADD2 with a broadcast bound,
+// no negation), so in yn terms
+//   D = [1/2 sgn(yn_l) - 1/2 sgn(yn_u)] + [sgn(yn_u) ch_u - sgn(yn_l) ch_l],
+//   w = y'_l E_l - y'_u E_u = yn_u E_u - yn_l E_l,
+// and the 0/1 bracket is 1 iff yn_u < 0 <= yn_l (sign bits, ALU pipe).
+__device__ __forceinline__ float2 ex2_2(const float2 yy) {
+  return make_float2(ex2_approx(-yy.x), ex2_approx(-yy.y));
+}
+__device__ __forceinline__ float hs_bit(float yn_u, float yn_l) {
+  const unsigned m = __float_as_uint(yn_u) & ~__float_as_uint(yn_l);
+  return __uint_as_float((unsigned)((int)m >> 31) & 0x3f800000u);
+}
+
+template <bool GRAD>
+__device__ __forceinline__ float2 phi_normal2(const float2 yu, const float2 yl, const float2 Eu, const float2 El,
+                                              float2& w) {
+  const float2 du = __ffma2_rn(make_float2(fabsf(yu.x), fabsf(yu.y)), f2(kPprime), f2(1.0f));
+  const float2 dl = __ffma2_rn(make_float2(fabsf(yl.x), fabsf(yl.y)), f2(kPprime), f2(1.0f));
+  const float2 pr = __fmul2_rn(du, dl);
+  const float2 r = make_float2(rcp_approx(pr.x), rcp_approx(pr.y));  // one MUFU.RCP per point and dimension
+  const float2 tu = __fmul2_rn(dl, r), tl = __fmul2_rn(du, r);
+  float2 qu = f2(0.5f * kde_phi_q(KDE_PHI_DEG)), ql = qu;
+#pragma unroll
+  for (int k = KDE_PHI_DEG - 1; k >= 0; --k) {
+    qu = __ffma2_rn(qu, tu, f2(0.5f * kde_phi_q(k)));
+    ql = __ffma2_rn(ql, tl, f2(0.5f * kde_phi_q(k)));
+  }
+  if (GRAD) {
+    const float2 m = __fmul2_rn(yl, El);
+    w = __ffma2_rn(yu, Eu, make_float2(-m.x, -m.y));
+  }
+  const float2 hs = make_float2(hs_bit(yu.x, yl.x), hs_bit(yu.y, yl.y));
+  const float2 Eus = make_float2(copysignf(Eu.x, yu.x), copysignf(Eu.y, yu.y));
+  const float2 Els = make_float2(copysignf(El.x, yl.x), copysignf(El.y, yl.y));
+  return __ffma2_rn(qu, Eus, __ffma2_rn(make_float2(-ql.x, -ql.y), Els, hs));
+}
+
+// narrow path for two points: nodes yn_1,2 = (t - l) ap - hd (1 +- 1/sqrt3) (weights hd)
+template <bool GRAD>
+__device__ __forceinline__ float2 phi_narrow2(const float2 y1, const float2 y2, const float2 E1, const float2 E2,
+                                              float hd, float2& w) {
+  const float2 s = __fadd2_rn(E1, E2);
+  if (GRAD) {
+    const float2 yy1 = __fmul2_rn(y1, y1), yy2 = __fmul2_rn(y2, y2);
+    const float2 m = __ffma2_rn(E1, yy1, __fmul2_rn(E2, yy2));
+    w = __fmul2_rn(f2(-hd), __ffma2_rn(f2(-kTwoLn2), m, s));
+  }
+  return __fmul2_rn(f2(hd * kInvSqrtPiLog2e), s);
+}
+
+template <bool GRAD, bool GENERAL>
+__device__ __forceinline__ float2 phi_diff2(const BoxDim& bd, const float2 t, float ap, float2& w) {
+  float2 yu, yl;
+  if (GENERAL) {  // narrow boxes have b = (l, l); a normal box has hd = 0 and the offsets vanish
+    const float2 tu = __fadd2_rn(t, f2(-bd.b.x)), tl = __fadd2_rn(t, f2(-bd.b.y));
+    yu = __ffma2_rn(tu, f2(ap), f2(-bd.hd * (1.0f + kGaussC)));
+    yl = __ffma2_rn(tl, f2(ap), f2(-bd.hd * (1.0f - kGaussC)));
+  } else {
+    yu = __fmul2_rn(__fadd2_rn(t, f2(-bd.b.x)), f2(ap));
+    yl = __fmul2_rn(__fadd2_rn(t, f2(-bd.b.y)), f2(ap));
+  }
+  const float2 Eu = ex2_2(__fmul2_rn(yu, yu)), El = ex2_2(__fmul2_rn(yl, yl));
+  if (GENERAL && bd.hd > 0.0f) return phi_narrow2<GRAD>(yu, yl, Eu, El, bd.hd, w);
+  return phi_normal2<GRAD>(yu, yl, Eu, El, w);
 }
 
 }  // namespace kde

@@ -31,14 +31,45 @@ template <int D>
 struct QT_for {
   static constexpr int value = 1;
 };
+// (KDE_TUNE_* macros override the measured defaults for tuning builds: tools/kbench.cu)
 template <int D>
-struct PU_for {  // points per inner iteration
-  static constexpr int value = (D <= 3 || (D >= 7 && D <= 8)) ? 2 : 1;
+struct PU_for {  // point pairs per inner iteration
+#ifdef KDE_TUNE_PU
+  static constexpr int value = KDE_TUNE_PU;
+#else
+  static constexpr int value = 2;
+#endif
 };
 template <int D>
 struct MINB_for {
+#ifdef KDE_TUNE_MINB
+  static constexpr int value = KDE_TUNE_MINB;
+#else
   static constexpr int value = D <= 6 ? 4 : (D <= 12 ? 2 : 1);
+#endif
 };
+// single-box TMA scan: points per tile, tiles in flight, resident CTAs per SM
+// (measured on B200 with tools/kbench.cu, profiles/r01_tune_single_ws.jsonl:
+// 2048-point tiles; 2 stages x 2 CTAs up to d = 5, 3 stages x 1 CTA above)
+#ifndef KDE_TUNE_SINGLE_TILE
+#define KDE_TUNE_SINGLE_TILE 2048
+#endif
+constexpr int kSingleTile = KDE_TUNE_SINGLE_TILE;
+static_assert(kColAlign % kSingleTile == 0, "TMA tiles of the single-box scan must not cross the padded column end");
+__host__ __device__ constexpr int single_stages(int d) {
+#ifdef KDE_TUNE_SINGLE_STAGES
+  return (void)d, KDE_TUNE_SINGLE_STAGES;
+#else
+  return d <= 5 ? 2 : 3;
+#endif
+}
+__host__ __device__ constexpr int single_tma_occ(int d) {
+#ifdef KDE_TUNE_SINGLE_OCC
+  return (void)d, KDE_TUNE_SINGLE_OCC;
+#else
+  return d <= 5 ? 2 : 1;
+#endif
+}
 
 constexpr int kSingleThreads = 256;
 constexpr int kBatchedThreads = 256;
@@ -48,7 +79,10 @@ constexpr int kSingleFlushPts = 16;  // single-box scan: fp32 partials flushed e
 
 // resident 256-thread CTAs per SM for the single-box scan (register budget)
 // (measured on B200 by tools/tune_single.cu, profiles/r01_tune_single*.jsonl)
-__host__ __device__ constexpr bool single_uses_tma(int d) { return d <= 8; }
+#ifndef KDE_TUNE_SINGLE_TMA_MAXD
+#define KDE_TUNE_SINGLE_TMA_MAXD 8
+#endif
+__host__ __device__ constexpr bool single_uses_tma(int d) { return d <= KDE_TUNE_SINGLE_TMA_MAXD; }
 __host__ __device__ constexpr int single_occ(int d, bool grad) {
   return grad ? (d <= 3 ? 4 : (d <= 10 ? 3 : 1)) : (d <= 10 ? 4 : (d <= 14 ? 2 : 1));
 }
@@ -86,6 +120,39 @@ __device__ __forceinline__ float point_box(const BoxDim (&bd)[D], const float (&
   return c;
 }
 
+// point_box for two points at once (float2 lanes = points, see phi_diff2):
+// s2[k] holds per-lane fp32 partial sums; `valid` is 1 or 0 per point and
+// enters as the first factor of the product, so a padding point contributes
+// exactly 0 to every sum.  Returns (p^(i0), p^(i1)).
+template <int D, bool GRAD, int MODE>
+__device__ __forceinline__ float2 point_box2(const BoxDim (&bd)[D], const float2 (&t)[D], const float (&ap)[D],
+                                             float2* s2, const float2 valid) {
+  float2 Dv[D], wv[D];
+#pragma unroll
+  for (int j = 0; j < D; ++j) {
+    if (MODE == 2) {
+      Dv[j].x = phi_epan<GRAD>(bd[j], t[j].x, ap[j], wv[j].x);
+      Dv[j].y = phi_epan<GRAD>(bd[j], t[j].y, ap[j], wv[j].y);
+    } else {
+      Dv[j] = phi_diff2<GRAD, MODE == 1>(bd[j], t[j], ap[j], wv[j]);
+    }
+  }
+  float2 pre[D + 1];
+  pre[0] = valid;
+#pragma unroll
+  for (int j = 0; j < D; ++j) pre[j + 1] = __fmul2_rn(pre[j], Dv[j]);
+  s2[0] = __fadd2_rn(s2[0], pre[D]);
+  if (GRAD) {
+    float2 suf = f2(1.0f);
+#pragma unroll
+    for (int j = D - 1; j >= 0; --j) {
+      s2[1 + j] = __ffma2_rn(wv[j], j == D - 1 ? pre[j] : __fmul2_rn(pre[j], suf), s2[1 + j]);
+      if (j > 0) suf = j == D - 1 ? Dv[j] : __fmul2_rn(suf, Dv[j]);
+    }
+  }
+  return pre[D];
+}
+
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
@@ -95,9 +162,9 @@ __device__ __forceinline__ double warp_sum(double v) {
 // Block reduction of the per-thread fp64 sums (fixed order), one fp64 partial
 // per block, and a deterministic second pass by the last block to finish
 // (fixed strided order + fixed tree) that also finalises p_hat, dp_hat/dh.
-template <int NA>
+template <int NA, int NT = kSingleThreads>
 __device__ __forceinline__ void single_reduce_finalize(const ScanSingleArgs& a, const double (&acc)[NA]) {
-  __shared__ double red[kSingleThreads / 32][NA];
+  __shared__ double red[NT / 32][NA];
   __shared__ bool am_last;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
 #pragma unroll
@@ -109,7 +176,7 @@ __device__ __forceinline__ void single_reduce_finalize(const ScanSingleArgs& a, 
   if (threadIdx.x < NA) {
     double t = 0.0;
 #pragma unroll
-    for (int w = 0; w < kSingleThreads / 32; ++w) t += red[w][threadIdx.x];
+    for (int w = 0; w < NT / 32; ++w) t += red[w][threadIdx.x];
     a.block_partials[(int64_t)blockIdx.x * NA + threadIdx.x] = t;
     __threadfence();
   }
@@ -121,7 +188,7 @@ __device__ __forceinline__ void single_reduce_finalize(const ScanSingleArgs& a, 
   // deterministic second pass over the block partials (fixed strided order + fixed tree)
   for (int k = 0; k < NA; ++k) {
     double t = 0.0;
-    for (int b = threadIdx.x; b < (int)gridDim.x; b += kSingleThreads) t += __ldcg(a.block_partials + (int64_t)b * NA + k);
+    for (int b = threadIdx.x; b < (int)gridDim.x; b += NT) t += __ldcg(a.block_partials + (int64_t)b * NA + k);
     t = warp_sum(t);
     __syncthreads();
     if (lane == 0) red[warp][0] = t;
@@ -129,7 +196,7 @@ __device__ __forceinline__ void single_reduce_finalize(const ScanSingleArgs& a, 
     if (threadIdx.x == 0) {
       double tot = 0.0;
 #pragma unroll
-      for (int w = 0; w < kSingleThreads / 32; ++w) tot += red[w][0];
+      for (int w = 0; w < NT / 32; ++w) tot += red[w][0];
       a.sums_out[k] = tot;
       const double fin = k == 0 ? tot / a.n_global : tot * a.consts->gconst[k - 1] / a.n_global;
       if (a.fin_out) a.fin_out[k] = fin;
@@ -147,11 +214,19 @@ __device__ __forceinline__ void single_reduce_finalize(const ScanSingleArgs& a, 
 // vector loads, coalesced across the warp).
 template <int D, bool GRAD>
 struct SingleVW {
+#ifdef KDE_TUNE_SINGLE_VW
+  static constexpr int value = KDE_TUNE_SINGLE_VW;
+#else
   static constexpr int value = 2;
+#endif
 };
 template <int D, bool GRAD>
 struct SinglePF {  // register double-buffered prefetch: spills, measured slower (tools/tune_single.cu)
+#ifdef KDE_TUNE_SINGLE_PF
+  static constexpr bool value = KDE_TUNE_SINGLE_PF;
+#else
   static constexpr bool value = false;
+#endif
 };
 
 template <int VW>
@@ -181,21 +256,27 @@ __device__ __forceinline__ void stcs_v(float4* p, const float* c) { __stcs(p, ma
 
 template <int D, bool GRAD, int MODE, int VW>
 __device__ __forceinline__ void single_group(const typename VecT<VW>::type (&tv)[D], const float4* __restrict__ smc,
-                                             float* s, float* c_out, int64_t v, int valid) {
+                                             float2* s2, float* c_out, int64_t v, int valid) {
+  static_assert(VW == 2 || VW == 4, "points are processed in pairs");
+  BoxDim bd[D];
+  float ap[D];
+#pragma unroll
+  for (int j = 0; j < D; ++j) {
+    const float4 c = smc[j];
+    bd[j].b = make_float2(c.x, c.y);
+    bd[j].hd = c.z;
+    ap[j] = c.w;
+  }
   float cs[VW];
 #pragma unroll
-  for (int p = 0; p < VW; ++p) {
-    BoxDim bd[D];
-    float ap[D], t[D];
+  for (int p = 0; p < VW; p += 2) {
+    float2 t[D];
 #pragma unroll
-    for (int j = 0; j < D; ++j) {
-      const float4 c = smc[j];
-      bd[j].b = make_float2(c.x, c.y);
-      bd[j].hd = c.z;
-      ap[j] = c.w;
-      t[j] = vcomp(tv[j], p);
-    }
-    cs[p] = point_box<D, GRAD, MODE>(bd, t, ap, s, p < valid);
+    for (int j = 0; j < D; ++j) t[j] = make_float2(vcomp(tv[j], p), vcomp(tv[j], p + 1));
+    const float2 c = point_box2<D, GRAD, MODE>(bd, t, ap, s2,
+                                               make_float2(p < valid ? 1.0f : 0.0f, p + 1 < valid ? 1.0f : 0.0f));
+    cs[p] = c.x;
+    cs[p + 1] = c.y;
   }
   if (c_out) stcs_v(reinterpret_cast<typename VecT<VW>::type*>(c_out) + v, cs);
 }
@@ -254,9 +335,9 @@ __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const 
       for (int j = 0; j < D; ++j) cur[j] = ldcs_v(col + j * ldv + v);
     }
     while (v < nfull) {
-      float s[NA];
+      float2 s[NA];
 #pragma unroll
-      for (int k = 0; k < NA; ++k) s[k] = 0.0f;
+      for (int k = 0; k < NA; ++k) s[k] = f2(0.0f);
 #pragma unroll 1
       for (int u = 0; u < kGroups && v < nfull; u += 2) {
         int64_t vn = v + stride;
@@ -276,13 +357,13 @@ __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const 
         v = vn;
       }
 #pragma unroll
-      for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
+      for (int k = 0; k < NA; ++k) acc[k] += (double)s[k].x + (double)s[k].y;
     }
   } else {
     while (v < nfull) {
-      float s[NA];
+      float2 s[NA];
 #pragma unroll
-      for (int k = 0; k < NA; ++k) s[k] = 0.0f;
+      for (int k = 0; k < NA; ++k) s[k] = f2(0.0f);
 #pragma unroll 1
       for (int u = 0; u < kGroups && v < nfull; ++u, v += stride) {
         V t0[D];
@@ -291,7 +372,7 @@ __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const 
         single_group<D, GRAD, MODE, VW>(t0, smc, s, a.c_out, v, VW);
       }
 #pragma unroll
-      for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
+      for (int k = 0; k < NA; ++k) acc[k] += (double)s[k].x + (double)s[k].y;
     }
   }
   // the ragged tail group (n % VW points) belongs to the thread that reaches v == nfull
@@ -300,12 +381,12 @@ __device__ __forceinline__ void scan_single_body(const ScanSingleArgs& a, const 
     V t0[D];
 #pragma unroll
     for (int j = 0; j < D; ++j) t0[j] = ldcs_v(col + j * ldv + v);
-    float s[NA];
+    float2 s[NA];
 #pragma unroll
-    for (int k = 0; k < NA; ++k) s[k] = 0.0f;
+    for (int k = 0; k < NA; ++k) s[k] = f2(0.0f);
     single_group<D, GRAD, MODE, VW>(t0, smc, s, a.c_out, v, valid);
 #pragma unroll
-    for (int k = 0; k < NA; ++k) acc[k] += (double)s[k];
+    for (int k = 0; k < NA; ++k) acc[k] += (double)s[k].x + (double)s[k].y;
   }
 
   single_reduce_finalize<NA>(a, acc);
@@ -320,6 +401,9 @@ __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
 }
 __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 __device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity) {
   asm volatile(
@@ -338,46 +422,51 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
 }
 
 // Accumulate every point of one shared-memory tile against the thread's QT
-// boxes.  No barriers inside, so the GENERAL (narrow-dimension) and fast
-// variants can be chosen per warp.
+// boxes.  The thread takes point PAIRS (2pp, 2pp + 1), pp = phase, phase + R,
+// ... (one LDS.64 per column and pair; see point_box2).  No barriers inside,
+// so the GENERAL (narrow-dimension) and fast variants can be chosen per warp.
 template <int D, bool GRAD, int MODE, int QT, int PU>
 __device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, int phase, int R, double* accsh,
                                                      const BoxDim (&bd)[QT][D], const float (&ap)[D]) {
   constexpr int NA = GRAD ? D + 1 : 1;
+  constexpr int kFlushPairs = kFlushPts / 2;
   const int tid = threadIdx.x;
-  // this thread's points of the tile: phase, phase + R, phase + 2R, ...
-  const int mine = npts > phase ? (npts - phase + R - 1) / R : 0;
-  for (int m0 = 0; m0 < mine; m0 += kFlushPts) {
-    const int me = min(m0 + kFlushPts, mine);
-    float s[QT][NA];
+  const int npairs = (npts + 1) >> 1;
+  const int mine = npairs > phase ? (npairs - phase + R - 1) / R : 0;
+  for (int m0 = 0; m0 < mine; m0 += kFlushPairs) {
+    const int me = min(m0 + kFlushPairs, mine);
+    float2 s[QT][NA];
 #pragma unroll
     for (int qq = 0; qq < QT; ++qq)
 #pragma unroll
-      for (int kk = 0; kk < NA; ++kk) s[qq][kk] = 0.0f;
+      for (int kk = 0; kk < NA; ++kk) s[qq][kk] = f2(0.0f);
     int m = m0;
-    for (; m + PU <= me; m += PU) {  // PU points per iteration: more independent chains per warp
+    for (; m + PU <= me; m += PU) {  // PU pairs per iteration: more independent chains per warp
 #pragma unroll
       for (int u = 0; u < PU; ++u) {
-        const int p = phase + (m + u) * R;
-        float t[D];
+        const int pp = phase + (m + u) * R;
+        float2 t[D];
 #pragma unroll
-        for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
+        for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * kTilePts + 2 * pp);
+        const float2 valid = make_float2(1.0f, 2 * pp + 1 < npts ? 1.0f : 0.0f);
 #pragma unroll
-        for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, MODE>(bd[qq], t, ap, s[qq], true);
+        for (int qq = 0; qq < QT; ++qq) point_box2<D, GRAD, MODE>(bd[qq], t, ap, s[qq], valid);
       }
     }
     for (; m < me; ++m) {
-      const int p = phase + m * R;
-      float t[D];
+      const int pp = phase + m * R;
+      float2 t[D];
 #pragma unroll
-      for (int j = 0; j < D; ++j) t[j] = tl[j * kTilePts + p];
+      for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * kTilePts + 2 * pp);
+      const float2 valid = make_float2(1.0f, 2 * pp + 1 < npts ? 1.0f : 0.0f);
 #pragma unroll
-      for (int qq = 0; qq < QT; ++qq) point_box<D, GRAD, MODE>(bd[qq], t, ap, s[qq], true);
+      for (int qq = 0; qq < QT; ++qq) point_box2<D, GRAD, MODE>(bd[qq], t, ap, s[qq], valid);
     }
 #pragma unroll
     for (int qq = 0; qq < QT; ++qq)
 #pragma unroll
-      for (int kk = 0; kk < NA; ++kk) accsh[(qq * NA + kk) * kBatchedThreads + tid] += (double)s[qq][kk];
+      for (int kk = 0; kk < NA; ++kk)
+        accsh[(qq * NA + kk) * kBatchedThreads + tid] += (double)s[qq][kk].x + (double)s[qq][kk].y;
   }
 }
 
@@ -551,13 +640,14 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
 template <int D, bool GRAD, int TILE, int STAGES, int OCC>
 cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStream_t s);
 
-// d <= 8: TMA-pipelined variant (1024-point tiles, 3 stages, 2 CTAs/SM);
+// d <= 8: TMA-pipelined, warp-specialised variant (kSingleTile-point tiles, single_stages(d) stages,
+// single_tma_occ(d) CTAs/SM);
 // d > 8: register-streaming variant (measured faster or equal there).
 template <int D>
 cudaError_t launch_single_t(bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s) {
   if (single_uses_tma(D)) {
-    return grad ? launch_single_tma_variant<D, true, 1024, 3, 2>(a, grid, s)
-                : launch_single_tma_variant<D, false, 1024, 3, 2>(a, grid, s);
+    return grad ? launch_single_tma_variant<D, true, kSingleTile, single_stages(D), single_tma_occ(D)>(a, grid, s)
+                : launch_single_tma_variant<D, false, kSingleTile, single_stages(D), single_tma_occ(D)>(a, grid, s);
   }
   if (grad)
     scan_single_kernel<D, true><<<grid, kSingleThreads, 0, s>>>(a);

@@ -34,8 +34,8 @@ cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int 
 // ~3 resident CTAs of 256 threads per SM, never more CTAs than 8-point work items.
 int scan_single_grid(int d, bool grad, int64_t n, int num_sms) {
   if (single_uses_tma(d)) {  // one contiguous chunk of >= 1 tile per CTA
-    int64_t grid = (int64_t)num_sms * 2;
-    const int64_t ntiles = (n + 1023) / 1024;
+    int64_t grid = (int64_t)num_sms * single_tma_occ(d);
+    const int64_t ntiles = (n + kSingleTile - 1) / kSingleTile;
     if (grid > ntiles) grid = ntiles;
     return (int)(grid < 1 ? 1 : grid);
   }

@@ -1,31 +1,44 @@
 // scan_single_tma.cuh -- single-box scan with the sample streamed through
 // shared memory by TMA bulk copies (included at the end of scan.cuh).
 //
-// Each CTA owns a contiguous chunk of the sample and walks it in tiles of
-// TILE points x d columns.  One elected thread keeps STAGES tiles in flight
-// (cp.async.bulk global -> shared, completion on an mbarrier with expect_tx),
-// so HBM requests are decoupled from the registers and latency of the compute
-// warps: the memory system sees STAGES * TILE * 4d bytes outstanding per CTA
-// while every thread computes on its points of the current tile.  A stage is
-// reused after the CTA barrier that ends the tile that read it.
+// Warp-specialised pipeline.  Each CTA owns a contiguous chunk of the sample
+// and walks it in tiles of TILE points x d columns held in a ring of STAGES
+// shared-memory stages.  A ninth (producer) warp keeps the ring full: for each
+// tile it waits until the stage is EMPTY (an mbarrier every compute warp
+// arrives on after its last read), then issues the d cp.async.bulk copies that
+// complete on the stage's FULL mbarrier (expect_tx).  The 8 compute warps only
+// wait on FULL and never on each other -- there is no CTA-wide barrier in the
+// tile loop, so warps drift out of phase and the FMA and MUFU pipes see a
+// mixed instruction stream instead of synchronised bursts.
 #pragma once
 
 namespace kde {
 
+constexpr int kSingleComputeWarps = kSingleThreads / 32;
+constexpr int kSingleTmaThreads = kSingleThreads + 32;  // + producer warp
+
 template <int D, int TILE, int STAGES>
 constexpr size_t single_tma_smem_bytes() {
-  return (size_t)STAGES * D * TILE * sizeof(float) + STAGES * sizeof(uint64_t);
+  return (size_t)STAGES * D * TILE * sizeof(float) + 2 * STAGES * sizeof(uint64_t);
 }
 
 template <int D, bool GRAD, int MODE, int TILE, int STAGES>
 __device__ __forceinline__ void scan_single_tma_body(const ScanSingleArgs& a, const float4* smc, float* tiles,
-                                                     uint64_t* full, int64_t c0, int64_t c1, int ntiles) {
+                                                     uint64_t* full, uint64_t* empty, int64_t c0, int64_t c1,
+                                                     int ntiles, double* acc) {
   constexpr int NA = GRAD ? D + 1 : 1;
   constexpr int PPT = TILE / kSingleThreads;  // points per thread per tile
+  static_assert(PPT % 2 == 0, "points are processed in pairs");
   const int tid = threadIdx.x;
-  double acc[NA];
+  BoxDim bd[D];
+  float ap[D];
 #pragma unroll
-  for (int k = 0; k < NA; ++k) acc[k] = 0.0;
+  for (int j = 0; j < D; ++j) {
+    const float4 c = smc[j];
+    bd[j].b = make_float2(c.x, c.y);
+    bd[j].hd = c.z;
+    ap[j] = c.w;
+  }
   for (int k = 0; k < ntiles; ++k) {
     const int st = k % STAGES;
     mbar_wait_parity(&full[st], (uint32_t)((k / STAGES) & 1));
@@ -33,52 +46,43 @@ __device__ __forceinline__ void scan_single_tma_body(const ScanSingleArgs& a, co
     const int64_t base = c0 + (int64_t)k * TILE;
     const int64_t rem = c1 - base;
     const int npts = rem < TILE ? (int)rem : TILE;
-    float s[NA];
+    float2 s[NA];
 #pragma unroll
-    for (int kk = 0; kk < NA; ++kk) s[kk] = 0.0f;
-    BoxDim bd[D];
-    float ap[D];
+    for (int kk = 0; kk < NA; ++kk) s[kk] = f2(0.0f);
+    // point pairs (2pp, 2pp + 1), pp = tid + r * threads: one LDS.64 per column and pair
 #pragma unroll
-    for (int j = 0; j < D; ++j) {
-      const float4 c = smc[j];
-      bd[j].b = make_float2(c.x, c.y);
-      bd[j].hd = c.z;
-      ap[j] = c.w;
+    for (int r = 0; r < PPT / 2; ++r) {
+      const int pp = tid + r * kSingleThreads;
+      float2 t[D];
+#pragma unroll
+      for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * TILE + 2 * pp);
+      const float2 valid = make_float2(2 * pp < npts ? 1.0f : 0.0f, 2 * pp + 1 < npts ? 1.0f : 0.0f);
+      const float2 c = point_box2<D, GRAD, MODE>(bd, t, ap, s, valid);
+      if (a.c_out) {
+        if (2 * pp + 1 < npts)
+          __stcs(reinterpret_cast<float2*>(a.c_out + base + 2 * pp), c);
+        else if (2 * pp < npts)
+          __stcs(a.c_out + base + 2 * pp, c.x);
+      }
     }
+    __syncwarp();
+    if ((tid & 31) == 0) mbar_arrive(&empty[st]);  // this warp is done reading stage st
 #pragma unroll
-    for (int r = 0; r < PPT; ++r) {
-      const int p = tid + r * kSingleThreads;
-      const bool valid = p < npts;
-      float t[D];
-#pragma unroll
-      for (int j = 0; j < D; ++j) t[j] = tl[j * TILE + p];
-      const float c = point_box<D, GRAD, MODE>(bd, t, ap, s, valid);
-      if (a.c_out && valid) __stcs(a.c_out + base + p, c);
-    }
-#pragma unroll
-    for (int kk = 0; kk < NA; ++kk) acc[kk] += (double)s[kk];
-    __syncthreads();  // every thread is done with stage st
-    if (tid == 0 && k + STAGES < ntiles) {
-      const int64_t nb = c0 + (int64_t)(k + STAGES) * TILE;
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-      mbar_arrive_expect_tx(&full[st], (uint32_t)(D * TILE * sizeof(float)));
-#pragma unroll
-      for (int j = 0; j < D; ++j)
-        bulk_g2s(tiles + ((size_t)st * D + j) * TILE, a.cols + (int64_t)j * a.ld + nb, (uint32_t)(TILE * sizeof(float)),
-                 &full[st]);
-    }
+    for (int kk = 0; kk < NA; ++kk) acc[kk] += (double)s[kk].x + (double)s[kk].y;
   }
-  single_reduce_finalize<NA>(a, acc);
 }
 
 template <int D, bool GRAD, int TILE, int STAGES, int OCC>
-__global__ void __launch_bounds__(kSingleThreads, OCC) scan_single_tma_kernel(const ScanSingleArgs a) {
+__global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel(const ScanSingleArgs a) {
+  constexpr int NA = GRAD ? D + 1 : 1;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   float* tiles = reinterpret_cast<float*>(smem_raw);
   uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + (size_t)STAGES * D * TILE * sizeof(float));
+  uint64_t* empty = full + STAGES;
   __shared__ float4 smc[D];
   __shared__ int narrow_s;
   const int tid = threadIdx.x;
+  const bool producer = tid >= kSingleThreads;
   // contiguous chunk of this CTA, a multiple of TILE points
   const int64_t ntile_total = (a.n + TILE - 1) / TILE;
   const int64_t tiles_per = (ntile_total + gridDim.x - 1) / gridDim.x;
@@ -87,20 +91,13 @@ __global__ void __launch_bounds__(kSingleThreads, OCC) scan_single_tma_kernel(co
   const int ntiles = c1 > c0 ? (int)((c1 - c0 + TILE - 1) / TILE) : 0;
   if (tid == 0) {
     narrow_s = 0;
-    for (int st = 0; st < STAGES; ++st) mbar_init(&full[st], 1);
+    for (int st = 0; st < STAGES; ++st) {
+      mbar_init(&full[st], 1);
+      mbar_init(&empty[st], kSingleComputeWarps);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
-  if (tid == 0) {
-    for (int k = 0; k < STAGES && k < ntiles; ++k) {
-      const int64_t nb = c0 + (int64_t)k * TILE;
-      mbar_arrive_expect_tx(&full[k], (uint32_t)(D * TILE * sizeof(float)));
-#pragma unroll
-      for (int j = 0; j < D; ++j)
-        bulk_g2s(tiles + ((size_t)k * D + j) * TILE, a.cols + (int64_t)j * a.ld + nb, (uint32_t)(TILE * sizeof(float)),
-                 &full[k]);
-    }
-  }
   if (tid < D) {
     const int j = tid;
     const float ap = a.consts->ap[j];
@@ -113,12 +110,30 @@ __global__ void __launch_bounds__(kSingleThreads, OCC) scan_single_tma_kernel(co
     if (!epan && bd.hd > 0.0f) atomicOr(&narrow_s, 1);
   }
   __syncthreads();
-  if (a.consts->kernel == kEpanechnikov)
-    scan_single_tma_body<D, GRAD, 2, TILE, STAGES>(a, smc, tiles, full, c0, c1, ntiles);
-  else if (narrow_s)
-    scan_single_tma_body<D, GRAD, 1, TILE, STAGES>(a, smc, tiles, full, c0, c1, ntiles);
-  else
-    scan_single_tma_body<D, GRAD, 0, TILE, STAGES>(a, smc, tiles, full, c0, c1, ntiles);
+  double acc[NA];
+#pragma unroll
+  for (int k = 0; k < NA; ++k) acc[k] = 0.0;
+  if (producer) {
+    if (tid == kSingleThreads) {
+      for (int k = 0; k < ntiles; ++k) {
+        const int st = k % STAGES;
+        if (k >= STAGES) mbar_wait_parity(&empty[st], (uint32_t)((k / STAGES - 1) & 1));
+        const int64_t nb = c0 + (int64_t)k * TILE;
+        mbar_arrive_expect_tx(&full[st], (uint32_t)(D * TILE * sizeof(float)));
+#pragma unroll
+        for (int j = 0; j < D; ++j)
+          bulk_g2s(tiles + ((size_t)st * D + j) * TILE, a.cols + (int64_t)j * a.ld + nb,
+                   (uint32_t)(TILE * sizeof(float)), &full[st]);
+      }
+    }
+  } else if (a.consts->kernel == kEpanechnikov) {
+    scan_single_tma_body<D, GRAD, 2, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
+  } else if (narrow_s) {
+    scan_single_tma_body<D, GRAD, 1, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
+  } else {
+    scan_single_tma_body<D, GRAD, 0, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
+  }
+  single_reduce_finalize<NA, kSingleTmaThreads>(a, acc);
 }
 
 template <int D, bool GRAD, int TILE, int STAGES, int OCC>
@@ -131,7 +146,7 @@ cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStr
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC><<<grid, kSingleThreads, smem, s>>>(a);
+  scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC><<<grid, kSingleTmaThreads, smem, s>>>(a);
   return cudaGetLastError();
 }
 
