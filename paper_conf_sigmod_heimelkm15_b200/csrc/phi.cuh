@@ -224,6 +224,26 @@ __device__ __forceinline__ float2 phi_narrow2(const float2 y1, const float2 y2, 
   return __fmul2_rn(f2(hd * kInvSqrtPiLog2e), s);
 }
 
+// Epanechnikov (reading R14) for two points, float2 lanes = points.  In the
+// negated coordinates a = (t - u)/h <= b = (t - l)/h (clamped to [-1, 1]) the
+// formulas of phi_epan are unchanged: Delta = b - a, S = a^2 + a b + b^2,
+// D = Delta (3 - S)/4, w = Delta (1 - S); Delta is the cancellation-free
+// (u - l)/h (bd.hd) when neither bound is clamped.
+template <bool GRAD>
+__device__ __forceinline__ float2 phi_epan2(const BoxDim& bd, const float2 t, float ih, float2& w) {
+  const float2 va = __fmul2_rn(__fadd2_rn(t, f2(-bd.b.x)), f2(ih));
+  const float2 vb = __fmul2_rn(__fadd2_rn(t, f2(-bd.b.y)), f2(ih));
+  const float2 a = make_float2(fminf(fmaxf(va.x, -1.0f), 1.0f), fminf(fmaxf(va.y, -1.0f), 1.0f));
+  const float2 b = make_float2(fminf(fmaxf(vb.x, -1.0f), 1.0f), fminf(fmaxf(vb.y, -1.0f), 1.0f));
+  const float2 dc = __fadd2_rn(b, make_float2(-a.x, -a.y));
+  // both bounds inside the support (|a|, |b| <= 1, unclamped) -> the exact (u - l)/h
+  const float2 dl = make_float2(fmaxf(fabsf(va.x), fabsf(vb.x)) <= 1.0f ? bd.hd : dc.x,
+                                fmaxf(fabsf(va.y), fabsf(vb.y)) <= 1.0f ? bd.hd : dc.y);
+  const float2 S = __ffma2_rn(a, __fadd2_rn(a, b), __fmul2_rn(b, b));
+  if (GRAD) w = __ffma2_rn(make_float2(-S.x, -S.y), dl, dl);
+  return __fmul2_rn(__ffma2_rn(S, f2(-0.25f), f2(0.75f)), dl);
+}
+
 template <bool GRAD, bool GENERAL>
 __device__ __forceinline__ float2 phi_diff2(const BoxDim& bd, const float2 t, float ap, float2& w) {
   float2 yu, yl;

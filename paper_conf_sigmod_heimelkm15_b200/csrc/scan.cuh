@@ -131,8 +131,7 @@ __device__ __forceinline__ float2 point_box2(const BoxDim (&bd)[D], const float2
 #pragma unroll
   for (int j = 0; j < D; ++j) {
     if (MODE == 2) {
-      Dv[j].x = phi_epan<GRAD>(bd[j], t[j].x, ap[j], wv[j].x);
-      Dv[j].y = phi_epan<GRAD>(bd[j], t[j].y, ap[j], wv[j].y);
+      Dv[j] = phi_epan2<GRAD>(bd[j], t[j], ap[j], wv[j]);
     } else {
       Dv[j] = phi_diff2<GRAD, MODE == 1>(bd[j], t[j], ap[j], wv[j]);
     }

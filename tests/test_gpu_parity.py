@@ -144,6 +144,35 @@ def test_small_bandwidth_degrades_to_exact_count():
     assert m.estimate(lo[:1], hi[:1])[0] == cnt[0] / len(S)
 
 
+@pytest.mark.parametrize("kernel", ["gauss", "epan"])
+def test_points_exactly_on_box_faces(kernel):
+    """Integer data and integer box bounds: many points sit exactly on a face (t == l or t == u),
+    where (t - b) a' is +0 and the sign-bit bracket of phi.cuh decides the side; ragged pair tail."""
+    g = synth.rng(61)
+    S = g.integers(-6, 7, size=(30001, 3)).astype(np.float32)
+    h = np.array([0.7, 1.3, 2.1])
+    lo = g.integers(-6, 1, size=(40, 3)).astype(np.float32)
+    hi = (lo + g.integers(0, 7, size=(40, 3))).astype(np.float32)
+    if kernel == "epan":
+        h = h * np.sqrt(5.0)
+    m = model(S, h)
+    if kernel == "epan":
+        m.set_kernel("epan")
+        m.bandwidth = h
+        est_o, g_o = oracle.epan_estimate_grad(S, h, lo, hi)
+        mabs = oracle.epan_grad_abs_scale(S, h, lo, hi)
+    else:
+        est_o, g_o = oracle.estimate_grad(S, h, lo, hi)
+        mabs = oracle.grad_abs_scale(S, h, lo, hi)
+    est, gr = m.estimate(lo, hi, grad=True)
+    sel_ok(est, est_o)
+    grad_ok(gr, g_o, mabs, h)
+    for k in range(0, 40, 7):
+        e1, g1 = m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+        sel_ok(e1, est_o[k:k + 1])
+        grad_ok(g1, g_o[k:k + 1], mabs[k:k + 1], h)
+
+
 def test_large_offset_data():
     """Subtract-then-scale argument formation keeps accuracy for data offset by 1e4."""
     S = (synth.make_data("gauss", 40000, 3, seed=7) + np.float32(1e4)).astype(np.float32)
