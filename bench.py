@@ -258,6 +258,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
         m.set_kernel("epan")
         m.bandwidth = m.bandwidth * np.sqrt(5.0)  # variance-matched to Scott's Gaussian bandwidth
     h = m.bandwidth
+    m.cull = not args.no_cull
 
     stream = torch.cuda.Stream(device=dev)
     d_lo = torch.from_numpy(lo).to(dev)
@@ -431,7 +432,8 @@ def run_cuda(args, cfg, rank, world, local_rank):
         achieved = alg_bytes / (avg_scan_ms * 1e-3) / 1e9
         peak = _measured_hbm()
         roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": _traffic(args.config), "kernel": f"{'scan_single_tma_kernel' if d <= 8 else 'scan_single_kernel'}<{d},{'grad' if cfg.get('grad') else 'est'}>",
+                "traffic": _traffic(args.config), "kernel": (f"scan_single_tma_kernel<{d},{'grad' if cfg.get('grad') else 'est'},cull>" if not args.no_cull else
+                           f"{'scan_single_tma_kernel' if d <= 8 else 'scan_single_kernel'}<{d},{'grad' if cfg.get('grad') else 'est'}>"),
                 "algorithmic": f"4*d bytes/point{' + 4 B/point retained' if cfg.get('retain') else ''} x {n} points per launch",
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
     elif cfg.get("kernel") == "epan":
@@ -469,6 +471,8 @@ def run_cuda(args, cfg, rank, world, local_rank):
         "config": {"workload": cfg["desc"], "d": d, "n_per_gpu": n, "n_global": n_global, "q": q,
                    "l2": "flushed between timed steps" if flush_l2 else "sample larger than L2",
                    "cuda_graph": bool(graphs is not None),
+                   "cull": (None if cfg["path"] == "batched" else
+                            ("off" if args.no_cull else "on: points with contribution provably < 2^-64 skipped")),
                    "clock_sampling": "nvidia-smi every 100 ms over the timed steps"
                                      + (f" + {soak} identical untimed soak steps (timed region < 1 s)" if soak else ""),
                    "accumulation": "fp32 per <=32 points, fp64 above"},
@@ -508,6 +512,8 @@ def main():
     ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="cuda", choices=["cuda", "reference"])
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
+    ap.add_argument("--no-cull", action="store_true",
+                    help="single-box scans evaluate every point (kde_set_cull(0)); default culls provably < 2^-64")
     ap.add_argument("--no-graph", action="store_true", help="stream configs: launch eagerly instead of CUDA graphs")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of all-core oracle work")
     args = ap.parse_args()

@@ -170,6 +170,18 @@ kde_status kde_get_kernel(const kde_model *m, int32_t *kernel);
  * buffer").  Default off. */
 kde_status kde_set_retain(kde_model *m, int32_t on);
 
+/* kde_set_cull / kde_get_cull -- on != 0 (the default): the single-box scan
+ * (q == 1) skips every point whose product of eq. (13) factors is provably
+ * below 2^-64: with o_j the distance of the point OUTSIDE the box in dimension
+ * j in units of sqrt2 h_j / sqrt(log2 e), D_j <= 1/2 erfc(z_j) <= 2^{-o_j^2}, so
+ * sum_j o_j^2 >= 64 bounds its contribution to p_hat by 2^-64 and to each
+ * dp_hat/dh_j by 15 * 2^-64 / (sqrt(pi) sqrt(log2 e) h_j).  A
+ * skipped point's retained p^(i) is 0.  Points inside the box are never
+ * skipped.  on == 0: every point is evaluated.  Errors: none (KDE_EINVAL for
+ * a NULL model). */
+kde_status kde_set_cull(kde_model *m, int32_t on);
+kde_status kde_get_cull(const kde_model *m, int32_t *on);
+
 /* ---------------------------------------------------------------- hot path */
 /* kde_estimate_batch -- selectivity estimates for q boxes, eq. (2)+(13):
  *   est[k]        = p_hat_H(Omega_k) = (1/s) sum_i prod_j [Phi((u_kj - t_ij)/h_j) - Phi((l_kj - t_ij)/h_j)]

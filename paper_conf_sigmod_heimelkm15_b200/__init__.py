@@ -36,7 +36,7 @@ ABI_SYMBOLS = (
     "kde_get_karma", "kde_set_karma", "kde_get_sample", "kde_get_contributions", "kde_get_online_state",
     "kde_set_online_state", "kde_synchronize", "kde_count_in_box_dev", "kde_set_profiling", "kde_get_profile",
     "kde_karma_update_dev", "kde_online_update_dev", "kde_replace_points_dev", "kde_stream_step_dev",
-    "kde_set_kernel", "kde_get_kernel",
+    "kde_set_kernel", "kde_get_kernel", "kde_set_cull", "kde_get_cull",
 )
 
 
@@ -102,6 +102,8 @@ def lib() -> ctypes.CDLL:
         "kde_set_retain": (ctypes.c_int, [P, i32]),
         "kde_set_kernel": (ctypes.c_int, [P, i32]),
         "kde_get_kernel": (ctypes.c_int, [P, P]),
+        "kde_set_cull": (ctypes.c_int, [P, i32]),
+        "kde_get_cull": (ctypes.c_int, [P, P]),
         "kde_estimate_batch": (ctypes.c_int, [P, P, P, i64, P, P]),
         "kde_estimate_batch_dev": (ctypes.c_int, [P, P, P, i64, P, P, P]),
         "kde_loss_and_grad": (ctypes.c_int, [P, P, P, P, i64, i32, f64, i32, P, P, P]),
@@ -223,6 +225,16 @@ def kde_get_kernel(m) -> int:
     k = ctypes.c_int32()
     _check(lib().kde_get_kernel(m, ctypes.byref(k)))
     return k.value
+
+
+def kde_set_cull(m, on: bool):
+    _check(lib().kde_set_cull(m, int(bool(on))))
+
+
+def kde_get_cull(m) -> bool:
+    k = ctypes.c_int32()
+    _check(lib().kde_get_cull(m, ctypes.byref(k)))
+    return bool(k.value)
 
 
 def kde_set_retain(m, on: bool):
@@ -432,6 +444,15 @@ class KDEModel:
 
     def set_retain(self, on=True):
         kde_set_retain(self.handle, on)
+
+    @property
+    def cull(self):
+        """single-box scan skips points whose contribution is provably < 2^-64 (default on)"""
+        return kde_get_cull(self.handle)
+
+    @cull.setter
+    def cull(self, on):
+        kde_set_cull(self.handle, on)
 
     def estimate(self, lo, hi, grad=False):
         return kde_estimate_batch(self.handle, lo, hi, self.d, grad)

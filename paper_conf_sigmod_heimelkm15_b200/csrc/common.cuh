@@ -85,6 +85,7 @@ struct ScanSingleArgs {
   double* est_out;        // nullable: p_hat (caller's buffer), world == 1
   double* dpdh_out;       // nullable: d x dp_hat/dh_j (caller's buffer), world == 1, GRAD only
   double n_global;        // s (results are divided by s, so s ones give exactly 1)
+  int cull;               // 1: skip points whose contribution is provably < 2^-64 (scan_single_tma.cuh)
 };
 
 // scan for many boxes: sample tiles staged in shared memory by TMA bulk
@@ -105,6 +106,6 @@ struct ScanBatchedArgs {
 cudaError_t launch_scan_single(int d, bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s);
 cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int num_sms, int* splits_out,
                                 cudaStream_t s, bool dry_run);
-int scan_single_grid(int d, bool grad, int64_t n, int num_sms);
+int scan_single_grid(int d, bool grad, int64_t n, int num_sms, bool cull);
 
 }  // namespace kde

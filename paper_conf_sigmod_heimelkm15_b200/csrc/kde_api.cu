@@ -80,6 +80,7 @@ struct kde_model {
 
   // retained single-box state
   bool retain = false;
+  bool cull = true;  // kde_set_cull: skip points whose contribution is provably < 2^-64 (single-box scan)
   bool ret_valid = false, ret_has_c = false, ret_has_grad = false;
   float ret_lo[kMaxDim], ret_hi[kMaxDim];
   uint64_t gen = 1;      // bumped whenever h or the sample changes
@@ -245,7 +246,8 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     a.est_out = m->world == 1 ? d_est : nullptr;
     a.dpdh_out = m->world == 1 ? d_dpdh : nullptr;
     a.n_global = (double)m->n_global;
-    const int grid = scan_single_grid(d, grad, m->n, m->num_sms);
+    a.cull = m->cull ? 1 : 0;
+    const int grid = scan_single_grid(d, grad, m->n, m->num_sms, m->cull);
     cudaEvent_t e1 = nullptr, e2 = nullptr;
     kde_status pst = prof_begin(m, s, &e1, &e2);
     if (pst != KDE_OK) return pst;
@@ -578,6 +580,18 @@ extern "C" kde_status kde_get_kernel(const kde_model* m, int32_t* kernel) {
 extern "C" kde_status kde_set_retain(kde_model* m, int32_t on) {
   CHECK_MODEL(m);
   m->retain = on != 0;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_set_cull(kde_model* m, int32_t on) {
+  CHECK_MODEL(m);
+  m->cull = on != 0;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_get_cull(const kde_model* m, int32_t* on) {
+  if (!m || !on) return fail(KDE_EINVAL, "NULL argument");
+  *on = m->cull ? 1 : 0;
   return KDE_OK;
 }
 

@@ -636,17 +636,31 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
 
 // ---------------------------------------------------------------- launchers
 // forward declaration (scan_single_tma.cuh, included below)
-template <int D, bool GRAD, int TILE, int STAGES, int OCC>
+template <int D, bool GRAD, int TILE, int STAGES, int OCC, bool CULL>
 cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStream_t s);
 
+// culled single-box scan (every d): TMA tiles + a per-warp ring of kept points.
+// Two stages; 2048-point tiles up to d = 8 (1024 above, shared-memory budget);
+// two CTAs per SM up to d = 5.
+__host__ __device__ constexpr int cull_tile(int d) { return d <= 8 ? 2048 : 1024; }
+__host__ __device__ constexpr int cull_stages(int d) { return (void)d, 2; }
+__host__ __device__ constexpr int cull_occ(int d) { return d <= 5 ? 2 : 1; }
+
+// cull on: the culled TMA variant;
 // d <= 8: TMA-pipelined, warp-specialised variant (kSingleTile-point tiles, single_stages(d) stages,
 // single_tma_occ(d) CTAs/SM);
 // d > 8: register-streaming variant (measured faster or equal there).
 template <int D>
 cudaError_t launch_single_t(bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s) {
-  if (single_uses_tma(D)) {
-    return grad ? launch_single_tma_variant<D, true, kSingleTile, single_stages(D), single_tma_occ(D)>(a, grid, s)
-                : launch_single_tma_variant<D, false, kSingleTile, single_stages(D), single_tma_occ(D)>(a, grid, s);
+  if (a.cull) {
+    return grad ? launch_single_tma_variant<D, true, cull_tile(D), cull_stages(D), cull_occ(D), true>(a, grid, s)
+                : launch_single_tma_variant<D, false, cull_tile(D), cull_stages(D), cull_occ(D), true>(a, grid, s);
+  }
+  if constexpr (single_uses_tma(D)) {
+    return grad
+               ? launch_single_tma_variant<D, true, kSingleTile, single_stages(D), single_tma_occ(D), false>(a, grid, s)
+               : launch_single_tma_variant<D, false, kSingleTile, single_stages(D), single_tma_occ(D), false>(a, grid,
+                                                                                                              s);
   }
   if (grad)
     scan_single_kernel<D, true><<<grid, kSingleThreads, 0, s>>>(a);

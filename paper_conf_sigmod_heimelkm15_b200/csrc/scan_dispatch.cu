@@ -32,7 +32,13 @@ cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int 
 }
 
 // ~3 resident CTAs of 256 threads per SM, never more CTAs than 8-point work items.
-int scan_single_grid(int d, bool grad, int64_t n, int num_sms) {
+int scan_single_grid(int d, bool grad, int64_t n, int num_sms, bool cull) {
+  if (cull) {  // culled TMA variant: one contiguous chunk of >= 1 tile per CTA
+    int64_t grid = (int64_t)num_sms * cull_occ(d);
+    const int64_t ntiles = (n + cull_tile(d) - 1) / cull_tile(d);
+    if (grid > ntiles) grid = ntiles;
+    return (int)(grid < 1 ? 1 : grid);
+  }
   if (single_uses_tma(d)) {  // one contiguous chunk of >= 1 tile per CTA
     int64_t grid = (int64_t)num_sms * single_tma_occ(d);
     const int64_t ntiles = (n + kSingleTile - 1) / kSingleTile;

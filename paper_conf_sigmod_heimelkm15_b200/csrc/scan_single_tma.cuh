@@ -72,14 +72,161 @@ __device__ __forceinline__ void scan_single_tma_body(const ScanSingleArgs& a, co
   }
 }
 
-template <int D, bool GRAD, int TILE, int STAGES, int OCC>
+// ---------------------------------------------------------------------------
+// Tail culling (DESIGN.md §8 "culled single-box scan").  For a point t and box
+// [l, u], let o_j = max(t_j - u_j, l_j - t_j, 0) sqrt(log2 e)/(sqrt2 h_j) be
+// the distance OUTSIDE the box in dimension j in y' units (y'^2 = z^2 log2 e).
+// Outside in dimension j, D_j <= 1/2 erfc(|z_j|) <= 1/2 e^{-z_j^2} = 2^{-o_j^2 - 1},
+// so p^(i) = prod_j D_j <= 2^{-sum_j o_j^2}, and every gradient term
+// |w_j| prod_{k!=j} D_k <= max(1, o_j) 2^{-sum_k o_k^2} (o_j <= 14 after bound
+// clamping).  A point with sum_j o_j^2 >= kCullY2 = 64 therefore changes p_hat
+// by at most 2^-64 and each dp_hat/dh_j by at most 15 * 2^-64 * gconst_j per
+// point: far below the fp32 rounding of the terms that are kept.  Such points
+// are skipped (their retained p^(i) is written as 0); the others go through a
+// per-warp ring of shared memory and are evaluated 64 at a time, so the
+// expensive Phi evaluation (FMA + MUFU dispatch bound, §8) runs only on the
+// points that can matter.  Points inside the box are never culled (o = 0), so
+// the eq. (20) test (c >= the largest contribution of an outside point) sees
+// every point it can flag.
+constexpr float kCullY2 = 64.0f;
+constexpr int kCullRing = 128;   // queued points per warp (< 64 left + one 64-point classification chunk)
+constexpr int kCullFlushChunks = 4;  // fp32 partials flushed to fp64 every 4 chunks (8 points per lane)
+
+template <int D>
+constexpr size_t cull_queue_bytes() {
+  return (size_t)kSingleComputeWarps * kCullRing * (D + 1) * sizeof(float);
+}
+
+template <int D, int TILE, int STAGES, bool CULL>
+constexpr size_t single_tma_kernel_smem() {
+  return single_tma_smem_bytes<D, TILE, STAGES>() + (CULL ? cull_queue_bytes<D>() : 0);
+}
+
+template <int D, bool GRAD, int MODE, int TILE, int STAGES>
+__device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, const float4* smc, const float2* scb,
+                                                      float* tiles, uint64_t* full, uint64_t* empty, float* queue,
+                                                      int64_t c0, int64_t c1, int ntiles, double* acc) {
+  constexpr int NA = GRAD ? D + 1 : 1;
+  constexpr int PPT = TILE / kSingleThreads;  // points per thread per tile
+  static_assert(PPT % 2 == 0, "points are classified in pairs");
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  float* qt = queue + (size_t)warp * kCullRing * (D + 1);  // [D][kCullRing] coordinates
+  int* qi = reinterpret_cast<int*>(qt + D * kCullRing);     // [kCullRing] point offset from c0
+  BoxDim bd[D];
+  float ap[D];
+  float2 cb[D];  // (u, l) of the clamped box, for the classification
+#pragma unroll
+  for (int j = 0; j < D; ++j) {
+    const float4 c = smc[j];
+    bd[j].b = make_float2(c.x, c.y);
+    bd[j].hd = c.z;
+    ap[j] = c.w;
+    cb[j] = scb[j];
+  }
+  const unsigned lt = (1u << lane) - 1u;
+  unsigned head = 0, tail = 0;  // warp-uniform ring positions (head is a multiple of 64)
+  int nproc = 0;
+  float2 s[NA];
+#pragma unroll
+  for (int kk = 0; kk < NA; ++kk) s[kk] = f2(0.0f);
+
+  // evaluate ring entries head + [0, 64): lane takes entries 2 lane, 2 lane + 1 (one LDS.64 per column)
+  auto process = [&](int cnt) {
+    const int e = (int)(head & (kCullRing - 1)) + 2 * lane;
+    const bool v0 = 2 * lane < cnt, v1 = 2 * lane + 1 < cnt;
+    float2 t[D];
+#pragma unroll
+    for (int j = 0; j < D; ++j) {
+      const float2 q = *reinterpret_cast<const float2*>(qt + j * kCullRing + e);
+      // stale ring slots may hold any bit pattern: replace them by a finite coordinate
+      t[j] = make_float2(v0 ? q.x : cb[j].x, v1 ? q.y : cb[j].x);
+    }
+    const float2 c = point_box2<D, GRAD, MODE>(bd, t, ap, s, make_float2(v0 ? 1.0f : 0.0f, v1 ? 1.0f : 0.0f));
+    if (a.c_out) {
+      const int2 ix = *reinterpret_cast<const int2*>(qi + e);
+      if (v0) __stcs(a.c_out + c0 + ix.x, c.x);
+      if (v1) __stcs(a.c_out + c0 + ix.y, c.y);
+    }
+    head += 64;
+    if (++nproc == kCullFlushChunks) {
+#pragma unroll
+      for (int kk = 0; kk < NA; ++kk) {
+        acc[kk] += (double)s[kk].x + (double)s[kk].y;
+        s[kk] = f2(0.0f);
+      }
+      nproc = 0;
+    }
+  };
+
+  for (int k = 0; k < ntiles; ++k) {
+    const int st = k % STAGES;
+    mbar_wait_parity(&full[st], (uint32_t)((k / STAGES) & 1));
+    const float* tl = tiles + (size_t)st * D * TILE;
+    const int64_t base = c0 + (int64_t)k * TILE;
+    const int64_t rem = c1 - base;
+    const int npts = rem < TILE ? (int)rem : TILE;
+#pragma unroll 1
+    for (int r = 0; r < PPT / 2; ++r) {
+      const int pp = tid + r * kSingleThreads;
+      float2 t[D];
+#pragma unroll
+      for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * TILE + 2 * pp);
+      // classification: o2 = sum_j (max(t - u, l - t, 0) ap)^2 (exact differences, then scale)
+      float2 o2 = f2(0.0f);
+#pragma unroll
+      for (int j = 0; j < D; ++j) {
+        const float2 ru = __fadd2_rn(t[j], f2(-cb[j].x));
+        const float2 rl = __fadd2_rn(f2(cb[j].y), make_float2(-t[j].x, -t[j].y));
+        const float2 rr = make_float2(fmaxf(fmaxf(ru.x, rl.x), 0.0f), fmaxf(fmaxf(ru.y, rl.y), 0.0f));
+        const float2 m = __fmul2_rn(rr, f2(ap[j]));
+        o2 = __ffma2_rn(m, m, o2);
+      }
+      const bool val0 = 2 * pp < npts, val1 = 2 * pp + 1 < npts;
+      const bool al0 = val0 && o2.x < kCullY2, al1 = val1 && o2.y < kCullY2;
+      if (a.c_out) {  // culled points retain 0; kept points are overwritten after evaluation (same warp, synced)
+        if (val1)
+          __stcs(reinterpret_cast<float2*>(a.c_out + base + 2 * pp), f2(0.0f));
+        else if (val0)
+          __stcs(a.c_out + base + 2 * pp, 0.0f);
+      }
+      __syncwarp();  // the previous chunk's ring reads are done before these writes
+      const unsigned m0 = __ballot_sync(0xffffffffu, al0), m1 = __ballot_sync(0xffffffffu, al1);
+      const int n0 = __popc(m0);
+      const int off = (int)(base - c0) + 2 * pp;
+      if (al0) {
+        const int pos = (int)((tail + __popc(m0 & lt)) & (kCullRing - 1));
+#pragma unroll
+        for (int j = 0; j < D; ++j) qt[j * kCullRing + pos] = t[j].x;
+        qi[pos] = off;
+      }
+      if (al1) {
+        const int pos = (int)((tail + n0 + __popc(m1 & lt)) & (kCullRing - 1));
+#pragma unroll
+        for (int j = 0; j < D; ++j) qt[j * kCullRing + pos] = t[j].y;
+        qi[pos] = off + 1;
+      }
+      tail += n0 + __popc(m1);
+      __syncwarp();
+      while (tail - head >= 64u) process(64);
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[st]);  // this warp is done reading stage st
+  }
+  if (tail != head) process((int)(tail - head));
+#pragma unroll
+  for (int kk = 0; kk < NA; ++kk) acc[kk] += (double)s[kk].x + (double)s[kk].y;
+}
+
+template <int D, bool GRAD, int TILE, int STAGES, int OCC, bool CULL>
 __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel(const ScanSingleArgs a) {
   constexpr int NA = GRAD ? D + 1 : 1;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   float* tiles = reinterpret_cast<float*>(smem_raw);
   uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + (size_t)STAGES * D * TILE * sizeof(float));
   uint64_t* empty = full + STAGES;
+  float* queue = reinterpret_cast<float*>(smem_raw + single_tma_smem_bytes<D, TILE, STAGES>());
   __shared__ float4 smc[D];
+  __shared__ float2 scb[D];
   __shared__ int narrow_s;
   const int tid = threadIdx.x;
   const bool producer = tid >= kSingleThreads;
@@ -108,6 +255,15 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
                                          a.consts->renc[2 * j + 1]);
     smc[j] = make_float4(bd.b.x, bd.b.y, bd.hd, ap);
     if (!epan && bd.hd > 0.0f) atomicOr(&narrow_s, 1);
+    if (CULL) {  // the clamped box of make_boxdim; an empty dimension (l == u) puts it above the range: all culled
+      const float tmin = fdec_range(a.consts->renc[2 * j]), tmax = fdec_range(a.consts->renc[2 * j + 1]);
+      const float m = kBoundMargin / ap;
+      float l = __ldg(a.lo + j), u = __ldg(a.hi + j);
+      const bool nonempty = (u - l) * ap > 0.0f;
+      l = fminf(fmaxf(l, tmin - m), tmax + m);
+      u = fminf(fmaxf(u, tmin - m), tmax + m);
+      scb[j] = nonempty ? make_float2(u, l) : make_float2(tmax + m, tmax + m);
+    }
   }
   __syncthreads();
   double acc[NA];
@@ -128,6 +284,11 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
     }
   } else if (a.consts->kernel == kEpanechnikov) {
     scan_single_tma_body<D, GRAD, 2, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
+  } else if (CULL) {
+    if (narrow_s)
+      scan_single_cull_body<D, GRAD, 1, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc);
+    else
+      scan_single_cull_body<D, GRAD, 0, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc);
   } else if (narrow_s) {
     scan_single_tma_body<D, GRAD, 1, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
   } else {
@@ -136,17 +297,18 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
   single_reduce_finalize<NA, kSingleTmaThreads>(a, acc);
 }
 
-template <int D, bool GRAD, int TILE, int STAGES, int OCC>
+template <int D, bool GRAD, int TILE, int STAGES, int OCC, bool CULL>
 cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStream_t s) {
-  constexpr size_t smem = single_tma_smem_bytes<D, TILE, STAGES>();
+  constexpr size_t smem = single_tma_kernel_smem<D, TILE, STAGES, CULL>();
+  static_assert(smem + 1024 <= 227 * 1024, "single-box scan shared memory");
   static bool attr_set = false;
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC>,
+    cudaError_t e = cudaFuncSetAttribute(scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC, CULL>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC><<<grid, kSingleTmaThreads, smem, s>>>(a);
+  scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC, CULL><<<grid, kSingleTmaThreads, smem, s>>>(a);
   return cudaGetLastError();
 }
 

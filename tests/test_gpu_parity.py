@@ -607,3 +607,70 @@ def test_epanechnikov_loss_karma_and_switch_back():
     m.set_kernel("gauss")
     m.bandwidth = h_g
     sel_ok(m.estimate(lo, hi), oracle.estimate(S, h_g, lo, hi))
+
+
+# ------------------------------------------------------------------ tail culling (single-box scan)
+@pytest.mark.parametrize("d,n,kernel", [(3, 70001, "gauss"), (5, 200003, "gauss"), (10, 50001, "gauss"),
+                                        (16, 9001, "gauss"), (5, 20011, "epan")])
+def test_cull_kept_points_bit_identical_and_bound(d, n, kernel):
+    """kde_set_cull: a culled point's retained p^(i) is 0 where the full
+    evaluation gives <= 2^-64; every kept point's p^(i) is bit-identical to the full
+    evaluation (same arithmetic); estimates and gradients of both settings pass the oracle."""
+    S = synth.make_data("gauss", n, d, seed=40 + d)
+    lo, hi = boxes_mix(S, 6, seed=41 + d)
+    lo2, hi2 = synth.mixed_workload(S, 8, seed=42 + d)
+    lo, hi = np.concatenate([lo, lo2]), np.concatenate([hi, hi2])
+    m = model(S)
+    if kernel == "epan":
+        m.set_kernel("epan")
+    h = m.bandwidth
+    m.set_retain(True)
+    if kernel == "epan":
+        est_o, g_o = oracle.epan_estimate_grad(S, h, lo, hi)
+        mabs = oracle.epan_grad_abs_scale(S, h, lo, hi)
+    else:
+        est_o, g_o = oracle.estimate_grad(S, h, lo, hi)
+        mabs = oracle.grad_abs_scale(S, h, lo, hi)
+    culled_any = 0
+    for k in range(len(lo)):
+        res = {}
+        for cull in (True, False):
+            m.cull = cull
+            e, g = m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+            sel_ok(e, est_o[k:k + 1])
+            grad_ok(g, g_o[k:k + 1], mabs[k:k + 1], h)
+            res[cull] = m.contributions()
+        c_on, c_off = res[True], res[False]
+        kept = c_on != 0.0
+        assert np.array_equal(c_on[kept], c_off[kept])
+        assert np.all(c_off[~kept] <= 2.0 ** -64)
+        culled_any += int(np.count_nonzero(~kept & (c_off > 0)))
+    assert m.cull is False
+    if kernel == "gauss":
+        assert culled_any > 0  # the workload does exercise culling of nonzero contributions
+
+
+def test_cull_far_box_and_inside_points_never_culled():
+    """A box ~12 bandwidths beyond the data in one dimension: every point is culled (estimate 0,
+    within the abs tolerance of the oracle's tail mass); a point exactly inside is never culled."""
+    S = synth.make_data("gauss", 30011, 4, seed=50)
+    m = model(S)
+    h = m.bandwidth
+    lo = S.min(0).astype(np.float64) - 1.0
+    hi = S.max(0).astype(np.float64) + 1.0
+    lo[2] = S[:, 2].max() + 12 * np.sqrt(2) * h[2]
+    hi[2] = lo[2] + 5 * h[2]
+    lo, hi = lo.astype(np.float32)[None], hi.astype(np.float32)[None]
+    est_o, g_o = oracle.estimate_grad(S, h, lo, hi)
+    e, g = m.estimate(lo, hi, grad=True)
+    assert e[0] == 0.0 and np.all(g == 0.0)
+    sel_ok(e, est_o)
+    grad_ok(g, g_o, oracle.grad_abs_scale(S, h, lo, hi), h)
+    # a tiny box around one sample point: that point is inside, its contribution is kept
+    i0 = 1234
+    lo1 = (S[i0] - 1e-3 * h).astype(np.float32)[None]
+    hi1 = (S[i0] + 1e-3 * h).astype(np.float32)[None]
+    m.set_retain(True)
+    e1 = m.estimate(lo1, hi1)
+    assert m.contributions()[i0] > 0.0
+    sel_ok(e1, oracle.estimate_grad(S, h, lo1, hi1)[0])
