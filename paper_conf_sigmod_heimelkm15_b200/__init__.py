@@ -19,7 +19,7 @@ from dataclasses import dataclass
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libkde.so")
+LIB_PATH = os.environ.get("KDE_LIB_PATH") or os.path.join(_HERE, "libkde.so")  # override: tuning builds
 
 KDE_OK, KDE_EINVAL, KDE_ENOMEM, KDE_ECUDA, KDE_ENCCL, KDE_ESTATE, KDE_ETRUNC = range(7)
 LOSS_SQUARED, LOSS_ABSOLUTE, LOSS_RELATIVE, LOSS_SQUARED_RELATIVE, LOSS_SQUARED_Q = range(5)

@@ -390,7 +390,7 @@ __global__ void karma_kernel(const float* __restrict__ cvals, double* __restrict
   }
 }
 
-__device__ void online_update_body(const double* __restrict__ ret, const double* __restrict__ p_ptr,
+__device__ __noinline__ void online_update_body(const double* __restrict__ ret, const double* __restrict__ p_ptr,
                                    const OnlineParamsDev& op, int d, OnlineState* st, DevConsts* c);
 
 // Ordered compaction of the karma flags: block b writes the ascending GLOBAL
@@ -505,8 +505,10 @@ __global__ void compact_fused_kernel(const uint32_t* __restrict__ bitmap, int64_
 // ret: [1+d] = (p_hat, dp/dh_j) of the retained query.  Adds L' dp/dh (x h in
 // log mode, eq. 18) to the mini-batch; every `minibatch` queries applies the
 // RMSprop / Rprop step of P:L179-183 and re-derives the constants.
-// One Listing 1 step, executed by one whole block (thread j < d owns dimension j).
-__device__ void online_update_body(const double* __restrict__ ret, const double* __restrict__ p_ptr,
+// One Listing 1 step, executed by one whole block (thread j < d owns dimension j).  Not inlined:
+// the standalone kernel and the fused streaming step run the same machine code, so their
+// bandwidths stay bit-identical (inlined copies may contract log/exp differently).
+__device__ __noinline__ void online_update_body(const double* __restrict__ ret, const double* __restrict__ p_ptr,
                                    const OnlineParamsDev& op, int d, OnlineState* st, DevConsts* c) {
   const int j = threadIdx.x;
   const double p = *p_ptr;

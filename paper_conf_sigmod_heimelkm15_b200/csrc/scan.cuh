@@ -642,9 +642,18 @@ cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStr
 // culled single-box scan (every d): TMA tiles + a per-warp ring of kept points.
 // Two stages; 2048-point tiles up to d = 8 (1024 above, shared-memory budget);
 // two CTAs per SM up to d = 5.
-__host__ __device__ constexpr int cull_tile(int d) { return d <= 8 ? 2048 : 1024; }
-__host__ __device__ constexpr int cull_stages(int d) { return (void)d, 2; }
-__host__ __device__ constexpr int cull_occ(int d) { return d <= 5 ? 2 : 1; }
+#ifndef KDE_TUNE_CULL_TILE
+#define KDE_TUNE_CULL_TILE(d) ((d) <= 8 ? 2048 : 1024)
+#endif
+#ifndef KDE_TUNE_CULL_STAGES
+#define KDE_TUNE_CULL_STAGES(d) 2
+#endif
+#ifndef KDE_TUNE_CULL_OCC
+#define KDE_TUNE_CULL_OCC(d) ((d) <= 5 ? 2 : 1)
+#endif
+__host__ __device__ constexpr int cull_tile(int d) { return KDE_TUNE_CULL_TILE(d); }
+__host__ __device__ constexpr int cull_stages(int d) { return (void)d, KDE_TUNE_CULL_STAGES(d); }
+__host__ __device__ constexpr int cull_occ(int d) { return KDE_TUNE_CULL_OCC(d); }
 
 // cull on: the culled TMA variant;
 // d <= 8: TMA-pipelined, warp-specialised variant (kSingleTile-point tiles, single_stages(d) stages,

@@ -88,9 +88,17 @@ __device__ __forceinline__ void scan_single_tma_body(const ScanSingleArgs& a, co
 // points that can matter.  Points inside the box are never culled (o = 0), so
 // the eq. (20) test (c >= the largest contribution of an outside point) sees
 // every point it can flag.
-constexpr float kCullY2 = 64.0f;
+constexpr float kCullY2 = 64.5f;  // 64 plus slack for the fp32 rounding of the o^2 sum
 constexpr int kCullRing = 128;   // queued points per warp (< 64 left + one 64-point classification chunk)
 constexpr int kCullFlushChunks = 4;  // fp32 partials flushed to fp64 every 4 chunks (8 points per lane)
+
+// st.shared.f32 under a predicate (no branch: culled lanes issue but do not store)
+__device__ __forceinline__ void st_shared_if(uint32_t addr, float v, bool p) {
+  asm volatile(
+      "{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q st.shared.f32 [%0], %1;\n\t}" ::"r"(addr), "f"(v),
+      "r"((uint32_t)p)
+      : "memory");
+}
 
 template <int D>
 constexpr size_t cull_queue_bytes() {
@@ -114,7 +122,7 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
   int* qi = reinterpret_cast<int*>(qt + D * kCullRing);     // [kCullRing] point offset from c0
   BoxDim bd[D];
   float ap[D];
-  float2 cb[D];  // (u, l) of the clamped box, for the classification
+  float2 cb[D];  // (c ap, hw' ap) of the clamped box, for the classification
 #pragma unroll
   for (int j = 0; j < D; ++j) {
     const float4 c = smc[j];
@@ -139,7 +147,7 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
     for (int j = 0; j < D; ++j) {
       const float2 q = *reinterpret_cast<const float2*>(qt + j * kCullRing + e);
       // stale ring slots may hold any bit pattern: replace them by a finite coordinate
-      t[j] = make_float2(v0 ? q.x : cb[j].x, v1 ? q.y : cb[j].x);
+      t[j] = make_float2(v0 ? q.x : bd[j].b.y, v1 ? q.y : bd[j].b.y);
     }
     const float2 c = point_box2<D, GRAD, MODE>(bd, t, ap, s, make_float2(v0 ? 1.0f : 0.0f, v1 ? 1.0f : 0.0f));
     if (a.c_out) {
@@ -171,15 +179,16 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
       float2 t[D];
 #pragma unroll
       for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * TILE + 2 * pp);
-      // classification: o2 = sum_j (max(t - u, l - t, 0) ap)^2 (exact differences, then scale)
+      // classification in scaled coordinates: y = t ap - c ap (one FFMA2), o = max(|y| - hw', 0),
+      // o2 = sum_j o^2; hw' is the half-width widened by a bound on the rounding of y (box setup),
+      // so o never exceeds the exact distance outside the box
       float2 o2 = f2(0.0f);
 #pragma unroll
       for (int j = 0; j < D; ++j) {
-        const float2 ru = __fadd2_rn(t[j], f2(-cb[j].x));
-        const float2 rl = __fadd2_rn(f2(cb[j].y), make_float2(-t[j].x, -t[j].y));
-        const float2 rr = make_float2(fmaxf(fmaxf(ru.x, rl.x), 0.0f), fmaxf(fmaxf(ru.y, rl.y), 0.0f));
-        const float2 m = __fmul2_rn(rr, f2(ap[j]));
-        o2 = __ffma2_rn(m, m, o2);
+        const float2 y = __ffma2_rn(t[j], f2(ap[j]), f2(-cb[j].x));
+        const float2 e = __fadd2_rn(make_float2(fabsf(y.x), fabsf(y.y)), f2(-cb[j].y));
+        const float2 r = make_float2(fmaxf(e.x, 0.0f), fmaxf(e.y, 0.0f));
+        o2 = __ffma2_rn(r, r, o2);
       }
       const bool val0 = 2 * pp < npts, val1 = 2 * pp + 1 < npts;
       const bool al0 = val0 && o2.x < kCullY2, al1 = val1 && o2.y < kCullY2;
@@ -190,22 +199,23 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
           __stcs(a.c_out + base + 2 * pp, 0.0f);
       }
       __syncwarp();  // the previous chunk's ring reads are done before these writes
+      // Branch-free compaction of the 64 candidates: the kept ones go to [tail, tail + nkeep)
+      // (x halves, then y halves, in lane order) with predicated shared stores.
       const unsigned m0 = __ballot_sync(0xffffffffu, al0), m1 = __ballot_sync(0xffffffffu, al1);
-      const int n0 = __popc(m0);
+      const int n0 = __popc(m0), nkeep = n0 + __popc(m1);
       const int off = (int)(base - c0) + 2 * pp;
-      if (al0) {
-        const int pos = (int)((tail + __popc(m0 & lt)) & (kCullRing - 1));
+      const uint32_t a0 = smem_u32(qt + ((tail + (unsigned)__popc(m0 & lt)) & (kCullRing - 1)));
+      const uint32_t a1 = smem_u32(qt + ((tail + (unsigned)(n0 + __popc(m1 & lt))) & (kCullRing - 1)));
 #pragma unroll
-        for (int j = 0; j < D; ++j) qt[j * kCullRing + pos] = t[j].x;
-        qi[pos] = off;
+      for (int j = 0; j < D; ++j) {
+        st_shared_if(a0 + j * kCullRing * 4, t[j].x, al0);
+        st_shared_if(a1 + j * kCullRing * 4, t[j].y, al1);
       }
-      if (al1) {
-        const int pos = (int)((tail + n0 + __popc(m1 & lt)) & (kCullRing - 1));
-#pragma unroll
-        for (int j = 0; j < D; ++j) qt[j * kCullRing + pos] = t[j].y;
-        qi[pos] = off + 1;
+      if (a.c_out) {
+        st_shared_if(a0 + D * kCullRing * 4, __int_as_float(off), al0);
+        st_shared_if(a1 + D * kCullRing * 4, __int_as_float(off + 1), al1);
       }
-      tail += n0 + __popc(m1);
+      tail += (unsigned)nkeep;
       __syncwarp();
       while (tail - head >= 64u) process(64);
     }
@@ -255,14 +265,20 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
                                          a.consts->renc[2 * j + 1]);
     smc[j] = make_float4(bd.b.x, bd.b.y, bd.hd, ap);
     if (!epan && bd.hd > 0.0f) atomicOr(&narrow_s, 1);
-    if (CULL) {  // the clamped box of make_boxdim; an empty dimension (l == u) puts it above the range: all culled
+    if (CULL) {  // the clamped box of make_boxdim as (c ap, hw ap + rounding margin); l == u: far above the range
       const float tmin = fdec_range(a.consts->renc[2 * j]), tmax = fdec_range(a.consts->renc[2 * j + 1]);
       const float m = kBoundMargin / ap;
       float l = __ldg(a.lo + j), u = __ldg(a.hi + j);
       const bool nonempty = (u - l) * ap > 0.0f;
       l = fminf(fmaxf(l, tmin - m), tmax + m);
       u = fminf(fmaxf(u, tmin - m), tmax + m);
-      scb[j] = nonempty ? make_float2(u, l) : make_float2(tmax + m, tmax + m);
+      const double c = nonempty ? 0.5 * ((double)u + (double)l) : (double)(tmax + m);
+      const double hw = nonempty ? 0.5 * ((double)u - (double)l) : 0.0;
+      const double cap = c * ap, hwap = hw * ap;
+      const double tabs = fmax(fabs((double)tmin), fabs((double)tmax)) * ap;
+      // |fl(t ap - fl(c ap)) - (t - c) ap| <= 2^-23 (|c ap| + tabs) (one rounding of c ap, one of the FFMA)
+      const double err = ldexp(2.0 * fabs(cap) + hwap + tabs, -22) + 1e-30;
+      scb[j] = make_float2((float)cap, (float)(hwap + err));
     }
   }
   __syncthreads();
