@@ -100,6 +100,7 @@ struct ScanBatchedArgs {
   int64_t split_len;      // points per split (multiple of the tile size)
   int qb;                 // boxes per CTA (power of two <= 256; 256/qb threads share a box)
   double* partials;       // [splits][1+d][q]
+  int cull;               // 1: per (box, point) tail culling (scan.cuh batched_tile_cull), qb == 256 only
 };
 
 // host-side launchers (scan_inst_*.cu)

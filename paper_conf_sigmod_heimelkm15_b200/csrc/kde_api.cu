@@ -262,6 +262,7 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     a.hi = d_hi;
     a.q = q;
     a.consts = m->consts;
+    a.cull = m->cull ? 1 : 0;
     a.split_len = 0;
     a.partials = nullptr;
     int splits = 1;

@@ -97,6 +97,41 @@ __device__ __forceinline__ BoxDim make_boxdim(float l, float u, float ap, unsign
   return r;
 }
 
+// Tail culling (reading R15, scan_single_tma.cuh): the box of make_boxdim (bounds clamped to the
+// column range widened by 14/ap) in scaled coordinates, (c ap, hw ap + margin), c / hw its centre /
+// half-width.  A point's distance outside the box in dimension j is then bounded from below by
+// max(|t ap - c ap| - hw', 0) as evaluated in fp32 (FFMA2 + FADD2): the margin covers the rounding of
+// c ap and of the FFMA, |fl(t ap - fl(c ap)) - (t - c) ap| <= 2^-23 (|c ap| + max|t| ap).  An empty
+// dimension (l == u, D = 0) becomes a point far above the range, so every point is culled.
+__device__ __forceinline__ float2 make_cullbox(float l, float u, float ap, unsigned rmin_enc, unsigned rmax_enc) {
+  const float tmin = fdec_range(rmin_enc), tmax = fdec_range(rmax_enc);
+  const float m = kBoundMargin / ap;
+  const bool nonempty = (u - l) * ap > 0.0f;
+  l = fminf(fmaxf(l, tmin - m), tmax + m);
+  u = fminf(fmaxf(u, tmin - m), tmax + m);
+  const double c = nonempty ? 0.5 * ((double)u + (double)l) : (double)(tmax + m);
+  const double hw = nonempty ? 0.5 * ((double)u - (double)l) : 0.0;
+  const double cap = c * ap, hwap = hw * ap;
+  const double tabs = fmax(fabs((double)tmin), fabs((double)tmax)) * ap;
+  const double err = ldexp(2.0 * fabs(cap) + hwap + tabs, -22) + 1e-30;
+  return make_float2((float)cap, (float)(hwap + err));
+}
+constexpr float kCullY2 = 64.5f;  // cull when sum_j o_j^2 >= 64 (+ slack for the fp32 rounding of the sum)
+
+// sum_j o_j^2 for two points (float2 lanes = points), o_j = max(|t ap - c ap| - hw', 0)
+template <int D>
+__device__ __forceinline__ float2 cull_o2(const float2 (&t)[D], const float (&ap)[D], const float2 (&cb)[D]) {
+  float2 o2 = f2(0.0f);
+#pragma unroll
+  for (int j = 0; j < D; ++j) {
+    const float2 y = __ffma2_rn(t[j], f2(ap[j]), f2(-cb[j].x));
+    const float2 e = __fadd2_rn(make_float2(fabsf(y.x), fabsf(y.y)), f2(-cb[j].y));
+    const float2 r = make_float2(fmaxf(e.x, 0.0f), fmaxf(e.y, 0.0f));
+    o2 = __ffma2_rn(r, r, o2);
+  }
+  return o2;
+}
+
 // erf-difference path: D = 1/2 [erf(z_u) - erf(z_l)], w = y'_l E_l - y'_u E_u.
 // One MUFU.RCP serves the pair: t_u = den_l / (den_u den_l), t_l = den_u / (den_u den_l)
 // (den = 1 + P'|y'| with |y'| bounded by the clamped bounds: the product stays finite for any

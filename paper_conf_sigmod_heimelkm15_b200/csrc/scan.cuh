@@ -469,6 +469,84 @@ __device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, 
   }
 }
 
+// Culled tile compute (reading R15, one box per thread, QB == 256): the thread
+// classifies all kTilePts points of the tile against its box (cull_o2, 3 packed
+// FMA-pipe + 2 ALU instructions per point pair and dimension, broadcast LDS.64),
+// keeping a 256-bit alive mask in registers, then walks its own alive points two at a
+// time (the warp iterates max over its lanes -- boxes are sorted by their kept
+// fraction within the CTA, see the kernel) with lane-varying LDS gathers from the tile.
+constexpr int kTileWords = kTilePts / 32;
+
+template <int D>
+__device__ __forceinline__ void cull_tile_mask(const float* tl, int npts, const float (&ap)[D], const float2 (&cb)[D],
+                                               unsigned (&mk)[kTileWords]) {
+#pragma unroll
+  for (int w = 0; w < kTileWords; ++w) {
+    unsigned m = 0u;
+#pragma unroll 4
+    for (int q = 0; q < 16; ++q) {
+      const int pp = 16 * w + q;
+      float2 t[D];
+#pragma unroll
+      for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * kTilePts + 2 * pp);
+      const float2 o2 = cull_o2<D>(t, ap, cb);
+      m |= (o2.x < kCullY2 ? 1u : 0u) << (2 * q);
+      m |= (o2.y < kCullY2 ? 1u : 0u) << (2 * q + 1);
+    }
+    const int v = npts - 32 * w;  // valid points in this word
+    mk[w] = v >= 32 ? m : (v > 0 ? m & ((1u << v) - 1u) : 0u);
+  }
+}
+
+__device__ __forceinline__ unsigned sel_word(const unsigned (&mk)[kTileWords], int w) {
+  unsigned r = mk[0];
+#pragma unroll
+  for (int i = 1; i < kTileWords; ++i) r = w == i ? mk[i] : r;
+  return r;
+}
+
+template <int D, bool GRAD, int MODE>
+__device__ __forceinline__ void batched_tile_cull(const float* tl, int npts, double* accsh, const BoxDim (&bd)[D],
+                                                  const float (&ap)[D], const float2 (&cb)[D]) {
+  constexpr int NA = GRAD ? D + 1 : 1;
+  constexpr int kFlushPairs = kFlushPts / 2;
+  const int tid = threadIdx.x;
+  unsigned mk[kTileWords];
+  cull_tile_mask<D>(tl, npts, ap, cb, mk);
+  int w = 0;
+  unsigned m = mk[0];
+  auto next = [&]() -> int {  // next alive point of this lane, -1 when exhausted
+    while (m == 0u && w < kTileWords - 1) m = sel_word(mk, ++w);
+    if (m == 0u) return -1;
+    const int b = __ffs(m) - 1;
+    m &= m - 1u;
+    return 32 * w + b;
+  };
+  float2 s[NA];
+#pragma unroll
+  for (int kk = 0; kk < NA; ++kk) s[kk] = f2(0.0f);
+  int it = 0;
+  while (true) {
+    const int p0 = next(), p1 = next();
+    if (!__any_sync(0xffffffffu, p0 >= 0)) break;
+    float2 t[D];
+#pragma unroll
+    for (int j = 0; j < D; ++j)  // masked points take a finite coordinate (the box bound)
+      t[j] = make_float2(p0 >= 0 ? tl[j * kTilePts + p0] : bd[j].b.y, p1 >= 0 ? tl[j * kTilePts + p1] : bd[j].b.y);
+    point_box2<D, GRAD, MODE>(bd, t, ap, s, make_float2(p0 >= 0 ? 1.0f : 0.0f, p1 >= 0 ? 1.0f : 0.0f));
+    if (++it == kFlushPairs) {
+#pragma unroll
+      for (int kk = 0; kk < NA; ++kk) {
+        accsh[kk * kBatchedThreads + tid] += (double)s[kk].x + (double)s[kk].y;
+        s[kk] = f2(0.0f);
+      }
+      it = 0;
+    }
+  }
+#pragma unroll
+  for (int kk = 0; kk < NA; ++kk) accsh[kk * kBatchedThreads + tid] += (double)s[kk].x + (double)s[kk].y;
+}
+
 // The tile loop of the batched scan: wait for tile k (TMA bulk copies
 // completing on bar[k&1]), prefetch tile k+1, compute (warp-uniform variant),
 // then the CTA barrier that releases the buffer -- barriers stay outside the
@@ -476,8 +554,8 @@ __device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, 
 template <int D, bool GRAD, int QT, int PU, typename Issue>
 __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const float* tile, uint64_t* bar,
                                               double* accsh, const BoxDim (&bd)[QT][D], const float (&ap)[D],
-                                              int64_t s0, int64_t s1, int ntiles, int mode, int phase, int R,
-                                              Issue& issue) {
+                                              const float2 (&cb)[D], bool cull, int64_t s0, int64_t s1,
+                                              int ntiles, int mode, int phase, int R, Issue& issue) {
   const int tid = threadIdx.x;
   for (int k = 0; k < ntiles; ++k) {
     const int buf = k & 1;
@@ -486,7 +564,11 @@ __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const fl
     const float* tl = tile + buf * D * kTilePts;
     const int64_t rem = s1 - (s0 + (int64_t)k * kTilePts);
     const int npts = rem < kTilePts ? (int)rem : kTilePts;
-    if (mode == 2)
+    if (cull && mode == 1)
+      batched_tile_cull<D, GRAD, 1>(tl, npts, accsh, bd[0], ap, cb);
+    else if (cull)
+      batched_tile_cull<D, GRAD, 0>(tl, npts, accsh, bd[0], ap, cb);
+    else if (mode == 2)
       batched_tile_compute<D, GRAD, 2, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
     else if (mode == 1)
       batched_tile_compute<D, GRAD, 1, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
@@ -609,6 +691,62 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
   };
   if (tid == 0 && ntiles > 0) issue(0);
 
+  // Culling (reading R15, large batches): sort the CTA's boxes by their kept fraction on the
+  // split's first tile (narrow-dimension boxes last), so that the lanes of a warp walk alive
+  // lists of similar length; each thread then takes the box perm_s[tid].
+  const bool cull = a.cull && QB == kBatchedThreads && !epan;
+  float2 cb[D];
+  if (cull) {
+    __shared__ int key_s[kBatchedThreads];
+    const int64_t q0 = min(qbase + tid, a.q - 1);
+#pragma unroll
+    for (int j = 0; j < D; ++j)
+      cb[j] = make_cullbox(__ldg(a.lo + q0 * D + j), __ldg(a.hi + q0 * D + j), ap[j], a.consts->renc[2 * j],
+                           a.consts->renc[2 * j + 1]);
+    int cnt = 0;
+    if (ntiles > 0) {
+      mbar_wait_parity(&bar[0], 0u);
+      const int64_t rem = s1 - s0;
+      unsigned mk[kTileWords];
+      cull_tile_mask<D>(tile, rem < kTilePts ? (int)rem : kTilePts, ap, cb, mk);
+#pragma unroll
+      for (int w = 0; w < kTileWords; ++w) cnt += __popc(mk[w]);
+    }
+    bool nar0 = false;
+#pragma unroll
+    for (int j = 0; j < D; ++j) {
+      const float dy = (__ldg(a.hi + q0 * D + j) - __ldg(a.lo + q0 * D + j)) * ap[j];
+      nar0 |= dy > 0.0f && dy < kNarrowY;
+    }
+    key_s[tid] = ((nar0 ? 512 : 0) + cnt) * kBatchedThreads + tid;  // unique keys: a deterministic order
+    __syncthreads();
+    for (int k = 2; k <= kBatchedThreads; k <<= 1)  // bitonic sort, ascending
+      for (int jj = k >> 1; jj > 0; jj >>= 1) {
+        const int ix = tid ^ jj;
+        if (ix > tid) {
+          const int x = key_s[tid], y = key_s[ix];
+          if (((tid & k) == 0) == (x > y)) {
+            key_s[tid] = y;
+            key_s[ix] = x;
+          }
+        }
+        __syncthreads();
+      }
+    const int sl = key_s[tid] % kBatchedThreads;
+    perm_s[tid] = sl;
+    int64_t qi = qbase + sl;
+    if (qi >= a.q) qi = a.q - 1;
+    narrow[0] = false;
+#pragma unroll
+    for (int j = 0; j < D; ++j) {
+      const float l = __ldg(a.lo + qi * D + j), u = __ldg(a.hi + qi * D + j);
+      bd[0][j] = make_boxdim(l, u, ap[j], a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
+      narrow[0] |= bd[0][j].hd > 0.0f;
+      cb[j] = make_cullbox(l, u, ap[j], a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
+    }
+    __syncthreads();
+  }
+
   // One warp-uniform variant for the whole split: boxes with a narrow
   // dimension (rare) switch the warp to the general per-dimension path, so
   // the common path stays branch-free and the QT boxes interleave for ILP.
@@ -616,7 +754,7 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
 #pragma unroll
   for (int qq = 0; qq < QT; ++qq) my_narrow |= narrow[qq];
   const int mode = epan ? 2 : (__any_sync(0xffffffffu, my_narrow) ? 1 : 0);
-  batched_tiles<D, GRAD, QT, PU>(a, tile, bar, accsh, bd, ap, s0, s1, ntiles, mode, phase, R, issue);
+  batched_tiles<D, GRAD, QT, PU>(a, tile, bar, accsh, bd, ap, cb, cull, s0, s1, ntiles, mode, phase, R, issue);
 
   // combine the R phases of each box in phase order, then
   // partials[(split*(NA) + comp) * q + qi]

@@ -88,7 +88,6 @@ __device__ __forceinline__ void scan_single_tma_body(const ScanSingleArgs& a, co
 // points that can matter.  Points inside the box are never culled (o = 0), so
 // the eq. (20) test (c >= the largest contribution of an outside point) sees
 // every point it can flag.
-constexpr float kCullY2 = 64.5f;  // 64 plus slack for the fp32 rounding of the o^2 sum
 constexpr int kCullRing = 128;   // queued points per warp (< 64 left + one 64-point classification chunk)
 constexpr int kCullFlushChunks = 4;  // fp32 partials flushed to fp64 every 4 chunks (8 points per lane)
 
@@ -179,17 +178,8 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
       float2 t[D];
 #pragma unroll
       for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * TILE + 2 * pp);
-      // classification in scaled coordinates: y = t ap - c ap (one FFMA2), o = max(|y| - hw', 0),
-      // o2 = sum_j o^2; hw' is the half-width widened by a bound on the rounding of y (box setup),
-      // so o never exceeds the exact distance outside the box
-      float2 o2 = f2(0.0f);
-#pragma unroll
-      for (int j = 0; j < D; ++j) {
-        const float2 y = __ffma2_rn(t[j], f2(ap[j]), f2(-cb[j].x));
-        const float2 e = __fadd2_rn(make_float2(fabsf(y.x), fabsf(y.y)), f2(-cb[j].y));
-        const float2 r = make_float2(fmaxf(e.x, 0.0f), fmaxf(e.y, 0.0f));
-        o2 = __ffma2_rn(r, r, o2);
-      }
+      // classification in scaled coordinates (make_cullbox / cull_o2, phi.cuh)
+      const float2 o2 = cull_o2<D>(t, ap, cb);
       const bool val0 = 2 * pp < npts, val1 = 2 * pp + 1 < npts;
       const bool al0 = val0 && o2.x < kCullY2, al1 = val1 && o2.y < kCullY2;
       if (a.c_out) {  // culled points retain 0; kept points are overwritten after evaluation (same warp, synced)
@@ -265,21 +255,7 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
                                          a.consts->renc[2 * j + 1]);
     smc[j] = make_float4(bd.b.x, bd.b.y, bd.hd, ap);
     if (!epan && bd.hd > 0.0f) atomicOr(&narrow_s, 1);
-    if (CULL) {  // the clamped box of make_boxdim as (c ap, hw ap + rounding margin); l == u: far above the range
-      const float tmin = fdec_range(a.consts->renc[2 * j]), tmax = fdec_range(a.consts->renc[2 * j + 1]);
-      const float m = kBoundMargin / ap;
-      float l = __ldg(a.lo + j), u = __ldg(a.hi + j);
-      const bool nonempty = (u - l) * ap > 0.0f;
-      l = fminf(fmaxf(l, tmin - m), tmax + m);
-      u = fminf(fmaxf(u, tmin - m), tmax + m);
-      const double c = nonempty ? 0.5 * ((double)u + (double)l) : (double)(tmax + m);
-      const double hw = nonempty ? 0.5 * ((double)u - (double)l) : 0.0;
-      const double cap = c * ap, hwap = hw * ap;
-      const double tabs = fmax(fabs((double)tmin), fabs((double)tmax)) * ap;
-      // |fl(t ap - fl(c ap)) - (t - c) ap| <= 2^-23 (|c ap| + tabs) (one rounding of c ap, one of the FFMA)
-      const double err = ldexp(2.0 * fabs(cap) + hwap + tabs, -22) + 1e-30;
-      scb[j] = make_float2((float)cap, (float)(hwap + err));
-    }
+    if (CULL) scb[j] = make_cullbox(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
   }
   __syncthreads();
   double acc[NA];
