@@ -450,8 +450,10 @@ def run_cuda(args, cfg, rank, world, local_rank):
         peak = sms * MUFU_PER_SM_CLK * SM_MAX_MHZ * 1e6 / (2 * d) / 1e9
         roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gpt·q/s",
                 "frac": achieved / peak, "traffic": _traffic(args.config),
-                "kernel": f"scan_batched_kernel<{d},grad>",
-                "algorithmic": f"{n} points x {q} boxes per launch; 2d MUFU.EX2 per point*box",
+                "kernel": f"scan_batched_kernel<{d},grad>{'' if args.no_cull else ' (culled)'}",
+                "algorithmic": f"{n} points x {q} boxes per launch; 2d MUFU.EX2 per point*box"
+                               + ("" if args.no_cull else " (brute-force count: culled pairs are counted as "
+                                  "evaluated, so frac is throughput against the unculled SFU ceiling)"),
                 "peak_source": f"SFU ceiling {sms} SMs x {MUFU_PER_SM_CLK} MUFU/clk x {SM_MAX_MHZ:.0f} MHz / (2d) "
                                "(guide unit counts; 16/clk/SM re-measured by tools/pipe_rates.cu)"}
     if clocks.get("sm_mhz"):
@@ -471,8 +473,8 @@ def run_cuda(args, cfg, rank, world, local_rank):
         "config": {"workload": cfg["desc"], "d": d, "n_per_gpu": n, "n_global": n_global, "q": q,
                    "l2": "flushed between timed steps" if flush_l2 else "sample larger than L2",
                    "cuda_graph": bool(graphs is not None),
-                   "cull": (None if cfg["path"] == "batched" else
-                            ("off" if args.no_cull else "on: points with contribution provably < 2^-64 skipped")),
+                   "cull": ("off" if args.no_cull or cfg.get("kernel") == "epan" else
+                            "on: (point, box) pairs whose contribution is provably < 2^-64 are skipped (DESIGN R15)"),
                    "clock_sampling": "nvidia-smi every 100 ms over the timed steps"
                                      + (f" + {soak} identical untimed soak steps (timed region < 1 s)" if soak else ""),
                    "accumulation": "fp32 per <=32 points, fp64 above"},

@@ -101,6 +101,7 @@ struct ScanBatchedArgs {
   int qb;                 // boxes per CTA (power of two <= 256; 256/qb threads share a box)
   double* partials;       // [splits][1+d][q]
   int cull;               // 1: per (box, point) tail culling (scan.cuh batched_tile_cull), qb == 256 only
+  const int* perm;        // nullable: CTA slot order -> box index (boxes sorted by their probed kept fraction)
 };
 
 // host-side launchers (scan_inst_*.cu)

@@ -64,6 +64,8 @@ struct kde_model {
   int64_t ocap = 0;
   double* partials = nullptr;
   size_t partials_cap = 0;           // bytes
+  void* order = nullptr;             // culled batched scan: box-order scratch (cull_order.cu)
+  size_t order_cap = 0;              // bytes
   double* gather = nullptr;          // [world][q][1+d]
   size_t gather_cap = 0;
   uint32_t* bitmap = nullptr;
@@ -265,6 +267,15 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     a.cull = m->cull ? 1 : 0;
     a.split_len = 0;
     a.partials = nullptr;
+    a.perm = nullptr;
+    if (m->cull && m->kernel == KDE_KERNEL_GAUSSIAN && q >= 256) {  // large batches: order boxes by probed cost
+      const size_t ob = cull_order_bytes(q);
+      kde_status st = ensure_bytes(&m->order, &m->order_cap, ob);
+      if (st != KDE_OK) return st;
+      int* perm = nullptr;
+      CUL(launch_cull_order(m->cols, m->ld, m->n, d, d_lo, d_hi, q, m->consts, m->order, m->order_cap, &perm, s));
+      a.perm = perm;
+    }
     int splits = 1;
     CU(launch_scan_batched(d, grad, a, m->num_sms, &splits, s, true));
     kde_status st = ensure_bytes((void**)&m->partials, &m->partials_cap, sizeof(double) * (size_t)splits * na * q);
@@ -351,6 +362,7 @@ static void free_model(kde_model* m) {
   cudaFree(m->qbuf);
   cudaFree(m->obuf);
   cudaFree(m->partials);
+  cudaFree(m->order);
   cudaFree(m->gather);
   cudaFree(m->bitmap);
   cudaFree(m->block_counts);

@@ -50,6 +50,11 @@ cudaError_t launch_moments_merge_ranks(const double* g, int world, int d, double
 cudaError_t launch_scott(const double* mom, int d, DevConsts* c, int* bad, cudaStream_t s);
 cudaError_t launch_set_consts(const double* h, int d, DevConsts* c, cudaStream_t s);
 cudaError_t launch_set_kernel_type(int kernel, int d, DevConsts* c, cudaStream_t s);
+// cull_order.cu: box order for the culled batched scan (probe counts + stable radix sort)
+size_t cull_order_bytes(int64_t q);
+cudaError_t launch_cull_order(const float* cols, int64_t ld, int64_t n, int d, const float* lo, const float* hi,
+                              int64_t q, const DevConsts* c, void* scratch, size_t scratch_bytes, int** perm_out,
+                              cudaStream_t s);
 cudaError_t launch_reduce_splits(const double* partials, int splits, int64_t q, int na, double* sums,
                                  cudaStream_t s);
 cudaError_t launch_combine_ranks(const double* gathered, int world, int64_t q, int na, double* sums,

@@ -547,21 +547,24 @@ __device__ __forceinline__ void batched_tile_cull(const float* tl, int npts, dou
   for (int kk = 0; kk < NA; ++kk) accsh[kk * kBatchedThreads + tid] += (double)s[kk].x + (double)s[kk].y;
 }
 
-// The tile loop of the batched scan: wait for tile k (TMA bulk copies
-// completing on bar[k&1]), prefetch tile k+1, compute (warp-uniform variant),
-// then the CTA barrier that releases the buffer -- barriers stay outside the
-// warp-divergent part.
+// The tile loop of the batched scan: a ring of kBatchedStages tile buffers
+// filled by TMA bulk copies (completing on full[stage]).  No CTA barrier:
+// each warp arrives on the stage's counter after its last read, and the
+// LAST warp out issues the copies of tile k + kBatchedStages into it, so warps
+// with less work (culling: boxes sorted by kept fraction) run ahead by up to
+// kBatchedStages - 1 tiles instead of waiting at every tile.
+constexpr int kBatchedStages = 4;
+
 template <int D, bool GRAD, int QT, int PU, typename Issue>
-__device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const float* tile, uint64_t* bar,
+__device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const float* tile, uint64_t* full, int* cnt,
                                               double* accsh, const BoxDim (&bd)[QT][D], const float (&ap)[D],
                                               const float2 (&cb)[D], bool cull, int64_t s0, int64_t s1,
                                               int ntiles, int mode, int phase, int R, Issue& issue) {
   const int tid = threadIdx.x;
   for (int k = 0; k < ntiles; ++k) {
-    const int buf = k & 1;
-    if (tid == 0 && k + 1 < ntiles) issue(k + 1);  // buffer buf^1 was released by the barrier ending tile k-1
-    mbar_wait_parity(&bar[buf], (uint32_t)((k >> 1) & 1));
-    const float* tl = tile + buf * D * kTilePts;
+    const int st = k % kBatchedStages;
+    mbar_wait_parity(&full[st], (uint32_t)((k / kBatchedStages) & 1));
+    const float* tl = tile + st * D * kTilePts;
     const int64_t rem = s1 - (s0 + (int64_t)k * kTilePts);
     const int npts = rem < kTilePts ? (int)rem : kTilePts;
     if (cull && mode == 1)
@@ -574,24 +577,33 @@ __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const fl
       batched_tile_compute<D, GRAD, 1, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
     else
       batched_tile_compute<D, GRAD, 0, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
-    __syncthreads();
+    __syncwarp();
+    if ((tid & 31) == 0) {
+      __threadfence_block();  // this warp's reads of the stage precede its arrival
+      if (atomicAdd(&cnt[st], 1) == kBatchedThreads / 32 - 1) {
+        cnt[st] = 0;
+        if (k + kBatchedStages < ntiles) issue(k + kBatchedStages);
+      }
+    }
   }
 }
 
 template <int D, bool GRAD, int QT = QT_for<D>::value>
 constexpr size_t batched_smem_bytes() {
   constexpr int NA = GRAD ? D + 1 : 1;
-  return 2ull * D * kTilePts * sizeof(float) + (size_t)QT * NA * kBatchedThreads * sizeof(double) + 16;
+  return (size_t)kBatchedStages * D * kTilePts * sizeof(float) + (size_t)QT * NA * kBatchedThreads * sizeof(double) +
+         kBatchedStages * (sizeof(uint64_t) + sizeof(int));
 }
 
 template <int D, bool GRAD, int QT = QT_for<D>::value, int MINB = MINB_for<D>::value, int PU = PU_for<D>::value>
 __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(const ScanBatchedArgs a) {
   constexpr int NA = GRAD ? D + 1 : 1;
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  float* tile = reinterpret_cast<float*>(smem_raw);                                   // [2][D][kTilePts]
-  double* accsh = reinterpret_cast<double*>(smem_raw + 2ull * D * kTilePts * sizeof(float));  // [QT*NA][threads]
+  float* tile = reinterpret_cast<float*>(smem_raw);  // [kBatchedStages][D][kTilePts]
+  double* accsh = reinterpret_cast<double*>(smem_raw + (size_t)kBatchedStages * D * kTilePts * sizeof(float));
   uint64_t* bar = reinterpret_cast<uint64_t*>(reinterpret_cast<unsigned char*>(accsh) +
-                                              (size_t)QT * NA * kBatchedThreads * sizeof(double));
+                                              (size_t)QT * NA * kBatchedThreads * sizeof(double));  // full[stages]
+  int* cnt = reinterpret_cast<int*>(bar + kBatchedStages);                                     // [stages]
   const int tid = threadIdx.x;
 
   // This CTA's QB boxes (slots 0..QB-1, box qbase + slot).  With QB < 256 each
@@ -616,6 +628,7 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
   if (tid < QB && !epan) {
     int64_t qi = qbase + tid;
     if (qi >= a.q) qi = a.q - 1;  // duplicate a valid box; its partial is never written
+    if (a.perm) qi = a.perm[qi];
 #pragma unroll
     for (int j = 0; j < D; ++j) {
       const float l = __ldg(a.lo + qi * D + j), u = __ldg(a.hi + qi * D + j);
@@ -655,6 +668,7 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
   {
     int64_t qi = qbase + perm_s[slot];
     if (qi >= a.q) qi = a.q - 1;
+    if (a.perm) qi = a.perm[qi];
     narrow[0] = false;
 #pragma unroll
     for (int j = 0; j < D; ++j) {
@@ -675,13 +689,15 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
   const int64_t s1 = min(a.n, s0 + a.split_len);
   const int ntiles = (int)((s1 - s0 + kTilePts - 1) / kTilePts);
   if (tid == 0) {
-    mbar_init(&bar[0], 1);
-    mbar_init(&bar[1], 1);
+    for (int st = 0; st < kBatchedStages; ++st) {
+      mbar_init(&bar[st], 1);
+      cnt[st] = 0;
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
   auto issue = [&](int k) {
-    const int buf = k & 1;
+    const int buf = k % kBatchedStages;
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     mbar_arrive_expect_tx(&bar[buf], (uint32_t)(D * kTilePts * sizeof(float)));
 #pragma unroll
@@ -689,7 +705,8 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
       bulk_g2s(tile + (buf * D + j) * kTilePts, a.cols + (int64_t)j * a.ld + s0 + (int64_t)k * kTilePts,
                (uint32_t)(kTilePts * sizeof(float)), &bar[buf]);
   };
-  if (tid == 0 && ntiles > 0) issue(0);
+  if (tid == 0)
+    for (int k = 0; k < kBatchedStages && k < ntiles; ++k) issue(k);
 
   // Culling (reading R15, large batches): sort the CTA's boxes by their kept fraction on the
   // split's first tile (narrow-dimension boxes last), so that the lanes of a warp walk alive
@@ -698,7 +715,8 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
   float2 cb[D];
   if (cull) {
     __shared__ int key_s[kBatchedThreads];
-    const int64_t q0 = min(qbase + tid, a.q - 1);
+    int64_t q0 = min(qbase + tid, a.q - 1);
+    if (a.perm) q0 = a.perm[q0];
 #pragma unroll
     for (int j = 0; j < D; ++j)
       cb[j] = make_cullbox(__ldg(a.lo + q0 * D + j), __ldg(a.hi + q0 * D + j), ap[j], a.consts->renc[2 * j],
@@ -736,6 +754,7 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
     perm_s[tid] = sl;
     int64_t qi = qbase + sl;
     if (qi >= a.q) qi = a.q - 1;
+    if (a.perm) qi = a.perm[qi];
     narrow[0] = false;
 #pragma unroll
     for (int j = 0; j < D; ++j) {
@@ -754,14 +773,15 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
 #pragma unroll
   for (int qq = 0; qq < QT; ++qq) my_narrow |= narrow[qq];
   const int mode = epan ? 2 : (__any_sync(0xffffffffu, my_narrow) ? 1 : 0);
-  batched_tiles<D, GRAD, QT, PU>(a, tile, bar, accsh, bd, ap, cb, cull, s0, s1, ntiles, mode, phase, R, issue);
+  batched_tiles<D, GRAD, QT, PU>(a, tile, bar, cnt, accsh, bd, ap, cb, cull, s0, s1, ntiles, mode, phase, R, issue);
 
   // combine the R phases of each box in phase order, then
   // partials[(split*(NA) + comp) * q + qi]
   if (R > 1) __syncthreads();
   if (tid < QB) {
-    const int64_t qi = qbase + perm_s[tid];
-    if (qi < a.q) {
+    const int64_t qs = qbase + perm_s[tid];
+    if (qs < a.q) {
+      const int64_t qi = a.perm ? a.perm[qs] : qs;
 #pragma unroll
       for (int kk = 0; kk < NA; ++kk) {
         double t = 0.0;
