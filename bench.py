@@ -473,7 +473,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
         "config": {"workload": cfg["desc"], "d": d, "n_per_gpu": n, "n_global": n_global, "q": q,
                    "l2": "flushed between timed steps" if flush_l2 else "sample larger than L2",
                    "cuda_graph": bool(graphs is not None),
-                   "cull": ("off" if args.no_cull or cfg.get("kernel") == "epan" else
+                   "cull": ("off" if args.no_cull else
                             "on: (point, box) pairs whose contribution is provably < 2^-64 are skipped (DESIGN R15)"),
                    "clock_sampling": "nvidia-smi every 100 ms over the timed steps"
                                      + (f" + {soak} identical untimed soak steps (timed region < 1 s)" if soak else ""),

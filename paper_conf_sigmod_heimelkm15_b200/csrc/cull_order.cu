@@ -32,15 +32,17 @@ __global__ void cull_probe_kernel(const float* __restrict__ cols, int64_t ld, in
     const float dy = (u - l) * ap[j];
     nar |= dy > 0.0f && dy < kNarrowY;
   }
+  const bool epan = c->kernel == kEpanechnikov;  // cull_score: max_j o_j < 1 instead of sum_j o_j^2 < kCullY2
+  if (epan) nar = false;
   unsigned cnt = 0;
   for (int p = 0; p < nprobe; ++p) {
     float o2 = 0.0f;
     for (int j = 0; j < d; ++j) {
       const float y = fmaf(__ldg(cols + (int64_t)j * ld + p), ap[j], -cb[j].x);
-      const float r = fmaxf(fabsf(y) - cb[j].y, 0.0f);
-      o2 = fmaf(r, r, o2);
+      const float e = fabsf(y) - cb[j].y;
+      o2 = epan ? fmaxf(o2, e) : fmaf(fmaxf(e, 0.0f), fmaxf(e, 0.0f), o2);
     }
-    cnt += o2 < kCullY2 ? 1u : 0u;
+    cnt += o2 < (epan ? cull_limit<true>() : cull_limit<false>()) ? 1u : 0u;
   }
   keys[i] = (nar ? (1u << 12) : 0u) + cnt;
   idx[i] = (int)i;

@@ -268,7 +268,7 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     a.split_len = 0;
     a.partials = nullptr;
     a.perm = nullptr;
-    if (m->cull && m->kernel == KDE_KERNEL_GAUSSIAN && q >= 256) {  // large batches: order boxes by probed cost
+    if (m->cull && q >= 256) {  // large batches: order boxes by probed cost
       const size_t ob = cull_order_bytes(q);
       kde_status st = ensure_bytes(&m->order, &m->order_cap, ob);
       if (st != KDE_OK) return st;

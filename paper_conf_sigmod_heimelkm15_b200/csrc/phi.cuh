@@ -118,19 +118,28 @@ __device__ __forceinline__ float2 make_cullbox(float l, float u, float ap, unsig
 }
 constexpr float kCullY2 = 64.5f;  // cull when sum_j o_j^2 >= 64 (+ slack for the fp32 rounding of the sum)
 
-// sum_j o_j^2 for two points (float2 lanes = points), o_j = max(|t ap - c ap| - hw', 0)
-template <int D>
-__device__ __forceinline__ float2 cull_o2(const float2 (&t)[D], const float (&ap)[D], const float2 (&cb)[D]) {
+// Cull score of two points (float2 lanes = points), with o_j = max(|t ap - c ap| - hw', 0):
+//   Gaussian:      sum_j o_j^2 (y' units), culled when >= kCullY2 (reading R15);
+//   Epanechnikov:  max_j o_j (units of h), culled when >= 1: the point is outside the kernel's
+//                  support in some dimension, so its contribution and gradient are exactly 0.
+template <int D, bool EPAN>
+__device__ __forceinline__ float2 cull_score(const float2 (&t)[D], const float (&ap)[D], const float2 (&cb)[D]) {
   float2 o2 = f2(0.0f);
 #pragma unroll
   for (int j = 0; j < D; ++j) {
     const float2 y = __ffma2_rn(t[j], f2(ap[j]), f2(-cb[j].x));
     const float2 e = __fadd2_rn(make_float2(fabsf(y.x), fabsf(y.y)), f2(-cb[j].y));
-    const float2 r = make_float2(fmaxf(e.x, 0.0f), fmaxf(e.y, 0.0f));
-    o2 = __ffma2_rn(r, r, o2);
+    if (EPAN) {
+      o2 = make_float2(fmaxf(o2.x, e.x), fmaxf(o2.y, e.y));
+    } else {
+      const float2 r = make_float2(fmaxf(e.x, 0.0f), fmaxf(e.y, 0.0f));
+      o2 = __ffma2_rn(r, r, o2);
+    }
   }
   return o2;
 }
+template <bool EPAN>
+__host__ __device__ constexpr float cull_limit() { return EPAN ? 1.0f : kCullY2; }
 
 // erf-difference path: D = 1/2 [erf(z_u) - erf(z_l)], w = y'_l E_l - y'_u E_u.
 // One MUFU.RCP serves the pair: t_u = den_l / (den_u den_l), t_l = den_u / (den_u den_l)

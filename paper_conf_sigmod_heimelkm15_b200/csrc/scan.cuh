@@ -477,7 +477,7 @@ __device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, 
 // fraction within the CTA, see the kernel) with lane-varying LDS gathers from the tile.
 constexpr int kTileWords = kTilePts / 32;
 
-template <int D>
+template <int D, bool EPAN>
 __device__ __forceinline__ void cull_tile_mask(const float* tl, int npts, const float (&ap)[D], const float2 (&cb)[D],
                                                unsigned (&mk)[kTileWords]) {
 #pragma unroll
@@ -489,9 +489,9 @@ __device__ __forceinline__ void cull_tile_mask(const float* tl, int npts, const 
       float2 t[D];
 #pragma unroll
       for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * kTilePts + 2 * pp);
-      const float2 o2 = cull_o2<D>(t, ap, cb);
-      m |= (o2.x < kCullY2 ? 1u : 0u) << (2 * q);
-      m |= (o2.y < kCullY2 ? 1u : 0u) << (2 * q + 1);
+      const float2 o2 = cull_score<D, EPAN>(t, ap, cb);
+      m |= (o2.x < cull_limit<EPAN>() ? 1u : 0u) << (2 * q);
+      m |= (o2.y < cull_limit<EPAN>() ? 1u : 0u) << (2 * q + 1);
     }
     const int v = npts - 32 * w;  // valid points in this word
     mk[w] = v >= 32 ? m : (v > 0 ? m & ((1u << v) - 1u) : 0u);
@@ -512,7 +512,7 @@ __device__ __forceinline__ void batched_tile_cull(const float* tl, int npts, dou
   constexpr int kFlushPairs = kFlushPts / 2;
   const int tid = threadIdx.x;
   unsigned mk[kTileWords];
-  cull_tile_mask<D>(tl, npts, ap, cb, mk);
+  cull_tile_mask<D, MODE == 2>(tl, npts, ap, cb, mk);
   int w = 0;
   unsigned m = mk[0];
   auto next = [&]() -> int {  // next alive point of this lane, -1 when exhausted
@@ -567,7 +567,9 @@ __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const fl
     const float* tl = tile + st * D * kTilePts;
     const int64_t rem = s1 - (s0 + (int64_t)k * kTilePts);
     const int npts = rem < kTilePts ? (int)rem : kTilePts;
-    if (cull && mode == 1)
+    if (cull && mode == 2)
+      batched_tile_cull<D, GRAD, 2>(tl, npts, accsh, bd[0], ap, cb);
+    else if (cull && mode == 1)
       batched_tile_cull<D, GRAD, 1>(tl, npts, accsh, bd[0], ap, cb);
     else if (cull)
       batched_tile_cull<D, GRAD, 0>(tl, npts, accsh, bd[0], ap, cb);
@@ -711,7 +713,7 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
   // Culling (reading R15, large batches): sort the CTA's boxes by their kept fraction on the
   // split's first tile (narrow-dimension boxes last), so that the lanes of a warp walk alive
   // lists of similar length; each thread then takes the box perm_s[tid].
-  const bool cull = a.cull && QB == kBatchedThreads && !epan;
+  const bool cull = a.cull && QB == kBatchedThreads;
   float2 cb[D];
   if (cull) {
     __shared__ int key_s[kBatchedThreads];
@@ -726,7 +728,10 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
       mbar_wait_parity(&bar[0], 0u);
       const int64_t rem = s1 - s0;
       unsigned mk[kTileWords];
-      cull_tile_mask<D>(tile, rem < kTilePts ? (int)rem : kTilePts, ap, cb, mk);
+      if (epan)
+        cull_tile_mask<D, true>(tile, rem < kTilePts ? (int)rem : kTilePts, ap, cb, mk);
+      else
+        cull_tile_mask<D, false>(tile, rem < kTilePts ? (int)rem : kTilePts, ap, cb, mk);
 #pragma unroll
       for (int w = 0; w < kTileWords; ++w) cnt += __popc(mk[w]);
     }
@@ -734,7 +739,7 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
 #pragma unroll
     for (int j = 0; j < D; ++j) {
       const float dy = (__ldg(a.hi + q0 * D + j) - __ldg(a.lo + q0 * D + j)) * ap[j];
-      nar0 |= dy > 0.0f && dy < kNarrowY;
+      nar0 |= !epan && dy > 0.0f && dy < kNarrowY;
     }
     key_s[tid] = ((nar0 ? 512 : 0) + cnt) * kBatchedThreads + tid;  // unique keys: a deterministic order
     __syncthreads();
@@ -759,8 +764,12 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
 #pragma unroll
     for (int j = 0; j < D; ++j) {
       const float l = __ldg(a.lo + qi * D + j), u = __ldg(a.hi + qi * D + j);
-      bd[0][j] = make_boxdim(l, u, ap[j], a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
-      narrow[0] |= bd[0][j].hd > 0.0f;
+      if (epan) {
+        bd[0][j] = make_boxdim<kEpanechnikov>(l, u, ap[j], a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
+      } else {
+        bd[0][j] = make_boxdim(l, u, ap[j], a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
+        narrow[0] |= bd[0][j].hd > 0.0f;
+      }
       cb[j] = make_cullbox(l, u, ap[j], a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
     }
     __syncthreads();

@@ -179,9 +179,9 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
 #pragma unroll
       for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * TILE + 2 * pp);
       // classification in scaled coordinates (make_cullbox / cull_o2, phi.cuh)
-      const float2 o2 = cull_o2<D>(t, ap, cb);
+      const float2 o2 = cull_score<D, MODE == 2>(t, ap, cb);
       const bool val0 = 2 * pp < npts, val1 = 2 * pp + 1 < npts;
-      const bool al0 = val0 && o2.x < kCullY2, al1 = val1 && o2.y < kCullY2;
+      const bool al0 = val0 && o2.x < cull_limit<MODE == 2>(), al1 = val1 && o2.y < cull_limit<MODE == 2>();
       if (a.c_out) {  // culled points retain 0; kept points are overwritten after evaluation (same warp, synced)
         if (val1)
           __stcs(reinterpret_cast<float2*>(a.c_out + base + 2 * pp), f2(0.0f));
@@ -274,6 +274,8 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
                    (uint32_t)(TILE * sizeof(float)), &full[st]);
       }
     }
+  } else if (CULL && a.consts->kernel == kEpanechnikov) {
+    scan_single_cull_body<D, GRAD, 2, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc);
   } else if (a.consts->kernel == kEpanechnikov) {
     scan_single_tma_body<D, GRAD, 2, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
   } else if (CULL) {

@@ -674,3 +674,36 @@ def test_cull_far_box_and_inside_points_never_culled():
     e1 = m.estimate(lo1, hi1)
     assert m.contributions()[i0] > 0.0
     sel_ok(e1, oracle.estimate_grad(S, h, lo1, hi1)[0])
+
+
+@pytest.mark.parametrize("kernel,d,n", [("gauss", 2, 40001), ("gauss", 5, 30011), ("gauss", 9, 9001),
+                                        ("epan", 3, 30011), ("epan", 6, 9001)])
+def test_batched_cull_matches_oracle_and_unculled(kernel, d, n):
+    """Batched scan with culling (q >= 256: probe order + CTA sort + alive-mask walk) and
+    without, against the oracle; special boxes (unbounded, empty, far, narrow) included."""
+    S = synth.make_data("gauss", n, d, seed=60 + d)
+    lo1, hi1 = synth.mixed_workload(S, 300, seed=61 + d)
+    lo2, hi2 = synth.special_boxes(S, seed=62 + d)
+    lo, hi = np.concatenate([lo1, lo2]), np.concatenate([hi1, hi2])
+    m = model(S)
+    if kernel == "epan":
+        m.set_kernel("epan")
+        m.bandwidth = m.bandwidth * np.sqrt(5.0)
+        h = m.bandwidth
+        est_o, g_o = oracle.epan_estimate_grad(S, h, lo, hi)
+        mabs = oracle.epan_grad_abs_scale(S, h, lo, hi)
+    else:
+        h = m.bandwidth
+        est_o, g_o = oracle.estimate_grad(S, h, lo, hi)
+        mabs = oracle.grad_abs_scale(S, h, lo, hi)
+    assert m.cull
+    e1, g1 = m.estimate(lo, hi, grad=True)
+    sel_ok(e1, est_o)
+    grad_ok(g1, g_o, mabs, h)
+    sel_ok(m.estimate(lo, hi), est_o)
+    e1b, g1b = m.estimate(lo, hi, grad=True)          # deterministic schedule: bitwise repeat
+    assert np.array_equal(e1, e1b) and np.array_equal(g1, g1b)
+    m.cull = False
+    e0, g0 = m.estimate(lo, hi, grad=True)
+    sel_ok(e0, est_o)
+    grad_ok(g0, g_o, mabs, h)
