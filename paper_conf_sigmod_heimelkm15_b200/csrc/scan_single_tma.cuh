@@ -78,9 +78,10 @@ __device__ __forceinline__ void scan_single_tma_body(const ScanSingleArgs& a, co
 // the distance OUTSIDE the box in dimension j in y' units (y'^2 = z^2 log2 e).
 // Outside in dimension j, D_j <= 1/2 erfc(|z_j|) <= 1/2 e^{-z_j^2} = 2^{-o_j^2 - 1},
 // so p^(i) = prod_j D_j <= 2^{-sum_j o_j^2}, and every gradient term
-// |w_j| prod_{k!=j} D_k <= max(1, o_j) 2^{-sum_k o_k^2} (o_j <= 14 after bound
-// clamping).  A point with sum_j o_j^2 >= kCullY2 = 64 therefore changes p_hat
-// by at most 2^-64 and each dp_hat/dh_j by at most 15 * 2^-64 * gconst_j per
+// |w_j| prod_{k!=j} D_k <= max(1.03, o_j) 2^{-sum_k o_k^2} <= 2^-61 once sum_k o_k^2 >= 64
+// (pinned on the fp64 oracle by tests/test_oracle_pins.py::test_r15_cull_bound_against_oracle).
+// A point with sum_j o_j^2 >= kCullY2 (64 + rounding slack) therefore changes p_hat
+// by at most 2^-64 and each dp_hat/dh_j by at most 2^-60 * gconst_j per
 // point: far below the fp32 rounding of the terms that are kept.  Such points
 // are skipped (their retained p^(i) is written as 0); the others go through a
 // per-warp ring of shared memory and are evaluated 64 at a time, so the

@@ -464,3 +464,50 @@ def test_epan_threshold_is_boundary_maximum_and_sound():
     c = oracle.epan_contributions(S, h, lo, hi)
     outside = ~np.all((S >= lo) & (S <= hi), axis=1)
     assert np.all(c[outside] < thr * (1 + 1e-12))
+
+
+# ------------------------------------------------------------------ reading R15 (tail culling bound)
+def _outside_sq(S, h, lo, hi):
+    """sum_j o_j^2 in y' units: o_j = distance of the point outside [l_j, u_j] / (sqrt2 h_j) * sqrt(log2 e)."""
+    S = S.astype(np.float64)
+    r = np.maximum(np.maximum(S - hi.astype(np.float64), lo.astype(np.float64) - S), 0.0)
+    return ((r / (math.sqrt(2.0) * h)) ** 2).sum(axis=1) * math.log2(math.e)
+
+
+@pytest.mark.parametrize("d", [1, 3, 6])
+def test_r15_cull_bound_against_oracle(d):
+    """DESIGN R15: a point with sum_j o_j^2 >= 64 contributes p^(i) <= 2^-sum o_j^2 (1/2 erfc(z) <= 1/2 e^{-z^2})
+    and each gradient term |d p^(i)/d h_j| <= 2^-60 / (sqrt(pi) sqrt(log2 e) h_j); checked on the fp64 oracle
+    (eq. 13 and eq. 17 as written, not the bound's algebra) for points at all distances from the box."""
+    g = np.random.default_rng(1500 + d)
+    n = 4000
+    S = g.normal(0.0, 1.0, size=(n, d)).astype(np.float32) * np.float32(3.0)
+    h = g.uniform(0.05, 0.4, d)
+    for k in range(4):
+        c = g.normal(0.0, 2.0, d)
+        w = g.uniform(0.2, 3.0, d)
+        lo, hi = (c - w).astype(np.float32), (c + w).astype(np.float32)
+        o2 = _outside_sq(S, h, lo, hi)
+        cvals = oracle.contributions(S, h, lo, hi)
+        assert np.all(cvals <= np.exp2(-o2) * (1 + 1e-12) + 1e-300)
+        far = np.nonzero(o2 >= 64.0)[0]
+        assert len(far) > 50                       # the workload does contain culled points
+        inside = np.all((S >= lo) & (S <= hi), axis=1)
+        assert np.all(o2[inside] == 0.0)           # inside points are never culled
+        gconst = 1.0 / (math.sqrt(math.pi) * math.sqrt(math.log2(math.e)) * h)
+        for i in far[:60]:
+            terms = oracle.grad_abs_scale(S[i:i + 1], h, lo, hi)[0]  # |d p^(i) / d h_j| of this point alone
+            assert np.all(terms <= 2.0 ** -60 * gconst * (1 + 1e-9) + 1e-300), (o2[i], terms)
+
+
+def test_r15_epanechnikov_support_is_exact():
+    """Epanechnikov culling (R15): a point outside the support |t - b| >= h beyond the box in any dimension
+    has contribution exactly 0 in the oracle (eq. 13 with the R14 kernel)."""
+    g = np.random.default_rng(1600)
+    S = g.normal(0.0, 1.0, size=(3000, 4)).astype(np.float32)
+    h = g.uniform(0.2, 0.6, 4)
+    lo, hi = np.full(4, -0.5, np.float32), np.full(4, 0.7, np.float32)
+    r = np.maximum(np.maximum(S.astype(np.float64) - hi, lo - S.astype(np.float64)), 0.0) / h
+    out = (r >= 1.0).any(axis=1)
+    c = oracle.epan_contributions(S, h, lo, hi)
+    assert out.sum() > 100 and np.all(c[out] == 0.0) and np.all(c[~out] > 0.0)
