@@ -553,7 +553,10 @@ __device__ __forceinline__ void batched_tile_cull(const float* tl, int npts, dou
 // LAST warp out issues the copies of tile k + kBatchedStages into it, so warps
 // with less work (culling: boxes sorted by kept fraction) run ahead by up to
 // kBatchedStages - 1 tiles instead of waiting at every tile.
-constexpr int kBatchedStages = 4;
+#ifndef KDE_TUNE_BATCHED_STAGES
+#define KDE_TUNE_BATCHED_STAGES 4
+#endif
+constexpr int kBatchedStages = KDE_TUNE_BATCHED_STAGES;
 
 template <int D, bool GRAD, int QT, int PU, typename Issue>
 __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const float* tile, uint64_t* full, int* cnt,
