@@ -40,7 +40,7 @@ __global__ void cull_probe_kernel(const float* __restrict__ cols, int64_t ld, in
     for (int j = 0; j < d; ++j) {
       const float y = fmaf(__ldg(cols + (int64_t)j * ld + p), ap[j], -cb[j].x);
       const float e = fabsf(y) - cb[j].y;
-      o2 = epan ? fmaxf(o2, e) : fmaf(fmaxf(e, 0.0f), fmaxf(e, 0.0f), o2);
+      o2 = epan ? fmaxf(o2, e) : fmaf(e + fabsf(e), e + fabsf(e), o2);  // as cull_score (phi.cuh)
     }
     cnt += o2 < (epan ? cull_limit<true>() : cull_limit<false>()) ? 1u : 0u;
   }

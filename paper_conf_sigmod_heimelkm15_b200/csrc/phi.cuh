@@ -119,7 +119,7 @@ __device__ __forceinline__ float2 make_cullbox(float l, float u, float ap, unsig
 constexpr float kCullY2 = 64.5f;  // cull when sum_j o_j^2 >= 64 (+ slack for the fp32 rounding of the sum)
 
 // Cull score of two points (float2 lanes = points), with o_j = max(|t ap - c ap| - hw', 0):
-//   Gaussian:      sum_j o_j^2 (y' units), culled when >= kCullY2 (reading R15);
+//   Gaussian:      4 sum_j o_j^2 (y' units), culled when >= 4 kCullY2 (reading R15);
 //   Epanechnikov:  max_j o_j (units of h), culled when >= 1: the point is outside the kernel's
 //                  support in some dimension, so its contribution and gradient are exactly 0.
 template <int D, bool EPAN>
@@ -131,15 +131,15 @@ __device__ __forceinline__ float2 cull_score(const float2 (&t)[D], const float (
     const float2 e = __fadd2_rn(make_float2(fabsf(y.x), fabsf(y.y)), f2(-cb[j].y));
     if (EPAN) {
       o2 = make_float2(fmaxf(o2.x, e.x), fmaxf(o2.y, e.y));
-    } else {
-      const float2 r = make_float2(fmaxf(e.x, 0.0f), fmaxf(e.y, 0.0f));
+    } else {  // r = e + |e| = 2 max(e, 0) exactly (one packed op instead of two FMNMX): the sum is 4 sum_j o_j^2
+      const float2 r = __fadd2_rn(e, make_float2(fabsf(e.x), fabsf(e.y)));
       o2 = __ffma2_rn(r, r, o2);
     }
   }
   return o2;
 }
 template <bool EPAN>
-__host__ __device__ constexpr float cull_limit() { return EPAN ? 1.0f : kCullY2; }
+__host__ __device__ constexpr float cull_limit() { return EPAN ? 1.0f : 4.0f * kCullY2; }
 
 // erf-difference path: D = 1/2 [erf(z_u) - erf(z_l)], w = y'_l E_l - y'_u E_u.
 // One MUFU.RCP serves the pair: t_u = den_l / (den_u den_l), t_l = den_u / (den_u den_l)

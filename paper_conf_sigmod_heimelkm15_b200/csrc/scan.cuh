@@ -489,9 +489,10 @@ __device__ __forceinline__ void cull_tile_mask(const float* tl, int npts, const 
       float2 t[D];
 #pragma unroll
       for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * kTilePts + 2 * pp);
-      const float2 o2 = cull_score<D, EPAN>(t, ap, cb);
-      m |= (o2.x < cull_limit<EPAN>() ? 1u : 0u) << (2 * q);
-      m |= (o2.y < cull_limit<EPAN>() ? 1u : 0u) << (2 * q + 1);
+      // kept <=> score - limit < 0: the sign bits are the mask bits (finite scores, exact sign)
+      const float2 u = __fadd2_rn(cull_score<D, EPAN>(t, ap, cb), f2(-cull_limit<EPAN>()));
+      m |= (__float_as_uint(u.x) >> 31) << (2 * q);
+      m |= (__float_as_uint(u.y) >> 31) << (2 * q + 1);
     }
     const int v = npts - 32 * w;  // valid points in this word
     mk[w] = v >= 32 ? m : (v > 0 ? m & ((1u << v) - 1u) : 0u);
