@@ -176,7 +176,7 @@ kde_status kde_set_retain(kde_model *m, int32_t on);
  * j in units of sqrt2 h_j / sqrt(log2 e), D_j <= 1/2 erfc(z_j) <= 2^{-o_j^2}, so
  * sum_j o_j^2 >= 64 bounds its contribution to p_hat by 2^-64 and to each
  * dp_hat/dh_j by 2^-60 / (sqrt(pi) sqrt(log2 e) h_j) (R15).  Both the
- * single-box scan and the batched scan (q >= 256) cull; for the Epanechnikov kernel
+ * single-box scan and the batched scan (batches that fill 256-box CTAs) cull; for the Epanechnikov kernel
  * a point outside the support in some dimension is skipped (exactly 0).  A
  * skipped point's retained p^(i) is 0.  Points inside the box are never
  * skipped.  on == 0: every point is evaluated.  Errors: none (KDE_EINVAL for

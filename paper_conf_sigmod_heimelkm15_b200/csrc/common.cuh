@@ -109,5 +109,6 @@ cudaError_t launch_scan_single(int d, bool grad, const ScanSingleArgs& a, int gr
 cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int num_sms, int* splits_out,
                                 cudaStream_t s, bool dry_run);
 int scan_single_grid(int d, bool grad, int64_t n, int num_sms, bool cull);
+bool batched_culls(int64_t q);
 
 }  // namespace kde

@@ -264,11 +264,11 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     a.hi = d_hi;
     a.q = q;
     a.consts = m->consts;
-    a.cull = m->cull ? 1 : 0;
+    a.cull = (m->cull && batched_culls(q)) ? 1 : 0;  // full CTAs only (measured: phased culling gains nothing)
     a.split_len = 0;
     a.partials = nullptr;
     a.perm = nullptr;
-    if (m->cull && q >= 256) {  // large batches: order boxes by probed cost
+    if (a.cull) {  // order boxes by probed cost
       const size_t ob = cull_order_bytes(q);
       kde_status st = ensure_bytes(&m->order, &m->order_cap, ob);
       if (st != KDE_OK) return st;

@@ -477,11 +477,14 @@ __device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, 
 // fraction within the CTA, see the kernel) with lane-varying LDS gathers from the tile.
 constexpr int kTileWords = kTilePts / 32;
 
+// phase / R: with R threads per box (small batches) the thread owns the words w = phase (mod R)
 template <int D, bool EPAN>
 __device__ __forceinline__ void cull_tile_mask(const float* tl, int npts, const float (&ap)[D], const float2 (&cb)[D],
-                                               unsigned (&mk)[kTileWords]) {
+                                               unsigned (&mk)[kTileWords], int phase = 0, int R = 1) {
 #pragma unroll
   for (int w = 0; w < kTileWords; ++w) {
+    mk[w] = 0u;
+    if ((w & (R - 1)) != phase) continue;  // warp-uniform: a warp holds one phase (QB >= 32)
     unsigned m = 0u;
 #pragma unroll 4
     for (int q = 0; q < 16; ++q) {
@@ -508,12 +511,12 @@ __device__ __forceinline__ unsigned sel_word(const unsigned (&mk)[kTileWords], i
 
 template <int D, bool GRAD, int MODE>
 __device__ __forceinline__ void batched_tile_cull(const float* tl, int npts, double* accsh, const BoxDim (&bd)[D],
-                                                  const float (&ap)[D], const float2 (&cb)[D]) {
+                                                  const float (&ap)[D], const float2 (&cb)[D], int phase, int R) {
   constexpr int NA = GRAD ? D + 1 : 1;
   constexpr int kFlushPairs = kFlushPts / 2;
   const int tid = threadIdx.x;
   unsigned mk[kTileWords];
-  cull_tile_mask<D, MODE == 2>(tl, npts, ap, cb, mk);
+  cull_tile_mask<D, MODE == 2>(tl, npts, ap, cb, mk, phase, R);
   int w = 0;
   unsigned m = mk[0];
   auto next = [&]() -> int {  // next alive point of this lane, -1 when exhausted
@@ -572,11 +575,11 @@ __device__ __forceinline__ void batched_tiles(const ScanBatchedArgs& a, const fl
     const int64_t rem = s1 - (s0 + (int64_t)k * kTilePts);
     const int npts = rem < kTilePts ? (int)rem : kTilePts;
     if (cull && mode == 2)
-      batched_tile_cull<D, GRAD, 2>(tl, npts, accsh, bd[0], ap, cb);
+      batched_tile_cull<D, GRAD, 2>(tl, npts, accsh, bd[0], ap, cb, phase, R);
     else if (cull && mode == 1)
-      batched_tile_cull<D, GRAD, 1>(tl, npts, accsh, bd[0], ap, cb);
+      batched_tile_cull<D, GRAD, 1>(tl, npts, accsh, bd[0], ap, cb, phase, R);
     else if (cull)
-      batched_tile_cull<D, GRAD, 0>(tl, npts, accsh, bd[0], ap, cb);
+      batched_tile_cull<D, GRAD, 0>(tl, npts, accsh, bd[0], ap, cb, phase, R);
     else if (mode == 2)
       batched_tile_compute<D, GRAD, 2, QT, PU>(tl, npts, phase, R, accsh, bd, ap);
     else if (mode == 1)
@@ -717,9 +720,20 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
   // Culling (reading R15, large batches): sort the CTA's boxes by their kept fraction on the
   // split's first tile (narrow-dimension boxes last), so that the lanes of a warp walk alive
   // lists of similar length; each thread then takes the box perm_s[tid].
-  const bool cull = a.cull && QB == kBatchedThreads;
+  // culling with R > 1 threads per box (phases own alternate mask words) is supported, but measured
+  // no faster than the unculled small-batch path, so the host enables it for full CTAs only
+  const bool cull = a.cull && QB >= 32;  // R <= kTileWords threads per box
   float2 cb[D];
-  if (cull) {
+  if (cull && R > 1) {  // small batches: the narrow/normal partition order, no re-sort
+    int64_t qi = qbase + perm_s[slot];
+    if (qi >= a.q) qi = a.q - 1;
+    if (a.perm) qi = a.perm[qi];
+#pragma unroll
+    for (int j = 0; j < D; ++j)
+      cb[j] = make_cullbox(__ldg(a.lo + qi * D + j), __ldg(a.hi + qi * D + j), ap[j], a.consts->renc[2 * j],
+                           a.consts->renc[2 * j + 1]);
+  }
+  if (cull && R == 1) {
     __shared__ int key_s[kBatchedThreads];
     int64_t q0 = min(qbase + tid, a.q - 1);
     if (a.perm) q0 = a.perm[q0];

@@ -31,6 +31,9 @@ cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int 
   return cudaErrorInvalidValue;
 }
 
+// the batched scan culls (and wants the probe order) when a CTA holds 256 boxes (one thread per box)
+bool batched_culls(int64_t q) { return batched_qb(q) == kBatchedThreads; }
+
 // ~3 resident CTAs of 256 threads per SM, never more CTAs than 8-point work items.
 int scan_single_grid(int d, bool grad, int64_t n, int num_sms, bool cull) {
   if (cull) {  // culled TMA variant: one contiguous chunk of >= 1 tile per CTA

@@ -486,10 +486,12 @@ def test_device_resident_stream_matches_host_path_and_oracle():
     assert np.array_equal(md.sample, mh.sample) and np.array_equal(mf.sample, mh.sample)
 
 
-def test_batched_mixed_narrow_and_normal_boxes():
+@pytest.mark.parametrize("q", [700, 768])
+def test_batched_mixed_narrow_and_normal_boxes(q):
     """Every third box has a dimension narrower than the Gauss-path threshold;
-    the CTA-local partition must return each box's result at its own index."""
-    n, d, q = 30000, 3, 700
+    the CTA-local partition (q = 700) or the culled path's probe order and sort
+    (q = 768, full 256-box CTAs) must return each box's result at its own index."""
+    n, d = 30000, 3
     S = synth.make_data("gauss", n, d, seed=50)
     m = model(S)
     h = m.bandwidth
@@ -682,8 +684,8 @@ def test_batched_cull_matches_oracle_and_unculled(kernel, d, n):
     """Batched scan with culling (q >= 256: probe order + CTA sort + alive-mask walk) and
     without, against the oracle; special boxes (unbounded, empty, far, narrow) included."""
     S = synth.make_data("gauss", n, d, seed=60 + d)
-    lo1, hi1 = synth.mixed_workload(S, 300, seed=61 + d)
     lo2, hi2 = synth.special_boxes(S, seed=62 + d)
+    lo1, hi1 = synth.mixed_workload(S, 512 - len(lo2), seed=61 + d)  # 512 boxes: full 256-box CTAs cull
     lo, hi = np.concatenate([lo1, lo2]), np.concatenate([hi1, hi2])
     m = model(S)
     if kernel == "epan":
