@@ -15,13 +15,16 @@ import paper_conf_sigmod_heimelkm15_b200 as K  # noqa: E402
 import synth  # noqa: E402
 
 
-def run(d, n, q):
+def run(d, n, q, kernel="gauss"):
+    """q = 0: a batch of exactly 512 boxes (full 256-box CTAs: the culled batched scan)."""
     S = synth.make_data("gauss", n, d, seed=d)
-    lo, hi = synth.mixed_workload(S, q, seed=d + 1)
     lo2, hi2 = synth.special_boxes(S, seed=d + 2)
+    lo, hi = synth.mixed_workload(S, q if q else 512 - len(lo2), seed=d + 1)
     lo, hi = np.concatenate([lo, lo2]), np.concatenate([hi, hi2])
     p = synth.true_selectivity_cpu(S, lo, hi)
     m = K.KDEModel.create(S)
+    if kernel == "epan":
+        m.set_kernel("epan")
     m.set_retain(True)
     m.estimate(lo, hi, grad=True)
     m.estimate(lo, hi)
@@ -57,6 +60,7 @@ def run(d, n, q):
 
 
 if __name__ == "__main__":
-    for d, n, q in [(3, 5003, 40), (10, 3001, 17), (13, 2053, 9)]:
-        run(d, n, q)
+    for d, n, q, kern in [(3, 5003, 40, "gauss"), (10, 3001, 17, "gauss"), (13, 2053, 9, "gauss"),
+                          (3, 9001, 0, "gauss"), (5, 4099, 0, "epan"), (10, 2051, 0, "gauss")]:
+        run(d, n, q, kern)
     print("sanitize run ok")
