@@ -348,7 +348,10 @@ __global__ void karma_kernel(const float* __restrict__ cvals, double* __restrict
   const double thr = thr_s;
   const int64_t base = (int64_t)blockIdx.x * kKarmaPts;
   constexpr int P = kKarmaPts / kKarmaThreads;
-  constexpr int PB = 8;  // points per load batch (PB loads of c and K in flight per thread)
+#ifndef KDE_TUNE_KARMA_PB
+#define KDE_TUNE_KARMA_PB 8
+#endif
+  constexpr int PB = KDE_TUNE_KARMA_PB;  // points per load batch (PB loads of c and K in flight per thread)
   const double inv_nm1 = 1.0 / (n_global - 1.0);
   int32_t my = 0;
 #pragma unroll 1

@@ -120,16 +120,32 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   float* qt = queue + (size_t)warp * kCullRing * (D + 1);  // [D][kCullRing] coordinates
   int* qi = reinterpret_cast<int*>(qt + D * kCullRing);     // [kCullRing] point offset from c0
+  // d >= 9: the box constants (5 d floats) are re-read from shared memory (broadcast) where they are
+  // used instead of living in registers for the whole scan, which keeps wide gradient scans at two
+  // CTAs per SM; narrower boxes keep them in registers.
+  constexpr bool kReload = D >= 9;
   BoxDim bd[D];
   float ap[D];
   float2 cb[D];  // (c ap, hw' ap) of the clamped box, for the classification
+  auto load_box = [&]() {
 #pragma unroll
-  for (int j = 0; j < D; ++j) {
-    const float4 c = smc[j];
-    bd[j].b = make_float2(c.x, c.y);
-    bd[j].hd = c.z;
-    ap[j] = c.w;
-    cb[j] = scb[j];
+    for (int j = 0; j < D; ++j) {
+      const float4 c = smc[j];
+      bd[j].b = make_float2(c.x, c.y);
+      bd[j].hd = c.z;
+      ap[j] = c.w;
+    }
+  };
+  auto load_cb = [&]() {
+#pragma unroll
+    for (int j = 0; j < D; ++j) {
+      cb[j] = scb[j];
+      ap[j] = smc[j].w;
+    }
+  };
+  if (!kReload) {
+    load_box();
+    load_cb();
   }
   const unsigned lt = (1u << lane) - 1u;
   unsigned head = 0, tail = 0;  // warp-uniform ring positions (head is a multiple of 64)
@@ -140,6 +156,7 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
 
   // evaluate ring entries head + [0, 64): lane takes entries 2 lane, 2 lane + 1 (one LDS.64 per column)
   auto process = [&](int cnt) {
+    if (kReload) load_box();
     const int e = (int)(head & (kCullRing - 1)) + 2 * lane;
     const bool v0 = 2 * lane < cnt, v1 = 2 * lane + 1 < cnt;
     float2 t[D];
@@ -179,7 +196,8 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
       float2 t[D];
 #pragma unroll
       for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * TILE + 2 * pp);
-      // classification in scaled coordinates (make_cullbox / cull_o2, phi.cuh)
+      if (kReload) load_cb();
+      // classification in scaled coordinates (make_cullbox / cull_score, phi.cuh)
       const float2 o2 = cull_score<D, MODE == 2>(t, ap, cb);
       const bool val0 = 2 * pp < npts, val1 = 2 * pp + 1 < npts;
       const bool al0 = val0 && o2.x < cull_limit<MODE == 2>(), al1 = val1 && o2.y < cull_limit<MODE == 2>();
