@@ -17,11 +17,13 @@ namespace kde {
 
 constexpr int kProbe = 1024;
 
+// one warp per box: the lanes split the probe points, the count is a warp sum
 __global__ void cull_probe_kernel(const float* __restrict__ cols, int64_t ld, int nprobe, int d,
                                   const float* __restrict__ lo, const float* __restrict__ hi, int64_t q,
                                   const DevConsts* __restrict__ c, unsigned* __restrict__ keys, int* __restrict__ idx) {
-  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= q) return;
+  const int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  if (i >= q) return;  // warp-uniform
   float2 cb[kMaxDim];
   float ap[kMaxDim];
   bool nar = false;
@@ -35,7 +37,7 @@ __global__ void cull_probe_kernel(const float* __restrict__ cols, int64_t ld, in
   const bool epan = c->kernel == kEpanechnikov;  // cull_score: max_j o_j < 1 instead of sum_j o_j^2 < kCullY2
   if (epan) nar = false;
   unsigned cnt = 0;
-  for (int p = 0; p < nprobe; ++p) {
+  for (int p = lane; p < nprobe; p += 32) {
     float o2 = 0.0f;
     for (int j = 0; j < d; ++j) {
       const float y = fmaf(__ldg(cols + (int64_t)j * ld + p), ap[j], -cb[j].x);
@@ -44,8 +46,11 @@ __global__ void cull_probe_kernel(const float* __restrict__ cols, int64_t ld, in
     }
     cnt += o2 < (epan ? cull_limit<true>() : cull_limit<false>()) ? 1u : 0u;
   }
-  keys[i] = (nar ? (1u << 12) : 0u) + cnt;
-  idx[i] = (int)i;
+  for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
+  if (lane == 0) {
+    keys[i] = (nar ? (1u << 12) : 0u) + cnt;
+    idx[i] = (int)i;
+  }
 }
 
 // scratch layout: keys_in [q] u32, keys_out [q] u32, idx_in [q] i32, perm [q] i32, cub temp
@@ -66,7 +71,7 @@ cudaError_t launch_cull_order(const float* cols, int64_t ld, int64_t n, int d, c
   void* temp = reinterpret_cast<void*>(((uintptr_t)(perm + q) + 255) & ~(uintptr_t)255);
   size_t temp_bytes = scratch_bytes - ((char*)temp - (char*)scratch);
   const int nprobe = (int)(n < kProbe ? n : kProbe);
-  cull_probe_kernel<<<(unsigned)((q + 127) / 128), 128, 0, s>>>(cols, ld, nprobe, d, lo, hi, q, c, kin, iin);
+  cull_probe_kernel<<<(unsigned)((q * 32 + 255) / 256), 256, 0, s>>>(cols, ld, nprobe, d, lo, hi, q, c, kin, iin);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   e = cub::DeviceRadixSort::SortPairs(temp, temp_bytes, kin, kout, iin, perm, (int)q, 0, 13, s);
