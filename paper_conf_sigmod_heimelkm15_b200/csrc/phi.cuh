@@ -116,6 +116,9 @@ __device__ __forceinline__ float2 make_cullbox(float l, float u, float ap, unsig
   const double err = ldexp(2.0 * fabs(cap) + hwap + tabs, -22) + 1e-30;
   return make_float2((float)cap, (float)(hwap + err));
 }
+// culling is only sound when the scaled box is representable in fp32 (|c ap|, hw' < 2^127): with
+// extreme bandwidths and offsets (e.g. h = 1e-30, |t| = 1e9) the caller disables it for that box
+__device__ __forceinline__ bool cullbox_ok(float2 cb) { return fabsf(cb.x) < 1.0e38f && cb.y < 1.0e38f; }
 constexpr float kCullY2 = 64.5f;  // cull when sum_j o_j^2 >= 64 (+ slack for the fp32 rounding of the sum)
 
 // Cull score of two points (float2 lanes = points), with o_j = max(|t ap - c ap| - hw', 0):

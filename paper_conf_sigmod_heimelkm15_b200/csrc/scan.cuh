@@ -480,7 +480,8 @@ constexpr int kTileWords = kTilePts / 32;
 // phase / R: with R threads per box (small batches) the thread owns the words w = phase (mod R)
 template <int D, bool EPAN>
 __device__ __forceinline__ void cull_tile_mask(const float* tl, int npts, const float (&ap)[D], const float2 (&cb)[D],
-                                               unsigned (&mk)[kTileWords], int phase = 0, int R = 1) {
+                                               unsigned (&mk)[kTileWords], int phase = 0, int R = 1,
+                                               bool keep_all = false) {
 #pragma unroll
   for (int w = 0; w < kTileWords; ++w) {
     mk[w] = 0u;
@@ -497,6 +498,7 @@ __device__ __forceinline__ void cull_tile_mask(const float* tl, int npts, const 
       m |= (__float_as_uint(u.x) >> 31) << (2 * q);
       m |= (__float_as_uint(u.y) >> 31) << (2 * q + 1);
     }
+    if (keep_all) m = 0xffffffffu;  // box not representable in fp32 scaled coordinates: no culling
     const int v = npts - 32 * w;  // valid points in this word
     mk[w] = v >= 32 ? m : (v > 0 ? m & ((1u << v) - 1u) : 0u);
   }
@@ -512,11 +514,14 @@ __device__ __forceinline__ unsigned sel_word(const unsigned (&mk)[kTileWords], i
 template <int D, bool GRAD, int MODE>
 __device__ __forceinline__ void batched_tile_cull(const float* tl, int npts, double* accsh, const BoxDim (&bd)[D],
                                                   const float (&ap)[D], const float2 (&cb)[D], int phase, int R) {
+  bool keep_all = false;
+#pragma unroll
+  for (int j = 0; j < D; ++j) keep_all |= !cullbox_ok(cb[j]);
   constexpr int NA = GRAD ? D + 1 : 1;
   constexpr int kFlushPairs = kFlushPts / 2;
   const int tid = threadIdx.x;
   unsigned mk[kTileWords];
-  cull_tile_mask<D, MODE == 2>(tl, npts, ap, cb, mk, phase, R);
+  cull_tile_mask<D, MODE == 2>(tl, npts, ap, cb, mk, phase, R, keep_all);
   int w = 0;
   unsigned m = mk[0];
   auto next = [&]() -> int {  // next alive point of this lane, -1 when exhausted

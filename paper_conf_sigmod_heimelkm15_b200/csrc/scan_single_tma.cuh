@@ -113,7 +113,7 @@ constexpr size_t single_tma_kernel_smem() {
 template <int D, bool GRAD, int MODE, int TILE, int STAGES>
 __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, const float4* smc, const float2* scb,
                                                       float* tiles, uint64_t* full, uint64_t* empty, float* queue,
-                                                      int64_t c0, int64_t c1, int ntiles, double* acc) {
+                                                      int64_t c0, int64_t c1, int ntiles, double* acc, bool keep_all) {
   constexpr int NA = GRAD ? D + 1 : 1;
   constexpr int PPT = TILE / kSingleThreads;  // points per thread per tile
   static_assert(PPT % 2 == 0, "points are classified in pairs");
@@ -200,7 +200,8 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
       // classification in scaled coordinates (make_cullbox / cull_score, phi.cuh)
       const float2 o2 = cull_score<D, MODE == 2>(t, ap, cb);
       const bool val0 = 2 * pp < npts, val1 = 2 * pp + 1 < npts;
-      const bool al0 = val0 && o2.x < cull_limit<MODE == 2>(), al1 = val1 && o2.y < cull_limit<MODE == 2>();
+      const bool al0 = val0 && (keep_all || o2.x < cull_limit<MODE == 2>()),
+                 al1 = val1 && (keep_all || o2.y < cull_limit<MODE == 2>());
       if (a.c_out) {  // culled points retain 0; kept points are overwritten after evaluation (same warp, synced)
         if (val1)
           __stcs(reinterpret_cast<float2*>(a.c_out + base + 2 * pp), f2(0.0f));
@@ -246,7 +247,7 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
   float* queue = reinterpret_cast<float*>(smem_raw + single_tma_smem_bytes<D, TILE, STAGES>());
   __shared__ float4 smc[D];
   __shared__ float2 scb[D];
-  __shared__ int narrow_s;
+  __shared__ int narrow_s, nocull_s;
   const int tid = threadIdx.x;
   const bool producer = tid >= kSingleThreads;
   // contiguous chunk of this CTA, a multiple of TILE points
@@ -257,6 +258,7 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
   const int ntiles = c1 > c0 ? (int)((c1 - c0 + TILE - 1) / TILE) : 0;
   if (tid == 0) {
     narrow_s = 0;
+    nocull_s = 0;
     for (int st = 0; st < STAGES; ++st) {
       mbar_init(&full[st], 1);
       mbar_init(&empty[st], kSingleComputeWarps);
@@ -274,7 +276,10 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
                                          a.consts->renc[2 * j + 1]);
     smc[j] = make_float4(bd.b.x, bd.b.y, bd.hd, ap);
     if (!epan && bd.hd > 0.0f) atomicOr(&narrow_s, 1);
-    if (CULL) scb[j] = make_cullbox(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
+    if (CULL) {
+      scb[j] = make_cullbox(__ldg(a.lo + j), __ldg(a.hi + j), ap, a.consts->renc[2 * j], a.consts->renc[2 * j + 1]);
+      if (!cullbox_ok(scb[j])) atomicOr(&nocull_s, 1);
+    }
   }
   __syncthreads();
   double acc[NA];
@@ -294,14 +299,17 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
       }
     }
   } else if (CULL && a.consts->kernel == kEpanechnikov) {
-    scan_single_cull_body<D, GRAD, 2, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc);
+    scan_single_cull_body<D, GRAD, 2, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc,
+                                                    nocull_s != 0);
   } else if (a.consts->kernel == kEpanechnikov) {
     scan_single_tma_body<D, GRAD, 2, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
   } else if (CULL) {
     if (narrow_s)
-      scan_single_cull_body<D, GRAD, 1, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc);
+      scan_single_cull_body<D, GRAD, 1, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc,
+                                                      nocull_s != 0);
     else
-      scan_single_cull_body<D, GRAD, 0, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc);
+      scan_single_cull_body<D, GRAD, 0, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc,
+                                                      nocull_s != 0);
   } else if (narrow_s) {
     scan_single_tma_body<D, GRAD, 1, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
   } else {

@@ -709,3 +709,24 @@ def test_batched_cull_matches_oracle_and_unculled(kernel, d, n):
     e0, g0 = m.estimate(lo, hi, grad=True)
     sel_ok(e0, est_o)
     grad_ok(g0, g_o, mabs, h)
+
+
+def test_cull_disabled_when_scaled_box_overflows():
+    """h = 1e-30 with coordinates near 1e9: c ap overflows fp32, so culling is disabled for those boxes
+    (cullbox_ok); estimates still equal the h -> 0 limit (exact count) and the oracle."""
+    g = synth.rng(77)
+    n, d = 5003, 2
+    # float32 spacing near 1e9 is 64: points on a 128 grid, bounds halfway between (exactly representable)
+    S = (1.0e9 + 128.0 * g.integers(0, 2000, size=(n, d))).astype(np.float32)
+    h = np.full(d, 1e-30)
+    m = model(S, h)
+    lo = (1.0e9 + 128.0 * g.integers(0, 1000, size=(512, d)) + 64.0).astype(np.float32)
+    hi = (lo.astype(np.float64) + 128.0 * g.integers(1, 800, size=(512, d))).astype(np.float32)
+    est_o, _ = oracle.estimate_grad(S, h, lo, hi)
+    cnt = np.array([np.all((S > lo[k]) & (S < hi[k]), axis=1).sum() for k in range(len(lo))]) / n
+    assert np.allclose(est_o, cnt, rtol=0, atol=1e-12)
+    for cull in (True, False):
+        m.cull = cull
+        sel_ok(m.estimate(lo, hi), est_o)                  # batched (512 boxes: full culled CTAs)
+        for k in (0, 7, 300):
+            sel_ok(m.estimate(lo[k:k + 1], hi[k:k + 1]), est_o[k:k + 1])
