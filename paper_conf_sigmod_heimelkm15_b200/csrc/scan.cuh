@@ -3,7 +3,8 @@
 //   S_j   = sum_i w_ij prod_{k!=j} D_ik                eq. (17), P:L545 (d p^(i)/d h_j = gconst_j S_j-term)
 // and optionally the retained per-point contributions p^(i).
 //
-// scan_single_kernel  (q == 1): HBM-streaming reduction.  Each thread owns
+// q == 1 with culling (default): scan_single_tma_kernel<..., CULL=1> (scan_single_tma.cuh).
+// scan_single_kernel  (q == 1, cull off, d > 8): HBM-streaming reduction.  Each thread owns
 //   float4 chunks of the SoA columns (coalesced 128-bit loads, streaming cache
 //   hint), fp32 math per point, fp32 sums over 8 points flushed to fp64,
 //   warp-shuffle + block reduction, and a deterministic last-block second pass
@@ -12,7 +13,10 @@
 //   (bounds in registers; 256/QB threads share a box and split its points)
 //   and one contiguous split of the sample; sample
 //   tiles of 256 points x d columns are staged into shared memory by TMA bulk
-//   copies (cp.async.bulk + mbarrier, double buffered) and read as broadcasts.
+//   copies (cp.async.bulk + mbarrier, a 4-stage ring refilled by the last warp
+//   out, no CTA barrier) and read as broadcasts.  Batches that fill 256-box CTAs
+//   are culled (reading R15): boxes ordered by a probed kept count (cull_order.cu)
+//   and re-sorted in the CTA, per-tile alive masks, lane-local alive walks.
 //   fp32 sums over 32 points are flushed into per-thread fp64 accumulators in
 //   shared memory; per-(split, box) partials go to global memory and are
 //   reduced in fixed split order by reduce_splits_kernel (kernels.cu).
