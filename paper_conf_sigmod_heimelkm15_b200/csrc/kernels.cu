@@ -330,7 +330,10 @@ __device__ double thr20_dev(const float* lo, const float* hi, int d, const DevCo
   return pmax * best;
 }
 
-__global__ void karma_kernel(const float* __restrict__ cvals, double* __restrict__ karma, int64_t n, double n_global,
+#ifndef KDE_TUNE_KARMA_MINB
+#define KDE_TUNE_KARMA_MINB 4  // 64 registers, 4 blocks per SM (r77 A/B: 26.7 -> 24.6 us at n = 2^22)
+#endif
+__global__ void __launch_bounds__(kKarmaThreads, KDE_TUNE_KARMA_MINB) karma_kernel(const float* __restrict__ cvals, double* __restrict__ karma, int64_t n, double n_global,
                              const double* __restrict__ phat_ptr, const double* __restrict__ p_ptr, KarmaParamsDev kp,
                              const float* lo,
                              const float* hi, int d, const DevConsts* c, uint32_t* __restrict__ bitmap,
@@ -402,12 +405,16 @@ __device__ __noinline__ void online_update_body(const double* __restrict__ ret, 
 // last block to finish writes the total and runs the optional tail of a
 // device-resident streaming step: the Listing 1 bandwidth update and the
 // replacement of the first min(total, cap) flagged points by tail.rows.
-__global__ void compact_fused_kernel(const uint32_t* __restrict__ bitmap, int64_t n, const int32_t* __restrict__ counts,
+#ifndef KDE_TUNE_COMPACT_MINB
+#define KDE_TUNE_COMPACT_MINB 8
+#endif
+__global__ void __launch_bounds__(kKarmaThreads, KDE_TUNE_COMPACT_MINB) compact_fused_kernel(const uint32_t* __restrict__ bitmap, int64_t n, const int32_t* __restrict__ counts,
                                      int nb, int64_t row_offset, int64_t* __restrict__ idx_out, int64_t cap,
                                      int64_t* __restrict__ total_out, unsigned* __restrict__ done, StreamTail tail) {
   constexpr int W = kKarmaPts / 32;  // bitmap words per block
   constexpr int WPL = W / 32;
   __shared__ int32_t wpre[W];
+  __shared__ uint32_t wbits[W];  // the block's bitmap words, read once by warp 0
   __shared__ int64_t red[kKarmaThreads / 32];
   __shared__ int64_t off_s;
   __shared__ bool last_s;
@@ -424,7 +431,9 @@ __global__ void compact_fused_kernel(const uint32_t* __restrict__ bitmap, int64_
 #pragma unroll
     for (int k = 0; k < WPL; ++k) {
       const int64_t w = wbase + WPL * lane + k;
-      c[k] = w < nwords ? __popc(bitmap[w]) : 0;
+      const uint32_t word = w < nwords ? bitmap[w] : 0u;
+      wbits[WPL * lane + k] = word;
+      c[k] = __popc(word);
       tot += c[k];
     }
     int incl = tot;
@@ -448,9 +457,9 @@ __global__ void compact_fused_kernel(const uint32_t* __restrict__ bitmap, int64_
   }
   __syncthreads();
   const int64_t off = off_s;
+#pragma unroll 4
   for (int w = warp; w < W; w += kKarmaThreads / 32) {
-    if (wbase + w >= nwords) break;
-    const uint32_t word = bitmap[wbase + w];
+    const uint32_t word = wbits[w];  // 0 past the end of the bitmap
     if (word & (1u << lane)) {
       const int64_t pos = off + wpre[w] + __popc(word & ((1u << lane) - 1u));
       if (pos < cap) idx_out[pos] = row_offset + (wbase + w) * 32 + lane;
@@ -486,15 +495,24 @@ __global__ void compact_fused_kernel(const uint32_t* __restrict__ bitmap, int64_
     }
     __syncthreads();
     const int64_t k = min(off_s, cap);
-    for (int64_t e = tid; e < k * tail.d; e += kKarmaThreads) {
-      const int64_t r = e / tail.d;
-      const int j = (int)(e - r * tail.d);
+    const float* __restrict__ rows = tail.rows;
+    float* __restrict__ cols = tail.cols;
+    // one flagged point per thread: its index and all d coordinates are loaded before any
+    // store, so the block waits for ~2 memory latencies instead of 2 per (point, dim) pass
+    for (int64_t r = tid; r < k; r += kKarmaThreads) {
       const int64_t i = __ldcg(idx_out + r) - row_offset;
-      const float x = tail.rows[e];
-      tail.cols[(int64_t)j * tail.ld + i] = x;
-      atomicMin(rmin + j, fenc(x));  // shared-memory range of the new rows
-      atomicMax(rmax + j, fenc(x));
-      if (j == 0) tail.karma[i] = tail.k_init;
+      float x[kMaxDim];
+#pragma unroll
+      for (int j = 0; j < kMaxDim; ++j) x[j] = j < tail.d ? rows[r * tail.d + j] : 0.0f;
+#pragma unroll
+      for (int j = 0; j < kMaxDim; ++j) {
+        if (j < tail.d) {
+          cols[(int64_t)j * tail.ld + i] = x[j];
+          atomicMin(rmin + j, fenc(x[j]));  // shared-memory range of the new rows
+          atomicMax(rmax + j, fenc(x[j]));
+        }
+      }
+      tail.karma[i] = tail.k_init;
     }
     __syncthreads();
     if (tid < tail.d && k > 0) {
