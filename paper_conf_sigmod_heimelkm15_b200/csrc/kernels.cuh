@@ -8,7 +8,10 @@
 namespace kde {
 
 constexpr int kKarmaThreads = 256;
-constexpr int kKarmaPts = 4096;  // contiguous points per karma block (16 passes, 2 load batches)
+#ifndef KDE_TUNE_KARMA_PTS
+#define KDE_TUNE_KARMA_PTS 4096
+#endif
+constexpr int kKarmaPts = KDE_TUNE_KARMA_PTS;  // contiguous points per karma block (4096: 16 passes, 2 load batches)
 inline int karma_blocks(int64_t n) { return (int)((n + kKarmaPts - 1) / kKarmaPts); }
 
 struct HVec {
