@@ -422,21 +422,28 @@ def test_c2_full_size_loss_grad_sampled():
 
 
 # ------------------------------------------------------------------ device-resident streaming step
-def test_device_resident_stream_matches_host_path_and_oracle():
+@pytest.mark.parametrize("many_flags", [False, True])
+def test_device_resident_stream_matches_host_path_and_oracle(many_flags):
     """NEXT-2 loop (estimate -> karma -> Listing 1 -> replacement) with device
     pointers only, bit-identical to the host-pointer calls step by step; the
-    first step's flags also match the oracle."""
+    first step's flags also match the oracle.  many_flags: threshold 0 and
+    cap = n, so thousands of points are replaced per step (the fused tail's
+    row-per-thread loop runs many strides)."""
     import torch
     n, d, steps, cap = 20000, 4, 24, 4096
+    if many_flags:
+        steps, cap = 6, n
     S = synth.make_data("gauss", n, d, seed=40)
     R = synth.make_data("gauss", 80000, d, seed=40)
     lo, hi = synth.workload(S, steps, seed=41, kind="DT")
     p = synth.true_selectivity_cpu(R, lo, hi)
     p[5] = 0.0
     pool = synth.replacement_rows(R, steps * cap, seed=42, step=0)
-    kp = K.karma_params(loss=K.LOSS_ABSOLUTE, threshold=-1.0 / (n - 1), k_max=4.0)
+    tau = 0.0 if many_flags else -1.0 / (n - 1)
+    kp = K.karma_params(loss=K.LOSS_ABSOLUTE, threshold=tau, k_max=4.0)
     op = K.online_params(minibatch=5, loss=K.LOSS_ABSOLUTE, log_bandwidth=True)
     mh, md, mf = model(S), model(S), model(S)
+    max_nf = 0
     mh.set_retain(True)
     md.set_retain(True)
     dev = torch.device("cuda")
@@ -457,11 +464,12 @@ def test_device_resident_stream_matches_host_path_and_oracle():
         e_h, g_h = mh.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
         idx, nf, trunc = mh.karma_update(lo[k], hi[k], p[k], kp)
         assert nf <= cap and not trunc
+        max_nf = max(max_nf, nf)
         if k == 0:
             c_o = oracle.contributions(S, h0, lo[0], hi[0])
             Ko = np.zeros(n)
-            idx_o = oracle.karma_update(c_o, c_o.mean(), p[0], K.LOSS_ABSOLUTE, 0.0, 4.0, -1.0 / (n - 1), np.inf, Ko)
-            amb = _karma_guard(Ko, -1.0 / (n - 1), c_o, np.inf, n)
+            idx_o = oracle.karma_update(c_o, c_o.mean(), p[0], K.LOSS_ABSOLUTE, 0.0, 4.0, tau, np.inf, Ko)
+            amb = _karma_guard(Ko, tau, c_o, np.inf, n)
             fo = np.zeros(n, bool); fo[idx_o] = True
             fg = np.zeros(n, bool); fg[idx] = True
             assert np.array_equal(fo[~amb], fg[~amb])
@@ -484,6 +492,8 @@ def test_device_resident_stream_matches_host_path_and_oracle():
         assert np.array_equal(md.bandwidth, mh.bandwidth)
     assert np.array_equal(md.karma, mh.karma) and np.array_equal(mf.karma, mh.karma)
     assert np.array_equal(md.sample, mh.sample) and np.array_equal(mf.sample, mh.sample)
+    if many_flags:
+        assert max_nf > 4 * 256  # several strides of the fused tail's replacement loop
 
 
 @pytest.mark.parametrize("q", [700, 768])
