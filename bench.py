@@ -1,25 +1,31 @@
 #!/usr/bin/env python
 """bench.py -- throughput of the KDE range-selectivity hot path on B200.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2|c3|c3s|c4|c5s] [--impl cuda|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3|c2|c4|c5|...] [--impl cuda|reference]
 
 A "step" is one pass of the hot path over one batch of synthetic input.  The
-default workload is BASELINE.json configs[1] ("c2"): d = 3, N = 2^20 sample
-points per GPU, a 10k-box batch, estimate + loss + bandwidth gradient
-(kde_loss_and_grad, eq. 5/14/17) -- the inner call of batch bandwidth
-optimisation.  With --gpus N > 1 (torchrun, one process per GPU) every rank
-holds its own 2^20-row shard of an N*2^20-row sample (weak scaling); the
-per-box partial sums are combined with NCCL inside libkde.
+default workload is BASELINE.json configs[2] ("c3", the largest single-GPU
+configuration): d = 5, N = 2^24 sample points per GPU (correlated Gaussian
+clusters), a 4096-box DT/DV/UT/UV batch, estimate + loss + bandwidth gradient
+(kde_loss_and_grad, eq. 5/14/17).  The same line carries the configs[2]
+single-query leg ("single_query": one DT box per step, the HBM-streaming scan)
+with its own roofline, so one run covers both north-star targets.
+
+--gpus N > 1 launches N ranks itself (torch.distributed.run) unless started by
+a launcher (WORLD_SIZE set, which must equal N).  c2/c3 scale weakly (N rows
+per GPU); c4 (configs[3]) is STRONG scaling: one 2^28-row sample, generated
+chunk-wise from one seed, split into contiguous row shards; per-box partial
+sums are combined inside libkde over peer device memory (--comm peer, default)
+or NCCL (--comm nccl).
 
 value   = point*query evaluations per second over the whole job
           (N_global * q / step time, max over ranks, CUDA events, inputs
-          resident in HBM, L2 flushed between timed steps).
-e2e     = the same metric through the host-pointer C-ABI call (bounds and
-          true selectivities copied host->device, loss + gradient copied back,
-          inside the timed region).
-roofline: the batched scan kernel against the SFU ceiling 148 SMs x 16
-          MUFU/clk x 1965 MHz / (2d) point*query/s (two exp per dimension are
-          the algorithmic minimum: Phi and the gradient share e^{-z^2}).
+          resident in HBM, L2 flushed between timed steps when the sample fits).
+e2e     = the same metric through the host-pointer C-ABI call (inputs copied
+          host->device and results device->host inside the timed region).
+roofline: the dominant kernel's own CUDA-event time (recorded inside libkde on
+          its stream) against the SFU ceiling 148 SMs x 16 MUFU/clk x 1965 MHz /
+          (2d) point*query/s (batched), or measured HBM bandwidth (single box).
 cpu_baseline / --impl reference: the fp64 C oracle (oracle/) as it stands,
           on the host cores, over a bounded sample of the same workload.
 """
@@ -28,6 +34,7 @@ from __future__ import annotations
 import argparse
 import json
 import os
+import socket
 import statistics
 import subprocess
 import sys
@@ -45,29 +52,35 @@ MUFU_PER_SM_CLK = 16
 SM_MAX_MHZ = 1965.0
 
 CONFIGS = {
-    # name: d, rows per GPU, boxes, path, description
+    # name: d, rows (per GPU, or global when strong), boxes, path, description
+    "c3": dict(d=5, n=1 << 24, q=4096, path="loss_grad", data="gauss", single_leg=True,
+               desc="configs[2]: d=5, N=2^24/GPU correlated Gaussian clusters, 4096-box DT/DV/UT/UV batch, "
+                    "estimate + L2 loss + bandwidth gradient; single_query leg: one DT box per step"),
     "c2": dict(d=3, n=1 << 20, q=10000, path="loss_grad", data="gauss",
                desc="configs[1]: d=3, N=2^20/GPU, 10k-box batch, estimate + L2 loss + bandwidth gradient"),
-    "c3": dict(d=5, n=1 << 24, q=4096, path="loss_grad", data="gauss",
-               desc="configs[2] batched: d=5, N=2^24/GPU, 4096-box DT/DV/UT/UV batch, estimate + gradient"),
     "c3s": dict(d=5, n=1 << 24, q=1, path="single", grad=False, retain=False, data="gauss",
                 desc="configs[2] single box: d=5, N=2^24/GPU, one DT box per step, estimate (HBM-streaming scan)"),
     "c3sg": dict(d=5, n=1 << 24, q=1, path="single", grad=True, retain=False, data="gauss",
                  desc="configs[2] single box: d=5, N=2^24/GPU, one DT box per step, estimate + bandwidth gradient"),
+    "c4": dict(d=8, n=1 << 28, q=4096, path="loss_grad", data="gauss_rows", strong=True,
+               desc="configs[3]: d=8, N=2^28 GLOBAL rows (one seed) split row-wise over the GPUs (strong scaling), "
+                    "4096-box batch, estimate + L2 loss + gradient, partials all-gathered + rank-order sum"),
+    "c4w": dict(d=8, n=1 << 25, q=4096, path="loss_grad", data="gauss",
+                desc="configs[3] per-GPU shard, weak: d=8, 2^25 rows/GPU, 4096 boxes, estimate + L2 loss + gradient"),
     "c5s": dict(d=10, n=1 << 22, q=1, path="single", grad=True, retain=True, data="gauss",
                 desc="configs[4] estimate step: d=10, N=2^22/GPU, one DT box, estimate + gradient + retained "
                      "contributions (Adaptive, P:L240)"),
-    "c5": dict(d=10, n=1 << 22, q=1, path="stream", grad=True, retain=True, data="gauss",
-               desc="configs[4] streaming step: d=10, N=2^22, one DT box per step: estimate + gradient + retained "
-                    "contributions, karma pass + compaction, Listing 1 bandwidth step, replacement of flagged points "
-                    "(device-resident kde_stream_step_dev: 3 kernels, single GPU)"),
+    "c5": dict(d=10, n=1 << 22, q=16, path="stream", grad=True, retain=True, data="stream",
+               desc="configs[4] streaming: d=10, N=2^22 sample of a cluster database (3 clusters x 2^22 rows, one "
+                    "new cluster inserted per cycle, the oldest deleted); one step = one 2^16-row insert chunk "
+                    "through the reservoir (kde_insert_rows) + 16 DT queries, each a device-resident streaming step "
+                    "(estimate + gradient + retained p^(i), karma + compaction, Listing 1 step, replacement; "
+                    "kde_stream_step_dev, CUDA graphs), single GPU"),
     "c2e": dict(d=3, n=1 << 20, q=10000, path="loss_grad", data="gauss", kernel="epan",
                 desc="configs[1] with the Epanechnikov product kernel (NEXT-4, reading R14): d=3, N=2^20/GPU, "
                      "10k-box batch, estimate + L2 loss + bandwidth gradient"),
     "c3se": dict(d=5, n=1 << 24, q=1, path="single", grad=False, retain=False, data="gauss", kernel="epan",
                  desc="configs[2] single box with the Epanechnikov product kernel: d=5, N=2^24/GPU, estimate"),
-    "c4": dict(d=8, n=1 << 25, q=4096, path="loss_grad", data="gauss",
-               desc="configs[3] per-GPU shard: d=8, 2^25 rows/GPU (2^28 at 8 GPUs), 4096 boxes, estimate + gradient + NCCL"),
 }
 
 
@@ -128,25 +141,45 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
-def make_inputs(cfg, rank: int, seed: int = 7):
-    """Seeded synthetic inputs: this rank's sample shard, the (replicated)
-    boxes and, for loss/grad, true selectivities counted on a database R."""
+def shard_of(cfg, rank: int, world: int):
+    """(row_offset, local rows, global rows) of this rank."""
+    from paper_conf_sigmod_heimelkm15_b200.dist import shard_range
+    if cfg.get("strong"):
+        off, k = shard_range(cfg["n"], rank, world)
+        return off, k, cfg["n"]
+    return rank * cfg["n"], cfg["n"], cfg["n"] * world
+
+
+def make_inputs(cfg, rank: int, world: int, seed: int = 7):
+    """Seeded synthetic inputs: this rank's sample shard S, a database R whose exact box
+    counts are the true selectivities, and the (replicated) boxes."""
     import synth
     d, n, q = cfg["d"], cfg["n"], cfg["q"]
-    if n <= (1 << 21):
+    off, k, n_global = shard_of(cfg, rank, world)
+    if cfg["data"] == "gauss_rows":
+        # one global sample generated chunk-wise from one seed: every world size sees the same rows
+        S = synth.gaussian_clusters_rows(n_global, d, seed, off, off + k)
+        R = synth.gaussian_clusters_rows(1 << 22, d, seed + 1, 0, 1 << 22)   # independent draw for the truths
+        Q = synth.gaussian_clusters_rows(n_global, d, seed, 0, 1 << 16)
+    elif n <= (1 << 21):
         # the "database" R has 4x the rows; the sample is a without-replacement draw from it
         R = synth.make_data(cfg["data"], 4 * n, d, seed=seed + 1000 * rank)
         S = R[synth.rng(seed, 500 + rank).choice(len(R), size=n, replace=False)]
+        Q = synth.make_data(cfg["data"], 1 << 16, d, seed=seed)
     else:
         # large samples: S is drawn directly; true selectivities are counted on a 2^22-row subsample
         S = synth.make_data(cfg["data"], n, d, seed=seed + 1000 * rank)
         R = S[synth.rng(seed, 600 + rank).choice(n, size=1 << 22, replace=False)]
-    Q = synth.make_data(cfg["data"], 1 << 16, d, seed=seed)  # rank-independent box generator
-    if q == 1:
-        lo, hi = synth.workload(Q, 64, seed + 1, "DT")
+        Q = synth.make_data(cfg["data"], 1 << 16, d, seed=seed)
+    if q == 1 or cfg.get("single_leg"):
+        lo1, hi1 = synth.workload(Q, 64, seed + 1, "DT")
     else:
+        lo1 = hi1 = None
+    if q > 1:
         lo, hi = synth.mixed_workload(Q, q, seed + 1)
-    return R, S, lo, hi
+    else:
+        lo, hi = lo1, hi1
+    return R, S, lo, hi, lo1, hi1
 
 
 def true_selectivities(R, lo, hi):
@@ -154,7 +187,7 @@ def true_selectivities(R, lo, hi):
     import torch
 
     import paper_conf_sigmod_heimelkm15_b200 as K
-    dR = torch.from_numpy(R).cuda()
+    dR = torch.from_numpy(np.ascontiguousarray(R)).cuda()
     dlo = torch.from_numpy(lo).cuda()
     dhi = torch.from_numpy(hi).cuda()
     cnt = torch.zeros(len(lo), dtype=torch.int64, device="cuda")
@@ -193,17 +226,30 @@ def cpu_oracle_rate(S, h, lo, hi, p, path, budget_s=12.0, per_step=False):
 def run_reference(args, cfg, rank, world):
     if rank != 0:
         return
-    R, S, lo, hi = make_inputs(cfg, 0)
     import oracle
     oracle.build()
+    if cfg["path"] == "stream":
+        import synth
+        sc = synth.StreamClusters(cfg["d"], 1 << 22, seed=11)
+        S = np.concatenate([sc.cluster_rows(c, 0, cfg["n"] // 3 + 1) for c in range(3)])[:cfg["n"]]
+        lo, hi = sc.queries([0, 1, 2], 64, seed=12)
+        p = None
+        sample_note = "first N/3 rows of each of the 3 initial clusters"
+    else:
+        c2 = dict(cfg)
+        if cfg.get("strong"):  # the oracle's rate is per point*query: a 2^24-row slice of the global sample
+            c2["n"] = 1 << 24
+        R, S, lo, hi, _, _ = make_inputs(c2, 0, 1)
+        p = np.clip(synth_true_cpu(R, lo, hi, cfg), 0, 1)
+        sample_note = "the rank-0 shard" if not cfg.get("strong") else "a 2^24-row slice of the 2^28-row sample"
     h = oracle.scott(S)
-    p = np.clip(synth_true_cpu(R, lo, hi, cfg), 0, 1)
     # size one step to ~3 s of all-core CPU work
-    rate, use, sample, dt, k = cpu_oracle_rate(S, h, lo, hi, p, cfg["path"], budget_s=3.0)
+    path = "single" if cfg["path"] in ("single", "stream") else cfg["path"]
+    rate, use, sample, dt, k = cpu_oracle_rate(S, h, lo, hi, p, path, budget_s=3.0)
     times = []
     for i in range(args.warmup + args.steps):
         t0 = time.perf_counter()
-        if cfg["path"] in ("single", "stream"):
+        if path == "single":
             oracle.estimate_grad(S, h, lo[:k], hi[:k])
         else:
             oracle.loss_and_grad(S, h, lo[:k], hi[:k], p[:k], 0, 0.0, False)
@@ -214,9 +260,10 @@ def run_reference(args, cfg, rank, world):
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": "point·query evals/s",
         "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": cfg["desc"], "d": cfg["d"], "n_per_gpu": cfg["n"], "q": cfg["q"],
-                   "reference_sample_boxes": k},
+        "higher_is_better": True, "scaling": "strong" if cfg.get("strong") else "weak", "vs_baseline": None,
+        "dtype": "f64", "data": "synthetic",
+        "config": {"workload": cfg["desc"], "d": cfg["d"], "n": cfg["n"], "q": cfg["q"],
+                   "reference_sample_boxes": k, "reference_sample_rows": len(S), "sample_rows": sample_note},
         "cpu_baseline": {"value": value, "unit": "point·query evals/s", "cores": use, "kind": "oracle",
                          "sample": sample},
         "e2e": {"value": value, "unit": "point·query evals/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -233,25 +280,109 @@ def synth_true_cpu(R, lo, hi, cfg):
 
 
 # ---------------------------------------------------------------- CUDA arm
+def timed_steps(step, steps, warmup, stream, m, K, flush=None, barrier=None, clock_index=0, min_region_s=1.0):
+    """W untimed warm-up steps, then `steps` steps bracketed by CUDA events on `stream` (the
+    launching stream), clocks sampled by nvidia-smi; short regions get an identical untimed soak
+    so the sampler sees the load.  libkde's profiling counters give the dominant kernel's time."""
+    import torch
+    with torch.cuda.stream(stream):
+        for i in range(warmup):
+            step(i)
+    torch.cuda.synchronize()
+    K.kde_set_profiling(m.handle, True)
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    if barrier:
+        barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(clock_index) as clk:
+        t_start = time.perf_counter()
+        with torch.cuda.stream(stream):
+            for i in range(steps):
+                if flush is not None:
+                    flush(i)
+                evs[i][0].record(stream)
+                step(warmup + i)
+                evs[i][1].record(stream)
+        torch.cuda.synchronize()
+        soak = 0
+        while time.perf_counter() - t_start < min_region_s and soak < 100000:
+            with torch.cuda.stream(stream):
+                for _ in range(8):
+                    step(warmup + steps + soak)
+                    soak += 1
+            torch.cuda.synchronize()
+    if barrier:
+        barrier()
+    torch.cuda.synchronize()
+    scan_ms, scan_launches, launches = K.kde_get_profile(m.handle)
+    K.kde_set_profiling(m.handle, False)
+    frac = steps / max(steps + soak, 1)  # the soak launched the same kernels: keep the timed steps' share
+    step_ms = [a.elapsed_time(b) for a, b in evs]
+    return dict(step_ms=step_ms, scan_ms=scan_ms * frac, scan_launches=int(round(scan_launches * frac)),
+                launches=int(round(launches * frac)), clocks=clk.summary(), soak=soak)
+
+
+def max_over_ranks(x, world, dev):
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([float(x)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def roofline_batched(cfg, args, n_local, q, avg_ms, sms, config_name):
+    d = cfg["d"]
+    achieved = n_local * q / (avg_ms * 1e-3) / 1e9
+    if cfg.get("kernel") == "epan":
+        peak = sms * 128 * SM_MAX_MHZ * 1e6 / (6 * d) / 1e9
+        return {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gpt·q/s", "frac": achieved / peak,
+                "traffic": _traffic(config_name), "kernel": f"scan_batched_kernel<{d},grad> (Epanechnikov)",
+                "algorithmic": f"{n_local} points x {q} boxes per launch; 6d FP32 ops per point*box",
+                "peak_source": f"FP32 ceiling {sms} SMs x 128 lanes x {SM_MAX_MHZ:.0f} MHz / (6d)"}
+    peak = sms * MUFU_PER_SM_CLK * SM_MAX_MHZ * 1e6 / (2 * d) / 1e9
+    return {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gpt·q/s", "frac": achieved / peak,
+            "traffic": _traffic(config_name),
+            "kernel": f"scan_batched_kernel<{d},grad>{'' if args.no_cull else ' (culled)'}",
+            "algorithmic": f"{n_local} points x {q} boxes per launch (per GPU); 2d MUFU.EX2 per point*box"
+                           + ("" if args.no_cull else " (brute-force count: culled pairs are counted as "
+                              "evaluated, so frac is throughput against the unculled SFU ceiling)"),
+            "peak_source": f"SFU ceiling {sms} SMs x {MUFU_PER_SM_CLK} MUFU/clk x {SM_MAX_MHZ:.0f} MHz / (2d) "
+                           "(guide unit counts; 16/clk/SM re-measured by tools/pipe_rates.cu)"}
+
+
+def roofline_single(d, n_local, grad, retain, avg_ms, cull, config_name):
+    alg_bytes = n_local * d * 4 + (n_local * 4 if retain else 0)  # 4d B/point read (+4 B/point retained c)
+    achieved = alg_bytes / (avg_ms * 1e-3) / 1e9
+    peak = _measured_hbm()
+    return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+            "traffic": _traffic(config_name),
+            "kernel": (f"scan_single_tma_kernel<{d},{'grad' if grad else 'est'},cull>" if cull else
+                       f"{'scan_single_tma_kernel' if d <= 8 else 'scan_single_kernel'}<{d},{'grad' if grad else 'est'}>"),
+            "algorithmic": f"4*d bytes/point{' + 4 B/point retained' if retain else ''} x {n_local} points per launch",
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
+
+
 def run_cuda(args, cfg, rank, world, local_rank):
     import torch
     import torch.distributed as dist
 
     import paper_conf_sigmod_heimelkm15_b200 as K
-    from paper_conf_sigmod_heimelkm15_b200.dist import exchange_unique_id
+    from paper_conf_sigmod_heimelkm15_b200.dist import create_sharded
 
     torch.cuda.set_device(local_rank)
     dev = torch.device("cuda", local_rank)
-    d, n, q = cfg["d"], cfg["n"], cfg["q"]
-    R, S, lo, hi = make_inputs(cfg, rank)
-    p = true_selectivities(R, lo, hi) if cfg["path"] != "single" else None
-    if cfg["path"] == "stream" and world > 1:
-        raise SystemExit("c5 (device-resident streaming) is single-GPU")
-
-    n_global = n * world
+    if cfg["path"] == "stream":
+        if world > 1:
+            raise SystemExit("c5 (device-resident streaming) is single-GPU")
+        return run_stream(args, cfg, dev)
+    d, q = cfg["d"], cfg["q"]
+    R, S, lo, hi, lo1, hi1 = make_inputs(cfg, rank, world)
+    off, n_local, n_global = shard_of(cfg, rank, world)
+    p = true_selectivities(R, lo, hi) if cfg["path"] == "loss_grad" else None
+    del R
     if world > 1:
-        nid = exchange_unique_id()
-        m = K.KDEModel.create_sharded(S, rank * n, n_global, None, nid, rank, world)
+        m = create_sharded(S, off, n_global, None, transport=args.comm)
     else:
         m = K.KDEModel.create(S)
     if cfg.get("kernel") == "epan":
@@ -259,10 +390,11 @@ def run_cuda(args, cfg, rank, world, local_rank):
         m.bandwidth = m.bandwidth * np.sqrt(5.0)  # variance-matched to Scott's Gaussian bandwidth
     h = m.bandwidth
     m.cull = not args.no_cull
+    if cfg.get("retain"):
+        m.set_retain(True)
 
     stream = torch.cuda.Stream(device=dev)
-    d_lo = torch.from_numpy(lo).to(dev)
-    d_hi = torch.from_numpy(hi).to(dev)
+    d_lo, d_hi = torch.from_numpy(lo).to(dev), torch.from_numpy(hi).to(dev)
     d_true = torch.from_numpy(p).to(dev) if p is not None else None
     d_loss = torch.zeros(1, dtype=torch.float64, device=dev)
     d_grad = torch.zeros(d, dtype=torch.float64, device=dev)
@@ -270,29 +402,12 @@ def run_cuda(args, cfg, rank, world, local_rank):
     d_dpdh = torch.zeros((q, d), dtype=torch.float64, device=dev)
     l2 = torch.cuda.get_device_properties(dev).L2_cache_size
     flush_buf = torch.empty(max(4 * l2, 256 << 20) // 4, dtype=torch.float32, device=dev)
-    flush_l2 = cfg["n"] * d * 4 < 2 * l2  # sample smaller than ~2x L2 -> flush between timed steps
+    flush_l2 = n_local * d * 4 < 2 * l2  # sample smaller than ~2x L2 -> flush between timed steps
+    flush = (lambda i: flush_buf.fill_(float(i))) if flush_l2 else None
+    barrier = dist.barrier if world > 1 else None
     nbox = len(lo)
 
-    if cfg.get("retain"):
-        m.set_retain(True)
-    use_graph = cfg["path"] == "stream" and not args.no_graph
-    if cfg["path"] == "stream":
-        cap = 1 << 16
-        kp = K.karma_params(loss=K.LOSS_ABSOLUTE, threshold=-1.0 / (n_global - 1), k_max=4.0)
-        op = K.online_params(minibatch=10, loss=K.LOSS_ABSOLUTE, log_bandwidth=True)
-        d_pool = torch.from_numpy(R).to(dev)  # replacement rows drawn from the database R
-        d_idx = torch.zeros(cap, dtype=torch.int64, device=dev)
-        d_cnt = torch.zeros(1, dtype=torch.int64, device=dev)
-        npool = len(R) - cap
-        flagged = []
-
     def step(i):
-        if cfg["path"] == "stream":
-            k = i % nbox
-            off = (k * 977) % npool
-            K.kde_stream_step_dev(m.handle, d_lo[k:k + 1], d_hi[k:k + 1], d_true[k:k + 1], kp, op, d_idx, d_cnt,
-                                  d_pool[off:off + cap], d_est[:1], d_dpdh[0], stream=stream)
-            return
         if cfg["path"] == "single":
             k = i % nbox
             K.kde_estimate_batch_dev(m.handle, d_lo[k:k + 1], d_hi[k:k + 1], d_est[:1],
@@ -301,88 +416,8 @@ def run_cuda(args, cfg, rank, world, local_rank):
             K.kde_loss_and_grad_dev(m.handle, d_lo, d_hi, d_true, d_loss, d_grad, K.LOSS_SQUARED, 0.0, False,
                                     stream=stream)
 
-    with torch.cuda.stream(stream):
-        for i in range(args.warmup):
-            step(i)
-    torch.cuda.synchronize()
-
-    graphs = None
-    prof_pre = None
-    if use_graph:
-        # launch-bound multi-kernel steps: one CUDA graph per box (the step's
-        # arguments depend only on the box index), replayed per step.  The scan
-        # kernel's own duration for the roofline is taken from profiled eager
-        # steps first (kernel events cannot be read back from a replayed graph).
-        K.kde_set_profiling(m.handle, True)
-        with torch.cuda.stream(stream):
-            for i in range(args.warmup, args.warmup + max(args.steps, 8)):
-                step(i)
-        torch.cuda.synchronize()
-        prof_pre = K.kde_get_profile(m.handle)
-        K.kde_set_profiling(m.handle, False)
-        graphs = []
-        for k in range(nbox):
-            g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g, stream=stream):
-                step(k)
-            graphs.append(g)
-        torch.cuda.synchronize()
-        # the first replay of a graph uploads it (~0.7 ms): replay each once, untimed
-        with torch.cuda.stream(stream):
-            for g in graphs:
-                g.replay()
-        torch.cuda.synchronize()
-
-        def step(i):  # noqa: F811
-            graphs[i % nbox].replay()
-
-    K.kde_set_profiling(m.handle, True)
-    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    with ClockSampler(local_rank) as clk:
-        t_start = time.perf_counter()
-        with torch.cuda.stream(stream):
-            for i in range(args.steps):
-                if flush_l2:
-                    flush_buf.fill_(float(i))
-                evs[i][0].record(stream)
-                step(i)
-                evs[i][1].record(stream)
-        torch.cuda.synchronize()
-        # short timed regions (< 1 s) are followed by an identical untimed soak so
-        # that nvidia-smi (100 ms period) samples the clocks under this load
-        soak = 0
-        while time.perf_counter() - t_start < 1.0 and soak < 100000:
-            with torch.cuda.stream(stream):
-                for _ in range(8):
-                    step(args.steps + soak)
-                    soak += 1
-            torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    scan_ms, scan_launches, launches = K.kde_get_profile(m.handle)
-    # the soak steps launched the same kernels: keep the timed steps' share
-    per_step = launches / max(args.steps + soak, 1)
-    launches = int(round(per_step * args.steps))
-    scan_ms *= args.steps / max(args.steps + soak, 1)
-    scan_launches = int(round(scan_launches * args.steps / max(args.steps + soak, 1)))
-    if graphs is not None:  # graph replays bypass libkde's host-side counters
-        ms_pre, sl_pre, l_pre = prof_pre
-        n_pre = max(args.steps, 8)
-        launches = int(round(l_pre / n_pre * args.steps))
-        scan_launches = int(round(sl_pre / n_pre * args.steps))
-        scan_ms = ms_pre / n_pre * args.steps
-    K.kde_set_profiling(m.handle, False)
-    step_ms = [a.elapsed_time(b) for a, b in evs]
-    tot_ms = sum(step_ms)
-    t = torch.tensor([tot_ms], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    tot_ms = float(t.item())
-    ms_per_step = tot_ms / args.steps
+    T = timed_steps(step, args.steps, args.warmup, stream, m, K, flush, barrier, local_rank)
+    ms_per_step = max_over_ranks(sum(T["step_ms"]), world, dev) / args.steps
     units_per_step = n_global * q
     value = units_per_step / (ms_per_step * 1e-3)
 
@@ -393,99 +428,244 @@ def run_cuda(args, cfg, rank, world, local_rank):
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     for i in range(e2e_steps):
-        if cfg["path"] == "stream":
-            k = i % nbox
-            m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
-            idx, nf, _ = m.karma_update(lo[k], hi[k], p[k], kp, cap=cap)
-            m.online_update(lo[k], hi[k], p[k], op)
-            off = (i * 977) % npool
-            m.replace_points(idx, R[off:off + len(idx)])
-            flagged.append(nf)
-        elif cfg["path"] == "single":
+        if cfg["path"] == "single":
             k = i % nbox
             m.estimate(lo[k:k + 1], hi[k:k + 1], grad=bool(cfg.get("grad")))
         else:
             m.loss_and_grad(lo, hi, p, K.LOSS_SQUARED, 0.0, False)
     torch.cuda.synchronize()
-    e2e_s = time.perf_counter() - t0
-    t = torch.tensor([e2e_s], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    e2e_s = float(t.item())
-    if cfg["path"] == "stream":
-        mean_flag = float(np.mean(flagged)) if flagged else 0.0
-        h2d = 2 * d * 4 * 3 + 8 * 2 + int(mean_flag * (8 + 4 * d))  # bounds (3 calls), true sel (2), replacement idx+rows
-        d2h = 8 * (1 + d) + int(mean_flag * 8) + 8 + 4  # estimate+gradient, flagged indices, count, update flag
-    elif cfg["path"] == "single":
+    e2e_s = max_over_ranks(time.perf_counter() - t0, world, dev)
+    if cfg["path"] == "single":
         h2d, d2h = 2 * d * 4, 8 * (1 + (d if cfg.get("grad") else 0))
     else:
         h2d, d2h = 2 * q * d * 4 + q * 8, 8 * (1 + d)
 
+    # ---------------- the configs[2] single-query leg on the same model (HBM-streaming scan)
+    single = None
+    if cfg.get("single_leg"):
+        d_lo1, d_hi1 = torch.from_numpy(lo1).to(dev), torch.from_numpy(hi1).to(dev)
+
+        def step1(i):
+            k = i % len(lo1)
+            K.kde_estimate_batch_dev(m.handle, d_lo1[k:k + 1], d_hi1[k:k + 1], d_est[:1], None, stream=stream)
+
+        T1 = timed_steps(step1, max(args.steps, 20), args.warmup, stream, m, K, None, barrier, local_rank)
+        ms1 = max_over_ranks(sum(T1["step_ms"]), world, dev) / len(T1["step_ms"])
+        if world > 1:
+            dist.barrier()
+        t0 = time.perf_counter()
+        for i in range(e2e_steps):
+            m.estimate(lo1[i % len(lo1):i % len(lo1) + 1], hi1[i % len(lo1):i % len(lo1) + 1])
+        e2e1 = max_over_ranks(time.perf_counter() - t0, world, dev)
+        avg1 = T1["scan_ms"] / max(T1["scan_launches"], 1)
+        roof1 = roofline_single(d, n_local, False, False, avg1, not args.no_cull, "c3s")
+        single = {"workload": "configs[2] single DT box per step, estimate (kde_estimate_batch_dev, q = 1)",
+                  "value": n_global / (ms1 * 1e-3), "unit": "point·query evals/s",
+                  "estimates_per_s": 1e3 / ms1, "ms_per_step": ms1, "steps": len(T1["step_ms"]),
+                  "e2e": {"value": n_global * e2e_steps / e2e1, "unit": "point·query evals/s",
+                          "h2d_bytes_per_step": 2 * d * 4, "d2h_bytes_per_step": 8, "steps": e2e_steps},
+                  "gpu_launches": T1["launches"], "roofline": roof1, "clocks": T1["clocks"],
+                  "step_ms": {"min": min(T1["step_ms"]), "median": statistics.median(T1["step_ms"]),
+                              "max": max(T1["step_ms"])}}
+
     if rank != 0:
         return
-    # ---------------- roofline of the dominant (scan) kernel, per GPU
-    clocks = clk.summary()
-    avg_scan_ms = scan_ms / max(scan_launches, 1)
+    clocks = T["clocks"]
+    avg_scan_ms = T["scan_ms"] / max(T["scan_launches"], 1)
     sms = torch.cuda.get_device_properties(dev).multi_processor_count
-    if cfg["path"] in ("single", "stream"):
-        alg_bytes = n * d * 4 + (n * 4 if cfg.get("retain") else 0)  # 4d B/point read (+4 B/point retained c)
-        achieved = alg_bytes / (avg_scan_ms * 1e-3) / 1e9
-        peak = _measured_hbm()
-        roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": _traffic(args.config), "kernel": (f"scan_single_tma_kernel<{d},{'grad' if cfg.get('grad') else 'est'},cull>" if not args.no_cull else
-                           f"{'scan_single_tma_kernel' if d <= 8 else 'scan_single_kernel'}<{d},{'grad' if cfg.get('grad') else 'est'}>"),
-                "algorithmic": f"4*d bytes/point{' + 4 B/point retained' if cfg.get('retain') else ''} x {n} points per launch",
-                "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
-    elif cfg.get("kernel") == "epan":
-        # no transcendental: the algorithmic minimum is the FP32 work, 6 FP32 ops per dimension
-        # (2 subtract-scale, 2 products of the S = a^2 + ab + b^2 form, 2 for D) -> FP32 ceiling
-        achieved = n * q / (avg_scan_ms * 1e-3) / 1e9
-        peak = sms * 128 * SM_MAX_MHZ * 1e6 / (6 * d) / 1e9
-        roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gpt·q/s", "frac": achieved / peak,
-                "traffic": _traffic(args.config), "kernel": f"scan_batched_kernel<{d},grad> (Epanechnikov)",
-                "algorithmic": f"{n} points x {q} boxes per launch; 6d FP32 ops per point*box",
-                "peak_source": f"FP32 ceiling {sms} SMs x 128 lanes x {SM_MAX_MHZ:.0f} MHz / (6d)"}
+    if cfg["path"] == "single":
+        roof = roofline_single(d, n_local, cfg.get("grad"), cfg.get("retain"), avg_scan_ms, not args.no_cull,
+                               args.config)
     else:
-        achieved = n * q / (avg_scan_ms * 1e-3) / 1e9
-        peak = sms * MUFU_PER_SM_CLK * SM_MAX_MHZ * 1e6 / (2 * d) / 1e9
-        roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gpt·q/s",
-                "frac": achieved / peak, "traffic": _traffic(args.config),
-                "kernel": f"scan_batched_kernel<{d},grad>{'' if args.no_cull else ' (culled)'}",
-                "algorithmic": f"{n} points x {q} boxes per launch; 2d MUFU.EX2 per point*box"
-                               + ("" if args.no_cull else " (brute-force count: culled pairs are counted as "
-                                  "evaluated, so frac is throughput against the unculled SFU ceiling)"),
-                "peak_source": f"SFU ceiling {sms} SMs x {MUFU_PER_SM_CLK} MUFU/clk x {SM_MAX_MHZ:.0f} MHz / (2d) "
-                               "(guide unit counts; 16/clk/SM re-measured by tools/pipe_rates.cu)"}
+        roof = roofline_batched(cfg, args, n_local, q, avg_scan_ms, sms, args.config)
     if clocks.get("sm_mhz"):
         roof["frac_at_measured_clock"] = roof["frac"] * SM_MAX_MHZ / clocks["sm_mhz"] if roof["bound"] == "alu" \
             else roof["frac"]
-
     cpu = None
     if world == 1 and not args.no_cpu:
         rate, use, sample, dt, k = cpu_oracle_rate(S, h, lo, hi, p, cfg["path"], budget_s=args.cpu_budget)
         cpu = {"value": rate, "unit": "point·query evals/s", "cores": use, "kind": "oracle", "sample": sample,
                "seconds": dt}
-
     line = {
         "metric": METRIC, "value": value, "unit": "point·query evals/s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
-        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-        "config": {"workload": cfg["desc"], "d": d, "n_per_gpu": n, "n_global": n_global, "q": q,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": "strong" if cfg.get("strong") else "weak", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic",
+        "config": {"workload": cfg["desc"], "d": d, "n_per_gpu": n_local, "n_global": n_global, "q": q,
+                   "comm": (args.comm if world > 1 else "none"),
                    "l2": "flushed between timed steps" if flush_l2 else "sample larger than L2",
-                   "cuda_graph": bool(graphs is not None),
                    "cull": ("off" if args.no_cull else
                             "on: (point, box) pairs whose contribution is provably < 2^-64 are skipped (DESIGN R15)"),
                    "clock_sampling": "nvidia-smi every 100 ms over the timed steps"
-                                     + (f" + {soak} identical untimed soak steps (timed region < 1 s)" if soak else ""),
+                                     + (f" + {T['soak']} identical untimed soak steps (timed region < 1 s)"
+                                        if T["soak"] else ""),
                    "accumulation": "fp32 per <=32 points, fp64 above"},
         "estimates_per_s": q / (ms_per_step * 1e-3),
-        **({"stream": {"queries_per_s": 1e3 / ms_per_step, "mean_flagged_per_query_e2e": float(np.mean(flagged))}}
-           if cfg["path"] == "stream" else {}),
         "e2e": {"value": units_per_step * e2e_steps / e2e_s, "unit": "point·query evals/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": e2e_steps},
-        "gpu_launches": launches, "scan_launches": scan_launches,
+        "gpu_launches": T["launches"], "scan_launches": T["scan_launches"],
         "roofline": roof, "cpu_baseline": cpu, "clocks": clocks,
-        "step_ms": {"min": min(step_ms), "median": statistics.median(step_ms), "max": max(step_ms)},
+        "step_ms": {"min": min(T["step_ms"]), "median": statistics.median(T["step_ms"]), "max": max(T["step_ms"])},
+    }
+    if single is not None:
+        line["single_query"] = single
+    print(json.dumps(line), flush=True)
+
+
+def run_stream(args, cfg, dev):
+    """configs[4]: reservoir inserts + device-resident streaming queries (single GPU)."""
+    import torch
+
+    import paper_conf_sigmod_heimelkm15_b200 as K
+    import synth
+    d, N = cfg["d"], cfg["n"]
+    rows = 1 << 22            # rows per database cluster
+    chunk = 1 << 16           # arrivals per insert chunk
+    qpc = cfg["q"]            # queries per chunk
+    cap = 1 << 16
+    res_seed = 0xC5
+    sc = synth.StreamClusters(d, rows, seed=11)
+    # initial database R0 = clusters 0, 1, 2; the sample is the reservoir after its 3 x 2^22 arrivals
+    base = np.concatenate([sc.cluster_rows(c) for c in range(3)])
+    n0 = len(base)
+    sl = K.kde_reservoir_select(res_seed, N, N, n0 - N)
+    content = np.arange(N)
+    ids = np.arange(N, n0)
+    ok = sl >= 0
+    rev_s, rev_i = sl[ok][::-1], ids[ok][::-1]
+    u, first = np.unique(rev_s, return_index=True)  # the last arrival per slot wins
+    content[u] = rev_i[first]
+    S = base[content]
+    m = K.KDEModel.create(S)
+    m.set_retain(True)
+    m.cull = not args.no_cull
+    # insert cycle 1: cluster 3 arrives in chunks; queries over the live clusters, newer ones more often
+    P = args.warmup + args.steps
+    new_rows = sc.cluster_rows(3, 0, min(rows, P * chunk))
+    live = [0, 1, 2, 3]
+    Qlo, Qhi = sc.queries(live, P * qpc, seed=13)
+    stream = torch.cuda.Stream(device=dev)
+    # true selectivities over the database at each chunk: the 3 base clusters + the inserted part of cluster 3
+    dbase = torch.from_numpy(base).to(dev)
+    p = np.empty(P * qpc)
+    for t in range(P):
+        sel = slice(t * qpc, (t + 1) * qpc)
+        dlo_t, dhi_t = torch.from_numpy(Qlo[sel]).to(dev), torch.from_numpy(Qhi[sel]).to(dev)
+        c0 = torch.zeros(qpc, dtype=torch.int64, device=dev)
+        K.kde_count_in_box_dev(dbase, dlo_t, dhi_t, c0)
+        ins = min(rows, (t + 1) * chunk)
+        c1 = torch.zeros(qpc, dtype=torch.int64, device=dev)
+        K.kde_count_in_box_dev(torch.from_numpy(new_rows[:ins]).to(dev), dlo_t, dhi_t, c1)
+        torch.cuda.synchronize()
+        p[sel] = ((c0 + c1).double() / (n0 + ins)).cpu().numpy()
+    del dbase
+    # replacement pool: rows of the current database
+    pool = np.concatenate([base[synth.rng(14).integers(0, n0, size=1 << 17)], new_rows[:chunk]])
+    d_pool = torch.from_numpy(pool).to(dev)
+    npool = len(pool) - cap
+    d_lo, d_hi = torch.from_numpy(Qlo).to(dev), torch.from_numpy(Qhi).to(dev)
+    d_true = torch.from_numpy(p).to(dev)
+    kp = K.karma_params(loss=K.LOSS_ABSOLUTE, threshold=-1.0 / (N - 1), k_max=4.0)
+    op = K.online_params(minibatch=10, loss=K.LOSS_ABSOLUTE, log_bandwidth=True)
+    d_idx = torch.zeros(cap, dtype=torch.int64, device=dev)
+    d_cnt = torch.zeros(1, dtype=torch.int64, device=dev)
+    d_est = torch.zeros(1, dtype=torch.float64, device=dev)
+    d_dpdh = torch.zeros(d, dtype=torch.float64, device=dev)
+    state = {"n_seen": n0, "written": []}
+
+    def query(qi):
+        off = (qi * 977) % npool
+        K.kde_stream_step_dev(m.handle, d_lo[qi:qi + 1], d_hi[qi:qi + 1], d_true[qi:qi + 1], kp, op, d_idx, d_cnt,
+                              d_pool[off:off + cap], d_est, d_dpdh, stream=stream)
+
+    # the chunk's 16 queries: one CUDA graph per chunk (launch-bound multi-kernel steps)
+    K.kde_set_profiling(m.handle, True)
+    with torch.cuda.stream(stream):
+        for qi in range(min(P * qpc, 64)):
+            query(qi)
+    torch.cuda.synchronize()
+    prof_pre = K.kde_get_profile(m.handle)
+    n_pre = min(P * qpc, 64)
+    K.kde_set_profiling(m.handle, False)
+    graphs = []
+    if not args.no_graph:
+        for t in range(P):
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=stream):
+                for qi in range(t * qpc, (t + 1) * qpc):
+                    query(qi)
+            graphs.append(g)
+        with torch.cuda.stream(stream):
+            for g in graphs:
+                g.replay()
+        torch.cuda.synchronize()
+
+    def step(i):
+        t = i % P
+        rows_t = new_rows[t * chunk:(t + 1) * chunk]
+        n_seen, nw = m.insert_rows(rows_t, res_seed, state["n_seen"])  # host decision, accepted rows only
+        state["n_seen"] = n_seen
+        state["written"].append(nw)
+        if graphs:
+            graphs[t].replay()
+        else:
+            for qi in range(t * qpc, (t + 1) * qpc):
+                query(qi)
+
+    T = timed_steps(step, args.steps, args.warmup, stream, m, K, None, None, 0)
+    ms_per_step = sum(T["step_ms"]) / args.steps
+    value = N * qpc / (ms_per_step * 1e-3)
+    launches = T["launches"] + int(round(prof_pre[2] / n_pre * qpc * args.steps)) if graphs else T["launches"]
+    avg_scan_ms = prof_pre[0] / max(prof_pre[1], 1)
+    written = float(np.mean(state["written"])) if state["written"] else 0.0
+
+    # e2e: the host-pointer calls (inserts, estimate + gradient, karma, Listing 1, replacement)
+    flagged = []
+    e2e_steps = max(1, min(args.steps, 5))
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for i in range(e2e_steps):
+        t = i % P
+        ns, _ = m.insert_rows(new_rows[t * chunk:(t + 1) * chunk], res_seed, state["n_seen"])
+        state["n_seen"] = ns
+        for qi in range(t * qpc, (t + 1) * qpc):
+            m.estimate(Qlo[qi:qi + 1], Qhi[qi:qi + 1], grad=True)
+            idx, nf, _ = m.karma_update(Qlo[qi], Qhi[qi], p[qi], kp, cap=cap)
+            m.online_update(Qlo[qi], Qhi[qi], p[qi], op)
+            off = (qi * 977) % npool
+            m.replace_points(idx, pool[off:off + len(idx)])
+            flagged.append(nf)
+    torch.cuda.synchronize()
+    e2e_s = time.perf_counter() - t0
+    mean_flag = float(np.mean(flagged)) if flagged else 0.0
+    h2d = int(written * (8 + 4 * d)) + qpc * (2 * d * 4 * 3 + 8 * 2 + int(mean_flag * (8 + 4 * d)))
+    d2h = qpc * (8 * (1 + d) + int(mean_flag * 8) + 8 + 4)
+    roof = roofline_single(d, N, True, True, avg_scan_ms, not args.no_cull, "c5s")
+    clocks = T["clocks"]
+    cpu = None
+    if not args.no_cpu:
+        h = m.bandwidth
+        rate, use, sample, dt, k = cpu_oracle_rate(S, h, Qlo, Qhi, None, "single", budget_s=args.cpu_budget)
+        cpu = {"value": rate, "unit": "point·query evals/s", "cores": use, "kind": "oracle", "sample": sample,
+               "seconds": dt}
+    line = {
+        "metric": METRIC, "value": value, "unit": "point·query evals/s", "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": cfg["desc"], "d": d, "n_per_gpu": N, "n_global": N, "q": qpc,
+                   "insert_chunk": chunk, "database_rows": n0 + P * chunk, "cuda_graph": bool(graphs),
+                   "l2": "sample larger than L2",
+                   "cull": "off" if args.no_cull else "on (DESIGN R15)",
+                   "clock_sampling": "nvidia-smi every 100 ms over the timed steps"
+                                     + (f" + {T['soak']} identical untimed soak steps" if T["soak"] else "")},
+        "estimates_per_s": qpc / (ms_per_step * 1e-3),
+        "stream": {"queries_per_s": qpc * 1e3 / ms_per_step, "inserts_per_s": chunk * 1e3 / ms_per_step,
+                   "rows_written_per_chunk": written, "mean_flagged_per_query_e2e": mean_flag},
+        "e2e": {"value": N * qpc * e2e_steps / e2e_s, "unit": "point·query evals/s",
+                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": e2e_steps,
+                "queries_per_s": qpc * e2e_steps / e2e_s},
+        "gpu_launches": launches, "roofline": roof, "cpu_baseline": cpu, "clocks": clocks,
+        "step_ms": {"min": min(T["step_ms"]), "median": statistics.median(T["step_ms"]), "max": max(T["step_ms"])},
     }
     print(json.dumps(line), flush=True)
 
@@ -506,24 +686,41 @@ def _traffic(config):
         return None
 
 
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="c2", choices=sorted(CONFIGS))
+    ap.add_argument("--config", default="c3", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="cuda", choices=["cuda", "reference"])
+    ap.add_argument("--comm", default="peer", choices=["peer", "nccl"],
+                    help="world > 1: all-gather of the partial sums over peer device memory (libkde) or NCCL")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-cull", action="store_true",
-                    help="single-box scans evaluate every point (kde_set_cull(0)); default culls provably < 2^-64")
+                    help="evaluate every (point, box) pair (kde_set_cull(0)); default culls provably < 2^-64")
     ap.add_argument("--no-graph", action="store_true", help="stream configs: launch eagerly instead of CUDA graphs")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of all-core oracle work")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        # launch one rank per GPU ourselves (the driver may also start us under torchrun)
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr", "127.0.0.1", "--master-port", str(_free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+        raise SystemExit(subprocess.call(cmd))
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE {world}")
     cfg = CONFIGS[args.config]
     if args.impl == "reference":
         run_reference(args, cfg, rank, world)

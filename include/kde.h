@@ -43,6 +43,19 @@ extern "C" {
 #define KDE_ABI_VERSION 1
 #define KDE_MAX_DIM 16          /* d in [1, KDE_MAX_DIM] */
 #define KDE_NCCL_ID_BYTES 128   /* sizeof(ncclUniqueId) */
+#define KDE_PEER_HANDLE_BYTES 64 /* sizeof(cudaIpcMemHandle_t) */
+
+/* How the ranks of a sharded model exchange their per-box partial sums, shard
+ * moments and karma index lists.  NCCL: ncclAllGather.
+ * PEER: the library's own all-gather over peer device memory -- every rank
+ * stores its payload straight into every peer's exchange window (NVLink /
+ * NVSwitch, CUDA IPC mappings) and release-stores an epoch flag; consumers
+ * acquire the flags (bounded wait) and combine in rank order. */
+typedef enum {
+    KDE_COMM_NONE = 0,
+    KDE_COMM_NCCL = 1,
+    KDE_COMM_PEER = 2
+} kde_comm;
 
 typedef struct kde_model kde_model;
 
@@ -143,6 +156,27 @@ kde_status kde_create_sharded(const float *local_rows, int64_t n_local, int64_t 
                               int64_t n_global, int32_t d, const double *h,
                               const void *nccl_id, int32_t rank, int32_t world, kde_model **out);
 
+/* kde_create_sharded_peer -- as kde_create_sharded, with the peer-memory
+ * exchange (KDE_COMM_PEER) instead of NCCL.  Two-phase: after this call every
+ * rank exports its window with kde_peer_handle, the caller all-gathers the
+ * world x KDE_PEER_HANDLE_BYTES handle bytes (any host transport) and every
+ * rank calls kde_peer_attach; until then every other call returns KDE_ESTATE.
+ * With h == NULL, Scott's rule over the global sample runs inside
+ * kde_peer_attach.  One process per rank; ranks may share a GPU (tests).
+ * Exchange waits are bounded (KDE_PEER_TIMEOUT_S, default 60 s): a rank that
+ * misses a collective call makes the others fail with KDE_ECUDA, never hang.
+ * Env KDE_PEER_SLOT_MB (default 4): window slot size; larger payloads are
+ * exchanged in slot-sized pieces.  Errors: as kde_create. */
+kde_status kde_create_sharded_peer(const float *local_rows, int64_t n_local, int64_t row_offset,
+                                   int64_t n_global, int32_t d, const double *h, int32_t rank,
+                                   int32_t world, kde_model **out);
+/* kde_peer_handle -- this rank's exchange-window handle (KDE_PEER_HANDLE_BYTES). */
+kde_status kde_peer_handle(kde_model *m, void *handle_out);
+/* kde_peer_attach -- collective: map every rank's window (handles: world x
+ * KDE_PEER_HANDLE_BYTES in rank order, host); runs the pending Scott's rule.
+ * Errors: KDE_ECUDA (mapping failed), KDE_ESTATE (already attached). */
+kde_status kde_peer_attach(kde_model *m, const void *handles);
+
 /* kde_get_unique_id -- writes an ncclUniqueId (KDE_NCCL_ID_BYTES bytes). */
 kde_status kde_get_unique_id(void *nccl_id_out);
 
@@ -170,17 +204,18 @@ kde_status kde_get_kernel(const kde_model *m, int32_t *kernel);
  * buffer").  Default off. */
 kde_status kde_set_retain(kde_model *m, int32_t on);
 
-/* kde_set_cull / kde_get_cull -- on != 0 (the default): the single-box scan
- * (q == 1) skips every point whose product of eq. (13) factors is provably
- * below 2^-64: with o_j the distance of the point OUTSIDE the box in dimension
- * j in units of sqrt2 h_j / sqrt(log2 e), D_j <= 1/2 erfc(z_j) <= 2^{-o_j^2}, so
- * sum_j o_j^2 >= 64 bounds its contribution to p_hat by 2^-64 and to each
- * dp_hat/dh_j by 2^-60 / (sqrt(pi) sqrt(log2 e) h_j) (R15).  Both the
- * single-box scan and the batched scan (batches that fill 256-box CTAs) cull; for the Epanechnikov kernel
- * a point outside the support in some dimension is skipped (exactly 0).  A
- * skipped point's retained p^(i) is 0.  Points inside the box are never
- * skipped.  on == 0: every point is evaluated.  Errors: none (KDE_EINVAL for
- * a NULL model). */
+/* kde_set_cull / kde_get_cull -- on != 0 (the default): the scans skip every
+ * (point, box) pair whose product of eq. (13) factors is provably below 2^-64.
+ * With o_j the distance of the point OUTSIDE the box in dimension j in units of
+ * sqrt2 h_j / sqrt(log2 e), D_j <= 1/2 erfc(z_j) <= 2^{-o_j^2}, so sum_j o_j^2 >= 64
+ * bounds its contribution to p_hat by 2^-64 and to each dp_hat/dh_j by
+ * 2^-60 / (sqrt(pi) sqrt(log2 e) h_j) (R15).  Which scans cull: the
+ * single-box scan (q == 1) always; the batched scan (q > 1) for batches that
+ * fill 256-box CTAs (smaller batches measured no faster culled).  For the
+ * Epanechnikov kernel a point outside the support in some dimension is skipped
+ * (its contribution is exactly 0).  A skipped point's retained p^(i) is 0.
+ * Points inside the box are never skipped.  on == 0: every pair is evaluated.
+ * Errors: none (KDE_EINVAL for a NULL model). */
 kde_status kde_set_cull(kde_model *m, int32_t on);
 kde_status kde_get_cull(const kde_model *m, int32_t *on);
 
@@ -240,6 +275,32 @@ kde_status kde_online_update(kde_model *m, const float *lo, const float *hi, dou
  * contributions.  Errors: KDE_EINVAL on duplicates, range, non-finite rows. */
 kde_status kde_replace_points(kde_model *m, const int64_t *idx, const float *rows, int64_t k,
                               double k_init);
+
+/* kde_reservoir_select -- the host's reservoir sampling decision for an
+ * insert-only workload (Section 4.2, P:L189 / P:L248: "reservoir sampling [43]
+ * adds newly inserted data to the sample with probability |S|/|R|, replacing a
+ * random point ... all decisions are made independently by the host").
+ * Algorithm R: arrival a = n_seen + r + 1 (1-based; arrivals 1..n_sample fill
+ * slots 0..n_sample-1) draws j uniform on [0, a) from a counter-based generator
+ *   z = SplitMix64 finaliser of (seed + a * 0x9E3779B97F4A7C15), j = floor(z a / 2^64),
+ * and takes slot j iff j < n_sample.  slot_out[r] = that slot or -1 (host,
+ * k int64, caller-owned).  Pure host code (no device, no model).
+ * Errors: KDE_EINVAL (n_sample < 1, n_seen < 0, k < 0, NULL slot_out). */
+kde_status kde_reservoir_select(uint64_t seed, int64_t n_sample, int64_t n_seen, int64_t k, int64_t *slot_out);
+
+/* kde_insert_rows -- insert-only maintenance of the sample: the k
+ * arriving rows (host row-major k x d fp32, copied) go through
+ * kde_reservoir_select(seed, n_global, *n_seen, k); ONLY the rows that enter
+ * the sample are transferred to the device and written (kde_replace_points
+ * semantics: karma reset to k_init, retained state invalidated).  When several
+ * arrivals of the chunk draw the same slot, the last one wins (the sequential
+ * result).  *n_seen (in/out): arrivals so far -- the sample itself counts as
+ * the first n_global (or more) -- advanced by k.  *n_written (optional): slots
+ * written.  Sharded models: every rank calls with the same rows and seed; each
+ * writes the slots of its shard.  Errors: KDE_EINVAL (non-finite rows, bad
+ * n_seen); state unchanged. */
+kde_status kde_insert_rows(kde_model *m, const float *rows, int64_t k, uint64_t seed, int64_t *n_seen,
+                           double k_init, int64_t *n_written);
 
 /* ---------------------------------------------------------------- device-resident feedback loop
  * Single-GPU (world == 1) device-pointer variants of the feedback calls, so a

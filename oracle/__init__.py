@@ -16,7 +16,12 @@ Parity status:
   scott                                      pinned (numpy population std)
   empty_region_threshold                     pinned (eq. 19 centre point, boundary max)
   karma_update                               pinned (brute-force leave-one-out)
-  online_apply (Listing 1 reconstruction)    PARITY UNPINNED (listing missing from PAPER.md)
+  online_apply (Listing 1 reconstruction)    the parts the prose fixes are pinned (rate x1.2 / x0.5 on
+                                             (dis)agreement, [1e-6, 50] clamps, mean SQUARE with alpha 0.9,
+                                             h/2 safeguard in linear mode only: hand traces); the listing
+                                             itself is missing from PAPER.md, so lr0 = 0.1 and the exact
+                                             step form (R6) stay PARITY UNPINNED
+  reservoir_* (Algorithm R, O11)             pinned (chi-square of inclusion frequencies, uniform draws)
   epan_* (Epanechnikov product kernel)       pinned (quadrature of the density, FD, closed forms);
                                              the kernel's bandwidth convention is reading R14
 """
@@ -69,6 +74,9 @@ def _L():
             "oracle_karma_update": (i64, [P, i64, f64, f64, i32, f64, f64, f64, f64, P, P, i64]),
             "oracle_online_accumulate": (None, [i32, P, P]),
             "oracle_online_apply": (None, [i32, i32, f64, f64, f64, f64, f64, i32, P, P, P, P, P]),
+            "oracle_reservoir_draw": (i64, [ctypes.c_uint64, i64]),
+            "oracle_reservoir_slots": (None, [ctypes.c_uint64, i64, i64, i64, P]),
+            "oracle_reservoir_run": (None, [ctypes.c_uint64, i64, i64, P]),
         }
         for name, (res, args) in sig.items():
             fn = getattr(_lib, name)
@@ -90,7 +98,9 @@ def _p(a):
 
 
 def set_threads(n: int) -> None:
-    """Set the OpenMP thread count used by estimate/estimate_grad (0 = default)."""
+    """Set the OpenMP thread count used by the oracle's loops (0 = all host cores)."""
+    if n <= 0:
+        n = os.cpu_count() or 1
     os.environ["OMP_NUM_THREADS"] = str(n)
     try:
         libgomp = ctypes.CDLL("libgomp.so.1")
@@ -232,6 +242,26 @@ def online_step(state: OnlineState, h: np.ndarray, grad, batch=10, alpha=0.9, lr
                              _p(h), _p(state.acc), _p(state.ms), _p(state.lr), _p(state.gprev))
     state.count = 0
     return True
+
+
+# ---------------------------------------------------------------- reservoir sampling (O11)
+def reservoir_draw(seed: int, a: int) -> int:
+    """Algorithm R draw of arrival a (1-based): uniform on [0, a) (counter-based)."""
+    return _L().oracle_reservoir_draw(seed, a)
+
+
+def reservoir_slots(seed: int, n_sample: int, n_seen: int, k: int) -> np.ndarray:
+    """Slot taken by each of the arrivals n_seen+1 .. n_seen+k, or -1."""
+    out = np.empty(k, dtype=np.int64)
+    _L().oracle_reservoir_slots(seed, n_sample, n_seen, k, _p(out))
+    return out
+
+
+def reservoir_run(seed: int, n_sample: int, n_total: int) -> np.ndarray:
+    """Final sample content (1-based arrival ids per slot) after n_total arrivals."""
+    out = np.empty(n_sample, dtype=np.int64)
+    _L().oracle_reservoir_run(seed, n_sample, n_total, _p(out))
+    return out
 
 
 # ---------------------------------------------------------------- Epanechnikov (NEXT-4, reading R14)

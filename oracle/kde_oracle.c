@@ -28,8 +28,11 @@
  *      square of (lambda + p); the true derivative of the printed loss
  *      is used (pinned by finite differences)
  *   R6 Listing 1 (adaptive bandwidth) is missing from the text; the
- *      update is reconstructed from the prose P:L179-183, L561.
- *      PARITY UNPINNED by the paper (no listing, no trace).
+ *      update is reconstructed from the prose P:L179-183, L561.  The
+ *      prose-fixed parts are pinned by hand traces; lr0 and the exact
+ *      step form stay PARITY UNPINNED (no listing, no trace).
+ *   R16 erf differences of eq. (13) with both arguments on one side of 0
+ *      are evaluated as the equal erfc difference (fp64 erf saturates)
  */
 #include <math.h>
 #include <stdint.h>
@@ -43,40 +46,57 @@
  * eq. (13): the i-th point's probability mass in the box
  *   p^(i) = 1/2^d * prod_j [ erf((u_j - t_j)/(sqrt2 h_j)) - erf((l_j - t_j)/(sqrt2 h_j)) ]
  * ------------------------------------------------------------------- */
+/* erf(b) - erf(a) for a <= b.  When both arguments have the same sign the
+ * difference is taken through the exact identity erf(b) - erf(a) = erfc(a) -
+ * erfc(b) (or erfc(-b) - erfc(-a)): fp64 erf saturates to +-1 beyond |z| ~ 5.9,
+ * so the plain difference would return 0 for a box in the far tail of a point
+ * (reading R16).  Same definition, no approximation. */
+static double erf_diff(double a, double b)
+{
+    if (a >= 0.0) return erfc(a) - erfc(b);
+    if (b <= 0.0) return erfc(-b) - erfc(-a);
+    return erf(b) - erf(a);
+}
+
 double oracle_point_mass(const float *t, int32_t d, const double *h,
                          const float *lo, const float *hi)
 {
     double prod = 1.0;
     for (int32_t j = 0; j < d; ++j) {
         double u = (double)hi[j], l = (double)lo[j], tj = (double)t[j];
-        double diff = erf((u - tj) / (OR_SQRT2 * h[j])) - erf((l - tj) / (OR_SQRT2 * h[j]));
+        double diff = erf_diff((l - tj) / (OR_SQRT2 * h[j]), (u - tj) / (OR_SQRT2 * h[j]));
         prod *= diff;
     }
     return prod / pow(2.0, (double)d);
 }
 
-/* eq. (13) for every sample point of one query (the retained buffer). */
+/* eq. (13) for every sample point of one query (the retained buffer).
+ * Each value depends only on its own point, so the loop over points runs on
+ * all host cores without changing any result. */
 void oracle_contributions(const float *sample, int64_t n, int32_t d, const double *h,
                           const float *lo, const float *hi, double *c_out)
 {
+    #pragma omp parallel for schedule(static)
     for (int64_t i = 0; i < n; ++i)
         c_out[i] = oracle_point_mass(sample + i * d, d, h, lo, hi);
 }
 
 /* ---------------------------------------------------------------------
- * eq. (2), P:L98-101: p_H(Omega) = (1/s) sum_i p^(i)(Omega), index order.
+ * Sums over the sample in index order, Neumaier-compensated (SURVEY.md
+ * §8(c) O3): the result is the fp64 rounding of the exact sum of the fp64
+ * terms up to ~2 ulp, independent of n.
  * ------------------------------------------------------------------- */
-void oracle_estimate(const float *sample, int64_t n, int32_t d, const double *h,
-                     const float *lo, const float *hi, int64_t q, double *est)
+typedef struct { double s, c; } nsum_t;
+
+static void nsum_add(nsum_t *a, double x)
 {
-    #pragma omp parallel for schedule(dynamic, 1)
-    for (int64_t k = 0; k < q; ++k) {
-        double sum = 0.0;
-        for (int64_t i = 0; i < n; ++i)
-            sum += oracle_point_mass(sample + i * d, d, h, lo + k * d, hi + k * d);
-        est[k] = sum / (double)n;
-    }
+    double t = a->s + x;
+    if (fabs(a->s) >= fabs(x)) a->c += (a->s - t) + x;
+    else                       a->c += (x - t) + a->s;
+    a->s = t;
 }
+
+static double nsum_get(const nsum_t *a) { return a->s + a->c; }
 
 /* x * exp(-x^2 / (2 h^2)) with the limit value 0 for infinite x (R3). */
 static double xexp(double x, double h)
@@ -85,81 +105,129 @@ static double xexp(double x, double h)
     return x * exp(-(x * x) / (2.0 * h * h));
 }
 
+/* Per-point terms of one query, written literally:
+ *   term[0]     = p^(i)                                            eq. (13)
+ *   term[1 + i] = [ (l_i - t_i) e^{-(l_i-t_i)^2/2h_i^2} - (u_i - t_i) e^{-(u_i-t_i)^2/2h_i^2} ]
+ *                 * prod_{k != i} [ erf((u_k - t_k)/(sqrt2 h_k)) - erf((l_k - t_k)/(sqrt2 h_k)) ]
+ *                                                                  eq. (17), P:L545-547 (summand)
+ * mode 1: the summand of eq. (17) in absolute value, |bracket| * |prod|
+ * (the tolerance scale m_ij = sum_j |d p^(i)/d h_i| of SURVEY.md §8(c)).
+ * The erf difference of dimension k is evaluated once per point and reused by
+ * the products over k != i (the same libm values the formula names; the
+ * product over k != i is still taken directly, O(d^2)). */
+static void point_terms(const float *t, int32_t d, const double *h, const float *l, const float *u,
+                        int mode, double *term)
+{
+    double diff[64];
+    for (int32_t k = 0; k < d; ++k)
+        diff[k] = erf_diff(((double)l[k] - (double)t[k]) / (OR_SQRT2 * h[k]),
+                           ((double)u[k] - (double)t[k]) / (OR_SQRT2 * h[k]));
+    double prod0 = 1.0;                                  /* eq. (13): the same factors, in order */
+    for (int32_t k = 0; k < d; ++k) prod0 *= diff[k];
+    term[0] = prod0 / pow(2.0, (double)d);
+    for (int32_t i = 0; i < d; ++i) {
+        double li = (double)l[i] - (double)t[i];
+        double ui = (double)u[i] - (double)t[i];
+        double bracket = xexp(li, h[i]) - xexp(ui, h[i]);
+        double prod = 1.0;
+        for (int32_t k = 0; k < d; ++k) {
+            if (k == i) continue;
+            prod *= diff[k];
+        }
+        term[1 + i] = mode == 1 ? fabs(bracket) * fabs(prod) : bracket * prod;
+    }
+}
+
+/* Driver shared by eq. (2) and eq. (17): sums[qq][0..d] = index-order Neumaier
+ * sums of the per-point terms.  Many small queries run one query per thread;
+ * a large sample is cut into fixed point chunks whose terms are computed by
+ * all threads and then added sequentially in index order, so every result is
+ * identical for any thread count. */
+#define OR_CHUNK 65536
+static void scan_queries(const float *sample, int64_t n, int32_t d, const double *h,
+                         const float *lo, const float *hi, int64_t q, int mode, double *sums)
+{
+    const int32_t na = 1 + d;
+    if (n < OR_CHUNK) {
+        #pragma omp parallel for schedule(dynamic, 1)
+        for (int64_t qq = 0; qq < q; ++qq) {
+            nsum_t acc[65];
+            double term[65];
+            for (int32_t k = 0; k < na; ++k) acc[k].s = acc[k].c = 0.0;
+            for (int64_t i = 0; i < n; ++i) {
+                point_terms(sample + i * d, d, h, lo + qq * d, hi + qq * d, mode, term);
+                for (int32_t k = 0; k < na; ++k) nsum_add(&acc[k], term[k]);
+            }
+            for (int32_t k = 0; k < na; ++k) sums[qq * na + k] = nsum_get(&acc[k]);
+        }
+        return;
+    }
+    double *buf = (double *)malloc(sizeof(double) * (size_t)OR_CHUNK * (size_t)na);
+    for (int64_t qq = 0; qq < q; ++qq) {
+        nsum_t acc[65];
+        for (int32_t k = 0; k < na; ++k) acc[k].s = acc[k].c = 0.0;
+        for (int64_t c0 = 0; c0 < n; c0 += OR_CHUNK) {
+            const int64_t m = n - c0 < OR_CHUNK ? n - c0 : OR_CHUNK;
+            #pragma omp parallel for schedule(static)
+            for (int64_t i = 0; i < m; ++i)
+                point_terms(sample + (c0 + i) * d, d, h, lo + qq * d, hi + qq * d, mode, buf + i * na);
+            for (int64_t i = 0; i < m; ++i)
+                for (int32_t k = 0; k < na; ++k) nsum_add(&acc[k], buf[i * na + k]);
+        }
+        for (int32_t k = 0; k < na; ++k) sums[qq * na + k] = nsum_get(&acc[k]);
+    }
+    free(buf);
+}
+
+/* ---------------------------------------------------------------------
+ * eq. (2), P:L98-101: p_H(Omega) = (1/s) sum_i p^(i)(Omega), index order.
+ * ------------------------------------------------------------------- */
+void oracle_estimate(const float *sample, int64_t n, int32_t d, const double *h,
+                     const float *lo, const float *hi, int64_t q, double *est)
+{
+    double *sums = (double *)malloc(sizeof(double) * (size_t)q * (size_t)(1 + d));
+    scan_queries(sample, n, d, h, lo, hi, q, 0, sums);
+    for (int64_t k = 0; k < q; ++k) est[k] = sums[k * (1 + d)] / (double)n;
+    free(sums);
+}
+
 /* ---------------------------------------------------------------------
  * eq. (17), written literally:
  *   dp/dh_i = sqrt2 / (sqrtpi h_i^2 2^d s) * sum_j [ (l_i - t_i) e^{-(l_i-t_i)^2/2h_i^2}
  *                                                - (u_i - t_i) e^{-(u_i-t_i)^2/2h_i^2} ]
  *             * prod_{k != i} [ erf((u_k - t_k)/(sqrt2 h_k)) - erf((l_k - t_k)/(sqrt2 h_k)) ]
- * Also returns the estimate (eq. 2) of the same query.  The product over
- * k != i is recomputed for every i (O(d^2)), exactly as written.
+ * Also returns the estimate (eq. 2) of the same query.
  * ------------------------------------------------------------------- */
 void oracle_estimate_grad(const float *sample, int64_t n, int32_t d, const double *h,
                           const float *lo, const float *hi, int64_t q,
                           double *est, double *dpdh)
 {
-    #pragma omp parallel for schedule(dynamic, 1)
+    double *sums = (double *)malloc(sizeof(double) * (size_t)q * (size_t)(1 + d));
+    scan_queries(sample, n, d, h, lo, hi, q, 0, sums);
     for (int64_t qq = 0; qq < q; ++qq) {
-        const float *l = lo + qq * d, *u = hi + qq * d;
-        double sum = 0.0;
-        double gsum[64];
-        for (int32_t i = 0; i < d; ++i) gsum[i] = 0.0;
-        for (int64_t j = 0; j < n; ++j) {
-            const float *t = sample + j * d;
-            sum += oracle_point_mass(t, d, h, l, u);
-            for (int32_t i = 0; i < d; ++i) {
-                double li = (double)l[i] - (double)t[i];
-                double ui = (double)u[i] - (double)t[i];
-                double bracket = xexp(li, h[i]) - xexp(ui, h[i]);
-                double prod = 1.0;
-                for (int32_t k = 0; k < d; ++k) {
-                    if (k == i) continue;
-                    prod *= erf(((double)u[k] - (double)t[k]) / (OR_SQRT2 * h[k]))
-                          - erf(((double)l[k] - (double)t[k]) / (OR_SQRT2 * h[k]));
-                }
-                gsum[i] += bracket * prod;
-            }
-        }
-        est[qq] = sum / (double)n;
+        est[qq] = sums[qq * (1 + d)] / (double)n;
         for (int32_t i = 0; i < d; ++i)
             dpdh[qq * d + i] = OR_SQRT2 / (OR_SQRTPI * h[i] * h[i] * pow(2.0, (double)d) * (double)n)
-                               * gsum[i];
+                               * sums[qq * (1 + d) + 1 + i];
     }
+    free(sums);
 }
 
 /* Gradient magnitude scale used by the parity tolerance (test infrastructure,
- * not a paper quantity):
- *   m_ij = sqrt2 / (sqrtpi h_i^2 2^d s) * sum_j ( |(l_i - t_i) e^{..}| + |(u_i - t_i) e^{..}| )
- *                                             * | prod_{k != i} [...] |
- * i.e. eq. (17) with both terms of the bracket and every per-point term taken
- * in absolute value -- the condition-number scale of evaluating eq. (17) in
- * finite precision (the bracket cancels when both bounds give equal terms). */
+ * not a paper quantity), SURVEY.md §8(c) "Parity criteria":
+ *   m_ij = (1/s) sum_j |d p^(i)/d h_i|
+ *        = sqrt2 / (sqrtpi h_i^2 2^d s) * sum_j |bracket_ij| * |prod_{k != i} [...]|
+ * i.e. eq. (17) with every per-point summand in absolute value. */
 void oracle_grad_abs_scale(const float *sample, int64_t n, int32_t d, const double *h,
                            const float *lo, const float *hi, int64_t q, double *mabs)
 {
-    #pragma omp parallel for schedule(dynamic, 1)
-    for (int64_t qq = 0; qq < q; ++qq) {
-        const float *l = lo + qq * d, *u = hi + qq * d;
-        double gsum[64];
-        for (int32_t i = 0; i < d; ++i) gsum[i] = 0.0;
-        for (int64_t j = 0; j < n; ++j) {
-            const float *t = sample + j * d;
-            for (int32_t i = 0; i < d; ++i) {
-                double li = (double)l[i] - (double)t[i];
-                double ui = (double)u[i] - (double)t[i];
-                double bracket = fabs(xexp(li, h[i])) + fabs(xexp(ui, h[i]));
-                double prod = 1.0;
-                for (int32_t k = 0; k < d; ++k) {
-                    if (k == i) continue;
-                    prod *= erf(((double)u[k] - (double)t[k]) / (OR_SQRT2 * h[k]))
-                          - erf(((double)l[k] - (double)t[k]) / (OR_SQRT2 * h[k]));
-                }
-                gsum[i] += bracket * fabs(prod);
-            }
-        }
+    double *sums = (double *)malloc(sizeof(double) * (size_t)q * (size_t)(1 + d));
+    scan_queries(sample, n, d, h, lo, hi, q, 1, sums);
+    for (int64_t qq = 0; qq < q; ++qq)
         for (int32_t i = 0; i < d; ++i)
             mabs[qq * d + i] = OR_SQRT2 / (OR_SQRTPI * h[i] * h[i] * pow(2.0, (double)d) * (double)n)
-                               * gsum[i];
-    }
+                               * sums[qq * (1 + d) + 1 + i];
+    free(sums);
 }
 
 /* ---------------------------------------------------------------------
@@ -467,4 +535,50 @@ double oracle_epan_empty_region_threshold(int32_t d, const double *h, const floa
     if (pmax_out) *pmax_out = disabled ? 0.0 : pmax;
     if (disabled || !(pmax > 0.0)) return INFINITY;
     return pmax * best;
+}
+
+/* =====================================================================
+ * Reservoir sampling for insert-only workloads (Section 4.2, P:L189 / P:L248:
+ * "the well-known reservoir sampling algorithm [43]" adds a newly inserted tuple
+ * with probability |S|/|R|, replacing a random point).  Algorithm R, SURVEY.md
+ * §8(c) O11: the a-th arriving tuple (a = 1, 2, ...; the first N arrivals fill
+ * the sample) draws j uniformly from [0, a) and replaces slot j if j < N.
+ * The random draw is a counter-based generator both sides implement from its
+ * definition (random numbers the method draws):
+ *   z = SplitMix64 finaliser of (seed + a * 0x9E3779B97F4A7C15),
+ *   j = floor(z * a / 2^64)            (multiply-shift onto [0, a)).
+ * ===================================================================== */
+static uint64_t or_splitmix(uint64_t seed, uint64_t a)
+{
+    uint64_t z = seed + a * 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+/* uniform draw of arrival a in [0, a) */
+int64_t oracle_reservoir_draw(uint64_t seed, int64_t a)
+{
+    return (int64_t)(((unsigned __int128)or_splitmix(seed, (uint64_t)a) * (unsigned __int128)(uint64_t)a) >> 64);
+}
+
+/* slot taken by each of k arrivals a = n_seen + 1 .. n_seen + k, or -1 (not sampled) */
+void oracle_reservoir_slots(uint64_t seed, int64_t n_sample, int64_t n_seen, int64_t k, int64_t *slot_out)
+{
+    for (int64_t r = 0; r < k; ++r) {
+        const int64_t a = n_seen + r + 1;
+        if (a <= n_sample) { slot_out[r] = a - 1; continue; }   /* the first N arrivals fill the sample */
+        const int64_t j = oracle_reservoir_draw(seed, a);
+        slot_out[r] = j < n_sample ? j : -1;
+    }
+}
+
+/* Run Algorithm R over arrivals 1..n_total: content[i] = id (1-based arrival) in slot i */
+void oracle_reservoir_run(uint64_t seed, int64_t n_sample, int64_t n_total, int64_t *content)
+{
+    for (int64_t a = 1; a <= n_total; ++a) {
+        if (a <= n_sample) { content[a - 1] = a; continue; }
+        const int64_t j = oracle_reservoir_draw(seed, a);
+        if (j < n_sample) content[j] = a;
+    }
 }

@@ -26,6 +26,7 @@ LOSS_SQUARED, LOSS_ABSOLUTE, LOSS_RELATIVE, LOSS_SQUARED_RELATIVE, LOSS_SQUARED_
 KERNEL_GAUSSIAN, KERNEL_EPANECHNIKOV = 0, 1
 KDE_MAX_DIM = 16
 KDE_NCCL_ID_BYTES = 128
+KDE_PEER_HANDLE_BYTES = 64
 
 # every symbol include/kde.h declares (checked by tests/test_abi.py)
 ABI_SYMBOLS = (
@@ -36,7 +37,8 @@ ABI_SYMBOLS = (
     "kde_get_karma", "kde_set_karma", "kde_get_sample", "kde_get_contributions", "kde_get_online_state",
     "kde_set_online_state", "kde_synchronize", "kde_count_in_box_dev", "kde_set_profiling", "kde_get_profile",
     "kde_karma_update_dev", "kde_online_update_dev", "kde_replace_points_dev", "kde_stream_step_dev",
-    "kde_set_kernel", "kde_get_kernel", "kde_set_cull", "kde_get_cull",
+    "kde_set_kernel", "kde_get_kernel", "kde_set_cull", "kde_get_cull", "kde_reservoir_select", "kde_insert_rows",
+    "kde_create_sharded_peer", "kde_peer_handle", "kde_peer_attach",
 )
 
 
@@ -95,6 +97,9 @@ def lib() -> ctypes.CDLL:
         "kde_create": (ctypes.c_int, [P, i64, i32, P, PP]),
         "kde_create_sharded": (ctypes.c_int, [P, i64, i64, i64, i32, P, P, i32, i32, PP]),
         "kde_get_unique_id": (ctypes.c_int, [P]),
+        "kde_create_sharded_peer": (ctypes.c_int, [P, i64, i64, i64, i32, P, i32, i32, PP]),
+        "kde_peer_handle": (ctypes.c_int, [P, P]),
+        "kde_peer_attach": (ctypes.c_int, [P, P]),
         "kde_destroy": (None, [P]),
         "kde_get_info": (ctypes.c_int, [P, P, P, P, P, P]),
         "kde_get_bandwidth": (ctypes.c_int, [P, P]),
@@ -111,6 +116,8 @@ def lib() -> ctypes.CDLL:
         "kde_karma_update": (ctypes.c_int, [P, P, P, f64, ctypes.POINTER(KarmaParams), P, i64, P]),
         "kde_online_update": (ctypes.c_int, [P, P, P, f64, ctypes.POINTER(OnlineParams), P]),
         "kde_replace_points": (ctypes.c_int, [P, P, P, i64, f64]),
+        "kde_reservoir_select": (ctypes.c_int, [ctypes.c_uint64, i64, i64, i64, P]),
+        "kde_insert_rows": (ctypes.c_int, [P, P, i64, ctypes.c_uint64, P, f64, P]),
         "kde_get_karma": (ctypes.c_int, [P, P]),
         "kde_set_karma": (ctypes.c_int, [P, P]),
         "kde_get_sample": (ctypes.c_int, [P, P]),
@@ -156,9 +163,36 @@ def _p(a):
     return None if a is None else a.ctypes.data_as(ctypes.c_void_p)
 
 
-def _tp(t):
-    """device pointer of a torch tensor (plumbing only)."""
-    return None if t is None else ctypes.c_void_p(t.data_ptr())
+def _tp(t, dtype=None, numel=None, name="tensor"):
+    """Device pointer of a torch tensor (plumbing only).  The C side cannot see
+    dtype, layout or extent, so they are checked here: a CUDA tensor, contiguous,
+    of the expected dtype ("f32" / "f64" / "i64") and with at least `numel` elements."""
+    if t is None:
+        return None
+    if not getattr(t, "is_cuda", False):
+        raise KDEError(KDE_EINVAL, f"{name} must be a CUDA tensor")
+    if not t.is_contiguous():
+        raise KDEError(KDE_EINVAL, f"{name} must be contiguous")
+    if dtype is not None:
+        want = {"f32": "torch.float32", "f64": "torch.float64", "i64": "torch.int64"}[dtype]
+        if str(t.dtype) != want:
+            raise KDEError(KDE_EINVAL, f"{name} must be {want}, got {t.dtype}")
+    if numel is not None and t.numel() < numel:
+        raise KDEError(KDE_EINVAL, f"{name} has {t.numel()} elements, needs >= {numel}")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+def _dim(m) -> int:
+    return kde_get_info(m)["d"]
+
+
+def _bounds(d_lo, d_hi, d, q=None):
+    """(q, d) fp32 device bounds of identical shape; returns q."""
+    if d_lo.shape != d_hi.shape:
+        raise KDEError(KDE_EINVAL, "lo and hi must have the same shape")
+    if d_lo.numel() % d != 0 or (q is not None and d_lo.numel() != q * d):
+        raise KDEError(KDE_EINVAL, f"bounds must hold q x {d} values, got shape {tuple(d_lo.shape)}")
+    return d_lo.numel() // d
 
 
 def _stream_ptr(stream):
@@ -193,6 +227,28 @@ def kde_create_sharded(local_rows, row_offset: int, n_global: int, h, nccl_id: b
     _check(lib().kde_create_sharded(_p(local_rows), n, row_offset, n_global, d, _p(hh), idb, rank, world,
                                     ctypes.byref(out)))
     return out
+
+
+def kde_create_sharded_peer(local_rows, row_offset: int, n_global: int, h, rank: int, world: int):
+    """Phase 1 of a peer-transport sharded model (kde_peer_handle / kde_peer_attach follow)."""
+    local_rows = _f32(local_rows)
+    n, d = local_rows.shape
+    hh = None if h is None else _f64(h)
+    out = ctypes.c_void_p()
+    _check(lib().kde_create_sharded_peer(_p(local_rows), n, row_offset, n_global, d, _p(hh), rank, world,
+                                         ctypes.byref(out)))
+    return out
+
+
+def kde_peer_handle(m) -> bytes:
+    buf = (ctypes.c_char * KDE_PEER_HANDLE_BYTES)()
+    _check(lib().kde_peer_handle(m, buf))
+    return bytes(buf)
+
+
+def kde_peer_attach(m, handles: bytes):
+    buf = ctypes.create_string_buffer(handles, len(handles))
+    _check(lib().kde_peer_attach(m, buf))
 
 
 def kde_destroy(m):
@@ -254,8 +310,11 @@ def kde_estimate_batch(m, lo, hi, d, grad=False):
 
 def kde_estimate_batch_dev(m, d_lo, d_hi, d_est, d_dpdh=None, stream=None):
     """Device-pointer variant (torch CUDA tensors; plumbing only): enqueue only."""
-    q = d_lo.shape[0]
-    _check(lib().kde_estimate_batch_dev(m, _tp(d_lo), _tp(d_hi), q, _tp(d_est), _tp(d_dpdh), _stream_ptr(stream)))
+    d = _dim(m)
+    q = _bounds(d_lo, d_hi, d)
+    _check(lib().kde_estimate_batch_dev(m, _tp(d_lo, "f32", name="d_lo"), _tp(d_hi, "f32", name="d_hi"), q,
+                                        _tp(d_est, "f64", q, "d_est"), _tp(d_dpdh, "f64", q * d, "d_dpdh"),
+                                        _stream_ptr(stream)))
 
 
 def kde_loss_and_grad(m, lo, hi, true_sel, d, loss=LOSS_SQUARED, lam=0.0, log_bandwidth=False, return_est=False):
@@ -274,9 +333,12 @@ def kde_loss_and_grad(m, lo, hi, true_sel, d, loss=LOSS_SQUARED, lam=0.0, log_ba
 
 def kde_loss_and_grad_dev(m, d_lo, d_hi, d_true, d_loss, d_grad, loss=LOSS_SQUARED, lam=0.0, log_bandwidth=False,
                           d_est=None, stream=None):
-    q = d_lo.shape[0]
-    _check(lib().kde_loss_and_grad_dev(m, _tp(d_lo), _tp(d_hi), _tp(d_true), q, loss, lam,
-                                       int(bool(log_bandwidth)), _tp(d_loss), _tp(d_grad), _tp(d_est),
+    d = _dim(m)
+    q = _bounds(d_lo, d_hi, d)
+    _check(lib().kde_loss_and_grad_dev(m, _tp(d_lo, "f32", name="d_lo"), _tp(d_hi, "f32", name="d_hi"),
+                                       _tp(d_true, "f64", q, "d_true"), q, loss, lam,
+                                       int(bool(log_bandwidth)), _tp(d_loss, "f64", 1, "d_loss"),
+                                       _tp(d_grad, "f64", d, "d_grad"), _tp(d_est, "f64", q, "d_est"),
                                        _stream_ptr(stream)))
 
 
@@ -301,17 +363,26 @@ def kde_online_update(m, lo, hi, true_sel: float, params: OnlineParams) -> bool:
 
 def kde_karma_update_dev(m, d_lo, d_hi, d_true, params: KarmaParams, d_idx, d_count, stream=None):
     """Device-resident karma pass (single GPU): enqueue only."""
-    _check(lib().kde_karma_update_dev(m, _tp(d_lo), _tp(d_hi), _tp(d_true), ctypes.byref(params), _tp(d_idx),
-                                      d_idx.numel(), _tp(d_count), _stream_ptr(stream)))
+    _bounds(d_lo, d_hi, _dim(m), 1)
+    _check(lib().kde_karma_update_dev(m, _tp(d_lo, "f32", name="d_lo"), _tp(d_hi, "f32", name="d_hi"),
+                                      _tp(d_true, "f64", 1, "d_true"), ctypes.byref(params),
+                                      _tp(d_idx, "i64", name="d_idx"), d_idx.numel(),
+                                      _tp(d_count, "i64", 1, "d_count"), _stream_ptr(stream)))
 
 
 def kde_online_update_dev(m, d_true, params: OnlineParams, stream=None):
-    _check(lib().kde_online_update_dev(m, _tp(d_true), ctypes.byref(params), _stream_ptr(stream)))
+    _check(lib().kde_online_update_dev(m, _tp(d_true, "f64", 1, "d_true"), ctypes.byref(params),
+                                       _stream_ptr(stream)))
 
 
 def kde_replace_points_dev(m, d_idx, d_rows, d_count, k_init=0.0, stream=None):
     """Rows d_rows[r] -> global index d_idx[r] for r < min(d_count, len(d_idx))."""
-    _check(lib().kde_replace_points_dev(m, _tp(d_idx), _tp(d_rows), _tp(d_count), d_idx.numel(), float(k_init),
+    d = _dim(m)
+    if d_rows.dim() != 2 or d_rows.shape[1] != d:
+        raise KDEError(KDE_EINVAL, f"d_rows must be (k, {d}), got {tuple(d_rows.shape)}")
+    _check(lib().kde_replace_points_dev(m, _tp(d_idx, "i64", name="d_idx"),
+                                        _tp(d_rows, "f32", d_idx.numel() * d, "d_rows"),
+                                        _tp(d_count, "i64", 1, "d_count"), d_idx.numel(), float(k_init),
                                         _stream_ptr(stream)))
 
 
@@ -319,9 +390,18 @@ def kde_stream_step_dev(m, d_lo, d_hi, d_true, kparams: KarmaParams, oparams, d_
                         d_dpdh, k_init=0.0, stream=None):
     """One device-resident streaming step (estimate + gradient + karma +
     Listing 1 + replacement) in three kernels; enqueue only."""
-    _check(lib().kde_stream_step_dev(m, _tp(d_lo), _tp(d_hi), _tp(d_true), ctypes.byref(kparams),
-                                     None if oparams is None else ctypes.byref(oparams), _tp(d_idx), d_idx.numel(),
-                                     _tp(d_count), _tp(d_rows), float(k_init), _tp(d_est), _tp(d_dpdh),
+    d = _dim(m)
+    _bounds(d_lo, d_hi, d, 1)
+    if d_rows is not None and (d_rows.dim() != 2 or d_rows.shape[1] != d):
+        raise KDEError(KDE_EINVAL, f"d_rows must be (k, {d}), got {tuple(d_rows.shape)}")
+    _check(lib().kde_stream_step_dev(m, _tp(d_lo, "f32", name="d_lo"), _tp(d_hi, "f32", name="d_hi"),
+                                     _tp(d_true, "f64", 1, "d_true"), ctypes.byref(kparams),
+                                     None if oparams is None else ctypes.byref(oparams),
+                                     _tp(d_idx, "i64", name="d_idx"), d_idx.numel(),
+                                     _tp(d_count, "i64", 1, "d_count"),
+                                     _tp(d_rows, "f32", d_idx.numel() * d, "d_rows"), float(k_init),
+                                     _tp(d_est, "f64", 1, "d_est"),
+                                     _tp(d_dpdh, "f64", d if oparams is not None else None, "d_dpdh"),
                                      _stream_ptr(stream)))
 
 
@@ -329,6 +409,23 @@ def kde_replace_points(m, idx, rows, k_init=0.0):
     idx = np.ascontiguousarray(idx, dtype=np.int64)
     rows = _f32(rows)
     _check(lib().kde_replace_points(m, _p(idx), _p(rows), len(idx), float(k_init)))
+
+
+def kde_reservoir_select(seed: int, n_sample: int, n_seen: int, k: int) -> np.ndarray:
+    """Algorithm R decisions of the host: slot per arrival n_seen+1 .. n_seen+k, or -1."""
+    out = np.empty(max(k, 1), dtype=np.int64)
+    _check(lib().kde_reservoir_select(seed, n_sample, n_seen, k, _p(out)))
+    return out[:k]
+
+
+def kde_insert_rows(m, rows, seed: int, n_seen: int, k_init=0.0):
+    """Insert k rows through the reservoir; returns (new n_seen, slots written)."""
+    rows = _f32(rows)
+    ns = ctypes.c_int64(n_seen)
+    nw = ctypes.c_int64()
+    _check(lib().kde_insert_rows(m, _p(rows), rows.shape[0], seed, ctypes.byref(ns), float(k_init),
+                                 ctypes.byref(nw)))
+    return ns.value, nw.value
 
 
 def kde_get_karma(m, n):
@@ -384,8 +481,9 @@ def kde_get_profile(m):
 def kde_count_in_box_dev(d_rows, d_lo, d_hi, d_counts, stream=None):
     """Harness only: exact counts of rows of R in each open box (the DBMS feedback)."""
     n, d = d_rows.shape
-    q = d_lo.shape[0]
-    _check(lib().kde_count_in_box_dev(_tp(d_rows), n, d, _tp(d_lo), _tp(d_hi), q, _tp(d_counts),
+    q = _bounds(d_lo, d_hi, d)
+    _check(lib().kde_count_in_box_dev(_tp(d_rows, "f32", name="d_rows"), n, d, _tp(d_lo, "f32", name="d_lo"),
+                                      _tp(d_hi, "f32", name="d_hi"), q, _tp(d_counts, "i64", q, "d_counts"),
                                       _stream_ptr(stream)))
 
 
@@ -410,6 +508,20 @@ class KDEModel:
     @classmethod
     def create_sharded(cls, local_rows, row_offset, n_global, h, nccl_id, rank, world):
         hd = kde_create_sharded(local_rows, row_offset, n_global, h, nccl_id, rank, world)
+        info = kde_get_info(hd)
+        return cls(hd, info["n_local"], info["n_global"], info["d"], rank, world)
+
+    @classmethod
+    def create_sharded_peer(cls, local_rows, row_offset, n_global, h, rank, world, all_gather_bytes):
+        """Peer-transport sharded model; all_gather_bytes(b: bytes) -> list of every rank's bytes
+        (host bootstrap, e.g. torch.distributed.all_gather_object)."""
+        hd = kde_create_sharded_peer(local_rows, row_offset, n_global, h, rank, world)
+        try:
+            if world > 1:
+                kde_peer_attach(hd, b"".join(all_gather_bytes(kde_peer_handle(hd))))
+        except Exception:
+            kde_destroy(hd)
+            raise
         info = kde_get_info(hd)
         return cls(hd, info["n_local"], info["n_global"], info["d"], rank, world)
 
@@ -469,6 +581,10 @@ class KDEModel:
 
     def replace_points(self, idx, rows, k_init=0.0):
         kde_replace_points(self.handle, idx, rows, k_init)
+
+    def insert_rows(self, rows, seed, n_seen, k_init=0.0):
+        """Reservoir inserts: returns (new n_seen, slots written)."""
+        return kde_insert_rows(self.handle, rows, seed, n_seen, k_init)
 
     @property
     def karma(self):

@@ -6,6 +6,7 @@
 // Every numeric step runs in the kernels of scan.cuh / kernels.cu; this file
 // only moves arguments, validates them and orders launches on one stream.
 #include <algorithm>
+#include <climits>
 #include <cstddef>
 #include <cmath>
 #include <cstdarg>
@@ -44,7 +45,13 @@ struct kde_model {
   int64_t row_offset = 0;
   int64_t ld = 0;        // padded column length
   int rank = 0, world = 1;
-  ncclComm_t comm = nullptr;
+  int comm_kind = KDE_COMM_NONE;   // how world > 1 ranks exchange (kde_comm)
+  ncclComm_t comm = nullptr;       // KDE_COMM_NCCL
+  bool attached = true;            // KDE_COMM_PEER: false until kde_peer_attach
+  bool h_pending = false;          // KDE_COMM_PEER without h: Scott's rule runs in kde_peer_attach
+  char* xwin = nullptr;            // KDE_COMM_PEER: this rank's exchange window (peer.cu)
+  size_t xwin_bytes = 0;
+  PeerArgs pa;                     // mapped windows of every rank + device epoch / counters / error flag
   bool poisoned = false;
 
   float* cols = nullptr;       // [d][ld]
@@ -70,6 +77,7 @@ struct kde_model {
   size_t gather_cap = 0;
   uint32_t* bitmap = nullptr;
   int32_t* block_counts = nullptr;
+  int64_t* block_offsets = nullptr;  // [nkb + 1] exclusive offsets of the karma flags + total
   int64_t* offsets = nullptr;        // [0] = total flagged (karma compaction)
   unsigned* done = nullptr;          // compaction last-block counter (self-resetting)
   int64_t* idx_dev = nullptr;
@@ -79,6 +87,10 @@ struct kde_model {
   double* scal = nullptr;            // [8] device scalars (true selectivity staging)
   void* pinned = nullptr;            // pinned host staging
   size_t pinned_cap = 0;
+  void* rbuf = nullptr;              // replacement staging (idx + rows), grow-only
+  size_t rbuf_cap = 0;
+  void* kbuf = nullptr;              // sharded karma gather: counts + index lists, grow-only
+  size_t kbuf_cap = 0;
 
   // retained single-box state
   bool retain = false;
@@ -127,6 +139,7 @@ struct kde_model {
   do {                                                                                     \
     if (!(m)) return fail(KDE_EINVAL, "model is NULL");                                   \
     if ((m)->poisoned) return fail(KDE_ESTATE, "model poisoned by an earlier CUDA/NCCL error"); \
+    if (!(m)->attached) return fail(KDE_ESTATE, "sharded model not attached (kde_peer_attach)"); \
   } while (0)
 
 struct DeviceGuard {
@@ -224,6 +237,33 @@ static kde_status prof_begin(kde_model* m, cudaStream_t s, cudaEvent_t* e1, cuda
   return KDE_OK;
 }
 
+// ------------------------------------------------------------------ exchange (world > 1)
+// recv[r * bytes ...] <- rank r's send[0, bytes) for every rank (an all-gather), over NCCL or
+// over peer device memory (peer.cu, chunked by the window slot).  Stream-ordered.
+static kde_status allgather(kde_model* m, const void* send, void* recv, size_t bytes, cudaStream_t s) {
+  if (m->comm_kind == KDE_COMM_NCCL) {
+    NC(ncclAllGather(send, recv, bytes, ncclChar, m->comm, s));
+    return KDE_OK;
+  }
+  for (size_t o = 0; o < bytes; o += m->pa.slot) {
+    const size_t len = std::min(m->pa.slot, bytes - o);
+    CUL(launch_peer_allgather((const char*)send + o, (char*)recv + o, len, bytes, m->pa, m->num_sms, s));
+  }
+  return KDE_OK;
+}
+
+// after a synchronizing host call: a timed-out peer wait poisons the model
+static kde_status check_peer(kde_model* m) {
+  if (m->comm_kind != KDE_COMM_PEER) return KDE_OK;
+  int err = 0;
+  CU(cudaMemcpy(&err, m->pa.err, sizeof(int), cudaMemcpyDeviceToHost));
+  if (err) {
+    m->poisoned = true;
+    return fail(KDE_ECUDA, "peer exchange timed out (a rank did not join a collective call)");
+  }
+  return KDE_OK;
+}
+
 // ------------------------------------------------------------------ scans
 // Raw sums for q boxes (device bounds) -> sums[q][na] combined over ranks.
 // For q == 1 also retains c (if c_out) and writes the finalised values to fin.
@@ -292,7 +332,8 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     const size_t bytes = sizeof(double) * (size_t)m->world * q * na;
     kde_status st = ensure_bytes((void**)&m->gather, &m->gather_cap, bytes);
     if (st != KDE_OK) return st;
-    NC(ncclAllGather(d_sums, m->gather, (size_t)q * na, ncclDouble, m->comm, s));
+    st = allgather(m, d_sums, m->gather, sizeof(double) * (size_t)q * na, s);
+    if (st != KDE_OK) return st;
     CUL(launch_combine_ranks(m->gather, m->world, q, na, d_sums, s));
   }
   return KDE_OK;
@@ -366,14 +407,23 @@ static void free_model(kde_model* m) {
   cudaFree(m->gather);
   cudaFree(m->bitmap);
   cudaFree(m->block_counts);
+  cudaFree(m->block_offsets);
   cudaFree(m->offsets);
   cudaFree(m->done);
   cudaFree(m->idx_dev);
   cudaFree(m->bad);
   cudaFree(m->scal);
+  cudaFree(m->rbuf);
   if (m->pinned) cudaFreeHost(m->pinned);
   for (cudaEvent_t e : m->ev) cudaEventDestroy(e);
   if (m->comm) ncclCommDestroy(m->comm);
+  if (m->comm_kind == KDE_COMM_PEER) {
+    for (int r = 0; r < m->world; ++r)
+      if (r != m->rank && m->pa.base[r]) cudaIpcCloseMemHandle(m->pa.base[r]);
+    cudaFree(m->xwin);
+    cudaFree(m->pa.epoch);  // epoch, counters and error flag share one allocation
+  }
+  cudaFree(m->kbuf);
   if (m->stream) cudaStreamDestroy(m->stream);
   delete m;
 }
@@ -381,8 +431,48 @@ static void free_model(kde_model* m) {
 extern "C" void kde_destroy(kde_model* m) { free_model(m); }
 
 // ------------------------------------------------------------------ ABI: create
+// Scott's rule (eq. 3) over the GLOBAL sample: per-shard moments, all-gathered and Chan-merged in
+// rank order (world > 1), then h_j = n^(-1/(d+4)) sigma_j on the device.
+static kde_status scott_bandwidth(kde_model* m) {
+  const int d = m->d;
+  cudaStream_t s = m->stream;
+  const int nb = moments_blocks(m->n);
+  double* part = nullptr;
+  CU(cudaMalloc(&part, sizeof(double) * ((size_t)nb * d * 3 + (size_t)d * 3 * (m->world + 1))));
+  double* mom = part + (size_t)nb * d * 3;
+  double* gath = mom + (size_t)d * 3;
+  kde_status st = KDE_OK;
+  cudaError_t e = launch_moments(m->cols, m->ld, m->n, d, part, mom, s);
+  ++m->launches;
+  if (e == cudaSuccess && m->world > 1) {
+    st = allgather(m, mom, gath, sizeof(double) * (size_t)d * 3, s);
+    if (st == KDE_OK) e = launch_moments_merge_ranks(gath, m->world, d, mom, s);
+  }
+  if (e == cudaSuccess && st == KDE_OK) e = launch_scott(mom, d, m->consts, m->bad, s);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  cudaFree(part);
+  if (st != KDE_OK) return st;
+  if (e != cudaSuccess) {
+    m->poisoned = true;
+    return fail(KDE_ECUDA, "Scott bandwidth: %s", cudaGetErrorString(e));
+  }
+  st = check_peer(m);
+  if (st != KDE_OK) return st;
+  int32_t bad = 0;
+  CU(cudaMemcpy(&bad, m->bad, sizeof(int32_t), cudaMemcpyDeviceToHost));
+  if (bad) return fail(KDE_EINVAL, "Scott's rule gives h outside [1e-30, 1e30] (constant column?)");
+  return KDE_OK;
+}
+
+static size_t peer_slot_bytes() {
+  size_t mb = 4;
+  if (const char* v = getenv("KDE_PEER_SLOT_MB")) mb = (size_t)std::max(1, atoi(v));
+  return mb << 20;
+}
+
 static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_offset, int64_t n_global, int32_t d,
-                              const double* h, const void* nccl_id, int32_t rank, int32_t world, kde_model** out) {
+                              const double* h, const void* nccl_id, int32_t rank, int32_t world, int comm_kind,
+                              kde_model** out) {
   if (!out) return fail(KDE_EINVAL, "out is NULL");
   if (d < 1 || d > KDE_MAX_DIM) return fail(KDE_EINVAL, "d = %d outside [1, %d]", d, KDE_MAX_DIM);
   if (world < 1 || rank < 0 || rank >= world) return fail(KDE_EINVAL, "bad rank/world %d/%d", rank, world);
@@ -391,7 +481,8 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
     return fail(KDE_EINVAL, "shard [%lld, %lld) outside [0, %lld) or empty", (long long)row_offset,
                 (long long)(row_offset + n_local), (long long)n_global);
   if (!rows) return fail(KDE_EINVAL, "sample is NULL");
-  if (world > 1 && !nccl_id) return fail(KDE_EINVAL, "nccl_id is NULL for world > 1");
+  if (world > 1 && comm_kind == KDE_COMM_NCCL && !nccl_id) return fail(KDE_EINVAL, "nccl_id is NULL for world > 1");
+  if (world > kMaxWorld) return fail(KDE_EINVAL, "world %d > %d", world, kMaxWorld);
   if (h)
     for (int j = 0; j < d; ++j)
       if (!h_ok(h[j])) return fail(KDE_EINVAL, "h[%d] = %g not finite in [1e-30, 1e30]", j, h[j]);
@@ -411,6 +502,7 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
   m->row_offset = row_offset;
   m->rank = rank;
   m->world = world;
+  m->comm_kind = world > 1 ? comm_kind : KDE_COMM_NONE;
   m->ld = (n_local + kColAlign - 1) / kColAlign * kColAlign;
 #define CUB(call)                                                                                   \
   do {                                                                                              \
@@ -421,7 +513,7 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
   } while (0)
   CUB(cudaStreamCreateWithFlags(&m->stream, cudaStreamNonBlocking));
   CUB(cudaMalloc(&m->cols, sizeof(float) * (size_t)d * m->ld));
-  CUB(cudaMalloc(&m->karma, sizeof(double) * (size_t)n_local));
+  CUB(cudaMalloc(&m->karma, sizeof(double) * (size_t)m->ld));  // padded: 128-bit karma loads
   CUB(cudaMalloc(&m->cret, sizeof(float) * (size_t)m->ld));
   CUB(cudaMalloc(&m->consts, sizeof(DevConsts)));
   CUB(cudaMalloc(&m->online, sizeof(OnlineState)));
@@ -435,23 +527,44 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
   const int nkb = karma_blocks(n_local);
   CUB(cudaMalloc(&m->bitmap, sizeof(uint32_t) * (size_t)nkb * (kKarmaPts / 32)));
   CUB(cudaMalloc(&m->block_counts, sizeof(int32_t) * (size_t)nkb));
+  CUB(cudaMalloc(&m->block_offsets, sizeof(int64_t) * ((size_t)nkb + 1)));
   CUB(cudaMalloc(&m->offsets, sizeof(int64_t) * 2));
-  CUB(cudaMalloc(&m->done, sizeof(unsigned)));
+  CUB(cudaMalloc(&m->done, 2 * sizeof(unsigned)));
   cudaStream_t s = m->stream;
   CUB(cudaMemsetAsync(m->cols, 0, sizeof(float) * (size_t)d * m->ld, s));
-  CUB(cudaMemsetAsync(m->karma, 0, sizeof(double) * (size_t)n_local, s));
+  CUB(cudaMemsetAsync(m->karma, 0, sizeof(double) * (size_t)m->ld, s));
   CUB(cudaMemsetAsync(m->cret, 0, sizeof(float) * (size_t)m->ld, s));
   CUB(cudaMemsetAsync(m->consts, 0, sizeof(DevConsts), s));
   CUB(cudaMemsetAsync(m->online, 0, sizeof(OnlineState), s));
   CUB(cudaMemsetAsync(m->counter, 0, sizeof(unsigned), s));
-  CUB(cudaMemsetAsync(m->done, 0, sizeof(unsigned), s));
+  CUB(cudaMemsetAsync(m->done, 0, 2 * sizeof(unsigned), s));
   CUB(cudaMemsetAsync(m->bad, 0, sizeof(int32_t), s));
 
-  if (world > 1) {
+  if (m->comm_kind == KDE_COMM_NCCL) {
     ncclUniqueId id;
     memcpy(&id, nccl_id, sizeof(id));
     ncclResult_t r = ncclCommInitRank(&m->comm, world, id, rank);
     if (r != ncclSuccess) return bail(fail(KDE_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r)));
+  } else if (m->comm_kind == KDE_COMM_PEER) {
+    // exchange window (flags + 2 parities x world slots), zeroed before its handle is exported
+    m->pa.slot = peer_slot_bytes();
+    m->xwin_bytes = kPeerFlagBytes + 2 * (size_t)world * m->pa.slot;
+    CUB(cudaMalloc(&m->xwin, m->xwin_bytes));
+    CUB(cudaMemsetAsync(m->xwin, 0, kPeerFlagBytes, s));
+    char* ctl = nullptr;  // epoch (8 B) | 2 arrival counters | error flag
+    CUB(cudaMalloc(&ctl, 64));
+    CUB(cudaMemsetAsync(ctl, 0, 64, s));
+    m->pa.epoch = reinterpret_cast<uint64_t*>(ctl);
+    m->pa.count = reinterpret_cast<unsigned*>(ctl + 8);
+    m->pa.err = reinterpret_cast<int*>(ctl + 16);
+    m->pa.rank = rank;
+    m->pa.world = world;
+    double tmo = 60.0;
+    if (const char* v = getenv("KDE_PEER_TIMEOUT_S")) tmo = atof(v);
+    m->pa.timeout_ns = (uint64_t)(tmo * 1e9);
+    for (int r = 0; r < kMaxWorld; ++r) m->pa.base[r] = nullptr;
+    m->pa.base[rank] = m->xwin;
+    m->attached = false;
   }
 
   // sample: host row-major -> device (chunked through a pinned buffer) -> SoA columns
@@ -496,31 +609,14 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
     CUB(launch_col_range(m->cols, m->ld, n_local, d, m->range_enc, m->consts, s));
   }
 
-  // bandwidth: caller's h, or Scott's rule (eq. 3) over the global sample
+  // bandwidth: caller's h, or Scott's rule (eq. 3) over the global sample (peer transport: after attach)
   if (h) {
     CUB(launch_set_consts(h, d, m->consts, s));
+  } else if (m->comm_kind == KDE_COMM_PEER) {
+    m->h_pending = true;
   } else {
-    const int nb = moments_blocks(n_local);
-    double* part = nullptr;
-    CUB(cudaMalloc(&part, sizeof(double) * ((size_t)nb * d * 3 + (size_t)d * 3 * (world + 1))));
-    double* mom = part + (size_t)nb * d * 3;
-    double* gath = mom + (size_t)d * 3;
-    cudaError_t e = launch_moments(m->cols, m->ld, n_local, d, part, mom, s);
-    if (e == cudaSuccess && world > 1) {
-      ncclResult_t r = ncclAllGather(mom, gath, (size_t)d * 3, ncclDouble, m->comm, s);
-      if (r != ncclSuccess) {
-        cudaFree(part);
-        return bail(fail(KDE_ENCCL, "moments allgather: %s", ncclGetErrorString(r)));
-      }
-      e = launch_moments_merge_ranks(gath, world, d, mom, s);
-    }
-    if (e == cudaSuccess) e = launch_scott(mom, d, m->consts, m->bad, s);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
-    cudaFree(part);
-    if (e != cudaSuccess) return bail(fail(KDE_ECUDA, "Scott bandwidth: %s", cudaGetErrorString(e)));
-    int32_t bad = 0;
-    CUB(cudaMemcpy(&bad, m->bad, sizeof(int32_t), cudaMemcpyDeviceToHost));
-    if (bad) return bail(fail(KDE_EINVAL, "Scott's rule gives h outside [1e-30, 1e30] (constant column?)"));
+    st = scott_bandwidth(m);
+    if (st != KDE_OK) return bail(st);
   }
   CUB(cudaStreamSynchronize(s));
 #undef CUB
@@ -529,13 +625,57 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
 }
 
 extern "C" kde_status kde_create(const float* sample, int64_t n, int32_t d, const double* h, kde_model** out) {
-  return create_impl(sample, n, 0, n, d, h, nullptr, 0, 1, out);
+  return create_impl(sample, n, 0, n, d, h, nullptr, 0, 1, KDE_COMM_NONE, out);
 }
 
 extern "C" kde_status kde_create_sharded(const float* local_rows, int64_t n_local, int64_t row_offset,
                                          int64_t n_global, int32_t d, const double* h, const void* nccl_id,
                                          int32_t rank, int32_t world, kde_model** out) {
-  return create_impl(local_rows, n_local, row_offset, n_global, d, h, nccl_id, rank, world, out);
+  return create_impl(local_rows, n_local, row_offset, n_global, d, h, nccl_id, rank, world, KDE_COMM_NCCL, out);
+}
+
+extern "C" kde_status kde_create_sharded_peer(const float* local_rows, int64_t n_local, int64_t row_offset,
+                                              int64_t n_global, int32_t d, const double* h, int32_t rank,
+                                              int32_t world, kde_model** out) {
+  return create_impl(local_rows, n_local, row_offset, n_global, d, h, nullptr, rank, world,
+                     world > 1 ? KDE_COMM_PEER : KDE_COMM_NONE, out);
+}
+
+extern "C" kde_status kde_peer_handle(kde_model* m, void* handle_out) {
+  if (!m || !handle_out) return fail(KDE_EINVAL, "NULL argument");
+  if (m->comm_kind != KDE_COMM_PEER) return fail(KDE_EINVAL, "model does not use the peer transport");
+  DeviceGuard g(m->device);
+  cudaIpcMemHandle_t hnd;
+  CU(cudaIpcGetMemHandle(&hnd, m->xwin));
+  static_assert(sizeof(hnd) == KDE_PEER_HANDLE_BYTES, "IPC handle size");
+  memcpy(handle_out, &hnd, sizeof(hnd));
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_peer_attach(kde_model* m, const void* handles) {
+  if (!m || !handles) return fail(KDE_EINVAL, "NULL argument");
+  if (m->comm_kind != KDE_COMM_PEER) return fail(KDE_EINVAL, "model does not use the peer transport");
+  if (m->attached) return fail(KDE_ESTATE, "already attached");
+  if (m->poisoned) return fail(KDE_ESTATE, "model poisoned by an earlier CUDA/NCCL error");
+  DeviceGuard g(m->device);
+  for (int r = 0; r < m->world; ++r) {
+    if (r == m->rank) continue;
+    cudaIpcMemHandle_t hnd;
+    memcpy(&hnd, (const char*)handles + (size_t)r * KDE_PEER_HANDLE_BYTES, sizeof(hnd));
+    void* p = nullptr;
+    CU(cudaIpcOpenMemHandle(&p, hnd, cudaIpcMemLazyEnablePeerAccess));
+    m->pa.base[r] = (char*)p;
+  }
+  m->attached = true;
+  if (m->h_pending) {  // Scott's rule needs the all-gather of the shard moments
+    m->h_pending = false;
+    kde_status st = scott_bandwidth(m);
+    if (st != KDE_OK) {
+      m->poisoned = true;
+      return st;
+    }
+  }
+  return KDE_OK;
 }
 
 extern "C" kde_status kde_get_info(const kde_model* m, int64_t* n_local, int64_t* n_global, int32_t* d,
@@ -664,6 +804,8 @@ extern "C" kde_status kde_estimate_batch(kde_model* m, const float* lo, const fl
     if (grad) CU(cudaMemcpyAsync(dest_dh, d_dpdh, sizeof(double) * q * m->d, cudaMemcpyDeviceToHost, m->stream));
   }
   CU(cudaStreamSynchronize(m->stream));
+  st = check_peer(m);
+  if (st != KDE_OK) return st;
   if (q == 1) note_retained(m, lo, hi, retain_c, grad);
   return KDE_OK;
 }
@@ -685,6 +827,9 @@ static kde_status loss_grad_dev_impl(kde_model* m, const float* d_lo, const floa
                                      double* d_grad, double* d_est_out, cudaStream_t s) {
   kde_status st = ensure_q(m, q);
   if (st != KDE_OK) return st;
+  // the scan below overwrites the retained (p_hat, dp_hat/dh) of a q == 1 batch: whatever box was
+  // retained before is no longer what m->ret holds (stale ret_valid after loss_and_grad)
+  m->ret_valid = false;
   double* d_est = d_est_out ? d_est_out : o_est(m);
   double* d_dpdh = o_dpdh(m);
   st = estimate_dev(m, d_lo, d_hi, q, d_est, d_dpdh, s, false);
@@ -716,7 +861,7 @@ extern "C" kde_status kde_loss_and_grad(kde_model* m, const float* lo, const flo
   CU(cudaMemcpyAsync(grad_out, o_grad(m), sizeof(double) * m->d, cudaMemcpyDeviceToHost, m->stream));
   if (est_out) CU(cudaMemcpyAsync(est_out, o_est(m), sizeof(double) * q, cudaMemcpyDeviceToHost, m->stream));
   CU(cudaStreamSynchronize(m->stream));
-  return KDE_OK;
+  return check_peer(m);
 }
 
 extern "C" kde_status kde_loss_and_grad_dev(kde_model* m, const float* d_lo, const float* d_hi,
@@ -832,7 +977,7 @@ extern "C" kde_status kde_karma_update(kde_model* m, const float* lo, const floa
   CU(cudaMemcpyAsync(m->scal, &true_sel, sizeof(double), cudaMemcpyHostToDevice, m->stream));
   m->launches += 1;  // karma + fused compaction
   CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, m->scal, kd, m->qbuf, m->qbuf + m->d, m->d,
-                  m->consts, m->bitmap, m->block_counts, m->done, m->row_offset, m->idx_dev, local_cap, m->offsets,
+                  m->consts, m->bitmap, m->block_counts, m->block_offsets, m->done, m->row_offset, m->idx_dev, local_cap, m->offsets,
                   StreamTail{}, m->stream));
   int64_t local_total = 0;
   CU(cudaMemcpyAsync(&local_total, m->offsets, sizeof(int64_t), cudaMemcpyDeviceToHost, m->stream));
@@ -844,22 +989,20 @@ extern "C" kde_status kde_karma_update(kde_model* m, const float* lo, const floa
     return local_total > idx_cap ? fail(KDE_ETRUNC, "%lld flagged > idx_cap %lld", (long long)local_total, (long long)idx_cap)
                                  : KDE_OK;
   }
-  // world > 1: gather counts, then the (ascending, rank-ordered) index lists
+  // world > 1: all-gather the counts, then the (ascending) index lists; concatenated in rank
+  // order they are the ascending GLOBAL list (contiguous row shards)
+  const size_t cnt_bytes = sizeof(int64_t) * (size_t)(m->world + 1);
+  st = ensure_bytes(&m->kbuf, &m->kbuf_cap, cnt_bytes);
+  if (st != KDE_OK) return st;
+  int64_t* d_cnt = (int64_t*)m->kbuf;  // [world] gathered + [1] own
+  CU(cudaMemcpyAsync(d_cnt + m->world, m->offsets, sizeof(int64_t), cudaMemcpyDeviceToDevice, m->stream));
+  st = allgather(m, d_cnt + m->world, d_cnt, sizeof(int64_t), m->stream);
+  if (st != KDE_OK) return st;
   std::vector<int64_t> counts(m->world);
-  {
-    int64_t* d_cnt = nullptr;
-    CU(cudaMalloc(&d_cnt, sizeof(int64_t) * (m->world + 1)));
-    CU(cudaMemcpyAsync(d_cnt + m->world, &local_total, sizeof(int64_t), cudaMemcpyHostToDevice, m->stream));
-    ncclResult_t r = ncclAllGather(d_cnt + m->world, d_cnt, 1, ncclInt64, m->comm, m->stream);
-    if (r != ncclSuccess) {
-      cudaFree(d_cnt);
-      m->poisoned = true;
-      return fail(KDE_ENCCL, "karma count allgather: %s", ncclGetErrorString(r));
-    }
-    CU(cudaMemcpyAsync(counts.data(), d_cnt, sizeof(int64_t) * m->world, cudaMemcpyDeviceToHost, m->stream));
-    CU(cudaStreamSynchronize(m->stream));
-    cudaFree(d_cnt);
-  }
+  CU(cudaMemcpyAsync(counts.data(), d_cnt, sizeof(int64_t) * m->world, cudaMemcpyDeviceToHost, m->stream));
+  CU(cudaStreamSynchronize(m->stream));
+  st = check_peer(m);
+  if (st != KDE_OK) return st;
   int64_t maxc = 0, total = 0;
   for (int64_t c : counts) {
     maxc = std::max(maxc, c);
@@ -867,27 +1010,28 @@ extern "C" kde_status kde_karma_update(kde_model* m, const float* lo, const floa
   }
   *n_flagged = total;
   if (maxc > 0) {
-    int64_t* d_all = nullptr;
-    CU(cudaMalloc(&d_all, sizeof(int64_t) * (size_t)maxc * (m->world + 1)));
-    int64_t* d_send = d_all + (size_t)maxc * m->world;
-    if (local_total > 0)
-      CU(cudaMemcpyAsync(d_send, m->idx_dev, sizeof(int64_t) * local_total, cudaMemcpyDeviceToDevice, m->stream));
-    ncclResult_t r = ncclAllGather(d_send, d_all, (size_t)maxc, ncclInt64, m->comm, m->stream);
-    if (r != ncclSuccess) {
-      cudaFree(d_all);
-      m->poisoned = true;
-      return fail(KDE_ENCCL, "karma index allgather: %s", ncclGetErrorString(r));
-    }
+    // only the first idx_cap indices are returned: no rank sends more than that
+    const int64_t send = std::min(maxc, std::max<int64_t>(idx_cap, 1));
+    st = ensure_bytes(&m->kbuf, &m->kbuf_cap, cnt_bytes + sizeof(int64_t) * (size_t)send * (m->world + 1));
+    if (st != KDE_OK) return st;
+    d_cnt = (int64_t*)m->kbuf;
+    int64_t* d_all = d_cnt + m->world + 1;
+    int64_t* d_send = d_all + (size_t)send * m->world;
+    const int64_t mine = std::min(local_total, send);
+    if (mine > 0) CU(cudaMemcpyAsync(d_send, m->idx_dev, sizeof(int64_t) * mine, cudaMemcpyDeviceToDevice, m->stream));
+    st = allgather(m, d_send, d_all, sizeof(int64_t) * (size_t)send, m->stream);
+    if (st != KDE_OK) return st;
     int64_t pos = 0;
     for (int rr = 0; rr < m->world && pos < idx_cap; ++rr) {
-      const int64_t k = std::min(counts[rr], idx_cap - pos);
+      const int64_t k = std::min(std::min(counts[rr], send), idx_cap - pos);
       if (k > 0)
-        CU(cudaMemcpyAsync(idx_out + pos, d_all + (size_t)rr * maxc, sizeof(int64_t) * k, cudaMemcpyDeviceToHost,
+        CU(cudaMemcpyAsync(idx_out + pos, d_all + (size_t)rr * send, sizeof(int64_t) * k, cudaMemcpyDeviceToHost,
                            m->stream));
       pos += k;
     }
     CU(cudaStreamSynchronize(m->stream));
-    cudaFree(d_all);
+    st = check_peer(m);
+    if (st != KDE_OK) return st;
   }
   return total > idx_cap ? fail(KDE_ETRUNC, "%lld flagged > idx_cap %lld", (long long)total, (long long)idx_cap) : KDE_OK;
 }
@@ -914,6 +1058,37 @@ extern "C" kde_status kde_online_update(kde_model* m, const float* lo, const flo
   return KDE_OK;
 }
 
+// Rows owned by this shard -> device staging (grow-only buffer, no per-call allocation) -> scatter.
+// idx are validated GLOBAL indices, unique; rows host row-major k x d.
+static kde_status replace_impl(kde_model* m, const int64_t* idx, const float* rows, int64_t k, double k_init) {
+  std::vector<int64_t> li;
+  std::vector<float> lr;
+  for (int64_t r = 0; r < k; ++r) {
+    const int64_t i = idx[r] - m->row_offset;
+    if (i >= 0 && i < m->n) {
+      li.push_back(i);
+      lr.insert(lr.end(), rows + r * m->d, rows + (r + 1) * m->d);
+    }
+  }
+  const int64_t kl = (int64_t)li.size();
+  if (kl > 0) {
+    const size_t ib = sizeof(int64_t) * kl, rb = sizeof(float) * kl * m->d;
+    kde_status st = ensure_pinned(m, ib + rb);
+    if (st != KDE_OK) return st;
+    st = ensure_bytes(&m->rbuf, &m->rbuf_cap, ib + rb);
+    if (st != KDE_OK) return st;
+    memcpy(m->pinned, li.data(), ib);
+    memcpy((char*)m->pinned + ib, lr.data(), rb);
+    CU(cudaMemcpyAsync(m->rbuf, m->pinned, ib + rb, cudaMemcpyHostToDevice, m->stream));
+    CUL(launch_row_range((const float*)((char*)m->rbuf + ib), kl, m->d, m->range_enc, m->consts, m->stream));
+    CUL(launch_scatter_rows((const int64_t*)m->rbuf, (const float*)((char*)m->rbuf + ib), kl, m->d, m->cols, m->ld,
+                           m->karma, k_init, m->stream));
+    CU(cudaStreamSynchronize(m->stream));  // the pinned staging buffer is reused by the next call
+  }
+  ++m->gen;
+  return KDE_OK;
+}
+
 extern "C" kde_status kde_replace_points(kde_model* m, const int64_t* idx, const float* rows, int64_t k,
                                          double k_init) {
   CHECK_MODEL(m);
@@ -929,34 +1104,51 @@ extern "C" kde_status kde_replace_points(kde_model* m, const int64_t* idx, const
   }
   for (int64_t e = 0; e < k * m->d; ++e)
     if (!std::isfinite(rows[e])) return fail(KDE_EINVAL, "non-finite value in replacement rows");
-  // rows owned by this shard
-  std::vector<int64_t> li;
-  std::vector<float> lr;
-  for (int64_t r = 0; r < k; ++r) {
-    const int64_t i = idx[r] - m->row_offset;
-    if (i >= 0 && i < m->n) {
-      li.push_back(i);
-      lr.insert(lr.end(), rows + r * m->d, rows + (r + 1) * m->d);
-    }
+  DeviceGuard g(m->device);
+  return replace_impl(m, idx, rows, k, k_init);
+}
+
+// ------------------------------------------------------------------ ABI: reservoir inserts
+extern "C" kde_status kde_reservoir_select(uint64_t seed, int64_t n_sample, int64_t n_seen, int64_t k,
+                                           int64_t* slot_out) {
+  if (n_sample < 1) return fail(KDE_EINVAL, "n_sample < 1");
+  if (n_seen < 0 || k < 0 || n_seen > INT64_MAX - k) return fail(KDE_EINVAL, "bad n_seen / k");
+  if (k > 0 && !slot_out) return fail(KDE_EINVAL, "slot_out is NULL");
+  reservoir_slots(seed, n_sample, n_seen, k, slot_out);
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_insert_rows(kde_model* m, const float* rows, int64_t k, uint64_t seed, int64_t* n_seen,
+                                      double k_init, int64_t* n_written) {
+  CHECK_MODEL(m);
+  if (k < 0 || !n_seen || *n_seen < 0 || *n_seen > INT64_MAX - k) return fail(KDE_EINVAL, "bad k / n_seen");
+  if (k > 0 && !rows) return fail(KDE_EINVAL, "rows is NULL");
+  if (!std::isfinite(k_init)) return fail(KDE_EINVAL, "k_init not finite");
+  for (int64_t e = 0; e < k * m->d; ++e)
+    if (!std::isfinite(rows[e])) return fail(KDE_EINVAL, "non-finite value in inserted rows");
+  std::vector<int64_t> slot((size_t)k);
+  reservoir_slots(seed, m->n_global, *n_seen, k, slot.data());
+  // several arrivals of one chunk may take the same slot: the last one wins (sequential semantics);
+  // only the winners are transferred
+  std::vector<std::pair<int64_t, int64_t>> win;  // (slot, arrival row)
+  win.reserve((size_t)k);
+  for (int64_t r = 0; r < k; ++r)
+    if (slot[r] >= 0) win.emplace_back(slot[r], r);
+  std::stable_sort(win.begin(), win.end(), [](const auto& a, const auto& b) { return a.first < b.first; });
+  std::vector<int64_t> idx;
+  std::vector<float> sel;
+  idx.reserve(win.size());
+  sel.reserve(win.size() * m->d);
+  for (size_t i = 0; i < win.size(); ++i) {
+    if (i + 1 < win.size() && win[i + 1].first == win[i].first) continue;  // a later arrival overwrites this slot
+    idx.push_back(win[i].first);
+    sel.insert(sel.end(), rows + win[i].second * m->d, rows + (win[i].second + 1) * m->d);
   }
   DeviceGuard g(m->device);
-  const int64_t kl = (int64_t)li.size();
-  if (kl > 0) {
-    const size_t ib = sizeof(int64_t) * kl, rb = sizeof(float) * kl * m->d;
-    kde_status st = ensure_pinned(m, ib + rb);
-    if (st != KDE_OK) return st;
-    void* dbuf = nullptr;
-    CU(cudaMalloc(&dbuf, ib + rb));
-    memcpy(m->pinned, li.data(), ib);
-    memcpy((char*)m->pinned + ib, lr.data(), rb);
-    CU(cudaMemcpyAsync(dbuf, m->pinned, ib + rb, cudaMemcpyHostToDevice, m->stream));
-    CUL(launch_row_range((const float*)((char*)dbuf + ib), kl, m->d, m->range_enc, m->consts, m->stream));
-    CUL(launch_scatter_rows((const int64_t*)dbuf, (const float*)((char*)dbuf + ib), kl, m->d, m->cols, m->ld,
-                           m->karma, k_init, m->stream));
-    CU(cudaStreamSynchronize(m->stream));
-    cudaFree(dbuf);
-  }
-  ++m->gen;
+  kde_status st = idx.empty() ? KDE_OK : replace_impl(m, idx.data(), sel.data(), (int64_t)idx.size(), k_init);
+  if (st != KDE_OK) return st;
+  *n_seen += k;
+  if (n_written) *n_written = (int64_t)idx.size();
   return KDE_OK;
 }
 
@@ -974,7 +1166,7 @@ extern "C" kde_status kde_karma_update_dev(kde_model* m, const float* d_lo, cons
   cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
   m->launches += 1;
   CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, d_true_sel, kd, d_lo, d_hi, m->d,
-                   m->consts, m->bitmap, m->block_counts, m->done, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
+                   m->consts, m->bitmap, m->block_counts, m->block_offsets, m->done, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
                    StreamTail{}, s));
   return KDE_OK;
 }
@@ -1050,7 +1242,7 @@ extern "C" kde_status kde_stream_step_dev(kde_model* m, const float* d_lo, const
   if (st != KDE_OK) return st;
   m->launches += 1;
   CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, d_true_sel, kd, d_lo, d_hi, m->d,
-                   m->consts, m->bitmap, m->block_counts, m->done, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
+                   m->consts, m->bitmap, m->block_counts, m->block_offsets, m->done, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
                    tail, s));
   ++m->gen;
   return KDE_OK;

@@ -331,68 +331,127 @@ __device__ double thr20_dev(const float* lo, const float* hi, int d, const DevCo
 }
 
 #ifndef KDE_TUNE_KARMA_MINB
-#define KDE_TUNE_KARMA_MINB 4  // 64 registers, 4 blocks per SM (r77 A/B: 26.7 -> 24.6 us at n = 2^22)
+#define KDE_TUNE_KARMA_MINB 4  // 64 registers, 4 blocks per SM
 #endif
-__global__ void __launch_bounds__(kKarmaThreads, KDE_TUNE_KARMA_MINB) karma_kernel(const float* __restrict__ cvals, double* __restrict__ karma, int64_t n, double n_global,
-                             const double* __restrict__ phat_ptr, const double* __restrict__ p_ptr, KarmaParamsDev kp,
-                             const float* lo,
-                             const float* hi, int d, const DevConsts* c, uint32_t* __restrict__ bitmap,
-                             int32_t* __restrict__ block_counts) {
+// Each block owns kKarmaPts contiguous points; a thread takes KV = 4 consecutive points per pass
+// (one float4 of p^(i), two double2 of K: 128-bit loads and stores, the karma array is padded to
+// the column length), all passes' loads issued before any arithmetic.  Flag bits are assembled
+// into index-order bitmap words with three shuffles (8 lanes x 4 points = one word).  The last
+// block to finish turns the per-block counts into exclusive offsets (one O(nb) scan), so the
+// compaction needs no prefix of its own.
+constexpr int kKarmaKV = 4;
+__global__ void __launch_bounds__(kKarmaThreads, KDE_TUNE_KARMA_MINB)
+    karma_kernel(const float* __restrict__ cvals, double* __restrict__ karma, int64_t n, double n_global,
+                 const double* __restrict__ phat_ptr, const double* __restrict__ p_ptr, KarmaParamsDev kp,
+                 const float* lo, const float* hi, int d, const DevConsts* c, uint32_t* __restrict__ bitmap,
+                 int32_t* __restrict__ block_counts, int64_t* __restrict__ block_offsets, unsigned* __restrict__ kdone,
+                 int nb) {
   __shared__ double thr_s;
   __shared__ int32_t wcount[kKarmaThreads / 32];
+  __shared__ bool last_s;
   const double p = *p_ptr;
   if (threadIdx.x == 0) thr_s = (kp.empty_region && p == 0.0) ? thr20_dev(lo, hi, d, c) : CUDART_INF;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  if (lane == 0) wcount[warp] = 0;
   __syncthreads();
   const double phat = *phat_ptr;
   double L_full, dummy;
   loss_eval(kp.loss, kp.lambda, phat, p, &L_full, &dummy);
   const double thr = thr_s;
   const int64_t base = (int64_t)blockIdx.x * kKarmaPts;
-  constexpr int P = kKarmaPts / kKarmaThreads;
+  constexpr int PASSES = kKarmaPts / (kKarmaThreads * kKarmaKV);
 #ifndef KDE_TUNE_KARMA_PB
-#define KDE_TUNE_KARMA_PB 8
+#define KDE_TUNE_KARMA_PB 2
 #endif
-  constexpr int PB = KDE_TUNE_KARMA_PB;  // points per load batch (PB loads of c and K in flight per thread)
+  constexpr int PB = KDE_TUNE_KARMA_PB;  // passes per load batch
+  static_assert(PASSES % PB == 0, "karma load batches");
   const double inv_nm1 = 1.0 / (n_global - 1.0);
   int32_t my = 0;
 #pragma unroll 1
-  for (int r0 = 0; r0 < P; r0 += PB) {
-    float cv[PB];
-    double kv[PB];
+  for (int r0 = 0; r0 < PASSES; r0 += PB) {
+    float4 cv[PB];
+    double2 kv[PB][2];
 #pragma unroll
     for (int r = 0; r < PB; ++r) {
-      const int64_t i = base + (r0 + r) * kKarmaThreads + threadIdx.x;
-      cv[r] = i < n ? cvals[i] : 0.0f;
-      kv[r] = i < n ? karma[i] : 0.0;
+      const int64_t i = base + ((int64_t)(r0 + r) * kKarmaThreads + threadIdx.x) * kKarmaKV;
+      if (i < n) {  // i is a multiple of 4; c and K are padded past n
+        cv[r] = __ldcs(reinterpret_cast<const float4*>(cvals + i));
+        kv[r][0] = __ldcs(reinterpret_cast<const double2*>(karma + i));
+        kv[r][1] = __ldcs(reinterpret_cast<const double2*>(karma + i + 2));
+      } else {
+        cv[r] = make_float4(0.f, 0.f, 0.f, 0.f);
+        kv[r][0] = kv[r][1] = make_double2(0.0, 0.0);
+      }
     }
 #pragma unroll
     for (int r = 0; r < PB; ++r) {
-      const int64_t i = base + (r0 + r) * kKarmaThreads + threadIdx.x;
-      bool flag = false;
-      if (i < n) {
-        const double ci = (double)cv[r];
-        const double p_minus = (phat * n_global - ci) * inv_nm1;  // eq. (6)
-        double L_minus;
-        loss_eval(kp.loss, kp.lambda, p_minus, p, &L_minus, &dummy);
-        const double k = fmin(kv[r] + (L_minus - L_full), kp.k_max);  // eq. (7)-(8)
-        karma[i] = k;
-        flag = (k < kp.threshold) || (ci >= thr);
+      const int64_t i = base + ((int64_t)(r0 + r) * kKarmaThreads + threadIdx.x) * kKarmaKV;
+      const float cc[4] = {cv[r].x, cv[r].y, cv[r].z, cv[r].w};
+      double kk[4] = {kv[r][0].x, kv[r][0].y, kv[r][1].x, kv[r][1].y};
+      unsigned nib = 0u;
+#pragma unroll
+      for (int v = 0; v < kKarmaKV; ++v) {
+        if (i + v < n) {
+          const double ci = (double)cc[v];
+          const double p_minus = (phat * n_global - ci) * inv_nm1;  // eq. (6)
+          double L_minus;
+          loss_eval(kp.loss, kp.lambda, p_minus, p, &L_minus, &dummy);
+          kk[v] = fmin(kk[v] + (L_minus - L_full), kp.k_max);  // eq. (7)-(8)
+          const bool flag = (kk[v] < kp.threshold) || (ci >= thr);
+          nib |= (unsigned)flag << v;
+        }
       }
-      const uint32_t word = __ballot_sync(0xffffffffu, flag);
-      if (lane == 0) {
-        bitmap[(base + (r0 + r) * kKarmaThreads + warp * 32) / 32] = word;
+      if (i < n) {
+        __stcs(reinterpret_cast<double2*>(karma + i), make_double2(kk[0], kk[1]));
+        __stcs(reinterpret_cast<double2*>(karma + i + 2), make_double2(kk[2], kk[3]));
+      }
+      // word w of this warp's 128 points = nibbles of lanes 8w .. 8w+7
+      unsigned word = nib << (4 * (lane & 7));
+      word |= __shfl_xor_sync(0xffffffffu, word, 1);
+      word |= __shfl_xor_sync(0xffffffffu, word, 2);
+      word |= __shfl_xor_sync(0xffffffffu, word, 4);
+      if ((lane & 7) == 0) {
+        const int64_t w0 = (base + ((int64_t)(r0 + r) * kKarmaThreads + warp * 32) * kKarmaKV) / 32;
+        bitmap[w0 + (lane >> 3)] = word;
         my += __popc(word);
       }
     }
   }
+  for (int o = 8; o < 32; o <<= 1) my += __shfl_xor_sync(0xffffffffu, my, o);
   if (lane == 0) wcount[warp] = my;
   __syncthreads();
   if (threadIdx.x == 0) {
     int32_t t = 0;
     for (int w = 0; w < kKarmaThreads / 32; ++w) t += wcount[w];
     block_counts[blockIdx.x] = t;
+    __threadfence();
+    last_s = atomicAdd(kdone, 1u) == (unsigned)nb - 1;
+  }
+  __syncthreads();
+  if (!last_s) return;
+  __threadfence();
+  // last block: exclusive offsets of the nb block counts, fixed order (each thread a contiguous run)
+  __shared__ int64_t run_s[kKarmaThreads];
+  const int per = (nb + kKarmaThreads - 1) / kKarmaThreads;
+  const int b0 = min(nb, (int)threadIdx.x * per), b1 = min(nb, b0 + per);
+  int64_t t = 0;
+  for (int b = b0; b < b1; ++b) t += __ldcg(block_counts + b);
+  run_s[threadIdx.x] = t;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    int64_t acc = 0;
+    for (int k = 0; k < kKarmaThreads; ++k) {
+      const int64_t v = run_s[k];
+      run_s[k] = acc;
+      acc += v;
+    }
+    block_offsets[nb] = acc;  // total
+    *kdone = 0u;
+  }
+  __syncthreads();
+  int64_t o = run_s[threadIdx.x];
+  for (int b = b0; b < b1; ++b) {
+    block_offsets[b] = o;
+    o += __ldcg(block_counts + b);
   }
 }
 
@@ -408,22 +467,17 @@ __device__ __noinline__ void online_update_body(const double* __restrict__ ret, 
 #ifndef KDE_TUNE_COMPACT_MINB
 #define KDE_TUNE_COMPACT_MINB 8
 #endif
-__global__ void __launch_bounds__(kKarmaThreads, KDE_TUNE_COMPACT_MINB) compact_fused_kernel(const uint32_t* __restrict__ bitmap, int64_t n, const int32_t* __restrict__ counts,
+__global__ void __launch_bounds__(kKarmaThreads, KDE_TUNE_COMPACT_MINB) compact_fused_kernel(const uint32_t* __restrict__ bitmap, int64_t n, const int64_t* __restrict__ block_offsets,
                                      int nb, int64_t row_offset, int64_t* __restrict__ idx_out, int64_t cap,
                                      int64_t* __restrict__ total_out, unsigned* __restrict__ done, StreamTail tail) {
   constexpr int W = kKarmaPts / 32;  // bitmap words per block
   constexpr int WPL = W / 32;
   __shared__ int32_t wpre[W];
   __shared__ uint32_t wbits[W];  // the block's bitmap words, read once by warp 0
-  __shared__ int64_t red[kKarmaThreads / 32];
   __shared__ int64_t off_s;
   __shared__ bool last_s;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  // block offset: fixed-order integer sum of the preceding block counts
-  int64_t o = 0;
-  for (int b = tid; b < (int)blockIdx.x; b += kKarmaThreads) o += counts[b];
-  for (int k = 16; k > 0; k >>= 1) o += __shfl_xor_sync(0xffffffffu, o, k);
-  if (lane == 0) red[warp] = o;
+  if (tid == 0) off_s = __ldg(block_offsets + blockIdx.x);  // exclusive offset (karma_kernel's last block)
   const int64_t wbase = (int64_t)blockIdx.x * W;
   const int64_t nwords = (n + 31) / 32;
   if (tid < 32) {  // exclusive prefix of the block's word popcounts
@@ -450,12 +504,6 @@ __global__ void __launch_bounds__(kKarmaThreads, KDE_TUNE_COMPACT_MINB) compact_
     }
   }
   __syncthreads();
-  if (tid == 0) {
-    int64_t t = 0;
-    for (int w = 0; w < kKarmaThreads / 32; ++w) t += red[w];
-    off_s = t;
-  }
-  __syncthreads();
   const int64_t off = off_s;
 #pragma unroll 4
   for (int w = warp; w < W; w += kKarmaThreads / 32) {
@@ -472,15 +520,8 @@ __global__ void __launch_bounds__(kKarmaThreads, KDE_TUNE_COMPACT_MINB) compact_
   __syncthreads();
   if (!last_s) return;
   __threadfence();
-  int64_t t = 0;
-  for (int b = tid; b < nb; b += kKarmaThreads) t += __ldcg(counts + b);
-  for (int k = 16; k > 0; k >>= 1) t += __shfl_xor_sync(0xffffffffu, t, k);
-  __syncthreads();
-  if (lane == 0) red[warp] = t;
-  __syncthreads();
   if (tid == 0) {
-    int64_t tot = 0;
-    for (int w = 0; w < kKarmaThreads / 32; ++w) tot += red[w];
+    const int64_t tot = __ldg(block_offsets + nb);
     off_s = tot;
     if (total_out) *total_out = tot;
     *done = 0u;
@@ -709,15 +750,16 @@ cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const do
 }
 cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, const double* p,
                          const KarmaParamsDev& kp, const float* lo, const float* hi, int d, const DevConsts* c,
-                         uint32_t* bitmap, int32_t* block_counts, unsigned* done, int64_t row_offset, int64_t* idx_out,
-                         int64_t cap, int64_t* total_out, const StreamTail& tail, cudaStream_t s) {
+                         uint32_t* bitmap, int32_t* block_counts, int64_t* block_offsets, unsigned* done,
+                         int64_t row_offset, int64_t* idx_out, int64_t cap, int64_t* total_out, const StreamTail& tail,
+                         cudaStream_t s) {
   const int nb = karma_blocks(n);
   if (nb == 0) return cudaSuccess;
   karma_kernel<<<nb, kKarmaThreads, 0, s>>>(cvals, karma, n, n_global, phat, p, kp, lo, hi, d, c, bitmap,
-                                            block_counts);
+                                            block_counts, block_offsets, done + 1, nb);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  compact_fused_kernel<<<nb, kKarmaThreads, 0, s>>>(bitmap, n, block_counts, nb, row_offset, idx_out, cap, total_out,
+  compact_fused_kernel<<<nb, kKarmaThreads, 0, s>>>(bitmap, n, block_offsets, nb, row_offset, idx_out, cap, total_out,
                                                     done, tail);
   KDE_LAUNCH_CHECK();
 }

@@ -67,13 +67,35 @@ cudaError_t launch_finalize(const double* sums, int64_t q, int d, int na, const 
 cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const double* true_sel, int64_t q, int d,
                                  int kind, double lambda, int log_bw, const DevConsts* c, double* loss_out,
                                  double* grad_out, cudaStream_t s);
+// karma pass + ordered compaction: block_counts int32 [nb], block_offsets int64 [nb + 1],
+// done: 2 self-resetting counters (compaction, karma); c and karma padded to a multiple of 4 points
 cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, const double* p,
                          const KarmaParamsDev& kp, const float* lo, const float* hi, int d, const DevConsts* c,
-                         uint32_t* bitmap, int32_t* block_counts, unsigned* done, int64_t row_offset, int64_t* idx_out,
-                         int64_t cap, int64_t* total_out, const StreamTail& tail, cudaStream_t s);
+                         uint32_t* bitmap, int32_t* block_counts, int64_t* block_offsets, unsigned* done,
+                         int64_t row_offset, int64_t* idx_out, int64_t cap, int64_t* total_out, const StreamTail& tail,
+                         cudaStream_t s);
 cudaError_t launch_online_update(const double* ret, const double* p, const OnlineParamsDev& op, int d, OnlineState* st,
                                  DevConsts* c, cudaStream_t s);
 cudaError_t launch_count_in_box(const float* rows, int64_t n, int d, const float* lo, const float* hi, int64_t q,
                                 unsigned long long* counts, int num_sms, cudaStream_t s);
+
+// reservoir.cu: Algorithm R decisions (host), slot or -1 per arrival n_seen+1 .. n_seen+k
+void reservoir_slots(uint64_t seed, int64_t n_sample, int64_t n_seen, int64_t k, int64_t* slot_out);
+
+// peer.cu: all-gather over peer device memory (the sharded model's exchange step without NCCL)
+constexpr int kMaxWorld = 32;
+constexpr size_t kPeerFlagBytes = (size_t)kMaxWorld * 128;  // one 128-byte line per source rank
+struct PeerArgs {
+  char* base[kMaxWorld];  // every rank's exchange window, mapped into this process (base[rank] = own)
+  int rank = 0, world = 1;
+  size_t slot = 0;        // bytes per (parity, source rank) slot, multiple of 256
+  uint64_t* epoch = nullptr;  // device: last completed exchange
+  unsigned* count = nullptr;  // device: 2 self-resetting block-arrival counters
+  int* err = nullptr;         // device: set to 1 when a wait times out
+  uint64_t timeout_ns = 0;
+};
+// dst + r * stride <- rank r's src (bytes <= pa.slot, multiples of 8), for every rank r
+cudaError_t launch_peer_allgather(const void* src, void* dst, size_t bytes, size_t stride, const PeerArgs& pa,
+                                  int num_sms, cudaStream_t s);
 
 }  // namespace kde

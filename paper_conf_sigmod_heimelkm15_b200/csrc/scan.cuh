@@ -21,6 +21,7 @@
 //   shared memory; per-(split, box) partials go to global memory and are
 //   reduced in fixed split order by reduce_splits_kernel (kernels.cu).
 #pragma once
+#include <atomic>
 #include <cstdint>
 #include <cuda_runtime.h>
 
@@ -154,6 +155,30 @@ __device__ __forceinline__ float2 point_box2(const BoxDim (&bd)[D], const float2
     }
   }
   return pre[D];
+}
+
+// GRAD variant of point_box2 with few live registers (the culled single-box scan at d >= 9):
+// the gradient term of dimension j is written w_j * p / D_j instead of w_j * prefix_j * suffix_j,
+// so only the d ratios r_j = w_j / D_j and the running product p are live, not the d factors,
+// d terms and d + 1 prefixes.  D_j == 0 (a factor flushed to zero) drops that term: then
+// |w_j| <= |y'| e^{-z^2} < 2^-120 as well, far below the culling floor (reading R15).
+template <int D, int MODE>
+__device__ __forceinline__ float2 point_box2_ratio(const BoxDim (&bd)[D], const float2 (&t)[D], const float (&ap)[D],
+                                                   float2* s2, const float2 valid) {
+  float2 r[D];
+  float2 p = valid;
+#pragma unroll
+  for (int j = 0; j < D; ++j) {
+    float2 w;
+    const float2 Dj = MODE == 2 ? phi_epan2<true>(bd[j], t[j], ap[j], w) : phi_diff2<true, MODE == 1>(bd[j], t[j], ap[j], w);
+    p = __fmul2_rn(p, Dj);
+    const float2 inv = make_float2(Dj.x != 0.0f ? rcp_approx(Dj.x) : 0.0f, Dj.y != 0.0f ? rcp_approx(Dj.y) : 0.0f);
+    r[j] = __fmul2_rn(w, inv);
+  }
+  s2[0] = __fadd2_rn(s2[0], p);
+#pragma unroll
+  for (int j = 0; j < D; ++j) s2[1 + j] = __ffma2_rn(r[j], p, s2[1 + j]);
+  return p;
 }
 
 __device__ __forceinline__ double warp_sum(double v) {
@@ -837,7 +862,7 @@ cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStr
 // Two stages; 2048-point tiles up to d = 8 (1024 above, shared-memory budget);
 // two CTAs per SM up to d = 5.
 #ifndef KDE_TUNE_CULL_TILE
-#define KDE_TUNE_CULL_TILE(d) ((d) <= 8 ? 2048 : 1024)
+#define KDE_TUNE_CULL_TILE(d) ((d) <= 8 ? 2048 : ((d) <= 12 ? 1024 : 512))
 #endif
 #ifndef KDE_TUNE_CULL_STAGES
 #define KDE_TUNE_CULL_STAGES(d) 2
@@ -882,12 +907,16 @@ cudaError_t launch_single_variant(const ScanSingleArgs& a, int grid, cudaStream_
 template <int D, bool GRAD, int QT = QT_for<D>::value, int MINB = MINB_for<D>::value, int PU = PU_for<D>::value>
 cudaError_t launch_batched_tg(const ScanBatchedArgs& a, dim3 grid, cudaStream_t s) {
   constexpr size_t smem = batched_smem_bytes<D, GRAD, QT>();
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(scan_batched_kernel<D, GRAD, QT, MINB, PU>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  // the attribute belongs to the device context: set it once per device (bit per ordinal)
+  static std::atomic<unsigned long long> attr_set{0ull};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  const unsigned long long bit = 1ull << (dev & 63);
+  if (!(attr_set.load(std::memory_order_acquire) & bit)) {
+    e = cudaFuncSetAttribute(scan_batched_kernel<D, GRAD, QT, MINB, PU>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    attr_set = true;
+    attr_set.fetch_or(bit, std::memory_order_acq_rel);
   }
   scan_batched_kernel<D, GRAD, QT, MINB, PU><<<grid, kBatchedThreads, smem, s>>>(a);
   return cudaGetLastError();

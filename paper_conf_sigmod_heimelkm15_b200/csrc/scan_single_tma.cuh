@@ -105,9 +105,17 @@ constexpr size_t cull_queue_bytes() {
   return (size_t)kSingleComputeWarps * kCullRing * (D + 1) * sizeof(float);
 }
 
-template <int D, int TILE, int STAGES, bool CULL>
+// d >= 9 gradient scans keep their fp64 per-thread sums in shared memory (stride kSingleThreads)
+// instead of registers, so two CTAs fit per SM (register budget 96/thread at 288 x 2 threads)
+template <int D, bool GRAD, bool CULL>
+__host__ __device__ constexpr bool acc_in_smem() {
+  return CULL && GRAD && D >= 9;
+}
+
+template <int D, int TILE, int STAGES, bool CULL, bool GRAD = false>
 constexpr size_t single_tma_kernel_smem() {
-  return single_tma_smem_bytes<D, TILE, STAGES>() + (CULL ? cull_queue_bytes<D>() : 0);
+  return single_tma_smem_bytes<D, TILE, STAGES>() + (CULL ? cull_queue_bytes<D>() : 0) +
+         (acc_in_smem<D, GRAD, CULL>() ? (size_t)(D + 1) * kSingleThreads * sizeof(double) : 0);
 }
 
 template <int D, bool GRAD, int MODE, int TILE, int STAGES>
@@ -115,6 +123,7 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
                                                       float* tiles, uint64_t* full, uint64_t* empty, float* queue,
                                                       int64_t c0, int64_t c1, int ntiles, double* acc, bool keep_all) {
   constexpr int NA = GRAD ? D + 1 : 1;
+  constexpr int AS = acc_in_smem<D, GRAD, true>() ? kSingleThreads : 1;  // stride of acc (shared memory or registers)
   constexpr int PPT = TILE / kSingleThreads;  // points per thread per tile
   static_assert(PPT % 2 == 0, "points are classified in pairs");
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -124,6 +133,7 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
   // used instead of living in registers for the whole scan, which keeps wide gradient scans at two
   // CTAs per SM; narrower boxes keep them in registers.
   constexpr bool kReload = D >= 9;
+  constexpr bool kRatio = D >= 9;  // few-register gradient form (point_box2_ratio): two CTAs per SM
   BoxDim bd[D];
   float ap[D];
   float2 cb[D];  // (c ap, hw' ap) of the clamped box, for the classification
@@ -166,7 +176,12 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
       // stale ring slots may hold any bit pattern: replace them by a finite coordinate
       t[j] = make_float2(v0 ? q.x : bd[j].b.y, v1 ? q.y : bd[j].b.y);
     }
-    const float2 c = point_box2<D, GRAD, MODE>(bd, t, ap, s, make_float2(v0 ? 1.0f : 0.0f, v1 ? 1.0f : 0.0f));
+    const float2 vv = make_float2(v0 ? 1.0f : 0.0f, v1 ? 1.0f : 0.0f);
+    float2 c;
+    if constexpr (GRAD && kRatio)
+      c = point_box2_ratio<D, MODE>(bd, t, ap, s, vv);
+    else
+      c = point_box2<D, GRAD, MODE>(bd, t, ap, s, vv);
     if (a.c_out) {
       const int2 ix = *reinterpret_cast<const int2*>(qi + e);
       if (v0) __stcs(a.c_out + c0 + ix.x, c.x);
@@ -176,7 +191,7 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
     if (++nproc == kCullFlushChunks) {
 #pragma unroll
       for (int kk = 0; kk < NA; ++kk) {
-        acc[kk] += (double)s[kk].x + (double)s[kk].y;
+        acc[kk * AS] += (double)s[kk].x + (double)s[kk].y;
         s[kk] = f2(0.0f);
       }
       nproc = 0;
@@ -234,7 +249,7 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
   }
   if (tail != head) process((int)(tail - head));
 #pragma unroll
-  for (int kk = 0; kk < NA; ++kk) acc[kk] += (double)s[kk].x + (double)s[kk].y;
+  for (int kk = 0; kk < NA; ++kk) acc[kk * AS] += (double)s[kk].x + (double)s[kk].y;
 }
 
 template <int D, bool GRAD, int TILE, int STAGES, int OCC, bool CULL>
@@ -285,6 +300,13 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
   double acc[NA];
 #pragma unroll
   for (int k = 0; k < NA; ++k) acc[k] = 0.0;
+  constexpr bool kAccSh = acc_in_smem<D, GRAD, CULL>();
+  double* accsh = reinterpret_cast<double*>(smem_raw + single_tma_smem_bytes<D, TILE, STAGES>() +
+                                            (CULL ? cull_queue_bytes<D>() : 0)) + tid;
+  if (kAccSh && !producer)
+#pragma unroll
+    for (int k = 0; k < NA; ++k) accsh[k * kSingleThreads] = 0.0;
+  double* accp = (kAccSh && !producer) ? accsh : acc;
   if (producer) {
     if (tid == kSingleThreads) {
       for (int k = 0; k < ntiles; ++k) {
@@ -299,35 +321,42 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
       }
     }
   } else if (CULL && a.consts->kernel == kEpanechnikov) {
-    scan_single_cull_body<D, GRAD, 2, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc,
+    scan_single_cull_body<D, GRAD, 2, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, accp,
                                                     nocull_s != 0);
   } else if (a.consts->kernel == kEpanechnikov) {
     scan_single_tma_body<D, GRAD, 2, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
   } else if (CULL) {
     if (narrow_s)
-      scan_single_cull_body<D, GRAD, 1, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc,
+      scan_single_cull_body<D, GRAD, 1, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, accp,
                                                       nocull_s != 0);
     else
-      scan_single_cull_body<D, GRAD, 0, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, acc,
+      scan_single_cull_body<D, GRAD, 0, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, accp,
                                                       nocull_s != 0);
   } else if (narrow_s) {
     scan_single_tma_body<D, GRAD, 1, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
   } else {
     scan_single_tma_body<D, GRAD, 0, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
   }
+  if (kAccSh && !producer)
+#pragma unroll
+    for (int k = 0; k < NA; ++k) acc[k] = accsh[k * kSingleThreads];
   single_reduce_finalize<NA, kSingleTmaThreads>(a, acc);
 }
 
 template <int D, bool GRAD, int TILE, int STAGES, int OCC, bool CULL>
 cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStream_t s) {
-  constexpr size_t smem = single_tma_kernel_smem<D, TILE, STAGES, CULL>();
+  constexpr size_t smem = single_tma_kernel_smem<D, TILE, STAGES, CULL, GRAD>();
   static_assert(smem + 1024 <= 227 * 1024, "single-box scan shared memory");
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC, CULL>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  // the attribute belongs to the device context: set it once per device (bit per ordinal)
+  static std::atomic<unsigned long long> attr_set{0ull};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  const unsigned long long bit = 1ull << (dev & 63);
+  if (!(attr_set.load(std::memory_order_acquire) & bit)) {
+    e = cudaFuncSetAttribute(scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC, CULL>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    attr_set = true;
+    attr_set.fetch_or(bit, std::memory_order_acq_rel);
   }
   scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC, CULL><<<grid, kSingleTmaThreads, smem, s>>>(a);
   return cudaGetLastError();

@@ -2,9 +2,10 @@
 
 The sample is split into contiguous row blocks, one per rank; query boxes,
 h and parameters are replicated; per-box partial sums (S_0, S_j) are combined
-inside libkde with an NCCL all-gather + fixed-order sum, so every rank gets
-identical, deterministic results.  torch.distributed is plumbing only: it
-bootstraps the process group and broadcasts the ncclUniqueId.
+inside libkde with an all-gather + fixed-order sum, so every rank gets
+identical, deterministic results.  The all-gather runs over peer device memory
+(libkde's own kernels, default) or NCCL.  torch.distributed is plumbing only: it
+bootstraps the process group and exchanges the IPC handles / ncclUniqueId.
 """
 from __future__ import annotations
 
@@ -30,9 +31,23 @@ def exchange_unique_id(get_id=kde_get_unique_id) -> bytes:
     return obj[0]
 
 
-def create_sharded(local_rows, row_offset: int, n_global: int, h=None) -> KDEModel:
-    """Collective: build this rank's shard of a model over n_global rows."""
+def all_gather_bytes(b: bytes):
+    """Every rank's bytes, in rank order, through the torch.distributed default group."""
+    import torch.distributed as dist
+    out = [None] * dist.get_world_size()
+    dist.all_gather_object(out, b)
+    return out
+
+
+def create_sharded(local_rows, row_offset: int, n_global: int, h=None, transport: str = "peer") -> KDEModel:
+    """Collective: build this rank's shard of a model over n_global rows.
+    transport "peer": the library's own exchange over peer device memory (IPC
+    handles all-gathered here); "nccl": ncclAllGather (ncclUniqueId broadcast here)."""
     import torch.distributed as dist
     rank, world = dist.get_rank(), dist.get_world_size()
+    if transport == "peer":
+        return KDEModel.create_sharded_peer(local_rows, row_offset, n_global, h, rank, world, all_gather_bytes)
+    if transport != "nccl":
+        raise ValueError(f"unknown transport {transport!r}")
     nid = exchange_unique_id() if world > 1 else None
     return KDEModel.create_sharded(local_rows, row_offset, n_global, h, nid, rank, world)

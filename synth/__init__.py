@@ -71,6 +71,83 @@ def gaussian_clusters(n: int, d: int, seed: int, n_clusters: int = 16, noise: fl
     return out[perm]
 
 
+def gaussian_clusters_rows(n_global: int, d: int, seed: int, row0: int, row1: int, n_clusters: int = 16,
+                           noise: float = 0.02, chunk: int = 1 << 20) -> np.ndarray:
+    """Rows [row0, row1) of a G-A-shaped sample of n_global rows, generated chunk by chunk
+    (chunk c = rows [c*chunk, (c+1)*chunk) from its own stream), so any rank can draw exactly its
+    contiguous shard and every world size sees the same global sample (strong scaling, C4).
+    Each row picks a cluster by Zipf(1) weight (prob 1-noise) or uniform noise over [-25, 125]^d."""
+    g = rng(seed, 40)
+    centres = g.uniform(0, 100, size=(n_clusters, d))
+    Ls = []
+    for _ in range(n_clusters):
+        Q = _random_orthogonal(g, d)
+        Ls.append(Q * g.uniform(1, 8, size=d))
+    w = 1.0 / np.arange(1, n_clusters + 1)
+    w = np.concatenate([(1.0 - noise) * w / w.sum(), [noise]])
+    out = np.empty((max(0, row1 - row0), d), dtype=np.float32)
+    for c in range(row0 // chunk, (row1 + chunk - 1) // chunk):
+        a, b = c * chunk, min(n_global, (c + 1) * chunk)
+        gc = rng(seed, 100000 + c)
+        lab = gc.choice(n_clusters + 1, size=b - a, p=w)
+        z = gc.standard_normal(size=(b - a, d))
+        x = np.empty((b - a, d))
+        for k in range(n_clusters):
+            sel = lab == k
+            x[sel] = centres[k] + z[sel] @ Ls[k].T
+        sel = lab == n_clusters
+        x[sel] = gc.uniform(-25.0, 125.0, size=(int(sel.sum()), d))
+        lo_, hi_ = max(a, row0), min(b, row1)
+        out[lo_ - row0:hi_ - row0] = x[lo_ - a:hi_ - a].astype(np.float32)
+    return out
+
+
+class StreamClusters:
+    """The insert/delete stream of configs[4] (after P:L367-373): the database
+    is a sequence of Gaussian clusters of `rows` rows each (cluster c: its own centre in [0, 100]^d,
+    rotation and scales U[1, 8]); cycle t inserts cluster t + 2 in chunks and deletes cluster t - 1.
+    Queries are DT boxes centred on rows of live clusters, cluster c drawn with P ~ 2^c (newer
+    clusters are asked more), sized to ~1% selectivity within their cluster."""
+
+    def __init__(self, d: int, rows: int, seed: int):
+        self.d, self.rows, self.seed = d, rows, seed
+
+    def _params(self, c: int):
+        g = rng(self.seed, 50000 + c)
+        return g.uniform(0, 100, size=self.d), _random_orthogonal(g, self.d) * g.uniform(1, 8, size=self.d)
+
+    def cluster_rows(self, c: int, a: int = 0, b: int | None = None) -> np.ndarray:
+        """Rows [a, b) of cluster c (generated in 2^16-row pieces from their own streams)."""
+        b = self.rows if b is None else b
+        centre, L = self._params(c)
+        piece = 1 << 16
+        out = np.empty((b - a, self.d), dtype=np.float32)
+        for p in range(a // piece, (b + piece - 1) // piece):
+            z = rng(self.seed, 60000 + 4096 * c + p).standard_normal(size=(piece, self.d))
+            x = (centre + z @ L.T).astype(np.float32)
+            lo_, hi_ = max(a, p * piece), min(b, (p + 1) * piece)
+            out[lo_ - a:hi_ - a] = x[lo_ - p * piece:hi_ - p * piece]
+        return out
+
+    def queries(self, live: list, q: int, seed: int):
+        """q DT boxes over the live clusters, cluster c with probability ~ 2^c."""
+        g = rng(seed, 70)
+        w = np.array([2.0 ** c for c in live])
+        pick = g.choice(len(live), size=q, p=w / w.sum())
+        lo = np.empty((q, self.d), np.float32)
+        hi = np.empty((q, self.d), np.float32)
+        for i, k in enumerate(pick):
+            c = live[k]
+            centre, L = self._params(c)
+            row = (centre + g.standard_normal(self.d) @ L.T)
+            # half-side in each axis: the cluster's per-axis sd times the 1%-volume factor
+            sd = np.sqrt((L ** 2).sum(axis=1))
+            half = sd * 0.5 * 0.01 ** (1.0 / self.d) * 4.0
+            lo[i] = (row - half).astype(np.float32)
+            hi[i] = (row + half).astype(np.float32)
+        return lo, hi
+
+
 def rect_clusters(n: int, d: int, seed: int, n_clusters: int = 10, noise: float = 0.1) -> np.ndarray:
     """G-B: hyper-rectangular clusters with uniform interiors plus uniform noise."""
     g = rng(seed, 2)

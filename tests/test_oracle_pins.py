@@ -78,7 +78,10 @@ def test_micro_scott():
 # --- closed forms and limits -------------------------------------------------
 
 @pytest.mark.parametrize("t,h,l,u", [(0.3, 0.7, -1.0, 2.0), (5.0, 0.1, 4.8, 5.05), (-2.0, 3.0, 1.0, 9.0),
-                                     (0.0, 1.0, -np.inf, 0.5), (1.0, 2.0, 0.0, np.inf)])
+                                     (0.0, 1.0, -np.inf, 0.5), (1.0, 2.0, 0.0, np.inf),
+                                     # far tails (reading R16): Phi(8) - Phi(7) = 1.3e-12, Phi(12) - Phi(9) = 1.1e-19
+                                     (0.0, 1.0, 7.0, 8.0), (0.0, 1.0, 9.0, 12.0), (0.0, 1.0, -12.0, -9.0),
+                                     (0.0, 0.5, 4.0, np.inf)])
 def test_d1_closed_form_vs_mpmath_ncdf(t, h, l, u):
     """d = 1, N = 1: eq. (13) is Phi((u-t)/h) - Phi((l-t)/h) (P:L480-482)."""
     mp.mp.dps = 40
@@ -349,6 +352,108 @@ def test_online_update_reduces_training_loss():
     assert L1 < L0
 
 
+def test_online_listing1_hand_trace_linear_mode():
+    """Listing 1 as the prose fixes it, d = 1, mini-batch 2, traced by hand:
+    average the mini-batch (line 12); running mean of the SQUARED gradient with alpha = 0.9
+    ("average magnitude", RMSprop [42], line 14); rate x1.2 when the directions agree and x0.5
+    when they do not (lines 15-16, first batch: no previous direction, rate kept); step
+    lr * g / sqrt(ms) (line 17); a step towards zero is limited to half the bandwidth."""
+    st = oracle.OnlineState(1, lr0=0.1)
+    h = np.array([0.4])
+    # batch 1: g = (0.2 + 0.4)/2 = 0.3, ms = 0.1 * 0.09 = 0.009, lr = 0.1 (no previous direction)
+    # step = 0.1 * 0.3 / sqrt(0.009) = 0.316228 > h/2 = 0.2  ->  h = 0.4 - 0.2 = 0.2 (safeguard)
+    assert not oracle.online_step(st, h, [0.2], batch=2, log_bw=False)
+    assert h[0] == 0.4
+    assert oracle.online_step(st, h, [0.4], batch=2, log_bw=False)
+    assert st.ms[0] == pytest.approx(0.009, rel=1e-15) and st.lr[0] == 0.1
+    assert h[0] == pytest.approx(0.2, rel=1e-15)
+    # batch 2: g = 0.01 agrees with 0.3 -> lr = 0.12; ms = 0.9 * 0.009 + 0.1 * 1e-4 = 0.00811
+    # step = 0.12 * 0.01 / sqrt(0.00811) = 0.0133250... < h/2  ->  h = 0.2 - step
+    oracle.online_step(st, h, [0.01], batch=2, log_bw=False)
+    oracle.online_step(st, h, [0.01], batch=2, log_bw=False)
+    assert st.lr[0] == pytest.approx(0.12, rel=1e-15)
+    assert st.ms[0] == pytest.approx(0.00811, rel=1e-14)
+    assert h[0] == pytest.approx(0.2 - 0.12 * 0.01 / math.sqrt(0.00811), rel=1e-14)
+    h2 = h[0]
+    # batch 3: g = -0.05 disagrees -> lr = 0.06; ms = 0.9 * 0.00811 + 0.1 * 0.0025 = 0.007549
+    # step = 0.06 * (-0.05) / sqrt(0.007549) < 0: a step away from zero is not limited
+    oracle.online_step(st, h, [-0.05], batch=2, log_bw=False)
+    oracle.online_step(st, h, [-0.05], batch=2, log_bw=False)
+    assert st.lr[0] == pytest.approx(0.06, rel=1e-15)
+    assert st.ms[0] == pytest.approx(0.007549, rel=1e-14)
+    assert h[0] == pytest.approx(h2 + 0.06 * 0.05 / math.sqrt(0.007549), rel=1e-14)
+    assert st.gprev[0] == pytest.approx(-0.05, rel=1e-15) and st.acc[0] == 0.0 and st.count == 0
+
+
+def test_online_listing1_log_mode_has_no_safeguard():
+    """eq. (18) / P:L561: in log mode the update is ln h <- ln h - step and the positivity
+    safeguard of line 17 is removed -- a step larger than h/2 (even than h) is taken in full."""
+    for lr0 in (0.1, 10.0):
+        st = oracle.OnlineState(1, lr0=lr0)
+        h = np.array([0.4])
+        oracle.online_step(st, h, [0.3], batch=1, log_bw=True)
+        step = lr0 * 0.3 / math.sqrt(0.1 * 0.09)          # ms = (1 - alpha) g^2
+        assert step > 0.2
+        assert h[0] == pytest.approx(0.4 * math.exp(-step), rel=1e-13)
+    # the same gradient in linear mode stops at h/2
+    st = oracle.OnlineState(1, lr0=10.0)
+    h = np.array([0.4])
+    oracle.online_step(st, h, [0.3], batch=1, log_bw=False)
+    assert h[0] == 0.2
+
+
+def test_online_listing1_rate_clamps():
+    """learning rates stay in [lambda_min, lambda_max] = [1e-6, 50]: forty agreeing
+    mini-batches saturate at exactly 50 (0.1 * 1.2^35 > 50), forty alternating ones at 1e-6."""
+    st = oracle.OnlineState(2, lr0=0.1)
+    h = np.array([0.4, 0.7])
+    rates = []
+    for k in range(40):
+        oracle.online_step(st, h, [1.0, (-1.0) ** k], batch=1, log_bw=False)
+        rates.append(st.lr.copy())
+    rates = np.array(rates)
+    assert rates[-1, 0] == 50.0 and rates[-1, 1] == 1e-6
+    # the k-th agreeing batch (k >= 1) multiplies by 1.2 until the cap
+    expect_up = np.minimum(0.1 * 1.2 ** np.arange(40), 50.0)
+    assert np.allclose(rates[:, 0], expect_up, rtol=1e-12, atol=0)
+    expect_dn = np.maximum(0.1 * 0.5 ** np.arange(40), 1e-6)
+    assert np.allclose(rates[:, 1], expect_dn, rtol=1e-12, atol=0)
+    assert np.all(h > 0)
+
+
+def test_karma_threshold_is_strict_at_equality():
+    """Reading R4: a point is flagged when its karma is BELOW the threshold
+    after the update; karma landing exactly on tau is kept.  Binary-exact values (N = 5, L1):
+    p^-(i) = (1.25 - c_i)/4, dK = |p^-(i) - 0.25|."""
+    c = np.array([0.25, 0.75, 0.0, 0.75, 0.5])
+    phat, p, tau = 0.25, 0.25, -0.5
+    karma = np.array([-0.625, -0.625, -0.5625, -0.6250001, 0.0])
+    idx = oracle.karma_update(c, phat, p, oracle.LOSS_ABSOLUTE, 0.0, 4.0, tau, np.inf, karma)
+    # dK = (0, 0.125, 0.0625, 0.125, 0.0625)
+    assert karma[1] == tau and karma[2] == tau           # exactly on the threshold: not flagged
+    assert karma[3] < tau                                 # just below: flagged
+    assert list(idx) == [0, 3]                            # point 0: -0.625 + 0 < tau
+
+
+def test_grad_abs_scale_is_sum_of_per_point_derivative_magnitudes():
+    """The gradient tolerance scale of SURVEY.md §8(c): m_j = (1/N) sum_i |d p^(i)/d h_j|,
+    each per-point derivative taken by central finite differences of eq. (13) alone (not eq. 17)."""
+    rng = np.random.default_rng(12)
+    S = rng.normal(size=(40, 3)).astype(np.float32)
+    h = np.array([0.35, 0.8, 1.3])
+    lo = np.array([0.1, -1.0, -np.inf], np.float32)
+    hi = np.array([0.9, 0.2, 0.4], np.float32)
+    m = oracle.grad_abs_scale(S, h, lo[None], hi[None])[0]
+    for j in range(3):
+        dh = 1e-6 * h[j]
+        hp, hm = h.copy(), h.copy()
+        hp[j] += dh; hm[j] -= dh
+        fd = (oracle.contributions(S, hp, lo, hi) - oracle.contributions(S, hm, lo, hi)) / (2 * dh)
+        assert m[j] == pytest.approx(np.abs(fd).mean(), rel=1e-6)
+        # and it is never below the magnitude of the gradient itself
+        assert m[j] >= abs(oracle.estimate_grad(S, h, lo[None], hi[None])[1][0, j]) * (1 - 1e-12)
+
+
 # --- property-based pins (hypothesis) ---------------------------------------------
 from hypothesis import given, settings, strategies as st  # noqa: E402
 
@@ -511,3 +616,59 @@ def test_r15_epanechnikov_support_is_exact():
     out = (r >= 1.0).any(axis=1)
     c = oracle.epan_contributions(S, h, lo, hi)
     assert out.sum() > 100 and np.all(c[out] == 0.0) and np.all(c[~out] > 0.0)
+
+
+# --- reservoir sampling (Algorithm R, O11) ---------------------------------------
+
+def test_reservoir_inclusion_frequencies_chi_square():
+    """After n = 10 N arrivals every arrival is in the sample with probability N / n (P:L248:
+    each insert enters with probability |S|/|R|): chi-square of the inclusion counts of the
+    200 arrival ids over 4000 seeds against the uniform expectation."""
+    from scipy.stats import chi2
+    Ns, n_total, T = 20, 200, 4000
+    counts = np.zeros(n_total + 1)
+    for seed in range(T):
+        content = oracle.reservoir_run(0x5EED0000 + seed, Ns, n_total)
+        assert len(set(content.tolist())) == Ns and content.min() >= 1 and content.max() <= n_total
+        counts[content] += 1
+    counts = counts[1:]
+    expect = T * Ns / n_total
+    stat = float(((counts - expect) ** 2 / expect).sum())
+    assert chi2.sf(stat, n_total - 1) > 1e-4, stat
+    # late and early arrivals alike (no drift with the arrival index)
+    assert abs(counts[:100].mean() - counts[100:].mean()) < 0.05 * expect
+
+
+def test_reservoir_draws_are_uniform_on_0_a():
+    """The a-th arrival draws j uniformly from [0, a): chi-square over 50000 draws for a = 7,
+    and j / a over a counter sweep is U(0, 1) (KS)."""
+    from scipy.stats import chi2, kstest
+    a = 7
+    js = np.array([oracle.reservoir_draw(s, a) for s in range(50000)])
+    assert js.min() == 0 and js.max() == a - 1
+    c = np.bincount(js, minlength=a)
+    stat = float(((c - 50000 / a) ** 2 / (50000 / a)).sum())
+    assert chi2.sf(stat, a - 1) > 1e-4
+    arr = np.arange(1000, 21000)
+    u = np.array([oracle.reservoir_draw(99, int(x)) for x in arr]) / arr
+    assert kstest(u, "uniform").pvalue > 1e-4
+
+
+def test_reservoir_slots_follow_algorithm_r():
+    """The first N arrivals fill slots 0..N-1 in order; afterwards arrival a takes slot j iff its
+    draw j < N; applying the per-chunk slot lists in order reproduces the whole-run content."""
+    Ns, seed = 64, 1234
+    first = oracle.reservoir_slots(seed, Ns, 0, Ns)
+    assert np.array_equal(first, np.arange(Ns))
+    content = np.arange(1, Ns + 1)
+    n_seen = Ns
+    for k in (1, 17, 300, 5000):
+        sl = oracle.reservoir_slots(seed, Ns, n_seen, k)
+        for r, j in enumerate(sl):
+            a = n_seen + r + 1
+            d = oracle.reservoir_draw(seed, a)
+            assert j == (d if d < Ns else -1)
+            if j >= 0:
+                content[j] = a
+        n_seen += k
+    assert np.array_equal(content, oracle.reservoir_run(seed, Ns, n_seen))

@@ -28,7 +28,8 @@ def main(name, macros):
     mine = {os.path.basename(x) + ".o" for x in scan_srcs}
     base = [o for o in glob.glob(os.path.join(B.OBJ, "*.o")) if not os.path.basename(o).startswith("scan_")
             and os.path.basename(o) not in mine]
-    lib = os.path.join(ROOT, "scratch", f"lib_{name}.so")
+    lib = os.path.join(ROOT, "variants", f"lib_{name}.so")
+    os.makedirs(os.path.dirname(lib), exist_ok=True)
     B._run(["nvcc"] + B.ARCH + ["-shared", "-o", lib] + objs + base +
            ["-L", libdir, "-l:libnccl.so.2", "-Xlinker", "-rpath=" + libdir, "-lcudart"])
     print(lib)

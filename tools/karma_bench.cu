@@ -39,24 +39,27 @@ int main(int argc, char** argv) {
   double *k, *phat, *p;
   uint32_t* bitmap;
   int32_t* counts;
+  int64_t* offsets;
   unsigned* done;
   int64_t *idx, *total;
   char* flush;
   const size_t flush_bytes = 512ull << 20;
-  CK(cudaMalloc(&c, n * 4));
-  CK(cudaMalloc(&k, n * 8));
+  const int64_t npad = (n + 2047) / 2048 * 2048;
+  CK(cudaMalloc(&c, npad * 4));
+  CK(cudaMalloc(&k, npad * 8));
   CK(cudaMalloc(&lo, 64));
   CK(cudaMalloc(&hi, 64));
   CK(cudaMalloc(&phat, 8));
   CK(cudaMalloc(&p, 8));
   CK(cudaMalloc(&bitmap, ((n + 31) / 32 + 1024) * 4));
   CK(cudaMalloc(&counts, (nb + 1) * 4));
-  CK(cudaMalloc(&done, 4));
+  CK(cudaMalloc(&offsets, (nb + 1) * 8));
+  CK(cudaMalloc(&done, 8));
   CK(cudaMalloc(&idx, n * 8));
   CK(cudaMalloc(&total, 8));
   CK(cudaMalloc(&flush, flush_bytes));
   CK(cudaMemcpy(c, hc.data(), n * 4, cudaMemcpyHostToDevice));
-  CK(cudaMemset(done, 0, 4));
+  CK(cudaMemset(done, 0, 8));
   const double hp = 1.0 / (double)n * 0.5, pp = 0.3;
   CK(cudaMemcpy(phat, &hp, 8, cudaMemcpyHostToDevice));
   CK(cudaMemcpy(p, &pp, 8, cudaMemcpyHostToDevice));
@@ -78,9 +81,10 @@ int main(int argc, char** argv) {
     CK(cudaMemcpyAsync(k, hk.data(), n * 8, cudaMemcpyHostToDevice, s));
     CK(cudaMemsetAsync(flush, r & 0xff, flush_bytes, s));
     CK(cudaEventRecord(e0, s));
-    karma_kernel<<<nb, kKarmaThreads, 0, s>>>(c, k, n, (double)n, phat, p, kp, lo, hi, 1, nullptr, bitmap, counts);
+    karma_kernel<<<nb, kKarmaThreads, 0, s>>>(c, k, n, (double)n, phat, p, kp, lo, hi, 1, nullptr, bitmap, counts,
+                                              offsets, done + 1, (int)nb);
     CK(cudaEventRecord(e1, s));
-    compact_fused_kernel<<<nb, kKarmaThreads, 0, s>>>(bitmap, n, counts, nb, 0, idx, n, total, done, tail);
+    compact_fused_kernel<<<nb, kKarmaThreads, 0, s>>>(bitmap, n, offsets, nb, 0, idx, n, total, done, tail);
     CK(cudaEventRecord(e2, s));
     CK(cudaStreamSynchronize(s));
     CK(cudaGetLastError());
