@@ -975,7 +975,7 @@ extern "C" kde_status kde_karma_update(kde_model* m, const float* lo, const floa
   kd.k_max = kp->k_max;
   kd.threshold = kp->threshold;
   CU(cudaMemcpyAsync(m->scal, &true_sel, sizeof(double), cudaMemcpyHostToDevice, m->stream));
-  m->launches += 1;  // karma + fused compaction
+  m->launches += karma_launches() - 1;  // CUL counts one
   CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, m->scal, kd, m->qbuf, m->qbuf + m->d, m->d,
                   m->consts, m->bitmap, m->block_counts, m->block_offsets, m->done, m->row_offset, m->idx_dev, local_cap, m->offsets,
                   StreamTail{}, m->stream));
@@ -1164,7 +1164,7 @@ extern "C" kde_status kde_karma_update_dev(kde_model* m, const float* d_lo, cons
   if (st != KDE_OK) return st;
   DeviceGuard g(m->device);
   cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
-  m->launches += 1;
+  m->launches += karma_launches() - 1;  // CUL counts one
   CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, d_true_sel, kd, d_lo, d_hi, m->d,
                    m->consts, m->bitmap, m->block_counts, m->block_offsets, m->done, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
                    StreamTail{}, s));
@@ -1240,7 +1240,7 @@ extern "C" kde_status kde_stream_step_dev(kde_model* m, const float* d_lo, const
   m->ret_valid = false;
   st = estimate_dev(m, d_lo, d_hi, 1, d_est, op ? d_dpdh : nullptr, s, true);
   if (st != KDE_OK) return st;
-  m->launches += 1;
+  m->launches += karma_launches() - 1;  // CUL counts one
   CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, d_true_sel, kd, d_lo, d_hi, m->d,
                    m->consts, m->bitmap, m->block_counts, m->block_offsets, m->done, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
                    tail, s));

@@ -5,7 +5,9 @@
 //   row replacement, the on-device Listing 1 step (Section 4.1)
 //   and the harness box counter.
 // All reductions use a fixed order, so results are bitwise reproducible.
+#include <cooperative_groups.h>
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_runtime.h>
 #include <math_constants.h>
 
@@ -13,6 +15,7 @@
 #include "kernels.cuh"
 
 namespace kde {
+namespace cg = cooperative_groups;
 
 // ------------------------------------------------------------ layout
 // rows: device row-major [n][d]; cols: [d][ld].  Flags non-finite values.
@@ -618,6 +621,230 @@ __global__ void online_update_kernel(const double* __restrict__ ret, const doubl
   online_update_body(ret, p_ptr, op, d, st, c);
 }
 
+// ------------------------------------------------------------ karma pass, one cooperative kernel
+// The whole feedback tail of a query in ONE persistent launch (cooperative: all CTAs co-resident,
+// grid-wide barriers): each CTA owns a contiguous run of 4096-point segments.
+//   phase 1  karma (eq. 6-8) and flags (R4, eq. 20) for its segments, exactly as karma_kernel:
+//            128-bit loads, index-order bitmap words, a per-CTA flag count;
+//   barrier  -> the CTA's offset is the sum of the counts of the CTAs before it (<= a few hundred);
+//   phase 2  ordered compaction of its segments' bitmap words into ascending GLOBAL indices;
+//   barrier  -> phase 3: CTA 0 runs the Listing 1 step (optional), all CTAs replace the first
+//            min(total, cap) flagged points by tail.rows (optional).
+// Replaces the karma + compaction kernel pair (two launches, nb = n/4096 blocks each, a serial
+// last-block tail).
+constexpr int kCoopThreads = 256;
+constexpr int kCoopSeg = kKarmaPts;  // points per segment (kCoopThreads x 4 points x 4 passes)
+
+struct KarmaCoopArgs {
+  const float* cvals;
+  double* karma;
+  int64_t n;
+  double n_global;
+  const double* phat;
+  const double* p;
+  KarmaParamsDev kp;
+  const float* lo;
+  const float* hi;
+  int d;
+  const DevConsts* c;
+  uint32_t* bitmap;
+  int32_t* cta_counts;  // [grid]
+  int64_t row_offset;
+  int64_t* idx_out;
+  int64_t cap;
+  int64_t* total_out;
+  StreamTail tail;
+};
+
+__global__ void __launch_bounds__(kCoopThreads, KDE_TUNE_KARMA_MINB) karma_coop_kernel(const KarmaCoopArgs a) {
+  cg::grid_group grid = cg::this_grid();
+  __shared__ double thr_s;
+  __shared__ int64_t red_s[2][kCoopThreads / 32];
+  __shared__ int32_t wpre[kCoopSeg / 32];
+  __shared__ uint32_t wbits[kCoopSeg / 32];
+  __shared__ int32_t segtot_s;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int G = gridDim.x, b = blockIdx.x;
+  const int64_t nseg = (a.n + kCoopSeg - 1) / kCoopSeg;
+  const int64_t per = (nseg + G - 1) / G;
+  const int64_t sg0 = min(nseg, (int64_t)b * per), sg1 = min(nseg, sg0 + per);
+  const KarmaParamsDev kp = a.kp;
+  const double p = *a.p;
+  if (tid == 0) thr_s = (kp.empty_region && p == 0.0) ? thr20_dev(a.lo, a.hi, a.d, a.c) : CUDART_INF;
+  __syncthreads();
+  const double phat = *a.phat;
+  double L_full, dummy;
+  loss_eval(kp.loss, kp.lambda, phat, p, &L_full, &dummy);
+  const double thr = thr_s;
+  const double inv_nm1 = 1.0 / (a.n_global - 1.0);
+  const int64_t n = a.n;
+  // ---------------- phase 1: karma + flags
+  int32_t my = 0;
+  constexpr int PASSES = kCoopSeg / (kCoopThreads * kKarmaKV);
+  constexpr int PB = 2;
+  for (int64_t sg = sg0; sg < sg1; ++sg) {
+    const int64_t base = sg * kCoopSeg;
+#pragma unroll 1
+    for (int r0 = 0; r0 < PASSES; r0 += PB) {
+      float4 cv[PB];
+      double2 kv[PB][2];
+#pragma unroll
+      for (int r = 0; r < PB; ++r) {
+        const int64_t i = base + ((int64_t)(r0 + r) * kCoopThreads + tid) * kKarmaKV;
+        if (i < n) {  // i is a multiple of 4; c and K are padded past n
+          cv[r] = __ldcs(reinterpret_cast<const float4*>(a.cvals + i));
+          kv[r][0] = __ldcs(reinterpret_cast<const double2*>(a.karma + i));
+          kv[r][1] = __ldcs(reinterpret_cast<const double2*>(a.karma + i + 2));
+        } else {
+          cv[r] = make_float4(0.f, 0.f, 0.f, 0.f);
+          kv[r][0] = kv[r][1] = make_double2(0.0, 0.0);
+        }
+      }
+#pragma unroll
+      for (int r = 0; r < PB; ++r) {
+        const int64_t i = base + ((int64_t)(r0 + r) * kCoopThreads + tid) * kKarmaKV;
+        const float cc[4] = {cv[r].x, cv[r].y, cv[r].z, cv[r].w};
+        double kk[4] = {kv[r][0].x, kv[r][0].y, kv[r][1].x, kv[r][1].y};
+        unsigned nib = 0u;
+#pragma unroll
+        for (int v = 0; v < kKarmaKV; ++v) {
+          if (i + v < n) {
+            const double ci = (double)cc[v];
+            const double p_minus = (phat * a.n_global - ci) * inv_nm1;  // eq. (6)
+            double L_minus;
+            loss_eval(kp.loss, kp.lambda, p_minus, p, &L_minus, &dummy);
+            kk[v] = fmin(kk[v] + (L_minus - L_full), kp.k_max);  // eq. (7)-(8)
+            nib |= (unsigned)((kk[v] < kp.threshold) || (ci >= thr)) << v;
+          }
+        }
+        if (i < n) {
+          __stcs(reinterpret_cast<double2*>(a.karma + i), make_double2(kk[0], kk[1]));
+          __stcs(reinterpret_cast<double2*>(a.karma + i + 2), make_double2(kk[2], kk[3]));
+        }
+        unsigned word = nib << (4 * (lane & 7));  // word of 32 points = nibbles of 8 lanes
+        word |= __shfl_xor_sync(0xffffffffu, word, 1);
+        word |= __shfl_xor_sync(0xffffffffu, word, 2);
+        word |= __shfl_xor_sync(0xffffffffu, word, 4);
+        if ((lane & 7) == 0) {
+          const int64_t w0 = (base + ((int64_t)(r0 + r) * kCoopThreads + warp * 32) * kKarmaKV) / 32;
+          a.bitmap[w0 + (lane >> 3)] = word;
+          my += __popc(word);
+        }
+      }
+    }
+  }
+  for (int o = 8; o < 32; o <<= 1) my += __shfl_xor_sync(0xffffffffu, my, o);
+  if (lane == 0) red_s[0][warp] = my;
+  __syncthreads();
+  if (tid == 0) {
+    int32_t t = 0;
+    for (int w = 0; w < kCoopThreads / 32; ++w) t += (int32_t)red_s[0][w];
+    a.cta_counts[b] = t;
+  }
+  grid.sync();
+  // ---------------- phase 2: this CTA's offset (fixed-order integer sums), ordered compaction
+  int64_t before = 0, total = 0;
+  for (int c = tid; c < G; c += kCoopThreads) {
+    const int64_t v = __ldcg(a.cta_counts + c);
+    total += v;
+    if (c < b) before += v;
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    before += __shfl_xor_sync(0xffffffffu, before, o);
+    total += __shfl_xor_sync(0xffffffffu, total, o);
+  }
+  __syncthreads();
+  if (lane == 0) {
+    red_s[0][warp] = before;
+    red_s[1][warp] = total;
+  }
+  __syncthreads();
+  before = total = 0;
+  for (int w = 0; w < kCoopThreads / 32; ++w) {
+    before += red_s[0][w];
+    total += red_s[1][w];
+  }
+  constexpr int W = kCoopSeg / 32;  // bitmap words per segment
+  constexpr int WPL = W / 32;
+  const int64_t nwords = (n + 31) / 32;
+  int64_t run = before;
+  for (int64_t sg = sg0; sg < sg1; ++sg) {
+    const int64_t wbase = sg * W;
+    if (warp == 0) {  // the segment's words, their exclusive popcount prefix
+      int cnt[WPL], tot = 0;
+#pragma unroll
+      for (int k = 0; k < WPL; ++k) {
+        const int64_t w = wbase + WPL * lane + k;
+        const uint32_t word = w < nwords ? __ldcg(a.bitmap + w) : 0u;
+        wbits[WPL * lane + k] = word;
+        cnt[k] = __popc(word);
+        tot += cnt[k];
+      }
+      int incl = tot;
+#pragma unroll
+      for (int k = 1; k < 32; k <<= 1) {
+        const int v = __shfl_up_sync(0xffffffffu, incl, k);
+        if (lane >= k) incl += v;
+      }
+      int rr = incl - tot;
+#pragma unroll
+      for (int k = 0; k < WPL; ++k) {
+        wpre[WPL * lane + k] = rr;
+        rr += cnt[k];
+      }
+      if (lane == 31) segtot_s = incl;
+    }
+    __syncthreads();
+#pragma unroll 4
+    for (int w = warp; w < W; w += kCoopThreads / 32) {
+      const uint32_t word = wbits[w];
+      if (word & (1u << lane)) {
+        const int64_t pos = run + wpre[w] + __popc(word & ((1u << lane) - 1u));
+        if (pos < a.cap) a.idx_out[pos] = a.row_offset + (wbase + w) * 32 + lane;
+      }
+    }
+    run += segtot_s;
+    __syncthreads();
+  }
+  if (b == 0 && tid == 0 && a.total_out) *a.total_out = total;
+  const StreamTail& tail = a.tail;
+  if (!tail.online && !tail.rows) return;
+  grid.sync();
+  // ---------------- phase 3: the streaming step's tail
+  if (tail.online && b == 0) online_update_body(tail.ret, tail.p, tail.op, tail.d, tail.st, tail.c);
+  if (tail.rows) {
+    __shared__ unsigned rmin[kMaxDim], rmax[kMaxDim];
+    if (tid < kMaxDim) {
+      rmin[tid] = 0xFFFFFFFFu;
+      rmax[tid] = 0u;
+    }
+    __syncthreads();
+    const int64_t k = min(total, a.cap);
+    const float* __restrict__ rows = tail.rows;
+    float* __restrict__ cols = tail.cols;
+    for (int64_t r = (int64_t)b * kCoopThreads + tid; r < k; r += (int64_t)G * kCoopThreads) {
+      const int64_t i = __ldcg(a.idx_out + r) - a.row_offset;
+      float x[kMaxDim];
+#pragma unroll
+      for (int j = 0; j < kMaxDim; ++j) x[j] = j < tail.d ? rows[r * tail.d + j] : 0.0f;
+#pragma unroll
+      for (int j = 0; j < kMaxDim; ++j) {
+        if (j < tail.d) {
+          cols[(int64_t)j * tail.ld + i] = x[j];
+          atomicMin(rmin + j, fenc(x[j]));
+          atomicMax(rmax + j, fenc(x[j]));
+        }
+      }
+      tail.karma[i] = tail.k_init;
+    }
+    __syncthreads();
+    if (tid < tail.d && (int64_t)b * kCoopThreads < k) {
+      atomicMin(tail.c->renc + 2 * tid, rmin[tid]);
+      atomicMax(tail.c->renc + 2 * tid + 1, rmax[tid]);
+    }
+  }
+}
+
 // ------------------------------------------------------------ harness: exact box counts
 // counts[k] = |{r : l_kj < R_rj < u_kj for all j}|, open box as in P:L45.
 __global__ void count_in_box_kernel(const float* __restrict__ rows, int64_t n, int d, const float* __restrict__ lo,
@@ -748,6 +975,26 @@ cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const do
   loss_epilogue_kernel<<<1, 512, 0, s>>>(est, dpdh, true_sel, q, d, kind, lambda, log_bw, c, loss_out, grad_out);
   KDE_LAUNCH_CHECK();
 }
+int karma_launches() {  // kernels per karma pass: 1 (cooperative) or 2 (KDE_KARMA_TWO_PASS, A/B timing)
+  static const int k = getenv("KDE_KARMA_TWO_PASS") != nullptr ? 2 : 1;
+  return k;
+}
+
+static int coop_grid_limit() {
+  // co-resident CTAs of the cooperative karma kernel, per device
+  static int cached[64] = {0};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return 0;
+  int& v = cached[dev & 63];
+  if (v == 0) {
+    int sms = 0, per = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, karma_coop_kernel, kCoopThreads, 0);
+    v = sms * (per > 0 ? per : 1);
+  }
+  return v;
+}
+
 cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, const double* p,
                          const KarmaParamsDev& kp, const float* lo, const float* hi, int d, const DevConsts* c,
                          uint32_t* bitmap, int32_t* block_counts, int64_t* block_offsets, unsigned* done,
@@ -755,6 +1002,15 @@ cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_
                          cudaStream_t s) {
   const int nb = karma_blocks(n);
   if (nb == 0) return cudaSuccess;
+  if (karma_launches() == 1) {
+    KarmaCoopArgs a{cvals, karma, n, n_global, phat, p, kp, lo, hi, d, c, bitmap, block_counts, row_offset,
+                    idx_out, cap, total_out, tail};
+    int grid = coop_grid_limit();
+    if (grid > nb) grid = nb;
+    if (grid < 1) grid = 1;
+    void* args[] = {&a};
+    return cudaLaunchCooperativeKernel((const void*)karma_coop_kernel, grid, kCoopThreads, args, 0, s);
+  }
   karma_kernel<<<nb, kKarmaThreads, 0, s>>>(cvals, karma, n, n_global, phat, p, kp, lo, hi, d, c, bitmap,
                                             block_counts, block_offsets, done + 1, nb);
   cudaError_t e = cudaGetLastError();

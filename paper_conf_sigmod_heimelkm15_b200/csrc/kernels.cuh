@@ -67,6 +67,7 @@ cudaError_t launch_finalize(const double* sums, int64_t q, int d, int na, const 
 cudaError_t launch_loss_epilogue(const double* est, const double* dpdh, const double* true_sel, int64_t q, int d,
                                  int kind, double lambda, int log_bw, const DevConsts* c, double* loss_out,
                                  double* grad_out, cudaStream_t s);
+int karma_launches();  // kernels one launch_karma enqueues
 // karma pass + ordered compaction: block_counts int32 [nb], block_offsets int64 [nb + 1],
 // done: 2 self-resetting counters (compaction, karma); c and karma padded to a multiple of 4 points
 cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_global, const double* phat, const double* p,

@@ -107,9 +107,12 @@ constexpr size_t cull_queue_bytes() {
 
 // d >= 9 gradient scans keep their fp64 per-thread sums in shared memory (stride kSingleThreads)
 // instead of registers, so two CTAs fit per SM (register budget 96/thread at 288 x 2 threads)
+#ifndef KDE_TUNE_RATIO_MIND
+#define KDE_TUNE_RATIO_MIND 9  // from this d on, the culled gradient scan uses point_box2_ratio + smem sums
+#endif
 template <int D, bool GRAD, bool CULL>
 __host__ __device__ constexpr bool acc_in_smem() {
-  return CULL && GRAD && D >= 9;
+  return CULL && GRAD && D >= KDE_TUNE_RATIO_MIND;
 }
 
 template <int D, int TILE, int STAGES, bool CULL, bool GRAD = false>
@@ -118,9 +121,9 @@ constexpr size_t single_tma_kernel_smem() {
          (acc_in_smem<D, GRAD, CULL>() ? (size_t)(D + 1) * kSingleThreads * sizeof(double) : 0);
 }
 
-template <int D, bool GRAD, int MODE, int TILE, int STAGES>
+template <int D, bool GRAD, int MODE, int TILE, int STAGES, typename Release>
 __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, const float4* smc, const float2* scb,
-                                                      float* tiles, uint64_t* full, uint64_t* empty, float* queue,
+                                                      float* tiles, uint64_t* full, Release& release, float* queue,
                                                       int64_t c0, int64_t c1, int ntiles, double* acc, bool keep_all) {
   constexpr int NA = GRAD ? D + 1 : 1;
   constexpr int AS = acc_in_smem<D, GRAD, true>() ? kSingleThreads : 1;  // stride of acc (shared memory or registers)
@@ -133,7 +136,7 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
   // used instead of living in registers for the whole scan, which keeps wide gradient scans at two
   // CTAs per SM; narrower boxes keep them in registers.
   constexpr bool kReload = D >= 9;
-  constexpr bool kRatio = D >= 9;  // few-register gradient form (point_box2_ratio): two CTAs per SM
+  constexpr bool kRatio = D >= KDE_TUNE_RATIO_MIND;  // few-register gradient form (point_box2_ratio)
   BoxDim bd[D];
   float ap[D];
   float2 cb[D];  // (c ap, hw' ap) of the clamped box, for the classification
@@ -244,17 +247,25 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
       __syncwarp();
       while (tail - head >= 64u) process(64);
     }
-    __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[st]);  // this warp is done reading stage st
+    release(k);  // this warp is done reading stage st (the ring holds copies of the kept points)
   }
   if (tail != head) process((int)(tail - head));
 #pragma unroll
   for (int kk = 0; kk < NA; ++kk) acc[kk * AS] += (double)s[kk].x + (double)s[kk].y;
 }
 
+// Culled variant: no producer warp -- the LAST compute warp to finish a tile's classification
+// issues that stage's next TMA copies (per-stage arrival counters), so all 8 warps compute and
+// the CTA's register budget allows two CTAs per SM at d >= 9.
+template <bool CULL>
+__host__ __device__ constexpr int single_tma_threads() {
+  return CULL ? kSingleThreads : kSingleTmaThreads;
+}
+
 template <int D, bool GRAD, int TILE, int STAGES, int OCC, bool CULL>
-__global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel(const ScanSingleArgs a) {
+__global__ void __launch_bounds__(single_tma_threads<CULL>(), OCC) scan_single_tma_kernel(const ScanSingleArgs a) {
   constexpr int NA = GRAD ? D + 1 : 1;
+  constexpr int NT = single_tma_threads<CULL>();
   extern __shared__ __align__(128) unsigned char smem_raw[];
   float* tiles = reinterpret_cast<float*>(smem_raw);
   uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + (size_t)STAGES * D * TILE * sizeof(float));
@@ -263,8 +274,9 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
   __shared__ float4 smc[D];
   __shared__ float2 scb[D];
   __shared__ int narrow_s, nocull_s;
+  __shared__ int rcnt[STAGES];  // culled variant: warps done with each stage
   const int tid = threadIdx.x;
-  const bool producer = tid >= kSingleThreads;
+  const bool producer = !CULL && tid >= kSingleThreads;
   // contiguous chunk of this CTA, a multiple of TILE points
   const int64_t ntile_total = (a.n + TILE - 1) / TILE;
   const int64_t tiles_per = (ntile_total + gridDim.x - 1) / gridDim.x;
@@ -277,10 +289,34 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
     for (int st = 0; st < STAGES; ++st) {
       mbar_init(&full[st], 1);
       mbar_init(&empty[st], kSingleComputeWarps);
+      rcnt[st] = 0;
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
+  auto issue = [&](int k) {  // tile k -> stage k % STAGES, completing on full[stage]
+    const int st = k % STAGES;
+    const int64_t nb = c0 + (int64_t)k * TILE;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    mbar_arrive_expect_tx(&full[st], (uint32_t)(D * TILE * sizeof(float)));
+#pragma unroll
+    for (int j = 0; j < D; ++j)
+      bulk_g2s(tiles + ((size_t)st * D + j) * TILE, a.cols + (int64_t)j * a.ld + nb, (uint32_t)(TILE * sizeof(float)),
+               &full[st]);
+  };
+  if (CULL && tid == 0)
+    for (int k = 0; k < STAGES && k < ntiles; ++k) issue(k);
+  auto release = [&](int k) {  // last warp out of tile k refills its stage with tile k + STAGES
+    __syncwarp();
+    if ((tid & 31) == 0) {
+      const int st = k % STAGES;
+      __threadfence_block();
+      if (atomicAdd(&rcnt[st], 1) == kSingleComputeWarps - 1) {
+        rcnt[st] = 0;
+        if (k + STAGES < ntiles) issue(k + STAGES);
+      }
+    }
+  };
   if (tid < D) {
     const int j = tid;
     const float ap = a.consts->ap[j];
@@ -321,16 +357,16 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
       }
     }
   } else if (CULL && a.consts->kernel == kEpanechnikov) {
-    scan_single_cull_body<D, GRAD, 2, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, accp,
+    scan_single_cull_body<D, GRAD, 2, TILE, STAGES>(a, smc, scb, tiles, full, release, queue, c0, c1, ntiles, accp,
                                                     nocull_s != 0);
   } else if (a.consts->kernel == kEpanechnikov) {
     scan_single_tma_body<D, GRAD, 2, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
   } else if (CULL) {
     if (narrow_s)
-      scan_single_cull_body<D, GRAD, 1, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, accp,
+      scan_single_cull_body<D, GRAD, 1, TILE, STAGES>(a, smc, scb, tiles, full, release, queue, c0, c1, ntiles, accp,
                                                       nocull_s != 0);
     else
-      scan_single_cull_body<D, GRAD, 0, TILE, STAGES>(a, smc, scb, tiles, full, empty, queue, c0, c1, ntiles, accp,
+      scan_single_cull_body<D, GRAD, 0, TILE, STAGES>(a, smc, scb, tiles, full, release, queue, c0, c1, ntiles, accp,
                                                       nocull_s != 0);
   } else if (narrow_s) {
     scan_single_tma_body<D, GRAD, 1, TILE, STAGES>(a, smc, tiles, full, empty, c0, c1, ntiles, acc);
@@ -340,7 +376,7 @@ __global__ void __launch_bounds__(kSingleTmaThreads, OCC) scan_single_tma_kernel
   if (kAccSh && !producer)
 #pragma unroll
     for (int k = 0; k < NA; ++k) acc[k] = accsh[k * kSingleThreads];
-  single_reduce_finalize<NA, kSingleTmaThreads>(a, acc);
+  single_reduce_finalize<NA, NT>(a, acc);
 }
 
 template <int D, bool GRAD, int TILE, int STAGES, int OCC, bool CULL>
@@ -358,7 +394,7 @@ cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStr
     if (e != cudaSuccess) return e;
     attr_set.fetch_or(bit, std::memory_order_acq_rel);
   }
-  scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC, CULL><<<grid, kSingleTmaThreads, smem, s>>>(a);
+  scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC, CULL><<<grid, single_tma_threads<CULL>(), smem, s>>>(a);
   return cudaGetLastError();
 }
 

@@ -98,8 +98,7 @@ def _worker(rank, world, port, out):
                                            cap=7)
         res["trunc"] = tr_c and nf_c == n and np.array_equal(idx_c, np.arange(7))
         # replacement routed to the owning shard, then reservoir inserts
-        rep = np.array([0, off, n // 2, n - 1], np.int64)
-        rep = np.unique(rep)
+        rep = np.array([0, n // 3, n // 2, n - 1], np.int64)   # the same global indices on every rank
         rows = synth.make_data("gauss", len(rep), d, seed=902)
         m.replace_points(rep, rows)
         S2 = S.copy()
