@@ -325,6 +325,8 @@ def timed_steps(step, steps, warmup, stream, m, K, flush=None, barrier=None, clo
 def max_over_ranks(x, world, dev):
     import torch
     import torch.distributed as dist
+    if world > 1 and dist.get_backend() == "gloo":
+        dev = "cpu"
     t = torch.tensor([float(x)], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -370,8 +372,9 @@ def run_cuda(args, cfg, rank, world, local_rank):
     import paper_conf_sigmod_heimelkm15_b200 as K
     from paper_conf_sigmod_heimelkm15_b200.dist import create_sharded
 
-    torch.cuda.set_device(local_rank)
-    dev = torch.device("cuda", local_rank)
+    gpu = 0 if args.share_gpu else local_rank
+    torch.cuda.set_device(gpu)
+    dev = torch.device("cuda", gpu)
     if cfg["path"] == "stream":
         if world > 1:
             raise SystemExit("c5 (device-resident streaming) is single-GPU")
@@ -416,7 +419,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
             K.kde_loss_and_grad_dev(m.handle, d_lo, d_hi, d_true, d_loss, d_grad, K.LOSS_SQUARED, 0.0, False,
                                     stream=stream)
 
-    T = timed_steps(step, args.steps, args.warmup, stream, m, K, flush, barrier, local_rank)
+    T = timed_steps(step, args.steps, args.warmup, stream, m, K, flush, barrier, gpu)
     ms_per_step = max_over_ranks(sum(T["step_ms"]), world, dev) / args.steps
     units_per_step = n_global * q
     value = units_per_step / (ms_per_step * 1e-3)
@@ -449,7 +452,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
             k = i % len(lo1)
             K.kde_estimate_batch_dev(m.handle, d_lo1[k:k + 1], d_hi1[k:k + 1], d_est[:1], None, stream=stream)
 
-        T1 = timed_steps(step1, max(args.steps, 20), args.warmup, stream, m, K, None, barrier, local_rank)
+        T1 = timed_steps(step1, max(args.steps, 20), args.warmup, stream, m, K, None, barrier, gpu)
         ms1 = max_over_ranks(sum(T1["step_ms"]), world, dev) / len(T1["step_ms"])
         if world > 1:
             dist.barrier()
@@ -493,6 +496,8 @@ def run_cuda(args, cfg, rank, world, local_rank):
         "data": "synthetic",
         "config": {"workload": cfg["desc"], "d": d, "n_per_gpu": n_local, "n_global": n_global, "q": q,
                    "comm": (args.comm if world > 1 else "none"),
+                   **({"shared_gpu": "all ranks on cuda:0 (time-sliced): a functional check of the world > 1 "
+                                     "path, NOT a scaling measurement"} if args.share_gpu else {}),
                    "l2": "flushed between timed steps" if flush_l2 else "sample larger than L2",
                    "cull": ("off" if args.no_cull else
                             "on: (point, box) pairs whose contribution is provably < 2^-64 are skipped (DESIGN R15)"),
@@ -708,6 +713,9 @@ def main():
                     help="evaluate every (point, box) pair (kde_set_cull(0)); default culls provably < 2^-64")
     ap.add_argument("--no-graph", action="store_true", help="stream configs: launch eagerly instead of CUDA graphs")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of all-core oracle work")
+    ap.add_argument("--share-gpu", action="store_true",
+                    help="run every rank on cuda:0 (gloo process group, peer transport): exercises the world > 1 "
+                         "path on a one-GPU box; not a scaling measurement")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -725,11 +733,17 @@ def main():
     if args.impl == "reference":
         run_reference(args, cfg, rank, world)
         return
+    if args.share_gpu and args.comm != "peer":
+        raise SystemExit("--share-gpu needs --comm peer (NCCL rejects two ranks on one GPU)")
     if world > 1:
         import torch
         import torch.distributed as dist
-        torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if args.share_gpu:
+            torch.cuda.set_device(0)
+            dist.init_process_group("gloo")
+        else:
+            torch.cuda.set_device(local_rank)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     try:
         run_cuda(args, cfg, rank, world, local_rank)
     finally:

@@ -296,8 +296,9 @@ kde_status kde_reservoir_select(uint64_t seed, int64_t n_sample, int64_t n_seen,
  * arrivals of the chunk draw the same slot, the last one wins (the sequential
  * result).  *n_seen (in/out): arrivals so far -- the sample itself counts as
  * the first n_global (or more) -- advanced by k.  *n_written (optional): slots
- * written.  Sharded models: every rank calls with the same rows and seed; each
- * writes the slots of its shard.  Errors: KDE_EINVAL (non-finite rows, bad
+ * of this shard written.  Sharded models: every rank calls with the same rows
+ * and seed; each writes the slots of its shard.  Host cost O(k) (a per-shard
+ * last-writer table resolves repeated slots).  Errors: KDE_EINVAL (non-finite rows, bad
  * n_seen); state unchanged. */
 kde_status kde_insert_rows(kde_model *m, const float *rows, int64_t k, uint64_t seed, int64_t *n_seen,
                            double k_init, int64_t *n_written);

@@ -89,6 +89,7 @@ struct kde_model {
   size_t pinned_cap = 0;
   void* rbuf = nullptr;              // replacement staging (idx + rows), grow-only
   size_t rbuf_cap = 0;
+  std::vector<int32_t> ins_last;     // kde_insert_rows: last arrival of a chunk per local slot (-1 = none)
   void* kbuf = nullptr;              // sharded karma gather: counts + index lists, grow-only
   size_t kbuf_cap = 0;
 
@@ -1124,29 +1125,38 @@ extern "C" kde_status kde_insert_rows(kde_model* m, const float* rows, int64_t k
   if (k < 0 || !n_seen || *n_seen < 0 || *n_seen > INT64_MAX - k) return fail(KDE_EINVAL, "bad k / n_seen");
   if (k > 0 && !rows) return fail(KDE_EINVAL, "rows is NULL");
   if (!std::isfinite(k_init)) return fail(KDE_EINVAL, "k_init not finite");
-  for (int64_t e = 0; e < k * m->d; ++e)
-    if (!std::isfinite(rows[e])) return fail(KDE_EINVAL, "non-finite value in inserted rows");
+  {  // every arriving value finite (branch-free exponent test, vectorisable)
+    const uint32_t* bits = reinterpret_cast<const uint32_t*>(rows);
+    uint32_t bad = 0;
+    for (int64_t e = 0; e < k * m->d; ++e) bad |= (uint32_t)((bits[e] & 0x7f800000u) == 0x7f800000u);
+    if (bad) return fail(KDE_EINVAL, "non-finite value in inserted rows");
+  }
   std::vector<int64_t> slot((size_t)k);
   reservoir_slots(seed, m->n_global, *n_seen, k, slot.data());
   // several arrivals of one chunk may take the same slot: the last one wins (sequential semantics);
-  // only the winners are transferred
-  std::vector<std::pair<int64_t, int64_t>> win;  // (slot, arrival row)
-  win.reserve((size_t)k);
-  for (int64_t r = 0; r < k; ++r)
-    if (slot[r] >= 0) win.emplace_back(slot[r], r);
-  std::stable_sort(win.begin(), win.end(), [](const auto& a, const auto& b) { return a.first < b.first; });
+  // only this shard's winners are transferred.  O(k) with a per-shard last-writer table.
+  if (m->ins_last.size() != (size_t)m->n) m->ins_last.assign((size_t)m->n, -1);
   std::vector<int64_t> idx;
   std::vector<float> sel;
-  idx.reserve(win.size());
-  sel.reserve(win.size() * m->d);
-  for (size_t i = 0; i < win.size(); ++i) {
-    if (i + 1 < win.size() && win[i + 1].first == win[i].first) continue;  // a later arrival overwrites this slot
-    idx.push_back(win[i].first);
-    sel.insert(sel.end(), rows + win[i].second * m->d, rows + (win[i].second + 1) * m->d);
+  for (int64_t r = 0; r < k; ++r) {
+    const int64_t i = slot[r] - m->row_offset;
+    if (slot[r] >= 0 && i >= 0 && i < m->n) m->ins_last[(size_t)i] = (int32_t)r;
+  }
+  for (int64_t r = 0; r < k; ++r) {
+    const int64_t i = slot[r] - m->row_offset;
+    if (slot[r] >= 0 && i >= 0 && i < m->n && m->ins_last[(size_t)i] == (int32_t)r) {
+      idx.push_back(slot[r]);
+      sel.insert(sel.end(), rows + r * m->d, rows + (r + 1) * m->d);
+    }
+  }
+  for (int64_t r = 0; r < k; ++r) {  // reset the touched entries
+    const int64_t i = slot[r] - m->row_offset;
+    if (slot[r] >= 0 && i >= 0 && i < m->n) m->ins_last[(size_t)i] = -1;
   }
   DeviceGuard g(m->device);
   kde_status st = idx.empty() ? KDE_OK : replace_impl(m, idx.data(), sel.data(), (int64_t)idx.size(), k_init);
   if (st != KDE_OK) return st;
+  ++m->gen;
   *n_seen += k;
   if (n_written) *n_written = (int64_t)idx.size();
   return KDE_OK;

@@ -71,13 +71,41 @@ __global__ void col_range_kernel(const float* __restrict__ cols, int64_t ld, int
   }
 }
 
-// widen the ranges by k host-supplied rows (row-major, device)
+// widen the ranges by k host-supplied rows (row-major, device): a block reduces its rows in
+// shared memory first, then one atomic per (block, column) -- not one per element
 __global__ void row_range_kernel(const float* __restrict__ rows, int64_t k, int d, unsigned* enc) {
-  const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (e >= k * d) return;
-  const int j = (int)(e % d);
-  atomicMin(enc + 2 * j, fenc(rows[e]));
-  atomicMax(enc + 2 * j + 1, fenc(rows[e]));
+  __shared__ unsigned smin[kMaxDim], smax[kMaxDim];
+  if (threadIdx.x < kMaxDim) {
+    smin[threadIdx.x] = 0xFFFFFFFFu;
+    smax[threadIdx.x] = 0u;
+  }
+  __syncthreads();
+  unsigned lmin[kMaxDim], lmax[kMaxDim];
+#pragma unroll
+  for (int j = 0; j < kMaxDim; ++j) {
+    lmin[j] = 0xFFFFFFFFu;
+    lmax[j] = 0u;
+  }
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < k; r += (int64_t)gridDim.x * blockDim.x) {
+#pragma unroll
+    for (int j = 0; j < kMaxDim; ++j)
+      if (j < d) {
+        const unsigned v = fenc(rows[r * d + j]);
+        lmin[j] = min(lmin[j], v);
+        lmax[j] = max(lmax[j], v);
+      }
+  }
+#pragma unroll
+  for (int j = 0; j < kMaxDim; ++j)
+    if (j < d) {
+      atomicMin(smin + j, lmin[j]);
+      atomicMax(smax + j, lmax[j]);
+    }
+  __syncthreads();
+  if (threadIdx.x < d) {
+    atomicMin(enc + 2 * threadIdx.x, smin[threadIdx.x]);
+    atomicMax(enc + 2 * threadIdx.x + 1, smax[threadIdx.x]);
+  }
 }
 
 
@@ -902,7 +930,9 @@ cudaError_t launch_col_range(const float* cols, int64_t ld, int64_t n, int d, un
 }
 cudaError_t launch_row_range(const float* rows, int64_t k, int d, unsigned* enc, DevConsts* c, cudaStream_t s) {
   if (k == 0) return cudaSuccess;
-  row_range_kernel<<<(unsigned)((k * d + 255) / 256), 256, 0, s>>>(rows, k, d, enc);
+  int64_t nb = (k + 255) / 256;
+  if (nb > 296) nb = 296;
+  row_range_kernel<<<(unsigned)nb, 256, 0, s>>>(rows, k, d, enc);
   KDE_LAUNCH_CHECK();
 }
 cudaError_t launch_scatter_rows_dev(const int64_t* idx_global, const float* rows, const int64_t* d_k, int64_t cap, int d,

@@ -69,3 +69,50 @@ def test_two_rank_gloo_combine_matches_full_estimate():
     assert len(out) == world
     for r in range(world):
         assert out[r] <= 1e-14
+
+
+def _worker_bootstrap(rank, world, port, out):
+    """The world > 1 host plumbing the GPU path relies on, on CPU: the strong-scaling sample
+    (every rank generates exactly its contiguous shard of ONE global sample), the IPC-handle
+    all-gather helper of dist.py, and libkde's host reservoir decision (identical on every rank)."""
+    import torch.distributed as dist
+
+    import bench
+    import paper_conf_sigmod_heimelkm15_b200 as K
+    import synth
+    from paper_conf_sigmod_heimelkm15_b200.dist import all_gather_bytes
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        cfg = dict(bench.CONFIGS["c4"], n=3_000_017, d=3)
+        off, k, n_global = bench.shard_of(cfg, rank, world)
+        shard = synth.gaussian_clusters_rows(n_global, 3, 7, off, off + k)
+        parts = [None] * world
+        dist.all_gather_object(parts, shard)
+        whole = synth.gaussian_clusters_rows(n_global, 3, 7, 0, n_global)
+        got = all_gather_bytes(bytes([rank]) * 64)           # the kde_peer_handle exchange
+        sel = K.kde_reservoir_select(99, n_global, n_global, 4096)
+        sels = [None] * world
+        dist.all_gather_object(sels, sel)
+        out[rank] = dict(strong=bool(np.array_equal(np.concatenate(parts), whole)),
+                         handles=got == [bytes([r]) * 64 for r in range(world)],
+                         reservoir=all(np.array_equal(s, sels[0]) for s in sels))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_two_rank_gloo_bootstrap_shards_and_reservoir():
+    world = 2
+    port = _free_port()
+    ctx = mp.get_context("spawn")
+    mgr = ctx.Manager()
+    out = mgr.dict()
+    procs = [ctx.Process(target=_worker_bootstrap, args=(r, world, port, out)) for r in range(world)]
+    for p in procs:
+        p.start()
+    for p in procs:
+        p.join(timeout=300)
+        assert p.exitcode == 0
+    for r in range(world):
+        assert out[r]["strong"] and out[r]["handles"] and out[r]["reservoir"], out[r]

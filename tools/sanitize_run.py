@@ -55,12 +55,23 @@ def run(d, n, q, kernel="gauss"):
     torch.cuda.synchronize()
     cnt = torch.zeros(len(lo), dtype=torch.int64, device=dev)
     K.kde_count_in_box_dev(torch.from_numpy(S).to(dev), dlo, dhi, cnt)
+    # device-resident streaming step (scan + cooperative karma / compaction / Listing 1 / replacement)
+    fest = torch.zeros(1, dtype=torch.float64, device=dev)
+    fg = torch.zeros(d, dtype=torch.float64, device=dev)
+    for k in range(3):
+        K.kde_stream_step_dev(m.handle, dlo[k:k + 1], dhi[k:k + 1], dp[k:k + 1], K.karma_params(threshold=0.0),
+                              K.online_params(minibatch=2), didx, dcnt, rows, fest, fg)
+    torch.cuda.synchronize()
+    # reservoir inserts (host decision, accepted rows only)
+    m.insert_rows(S[: min(n, 3000)][::-1].copy(), seed=5, n_seen=n)
+    m.estimate(lo[:1], hi[:1], grad=True)
     torch.cuda.synchronize()
     m.close()
 
 
 if __name__ == "__main__":
     for d, n, q, kern in [(3, 5003, 40, "gauss"), (10, 3001, 17, "gauss"), (13, 2053, 9, "gauss"),
-                          (3, 9001, 0, "gauss"), (5, 4099, 0, "epan"), (10, 2051, 0, "gauss")]:
+                          (3, 9001, 0, "gauss"), (5, 4099, 0, "epan"), (10, 2051, 0, "gauss"),
+                          (8, 20011, 0, "gauss"), (10, 40009, 33, "gauss"), (16, 9001, 5, "gauss")]:
         run(d, n, q, kern)
     print("sanitize run ok")
