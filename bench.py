@@ -713,6 +713,9 @@ def main():
                     help="evaluate every (point, box) pair (kde_set_cull(0)); default culls provably < 2^-64")
     ap.add_argument("--no-graph", action="store_true", help="stream configs: launch eagerly instead of CUDA graphs")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of all-core oracle work")
+    ap.add_argument("--rows", type=int, default=0,
+                    help="override the config's sample rows (per GPU, or global for strong configs); recorded in "
+                         "config -- for functional checks, not the named workload")
     ap.add_argument("--share-gpu", action="store_true",
                     help="run every rank on cuda:0 (gloo process group, peer transport): exercises the world > 1 "
                          "path on a one-GPU box; not a scaling measurement")
@@ -729,7 +732,10 @@ def main():
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE {world}")
-    cfg = CONFIGS[args.config]
+    cfg = dict(CONFIGS[args.config])
+    if args.rows:
+        cfg["n"] = args.rows
+        cfg["desc"] = cfg["desc"] + f" [rows overridden: {args.rows}]"
     if args.impl == "reference":
         run_reference(args, cfg, rank, world)
         return

@@ -30,6 +30,17 @@
  *  - Sharded models (one process per GPU): every rank calls every function
  *    collectively with identical query arguments; point indices are GLOBAL.
  *  - A model is externally synchronised (one thread at a time).
+ *
+ * Environment (read by the library)
+ *  - KDE_DEBUG_SYNC=1      synchronise after every kernel launch, so a fault
+ *                          is reported by the call that launched it (debug).
+ *  - KDE_PEER_TIMEOUT_S    bound on a peer-exchange wait (default 60 s).
+ *  - KDE_PEER_SLOT_MB      peer exchange window slot size (default 4 MiB).
+ *  - KDE_PEER_FUSED=0      peer transport: separate all-gather instead of the
+ *                          producer-tail push (A/B testing).
+ *  - KDE_KARMA_TWO_PASS=1  karma pass as two kernels instead of the
+ *                          cooperative one (A/B timing).
+ *  Every entry point that does device work opens an NVTX range named after it.
  */
 #ifndef KDE_H
 #define KDE_H

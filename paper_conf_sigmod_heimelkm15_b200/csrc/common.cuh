@@ -69,6 +69,21 @@ struct KarmaParamsDev {
   double lambda, k_max, threshold;
 };
 
+// Peer-memory exchange of a sharded model (peer.cu): every rank's exchange window mapped into
+// this process, the device-side epoch / arrival counters / error flag.  A window is
+//   [kPeerFlagBytes) flags: uint64 epoch per source rank (128 B apart) | [2][world][slot] data slots
+constexpr int kMaxWorld = 32;
+constexpr size_t kPeerFlagBytes = (size_t)kMaxWorld * 128;
+struct PeerArgs {
+  char* base[kMaxWorld];  // every rank's exchange window (base[rank] = own)
+  int rank = 0, world = 1;
+  size_t slot = 0;            // bytes per (parity, source rank) slot, multiple of 256
+  uint64_t* epoch = nullptr;  // device: last completed exchange
+  unsigned* count = nullptr;  // device: 4 self-resetting block-arrival counters
+  int* err = nullptr;         // device: set to 1 when a wait times out
+  uint64_t timeout_ns = 0;
+};
+
 // scan over the sample for ONE box (q == 1): HBM-streaming reduction.
 struct ScanSingleArgs {
   const float* cols;      // [d][ld] fp32 SoA sample
@@ -86,6 +101,7 @@ struct ScanSingleArgs {
   double* dpdh_out;       // nullable: d x dp_hat/dh_j (caller's buffer), world == 1, GRAD only
   double n_global;        // s (results are divided by s, so s ones give exactly 1)
   int cull;               // 1: skip points whose contribution is provably < 2^-64 (scan_single_tma.cuh)
+  const PeerArgs* peer;   // nullable (device): the last block pushes sums_out into every rank's window
 };
 
 // scan for many boxes: sample tiles staged in shared memory by TMA bulk

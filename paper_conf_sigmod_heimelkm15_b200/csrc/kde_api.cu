@@ -17,6 +17,7 @@
 
 #include <cuda_runtime.h>
 #include <nccl.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include "../../include/kde.h"
 #include "common.cuh"
@@ -52,6 +53,7 @@ struct kde_model {
   char* xwin = nullptr;            // KDE_COMM_PEER: this rank's exchange window (peer.cu)
   size_t xwin_bytes = 0;
   PeerArgs pa;                     // mapped windows of every rank + device epoch / counters / error flag
+  PeerArgs* pa_dev = nullptr;      // device copy of pa (read by the producers' fused push)
   bool poisoned = false;
 
   float* cols = nullptr;       // [d][ld]
@@ -121,11 +123,25 @@ struct kde_model {
     }                                                                                                \
   } while (0)
 
-#define CUL(call)   \
-  do {              \
-    ++m->launches;  \
-    CU(call);       \
+// KDE_DEBUG_SYNC=1: synchronise the stream after every launch so a faulting kernel is reported by
+// the call that launched it (debugging aid; off by default)
+static bool debug_sync() {
+  static const bool on = getenv("KDE_DEBUG_SYNC") && atoi(getenv("KDE_DEBUG_SYNC")) != 0;
+  return on;
+}
+#define CUL(call)                                         \
+  do {                                                    \
+    ++m->launches;                                        \
+    CU(call);                                             \
+    if (debug_sync()) CU(cudaDeviceSynchronize());        \
   } while (0)
+
+// NVTX range per ABI call (visible in Nsight Systems / ncu --nvtx; no cost without a tool attached)
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+#define KDE_RANGE() NvtxRange nvtx_range_(__func__)
 
 #define NC(call)                                                                                     \
   do {                                                                                               \
@@ -272,8 +288,16 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
                             double* d_sums, cudaStream_t s, double* d_est = nullptr, double* d_dpdh = nullptr) {
   const int d = m->d;
   const int na = grad ? d + 1 : 1;
+  // fused exchange (peer transport): the producer's tail pushes the final sums into every rank's
+  // window; one combine kernel follows (KDE_PEER_FUSED=0: the separate all-gather, for A/B tests)
+  const char* fenv = getenv("KDE_PEER_FUSED");
+  const PeerArgs* fused = (m->comm_kind == KDE_COMM_PEER && sizeof(double) * (size_t)q * na <= m->pa.slot &&
+                           !(fenv && atoi(fenv) == 0))
+                              ? m->pa_dev
+                              : nullptr;
   if (q == 1) {
     ScanSingleArgs a;
+    a.peer = fused;
     a.cols = m->cols;
     a.ld = m->ld;
     a.n = m->n;
@@ -327,9 +351,11 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     if (st != KDE_OK) return st;
     CUL(launch_scan_batched(d, grad, a, m->num_sms, &splits, s, false));
     if (e2) CU(cudaEventRecord(e2, s));
-    CUL(launch_reduce_splits(m->partials, splits, q, na, d_sums, s));
+    CUL(launch_reduce_splits(m->partials, splits, q, na, d_sums, fused, s));
   }
-  if (m->world > 1) {
+  if (fused) {
+    CUL(launch_peer_combine(d_sums, q * na, m->pa, m->num_sms, s));
+  } else if (m->world > 1) {
     const size_t bytes = sizeof(double) * (size_t)m->world * q * na;
     kde_status st = ensure_bytes((void**)&m->gather, &m->gather_cap, bytes);
     if (st != KDE_OK) return st;
@@ -423,6 +449,7 @@ static void free_model(kde_model* m) {
       if (r != m->rank && m->pa.base[r]) cudaIpcCloseMemHandle(m->pa.base[r]);
     cudaFree(m->xwin);
     cudaFree(m->pa.epoch);  // epoch, counters and error flag share one allocation
+    cudaFree(m->pa_dev);
   }
   cudaFree(m->kbuf);
   if (m->stream) cudaStreamDestroy(m->stream);
@@ -474,6 +501,7 @@ static size_t peer_slot_bytes() {
 static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_offset, int64_t n_global, int32_t d,
                               const double* h, const void* nccl_id, int32_t rank, int32_t world, int comm_kind,
                               kde_model** out) {
+  KDE_RANGE();
   if (!out) return fail(KDE_EINVAL, "out is NULL");
   if (d < 1 || d > KDE_MAX_DIM) return fail(KDE_EINVAL, "d = %d outside [1, %d]", d, KDE_MAX_DIM);
   if (world < 1 || rank < 0 || rank >= world) return fail(KDE_EINVAL, "bad rank/world %d/%d", rank, world);
@@ -527,7 +555,7 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
   CUB(cudaMalloc(&m->scal, sizeof(double) * 8));
   const int nkb = karma_blocks(n_local);
   CUB(cudaMalloc(&m->bitmap, sizeof(uint32_t) * (size_t)nkb * (kKarmaPts / 32)));
-  CUB(cudaMalloc(&m->block_counts, sizeof(int32_t) * (size_t)nkb));
+  CUB(cudaMalloc(&m->block_counts, sizeof(int32_t) * (size_t)nkb * 4));  // also the cooperative karma CTA counts (<= passes)
   CUB(cudaMalloc(&m->block_offsets, sizeof(int64_t) * ((size_t)nkb + 1)));
   CUB(cudaMalloc(&m->offsets, sizeof(int64_t) * 2));
   CUB(cudaMalloc(&m->done, 2 * sizeof(unsigned)));
@@ -556,8 +584,8 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
     CUB(cudaMalloc(&ctl, 64));
     CUB(cudaMemsetAsync(ctl, 0, 64, s));
     m->pa.epoch = reinterpret_cast<uint64_t*>(ctl);
-    m->pa.count = reinterpret_cast<unsigned*>(ctl + 8);
-    m->pa.err = reinterpret_cast<int*>(ctl + 16);
+    m->pa.count = reinterpret_cast<unsigned*>(ctl + 8);  // 4 counters
+    m->pa.err = reinterpret_cast<int*>(ctl + 32);
     m->pa.rank = rank;
     m->pa.world = world;
     double tmo = 60.0;
@@ -654,6 +682,7 @@ extern "C" kde_status kde_peer_handle(kde_model* m, void* handle_out) {
 }
 
 extern "C" kde_status kde_peer_attach(kde_model* m, const void* handles) {
+  KDE_RANGE();
   if (!m || !handles) return fail(KDE_EINVAL, "NULL argument");
   if (m->comm_kind != KDE_COMM_PEER) return fail(KDE_EINVAL, "model does not use the peer transport");
   if (m->attached) return fail(KDE_ESTATE, "already attached");
@@ -667,6 +696,8 @@ extern "C" kde_status kde_peer_attach(kde_model* m, const void* handles) {
     CU(cudaIpcOpenMemHandle(&p, hnd, cudaIpcMemLazyEnablePeerAccess));
     m->pa.base[r] = (char*)p;
   }
+  CU(cudaMalloc(&m->pa_dev, sizeof(PeerArgs)));
+  CU(cudaMemcpy(m->pa_dev, &m->pa, sizeof(PeerArgs), cudaMemcpyHostToDevice));
   m->attached = true;
   if (m->h_pending) {  // Scott's rule needs the all-gather of the shard moments
     m->h_pending = false;
@@ -781,6 +812,7 @@ static void note_retained(kde_model* m, const float* lo, const float* hi, bool h
 
 extern "C" kde_status kde_estimate_batch(kde_model* m, const float* lo, const float* hi, int64_t q, double* est,
                                          double* dest_dh) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   kde_status st = validate_bounds(lo, hi, q, m->d);
   if (st != KDE_OK) return st;
@@ -813,6 +845,7 @@ extern "C" kde_status kde_estimate_batch(kde_model* m, const float* lo, const fl
 
 extern "C" kde_status kde_estimate_batch_dev(kde_model* m, const float* d_lo, const float* d_hi, int64_t q,
                                              double* d_est, double* d_dest_dh, void* stream) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   if (q < 0) return fail(KDE_EINVAL, "q < 0");
   if (q == 0) return KDE_OK;
@@ -842,6 +875,7 @@ static kde_status loss_grad_dev_impl(kde_model* m, const float* d_lo, const floa
 extern "C" kde_status kde_loss_and_grad(kde_model* m, const float* lo, const float* hi, const double* true_sel,
                                         int64_t q, int32_t loss, double lambda, int32_t log_bandwidth,
                                         double* loss_out, double* grad_out, double* est_out) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   if (q < 1) return fail(KDE_EINVAL, "q must be >= 1");
   kde_status st = validate_bounds(lo, hi, q, m->d);
@@ -869,6 +903,7 @@ extern "C" kde_status kde_loss_and_grad_dev(kde_model* m, const float* d_lo, con
                                             const double* d_true_sel, int64_t q, int32_t loss, double lambda,
                                             int32_t log_bandwidth, double* d_loss, double* d_grad, double* d_est,
                                             void* stream) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   if (q < 1) return fail(KDE_EINVAL, "q must be >= 1");
   kde_status st = validate_loss(loss, lambda);
@@ -949,6 +984,7 @@ static kde_status ensure_retained(kde_model* m, const float* lo, const float* hi
 extern "C" kde_status kde_karma_update(kde_model* m, const float* lo, const float* hi, double true_sel,
                                        const kde_karma_params* kp, int64_t* idx_out, int64_t idx_cap,
                                        int64_t* n_flagged) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   kde_status st = validate_bounds(lo, hi, 1, m->d);
   if (st != KDE_OK) return st;
@@ -1039,6 +1075,7 @@ extern "C" kde_status kde_karma_update(kde_model* m, const float* lo, const floa
 
 extern "C" kde_status kde_online_update(kde_model* m, const float* lo, const float* hi, double true_sel,
                                         const kde_online_params* op, int32_t* updated) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   kde_status st = validate_bounds(lo, hi, 1, m->d);
   if (st != KDE_OK) return st;
@@ -1092,6 +1129,7 @@ static kde_status replace_impl(kde_model* m, const int64_t* idx, const float* ro
 
 extern "C" kde_status kde_replace_points(kde_model* m, const int64_t* idx, const float* rows, int64_t k,
                                          double k_init) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   if (k < 0) return fail(KDE_EINVAL, "k < 0");
   if (k == 0) return KDE_OK;
@@ -1121,6 +1159,7 @@ extern "C" kde_status kde_reservoir_select(uint64_t seed, int64_t n_sample, int6
 
 extern "C" kde_status kde_insert_rows(kde_model* m, const float* rows, int64_t k, uint64_t seed, int64_t* n_seen,
                                       double k_init, int64_t* n_written) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   if (k < 0 || !n_seen || *n_seen < 0 || *n_seen > INT64_MAX - k) return fail(KDE_EINVAL, "bad k / n_seen");
   if (k > 0 && !rows) return fail(KDE_EINVAL, "rows is NULL");
@@ -1165,6 +1204,7 @@ extern "C" kde_status kde_insert_rows(kde_model* m, const float* rows, int64_t k
 extern "C" kde_status kde_karma_update_dev(kde_model* m, const float* d_lo, const float* d_hi,
                                            const double* d_true_sel, const kde_karma_params* kp, int64_t* d_idx_out,
                                            int64_t idx_cap, int64_t* d_n_flagged, void* stream) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   if (m->world != 1) return fail(KDE_EINVAL, "device-resident feedback calls are single-GPU (world == 1)");
   if (!d_lo || !d_hi || !d_true_sel || !d_n_flagged || idx_cap < 0 || (idx_cap > 0 && !d_idx_out))
@@ -1183,6 +1223,7 @@ extern "C" kde_status kde_karma_update_dev(kde_model* m, const float* d_lo, cons
 
 extern "C" kde_status kde_online_update_dev(kde_model* m, const double* d_true_sel, const kde_online_params* op,
                                             void* stream) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   if (!d_true_sel) return fail(KDE_EINVAL, "NULL device pointer");
   DeviceGuard g(m->device);
@@ -1197,6 +1238,7 @@ extern "C" kde_status kde_online_update_dev(kde_model* m, const double* d_true_s
 
 extern "C" kde_status kde_replace_points_dev(kde_model* m, const int64_t* d_idx, const float* d_rows,
                                              const int64_t* d_k, int64_t cap, double k_init, void* stream) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   if (cap < 0 || (cap > 0 && (!d_idx || !d_rows || !d_k))) return fail(KDE_EINVAL, "NULL device pointer / cap");
   if (!std::isfinite(k_init)) return fail(KDE_EINVAL, "k_init not finite");
@@ -1218,6 +1260,7 @@ extern "C" kde_status kde_stream_step_dev(kde_model* m, const float* d_lo, const
                                           const kde_online_params* op, int64_t* d_idx_out, int64_t idx_cap,
                                           int64_t* d_n_flagged, const float* d_rows, double k_init, double* d_est,
                                           double* d_dpdh, void* stream) {
+  KDE_RANGE();
   CHECK_MODEL(m);
   if (m->world != 1) return fail(KDE_EINVAL, "device-resident streaming step is single-GPU (world == 1)");
   if (!d_lo || !d_hi || !d_true_sel || !d_n_flagged || !d_est || idx_cap < 0 || (idx_cap > 0 && !d_idx_out))

@@ -13,6 +13,7 @@
 
 #include "common.cuh"
 #include "kernels.cuh"
+#include "peer.cuh"
 
 namespace kde {
 namespace cg = cooperative_groups;
@@ -241,13 +242,27 @@ __global__ void set_consts_kernel(HVec hv, int d, DevConsts* c) {
 // sums[qi][k] = sum_{s in split order} partials[(s*NA + k)*q + qi]; with
 // finalisation (world == 1): est[qi] = S_0/N, dpdh[qi][j] = S_j gconst_j / N.
 __global__ void reduce_splits_kernel(const double* __restrict__ partials, int splits, int64_t q, int na,
-                                     double* __restrict__ sums) {
+                                     double* __restrict__ sums, const PeerArgs* __restrict__ peer) {
   const int64_t qi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (qi >= q) return;
-  for (int k = 0; k < na; ++k) {
-    double t = 0.0;
-    for (int s = 0; s < splits; ++s) t += partials[((int64_t)s * na + k) * q + qi];
-    sums[qi * na + k] = t;
+  const uint64_t pe = peer ? peer_next_epoch(*peer) : 0;
+  if (qi < q)
+    for (int k = 0; k < na; ++k) {
+      double t = 0.0;
+      for (int s = 0; s < splits; ++s) t += partials[((int64_t)s * na + k) * q + qi];
+      if (peer)
+        peer_store(*peer, pe, qi * na + k, t);  // fused exchange: straight into every rank's window
+      else
+        sums[qi * na + k] = t;
+    }
+  if (!peer) return;
+  __shared__ bool last_s;
+  __threadfence_system();
+  __syncthreads();
+  if (threadIdx.x == 0) last_s = atomicAdd(peer->count + 2, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (last_s && threadIdx.x == 0) {  // every block's stores are fenced: flags up
+    peer->count[2] = 0u;
+    peer_release(*peer, pe);
   }
 }
 
@@ -651,17 +666,17 @@ __global__ void online_update_kernel(const double* __restrict__ ret, const doubl
 
 // ------------------------------------------------------------ karma pass, one cooperative kernel
 // The whole feedback tail of a query in ONE persistent launch (cooperative: all CTAs co-resident,
-// grid-wide barriers): each CTA owns a contiguous run of 4096-point segments.
-//   phase 1  karma (eq. 6-8) and flags (R4, eq. 20) for its segments, exactly as karma_kernel:
-//            128-bit loads, index-order bitmap words, a per-CTA flag count;
-//   barrier  -> the CTA's offset is the sum of the counts of the CTAs before it (<= a few hundred);
-//   phase 2  ordered compaction of its segments' bitmap words into ascending GLOBAL indices;
-//   barrier  -> phase 3: CTA 0 runs the Listing 1 step (optional), all CTAs replace the first
-//            min(total, cap) flagged points by tail.rows (optional).
-// Replaces the karma + compaction kernel pair (two launches, nb = n/4096 blocks each, a serial
-// last-block tail).
+// grid-wide barriers).  The points are cut into passes of 1024 (256 threads x 4 consecutive points);
+// CTA b owns the contiguous passes [b P / G, (b + 1) P / G) -- balanced to one pass.
+//   phase 1  karma (eq. 6-8) and flags (R4, eq. 20): 128-bit loads of p^(i) and K, index-order
+//            bitmap words (8 lanes x 4 points per word), a per-CTA flag count;
+//   barrier  -> the CTA's offset is the sum of the counts of the CTAs before it;
+//   phase 2  ordered compaction of its bitmap words into ascending GLOBAL indices (128 words per
+//            step: warp 0 forms the popcount prefix, all warps write);
+//   barrier  -> phase 3 (streaming step only): CTA 0 runs the Listing 1 step, all CTAs replace the
+//            first min(total, cap) flagged points by tail.rows.
 constexpr int kCoopThreads = 256;
-constexpr int kCoopSeg = kKarmaPts;  // points per segment (kCoopThreads x 4 points x 4 passes)
+constexpr int kCoopPass = kCoopThreads * kKarmaKV;  // points per pass (32 bitmap words)
 
 struct KarmaCoopArgs {
   const float* cvals;
@@ -686,16 +701,18 @@ struct KarmaCoopArgs {
 
 __global__ void __launch_bounds__(kCoopThreads, KDE_TUNE_KARMA_MINB) karma_coop_kernel(const KarmaCoopArgs a) {
   cg::grid_group grid = cg::this_grid();
+  constexpr int W = 128;  // bitmap words per compaction step
+  constexpr int WPL = W / 32;
   __shared__ double thr_s;
   __shared__ int64_t red_s[2][kCoopThreads / 32];
-  __shared__ int32_t wpre[kCoopSeg / 32];
-  __shared__ uint32_t wbits[kCoopSeg / 32];
+  __shared__ int32_t wpre[W];
+  __shared__ uint32_t wbits[W];
   __shared__ int32_t segtot_s;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int G = gridDim.x, b = blockIdx.x;
-  const int64_t nseg = (a.n + kCoopSeg - 1) / kCoopSeg;
-  const int64_t per = (nseg + G - 1) / G;
-  const int64_t sg0 = min(nseg, (int64_t)b * per), sg1 = min(nseg, sg0 + per);
+  const int64_t n = a.n;
+  const int64_t P = (n + kCoopPass - 1) / kCoopPass;
+  const int64_t p0 = (int64_t)b * P / G, p1 = (int64_t)(b + 1) * P / G;
   const KarmaParamsDev kp = a.kp;
   const double p = *a.p;
   if (tid == 0) thr_s = (kp.empty_region && p == 0.0) ? thr20_dev(a.lo, a.hi, a.d, a.c) : CUDART_INF;
@@ -705,59 +722,57 @@ __global__ void __launch_bounds__(kCoopThreads, KDE_TUNE_KARMA_MINB) karma_coop_
   loss_eval(kp.loss, kp.lambda, phat, p, &L_full, &dummy);
   const double thr = thr_s;
   const double inv_nm1 = 1.0 / (a.n_global - 1.0);
-  const int64_t n = a.n;
   // ---------------- phase 1: karma + flags
   int32_t my = 0;
-  constexpr int PASSES = kCoopSeg / (kCoopThreads * kKarmaKV);
-  constexpr int PB = 2;
-  for (int64_t sg = sg0; sg < sg1; ++sg) {
-    const int64_t base = sg * kCoopSeg;
+#ifndef KDE_TUNE_COOP_PB
+#define KDE_TUNE_COOP_PB 2
+#endif
+  constexpr int PB = KDE_TUNE_COOP_PB;  // passes whose loads are in flight together
 #pragma unroll 1
-    for (int r0 = 0; r0 < PASSES; r0 += PB) {
-      float4 cv[PB];
-      double2 kv[PB][2];
+  for (int64_t q0 = p0; q0 < p1; q0 += PB) {
+    float4 cv[PB];
+    double2 kv[PB][2];
 #pragma unroll
-      for (int r = 0; r < PB; ++r) {
-        const int64_t i = base + ((int64_t)(r0 + r) * kCoopThreads + tid) * kKarmaKV;
-        if (i < n) {  // i is a multiple of 4; c and K are padded past n
-          cv[r] = __ldcs(reinterpret_cast<const float4*>(a.cvals + i));
-          kv[r][0] = __ldcs(reinterpret_cast<const double2*>(a.karma + i));
-          kv[r][1] = __ldcs(reinterpret_cast<const double2*>(a.karma + i + 2));
-        } else {
-          cv[r] = make_float4(0.f, 0.f, 0.f, 0.f);
-          kv[r][0] = kv[r][1] = make_double2(0.0, 0.0);
+    for (int r = 0; r < PB; ++r) {
+      const int64_t i = (q0 + r) * kCoopPass + (int64_t)tid * kKarmaKV;
+      if (q0 + r < p1 && i < n) {  // i is a multiple of 4; c and K are padded past n
+        cv[r] = __ldcs(reinterpret_cast<const float4*>(a.cvals + i));
+        kv[r][0] = __ldcs(reinterpret_cast<const double2*>(a.karma + i));
+        kv[r][1] = __ldcs(reinterpret_cast<const double2*>(a.karma + i + 2));
+      } else {
+        cv[r] = make_float4(0.f, 0.f, 0.f, 0.f);
+        kv[r][0] = kv[r][1] = make_double2(0.0, 0.0);
+      }
+    }
+#pragma unroll
+    for (int r = 0; r < PB; ++r) {
+      if (q0 + r >= p1) break;  // CTA-uniform
+      const int64_t i = (q0 + r) * kCoopPass + (int64_t)tid * kKarmaKV;
+      const float cc[4] = {cv[r].x, cv[r].y, cv[r].z, cv[r].w};
+      double kk[4] = {kv[r][0].x, kv[r][0].y, kv[r][1].x, kv[r][1].y};
+      unsigned nib = 0u;
+#pragma unroll
+      for (int v = 0; v < kKarmaKV; ++v) {
+        if (i + v < n) {
+          const double ci = (double)cc[v];
+          const double p_minus = (phat * a.n_global - ci) * inv_nm1;  // eq. (6)
+          double L_minus;
+          loss_eval(kp.loss, kp.lambda, p_minus, p, &L_minus, &dummy);
+          kk[v] = fmin(kk[v] + (L_minus - L_full), kp.k_max);  // eq. (7)-(8)
+          nib |= (unsigned)((kk[v] < kp.threshold) || (ci >= thr)) << v;
         }
       }
-#pragma unroll
-      for (int r = 0; r < PB; ++r) {
-        const int64_t i = base + ((int64_t)(r0 + r) * kCoopThreads + tid) * kKarmaKV;
-        const float cc[4] = {cv[r].x, cv[r].y, cv[r].z, cv[r].w};
-        double kk[4] = {kv[r][0].x, kv[r][0].y, kv[r][1].x, kv[r][1].y};
-        unsigned nib = 0u;
-#pragma unroll
-        for (int v = 0; v < kKarmaKV; ++v) {
-          if (i + v < n) {
-            const double ci = (double)cc[v];
-            const double p_minus = (phat * a.n_global - ci) * inv_nm1;  // eq. (6)
-            double L_minus;
-            loss_eval(kp.loss, kp.lambda, p_minus, p, &L_minus, &dummy);
-            kk[v] = fmin(kk[v] + (L_minus - L_full), kp.k_max);  // eq. (7)-(8)
-            nib |= (unsigned)((kk[v] < kp.threshold) || (ci >= thr)) << v;
-          }
-        }
-        if (i < n) {
-          __stcs(reinterpret_cast<double2*>(a.karma + i), make_double2(kk[0], kk[1]));
-          __stcs(reinterpret_cast<double2*>(a.karma + i + 2), make_double2(kk[2], kk[3]));
-        }
-        unsigned word = nib << (4 * (lane & 7));  // word of 32 points = nibbles of 8 lanes
-        word |= __shfl_xor_sync(0xffffffffu, word, 1);
-        word |= __shfl_xor_sync(0xffffffffu, word, 2);
-        word |= __shfl_xor_sync(0xffffffffu, word, 4);
-        if ((lane & 7) == 0) {
-          const int64_t w0 = (base + ((int64_t)(r0 + r) * kCoopThreads + warp * 32) * kKarmaKV) / 32;
-          a.bitmap[w0 + (lane >> 3)] = word;
-          my += __popc(word);
-        }
+      if (i < n) {
+        __stcs(reinterpret_cast<double2*>(a.karma + i), make_double2(kk[0], kk[1]));
+        __stcs(reinterpret_cast<double2*>(a.karma + i + 2), make_double2(kk[2], kk[3]));
+      }
+      unsigned word = nib << (4 * (lane & 7));  // word of 32 points = nibbles of 8 lanes
+      word |= __shfl_xor_sync(0xffffffffu, word, 1);
+      word |= __shfl_xor_sync(0xffffffffu, word, 2);
+      word |= __shfl_xor_sync(0xffffffffu, word, 4);
+      if ((lane & 7) == 0) {
+        a.bitmap[(q0 + r) * (kCoopPass / 32) + warp * 4 + (lane >> 3)] = word;
+        my += __popc(word);
       }
     }
   }
@@ -792,47 +807,47 @@ __global__ void __launch_bounds__(kCoopThreads, KDE_TUNE_KARMA_MINB) karma_coop_
     before += red_s[0][w];
     total += red_s[1][w];
   }
-  constexpr int W = kCoopSeg / 32;  // bitmap words per segment
-  constexpr int WPL = W / 32;
-  const int64_t nwords = (n + 31) / 32;
-  int64_t run = before;
-  for (int64_t sg = sg0; sg < sg1; ++sg) {
-    const int64_t wbase = sg * W;
-    if (warp == 0) {  // the segment's words, their exclusive popcount prefix
-      int cnt[WPL], tot = 0;
+  if (total > 0) {  // nothing flagged anywhere: no bitmap to walk
+    const int64_t nwords = (n + 31) / 32;
+    const int64_t w1 = min(p1 * (kCoopPass / 32), nwords);
+    int64_t run = before;
+    for (int64_t wb = p0 * (kCoopPass / 32); wb < w1; wb += W) {
+      if (warp == 0) {  // the step's words, their exclusive popcount prefix
+        int cnt[WPL], tot = 0;
 #pragma unroll
-      for (int k = 0; k < WPL; ++k) {
-        const int64_t w = wbase + WPL * lane + k;
-        const uint32_t word = w < nwords ? __ldcg(a.bitmap + w) : 0u;
-        wbits[WPL * lane + k] = word;
-        cnt[k] = __popc(word);
-        tot += cnt[k];
-      }
-      int incl = tot;
+        for (int k = 0; k < WPL; ++k) {
+          const int64_t w = wb + WPL * lane + k;
+          const uint32_t word = w < w1 ? __ldcg(a.bitmap + w) : 0u;
+          wbits[WPL * lane + k] = word;
+          cnt[k] = __popc(word);
+          tot += cnt[k];
+        }
+        int incl = tot;
 #pragma unroll
-      for (int k = 1; k < 32; k <<= 1) {
-        const int v = __shfl_up_sync(0xffffffffu, incl, k);
-        if (lane >= k) incl += v;
-      }
-      int rr = incl - tot;
+        for (int k = 1; k < 32; k <<= 1) {
+          const int v = __shfl_up_sync(0xffffffffu, incl, k);
+          if (lane >= k) incl += v;
+        }
+        int rr = incl - tot;
 #pragma unroll
-      for (int k = 0; k < WPL; ++k) {
-        wpre[WPL * lane + k] = rr;
-        rr += cnt[k];
+        for (int k = 0; k < WPL; ++k) {
+          wpre[WPL * lane + k] = rr;
+          rr += cnt[k];
+        }
+        if (lane == 31) segtot_s = incl;
       }
-      if (lane == 31) segtot_s = incl;
-    }
-    __syncthreads();
+      __syncthreads();
 #pragma unroll 4
-    for (int w = warp; w < W; w += kCoopThreads / 32) {
-      const uint32_t word = wbits[w];
-      if (word & (1u << lane)) {
-        const int64_t pos = run + wpre[w] + __popc(word & ((1u << lane) - 1u));
-        if (pos < a.cap) a.idx_out[pos] = a.row_offset + (wbase + w) * 32 + lane;
+      for (int w = warp; w < W; w += kCoopThreads / 32) {
+        const uint32_t word = wbits[w];
+        if (word & (1u << lane)) {
+          const int64_t pos = run + wpre[w] + __popc(word & ((1u << lane) - 1u));
+          if (pos < a.cap) a.idx_out[pos] = a.row_offset + (wb + w) * 32 + lane;
+        }
       }
+      run += segtot_s;
+      __syncthreads();
     }
-    run += segtot_s;
-    __syncthreads();
   }
   if (b == 0 && tid == 0 && a.total_out) *a.total_out = total;
   const StreamTail& tail = a.tail;
@@ -984,8 +999,8 @@ cudaError_t launch_set_consts(const double* h, int d, DevConsts* c, cudaStream_t
   KDE_LAUNCH_CHECK();
 }
 cudaError_t launch_reduce_splits(const double* partials, int splits, int64_t q, int na, double* sums,
-                                 cudaStream_t s) {
-  reduce_splits_kernel<<<(unsigned)((q + 255) / 256), 256, 0, s>>>(partials, splits, q, na, sums);
+                                 const PeerArgs* peer, cudaStream_t s) {
+  reduce_splits_kernel<<<(unsigned)((q + 255) / 256), 256, 0, s>>>(partials, splits, q, na, sums, peer);
   KDE_LAUNCH_CHECK();
 }
 cudaError_t launch_combine_ranks(const double* gathered, int world, int64_t q, int na, double* sums,
@@ -1036,7 +1051,8 @@ cudaError_t launch_karma(const float* cvals, double* karma, int64_t n, double n_
     KarmaCoopArgs a{cvals, karma, n, n_global, phat, p, kp, lo, hi, d, c, bitmap, block_counts, row_offset,
                     idx_out, cap, total_out, tail};
     int grid = coop_grid_limit();
-    if (grid > nb) grid = nb;
+    const int64_t passes = (n + kCoopPass - 1) / kCoopPass;
+    if (grid > passes) grid = (int)passes;
     if (grid < 1) grid = 1;
     void* args[] = {&a};
     return cudaLaunchCooperativeKernel((const void*)karma_coop_kernel, grid, kCoopThreads, args, 0, s);

@@ -58,8 +58,10 @@ size_t cull_order_bytes(int64_t q);
 cudaError_t launch_cull_order(const float* cols, int64_t ld, int64_t n, int d, const float* lo, const float* hi,
                               int64_t q, const DevConsts* c, void* scratch, size_t scratch_bytes, int** perm_out,
                               cudaStream_t s);
+// sums (or, with peer != NULL, slot [epoch parity][rank] of EVERY rank's exchange window: the fused
+// exchange) <- the fixed-order sum over splits
 cudaError_t launch_reduce_splits(const double* partials, int splits, int64_t q, int na, double* sums,
-                                 cudaStream_t s);
+                                 const PeerArgs* peer, cudaStream_t s);
 cudaError_t launch_combine_ranks(const double* gathered, int world, int64_t q, int na, double* sums,
                                  cudaStream_t s);
 cudaError_t launch_finalize(const double* sums, int64_t q, int d, int na, const DevConsts* c, double n_global,
@@ -83,20 +85,13 @@ cudaError_t launch_count_in_box(const float* rows, int64_t n, int d, const float
 // reservoir.cu: Algorithm R decisions (host), slot or -1 per arrival n_seen+1 .. n_seen+k
 void reservoir_slots(uint64_t seed, int64_t n_sample, int64_t n_seen, int64_t k, int64_t* slot_out);
 
-// peer.cu: all-gather over peer device memory (the sharded model's exchange step without NCCL)
-constexpr int kMaxWorld = 32;
-constexpr size_t kPeerFlagBytes = (size_t)kMaxWorld * 128;  // one 128-byte line per source rank
-struct PeerArgs {
-  char* base[kMaxWorld];  // every rank's exchange window, mapped into this process (base[rank] = own)
-  int rank = 0, world = 1;
-  size_t slot = 0;        // bytes per (parity, source rank) slot, multiple of 256
-  uint64_t* epoch = nullptr;  // device: last completed exchange
-  unsigned* count = nullptr;  // device: 2 self-resetting block-arrival counters
-  int* err = nullptr;         // device: set to 1 when a wait times out
-  uint64_t timeout_ns = 0;
-};
+// peer.cu: all-gather over peer device memory (the sharded model's exchange step without NCCL);
+// PeerArgs / kPeerFlagBytes live in common.cuh (the scan tails push into peer windows directly)
 // dst + r * stride <- rank r's src (bytes <= pa.slot, multiples of 8), for every rank r
 cudaError_t launch_peer_allgather(const void* src, void* dst, size_t bytes, size_t stride, const PeerArgs& pa,
                                   int num_sms, cudaStream_t s);
+// fused exchange, consumer side: wait for every rank's pushed slot of this epoch (count doubles,
+// pushed by the scan tail / reduce_splits), sum the slots in rank order into dst, publish the epoch
+cudaError_t launch_peer_combine(double* dst, int64_t count, const PeerArgs& pa, int num_sms, cudaStream_t s);
 
 }  // namespace kde

@@ -27,25 +27,12 @@
 
 #include "common.cuh"
 #include "kernels.cuh"
+#include "peer.cuh"
 
 namespace kde {
 
-__device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
-  uint64_t v;
-  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
-  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-__device__ __forceinline__ uint64_t globaltimer_ns() {
-  uint64_t t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
-
 __device__ __forceinline__ char* slot_ptr(char* win, int parity, int src, int world, size_t slot) {
-  return win + kPeerFlagBytes + ((size_t)parity * world + src) * slot;
+  return peer_slot(win, parity, src, world, slot);
 }
 
 __global__ void peer_push_kernel(const char* __restrict__ src, size_t bytes, PeerArgs pa) {
@@ -127,6 +114,53 @@ __global__ void peer_collect_kernel(char* __restrict__ dst, size_t bytes, size_t
     *pa.epoch = e;
     pa.count[1] = 0u;
   }
+}
+
+// fused exchange consumer: wait for every rank's epoch-e slot, rank-order sum into dst
+__global__ void peer_combine_kernel(double* __restrict__ dst, int64_t count, PeerArgs pa) {
+  __shared__ bool ok_s, last_s;
+  const uint64_t e = *pa.epoch + 1;
+  const int parity = (int)(e & 1);
+  char* mine = pa.base[pa.rank];
+  if (threadIdx.x == 0) {
+    bool ok = true;
+    const uint64_t t0 = globaltimer_ns();
+    for (int r = 0; r < pa.world && ok; ++r) {
+      const uint64_t* f = reinterpret_cast<const uint64_t*>(mine + (size_t)r * 128);
+      while (ld_acquire_sys(f) < e) {
+        if (globaltimer_ns() - t0 > pa.timeout_ns) {
+          ok = false;
+          atomicExch(pa.err, 1);
+          break;
+        }
+        __nanosleep(256);
+      }
+    }
+    ok_s = ok;
+  }
+  __syncthreads();
+  if (ok_s)
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x) {
+      double t = 0.0;
+      for (int r = 0; r < pa.world; ++r)
+        t += __ldcv(reinterpret_cast<const double*>(slot_ptr(mine, parity, r, pa.world, pa.slot)) + i);
+      dst[i] = t;
+    }
+  __syncthreads();
+  if (threadIdx.x == 0) last_s = atomicAdd(pa.count + 1, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (last_s && threadIdx.x == 0) {
+    *pa.epoch = e;
+    pa.count[1] = 0u;
+  }
+}
+
+cudaError_t launch_peer_combine(double* dst, int64_t count, const PeerArgs& pa, int num_sms, cudaStream_t s) {
+  int64_t grid = (count + 255) / 256;
+  if (grid > num_sms) grid = num_sms;
+  if (grid < 1) grid = 1;
+  peer_combine_kernel<<<(unsigned)grid, 256, 0, s>>>(dst, count, pa);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_peer_allgather(const void* src, void* dst, size_t bytes, size_t stride, const PeerArgs& pa,

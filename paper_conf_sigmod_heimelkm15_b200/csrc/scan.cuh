@@ -26,6 +26,7 @@
 #include <cuda_runtime.h>
 
 #include "common.cuh"
+#include "peer.cuh"
 #include "phi.cuh"
 
 namespace kde {
@@ -213,6 +214,9 @@ __device__ __forceinline__ void single_reduce_finalize(const ScanSingleArgs& a, 
   __syncthreads();
   if (!am_last) return;
   __threadfence();
+  // fused exchange (sharded model, peer transport): the final sums go straight into every rank's
+  // window slot of this epoch, then this rank's flag is released (peer.cuh)
+  const uint64_t pe = a.peer ? peer_next_epoch(*a.peer) : 0;
   // deterministic second pass over the block partials (fixed strided order + fixed tree)
   for (int k = 0; k < NA; ++k) {
     double t = 0.0;
@@ -226,13 +230,17 @@ __device__ __forceinline__ void single_reduce_finalize(const ScanSingleArgs& a, 
 #pragma unroll
       for (int w = 0; w < NT / 32; ++w) tot += red[w][0];
       a.sums_out[k] = tot;
+      if (a.peer) peer_store(*a.peer, pe, k, tot);
       const double fin = k == 0 ? tot / a.n_global : tot * a.consts->gconst[k - 1] / a.n_global;
       if (a.fin_out) a.fin_out[k] = fin;
       if (k == 0 && a.est_out) *a.est_out = fin;
       if (k > 0 && a.dpdh_out) a.dpdh_out[k - 1] = fin;
     }
   }
-  if (threadIdx.x == 0) *a.counter = 0u;
+  if (threadIdx.x == 0) {
+    if (a.peer) peer_release(*a.peer, pe);
+    *a.counter = 0u;
+  }
 }
 
 // ---------------------------------------------------------------- single box

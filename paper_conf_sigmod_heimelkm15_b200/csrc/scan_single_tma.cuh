@@ -16,6 +16,12 @@ namespace kde {
 
 constexpr int kSingleComputeWarps = kSingleThreads / 32;
 constexpr int kSingleTmaThreads = kSingleThreads + 32;  // + producer warp
+// compute warps of the culled variant (no producer warp); 16 at d = 9, 10 (one CTA per SM) measured
+// slower than 8 (c5s 80.9 vs 76.5 us, profiles/r02_experiments.md)
+#ifndef KDE_TUNE_CULL_WARPS
+#define KDE_TUNE_CULL_WARPS(d) 8
+#endif
+__host__ __device__ constexpr int cull_warps(int d) { return KDE_TUNE_CULL_WARPS(d); }
 
 template <int D, int TILE, int STAGES>
 constexpr size_t single_tma_smem_bytes() {
@@ -102,7 +108,7 @@ __device__ __forceinline__ void st_shared_if(uint32_t addr, float v, bool p) {
 
 template <int D>
 constexpr size_t cull_queue_bytes() {
-  return (size_t)kSingleComputeWarps * kCullRing * (D + 1) * sizeof(float);
+  return (size_t)cull_warps(D) * kCullRing * (D + 1) * sizeof(float);
 }
 
 // d >= 9 gradient scans keep their fp64 per-thread sums in shared memory (stride kSingleThreads)
@@ -118,7 +124,7 @@ __host__ __device__ constexpr bool acc_in_smem() {
 template <int D, int TILE, int STAGES, bool CULL, bool GRAD = false>
 constexpr size_t single_tma_kernel_smem() {
   return single_tma_smem_bytes<D, TILE, STAGES>() + (CULL ? cull_queue_bytes<D>() : 0) +
-         (acc_in_smem<D, GRAD, CULL>() ? (size_t)(D + 1) * kSingleThreads * sizeof(double) : 0);
+         (acc_in_smem<D, GRAD, CULL>() ? (size_t)(D + 1) * 32 * cull_warps(D) * sizeof(double) : 0);
 }
 
 template <int D, bool GRAD, int MODE, int TILE, int STAGES, typename Release>
@@ -126,8 +132,9 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
                                                       float* tiles, uint64_t* full, Release& release, float* queue,
                                                       int64_t c0, int64_t c1, int ntiles, double* acc, bool keep_all) {
   constexpr int NA = GRAD ? D + 1 : 1;
-  constexpr int AS = acc_in_smem<D, GRAD, true>() ? kSingleThreads : 1;  // stride of acc (shared memory or registers)
-  constexpr int PPT = TILE / kSingleThreads;  // points per thread per tile
+  constexpr int NT = 32 * cull_warps(D);
+  constexpr int AS = acc_in_smem<D, GRAD, true>() ? NT : 1;  // stride of acc (shared memory or registers)
+  constexpr int PPT = TILE / NT;  // points per thread per tile
   static_assert(PPT % 2 == 0, "points are classified in pairs");
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   float* qt = queue + (size_t)warp * kCullRing * (D + 1);  // [D][kCullRing] coordinates
@@ -210,7 +217,7 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
     const int npts = rem < TILE ? (int)rem : TILE;
 #pragma unroll 1
     for (int r = 0; r < PPT / 2; ++r) {
-      const int pp = tid + r * kSingleThreads;
+      const int pp = tid + r * NT;
       float2 t[D];
 #pragma unroll
       for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * TILE + 2 * pp);
@@ -257,15 +264,16 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
 // Culled variant: no producer warp -- the LAST compute warp to finish a tile's classification
 // issues that stage's next TMA copies (per-stage arrival counters), so all 8 warps compute and
 // the CTA's register budget allows two CTAs per SM at d >= 9.
-template <bool CULL>
+template <int D, bool CULL>
 __host__ __device__ constexpr int single_tma_threads() {
-  return CULL ? kSingleThreads : kSingleTmaThreads;
+  return CULL ? 32 * cull_warps(D) : kSingleTmaThreads;
 }
 
 template <int D, bool GRAD, int TILE, int STAGES, int OCC, bool CULL>
-__global__ void __launch_bounds__(single_tma_threads<CULL>(), OCC) scan_single_tma_kernel(const ScanSingleArgs a) {
+__global__ void __launch_bounds__(single_tma_threads<D, CULL>(), OCC) scan_single_tma_kernel(const ScanSingleArgs a) {
   constexpr int NA = GRAD ? D + 1 : 1;
-  constexpr int NT = single_tma_threads<CULL>();
+  constexpr int NT = single_tma_threads<D, CULL>();
+  constexpr int NW = CULL ? cull_warps(D) : kSingleComputeWarps;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   float* tiles = reinterpret_cast<float*>(smem_raw);
   uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + (size_t)STAGES * D * TILE * sizeof(float));
@@ -311,7 +319,7 @@ __global__ void __launch_bounds__(single_tma_threads<CULL>(), OCC) scan_single_t
     if ((tid & 31) == 0) {
       const int st = k % STAGES;
       __threadfence_block();
-      if (atomicAdd(&rcnt[st], 1) == kSingleComputeWarps - 1) {
+      if (atomicAdd(&rcnt[st], 1) == NW - 1) {
         rcnt[st] = 0;
         if (k + STAGES < ntiles) issue(k + STAGES);
       }
@@ -341,7 +349,7 @@ __global__ void __launch_bounds__(single_tma_threads<CULL>(), OCC) scan_single_t
                                             (CULL ? cull_queue_bytes<D>() : 0)) + tid;
   if (kAccSh && !producer)
 #pragma unroll
-    for (int k = 0; k < NA; ++k) accsh[k * kSingleThreads] = 0.0;
+    for (int k = 0; k < NA; ++k) accsh[k * NT] = 0.0;
   double* accp = (kAccSh && !producer) ? accsh : acc;
   if (producer) {
     if (tid == kSingleThreads) {
@@ -375,7 +383,7 @@ __global__ void __launch_bounds__(single_tma_threads<CULL>(), OCC) scan_single_t
   }
   if (kAccSh && !producer)
 #pragma unroll
-    for (int k = 0; k < NA; ++k) acc[k] = accsh[k * kSingleThreads];
+    for (int k = 0; k < NA; ++k) acc[k] = accsh[k * NT];
   single_reduce_finalize<NA, NT>(a, acc);
 }
 
@@ -394,7 +402,7 @@ cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStr
     if (e != cudaSuccess) return e;
     attr_set.fetch_or(bit, std::memory_order_acq_rel);
   }
-  scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC, CULL><<<grid, single_tma_threads<CULL>(), smem, s>>>(a);
+  scan_single_tma_kernel<D, GRAD, TILE, STAGES, OCC, CULL><<<grid, single_tma_threads<D, CULL>(), smem, s>>>(a);
   return cudaGetLastError();
 }
 

@@ -1,5 +1,6 @@
 """World > 1 on ONE GPU: 2 and 3 processes (one rank each) share cuda:0 and run the
-sharded model over the peer-memory exchange (KDE_COMM_PEER, peer.cu) -- the same
+sharded model over the peer-memory exchange (KDE_COMM_PEER, peer.cu; fused: the scan /
+reduce_splits tails push their sums into every rank's window, else a separate all-gather) -- the same
 consumers the NCCL path feeds: rank-order combine of the per-box sums
 (combine_ranks_kernel), Chan merge of the shard moments (moments_merge_ranks_kernel,
 Scott's rule over the global sample), the rank-ordered karma index gather, and
@@ -33,7 +34,7 @@ def _grad_ok(gpu, ora, scale, h, fscale=1.0):
     return bool(np.all(np.abs(np.asarray(gpu) - ora) <= 1e-4 * np.abs(ora) + 1e-4 * scale + floor))
 
 
-def _worker(rank, world, port, out):
+def _worker(rank, world, port, out, fused):
     import torch
     import torch.distributed as dist
 
@@ -44,6 +45,7 @@ def _worker(rank, world, port, out):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     os.environ.setdefault("KDE_PEER_TIMEOUT_S", "60")
+    os.environ["KDE_PEER_FUSED"] = "1" if fused else "0"  # producer-tail push vs separate all-gather
     torch.cuda.set_device(0)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     res = {}
@@ -119,8 +121,8 @@ def _worker(rank, world, port, out):
     out[rank] = res
 
 
-@pytest.mark.parametrize("world", [2, 3])
-def test_peer_exchange_multirank_on_one_gpu(world):
+@pytest.mark.parametrize("world,fused", [(2, True), (3, True), (2, False)])
+def test_peer_exchange_multirank_on_one_gpu(world, fused):
     import torch
     import torch.multiprocessing as mp
     if not torch.cuda.is_available():
@@ -129,7 +131,7 @@ def test_peer_exchange_multirank_on_one_gpu(world):
     ctx = mp.get_context("spawn")
     mgr = ctx.Manager()
     out = mgr.dict()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, out)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, out, fused)) for r in range(world)]
     for p in procs:
         p.start()
     for p in procs:
