@@ -142,7 +142,10 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
   // d >= 9: the box constants (5 d floats) are re-read from shared memory (broadcast) where they are
   // used instead of living in registers for the whole scan, which keeps wide gradient scans at two
   // CTAs per SM; narrower boxes keep them in registers.
-  constexpr bool kReload = D >= 9;
+#ifndef KDE_TUNE_RELOAD_MIND
+#define KDE_TUNE_RELOAD_MIND 9
+#endif
+  constexpr bool kReload = D >= KDE_TUNE_RELOAD_MIND;
   constexpr bool kRatio = D >= KDE_TUNE_RATIO_MIND;  // few-register gradient form (point_box2_ratio)
   BoxDim bd[D];
   float ap[D];
