@@ -675,8 +675,14 @@ __global__ void online_update_kernel(const double* __restrict__ ret, const doubl
 //            step: warp 0 forms the popcount prefix, all warps write);
 //   barrier  -> phase 3 (streaming step only): CTA 0 runs the Listing 1 step, all CTAs replace the
 //            first min(total, cap) flagged points by tail.rows.
-constexpr int kCoopThreads = 256;
-constexpr int kCoopPass = kCoopThreads * kKarmaKV;  // points per pass (32 bitmap words)
+#ifndef KDE_TUNE_COOP_THREADS
+#define KDE_TUNE_COOP_THREADS 256
+#endif
+#ifndef KDE_TUNE_COOP_MINB
+#define KDE_TUNE_COOP_MINB 4  // 64 registers, 4 CTAs per SM
+#endif
+constexpr int kCoopThreads = KDE_TUNE_COOP_THREADS;
+constexpr int kCoopPass = kCoopThreads * kKarmaKV;  // points per pass (kCoopThreads / 8 bitmap words)
 
 struct KarmaCoopArgs {
   const float* cvals;
@@ -699,7 +705,7 @@ struct KarmaCoopArgs {
   StreamTail tail;
 };
 
-__global__ void __launch_bounds__(kCoopThreads, KDE_TUNE_KARMA_MINB) karma_coop_kernel(const KarmaCoopArgs a) {
+__global__ void __launch_bounds__(kCoopThreads, KDE_TUNE_COOP_MINB) karma_coop_kernel(const KarmaCoopArgs a) {
   cg::grid_group grid = cg::this_grid();
   constexpr int W = 128;  // bitmap words per compaction step
   constexpr int WPL = W / 32;

@@ -867,10 +867,11 @@ template <int D, bool GRAD, int TILE, int STAGES, int OCC, bool CULL>
 cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStream_t s);
 
 // culled single-box scan (every d): TMA tiles + a per-warp ring of kept points.
-// Two stages; 2048-point tiles up to d = 8 (1024 above, shared-memory budget);
-// two CTAs per SM up to d = 5.
+// Two stages; 2048-point tiles up to d = 10 (8 KB bulk copies per column: 4 KB / 2 KB copies
+// measured 0.43 / 0.39 of HBM at d = 10 against 0.47, profiles/r02_experiments.md), 1024 / 512
+// above (shared-memory budget); two CTAs per SM up to d = 5.
 #ifndef KDE_TUNE_CULL_TILE
-#define KDE_TUNE_CULL_TILE(d) ((d) <= 8 ? 2048 : ((d) <= 12 ? 1024 : 512))
+#define KDE_TUNE_CULL_TILE(d) ((d) <= 10 ? 2048 : ((d) <= 12 ? 1024 : 512))
 #endif
 #ifndef KDE_TUNE_CULL_STAGES
 #define KDE_TUNE_CULL_STAGES(d) 2

@@ -114,7 +114,7 @@ constexpr size_t cull_queue_bytes() {
 // d >= 9 gradient scans keep their fp64 per-thread sums in shared memory (stride kSingleThreads)
 // instead of registers, so two CTAs fit per SM (register budget 96/thread at 288 x 2 threads)
 #ifndef KDE_TUNE_RATIO_MIND
-#define KDE_TUNE_RATIO_MIND 9  // from this d on, the culled gradient scan uses point_box2_ratio + smem sums
+#define KDE_TUNE_RATIO_MIND 17  // from this d on: point_box2_ratio + smem sums (off: measured no gain at one CTA per SM)
 #endif
 template <int D, bool GRAD, bool CULL>
 __host__ __device__ constexpr bool acc_in_smem() {
@@ -143,7 +143,7 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
   // used instead of living in registers for the whole scan, which keeps wide gradient scans at two
   // CTAs per SM; narrower boxes keep them in registers.
 #ifndef KDE_TUNE_RELOAD_MIND
-#define KDE_TUNE_RELOAD_MIND 9
+#define KDE_TUNE_RELOAD_MIND 13  // from this d on: box constants re-read from shared memory (register budget)
 #endif
   constexpr bool kReload = D >= KDE_TUNE_RELOAD_MIND;
   constexpr bool kRatio = D >= KDE_TUNE_RATIO_MIND;  // few-register gradient form (point_box2_ratio)
