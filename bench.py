@@ -319,7 +319,7 @@ def timed_steps(step, steps, warmup, stream, m, K, flush=None, barrier=None, clo
     frac = steps / max(steps + soak, 1)  # the soak launched the same kernels: keep the timed steps' share
     step_ms = [a.elapsed_time(b) for a, b in evs]
     return dict(step_ms=step_ms, scan_ms=scan_ms * frac, scan_launches=int(round(scan_launches * frac)),
-                launches=int(round(launches * frac)), clocks=clk.summary(), soak=soak)
+                launches=int(round(launches * frac)), clocks=clk.summary(), soak=soak, events=evs)
 
 
 def max_over_ranks(x, world, dev):
@@ -518,7 +518,11 @@ def run_cuda(args, cfg, rank, world, local_rank):
 
 
 def run_stream(args, cfg, dev):
-    """configs[4]: reservoir inserts + device-resident streaming queries (single GPU)."""
+    """configs[4]: reservoir inserts + deletes + device-resident streaming queries (single GPU).
+    Database: clusters of 2^22 rows; cycle c inserts cluster c + 3 in 2^16-row chunks (64 chunks)
+    through the reservoir, then deletes cluster c.  The timed steps cross the end of cycle 0: the
+    first PRE chunks of cluster 3 are inserted untimed, so the timed region sees the last chunks of
+    cycle 0, the deletion of cluster 0 and the first chunks of cluster 4."""
     import torch
 
     import paper_conf_sigmod_heimelkm15_b200 as K
@@ -526,12 +530,19 @@ def run_stream(args, cfg, dev):
     d, N = cfg["d"], cfg["n"]
     rows = 1 << 22            # rows per database cluster
     chunk = 1 << 16           # arrivals per insert chunk
+    per_cycle = rows // chunk
     qpc = cfg["q"]            # queries per chunk
     cap = 1 << 16
     res_seed = 0xC5
+    P = args.warmup + args.steps
+    PRE = max(0, per_cycle - 4)  # untimed prefill: the timed steps cross the cycle boundary
     sc = synth.StreamClusters(d, rows, seed=11)
-    # initial database R0 = clusters 0, 1, 2; the sample is the reservoir after its 3 x 2^22 arrivals
-    base = np.concatenate([sc.cluster_rows(c) for c in range(3)])
+    cl = {c: sc.cluster_rows(c) for c in range(4)}   # R0 = clusters 0..2; cluster 3 = cycle 0's inserts
+    n_c4 = max(0, PRE + P - per_cycle) * chunk
+    if n_c4:
+        cl[4] = sc.cluster_rows(4, 0, min(rows, n_c4))
+    # the sample: the reservoir after R0's 3 x 2^22 arrivals
+    base = np.concatenate([cl[0], cl[1], cl[2]])
     n0 = len(base)
     sl = K.kde_reservoir_select(res_seed, N, N, n0 - N)
     content = np.arange(N)
@@ -541,33 +552,52 @@ def run_stream(args, cfg, dev):
     u, first = np.unique(rev_s, return_index=True)  # the last arrival per slot wins
     content[u] = rev_i[first]
     S = base[content]
+    del base
     m = K.KDEModel.create(S)
     m.set_retain(True)
     m.cull = not args.no_cull
-    # insert cycle 1: cluster 3 arrives in chunks; queries over the live clusters, newer ones more often
-    P = args.warmup + args.steps
-    new_rows = sc.cluster_rows(3, 0, min(rows, P * chunk))
-    live = [0, 1, 2, 3]
-    Qlo, Qhi = sc.queries(live, P * qpc, seed=13)
-    stream = torch.cuda.Stream(device=dev)
-    # true selectivities over the database at each chunk: the 3 base clusters + the inserted part of cluster 3
-    dbase = torch.from_numpy(base).to(dev)
+    state = {"n_seen": n0, "written": []}
+
+    def chunk_rows(t):  # arrivals of global chunk t
+        c = 3 + t // per_cycle
+        a = (t % per_cycle) * chunk
+        return cl[c][a:a + chunk]
+
+    for t in range(PRE):  # untimed prefill of cycle 0
+        state["n_seen"], _ = m.insert_rows(chunk_rows(t), res_seed, state["n_seen"])
+
+    def live_after(t):  # (full clusters, partial cluster, inserted rows of it) after chunk t's insert
+        c = t // per_cycle
+        return [c, c + 1, c + 2], c + 3, (t % per_cycle + 1) * chunk
+
+    ts = [PRE + i for i in range(P)]
+    Qlo = np.empty((P * qpc, d), np.float32)
+    Qhi = np.empty((P * qpc, d), np.float32)
     p = np.empty(P * qpc)
-    for t in range(P):
-        sel = slice(t * qpc, (t + 1) * qpc)
-        dlo_t, dhi_t = torch.from_numpy(Qlo[sel]).to(dev), torch.from_numpy(Qhi[sel]).to(dev)
-        c0 = torch.zeros(qpc, dtype=torch.int64, device=dev)
-        K.kde_count_in_box_dev(dbase, dlo_t, dhi_t, c0)
-        ins = min(rows, (t + 1) * chunk)
-        c1 = torch.zeros(qpc, dtype=torch.int64, device=dev)
-        K.kde_count_in_box_dev(torch.from_numpy(new_rows[:ins]).to(dev), dlo_t, dhi_t, c1)
+    dcl = {}
+    for i, t in enumerate(ts):
+        full, part, ins = live_after(t)
+        lo_t, hi_t = sc.queries(full + [part], qpc, seed=1000 + t)
+        Qlo[i * qpc:(i + 1) * qpc], Qhi[i * qpc:(i + 1) * qpc] = lo_t, hi_t
+        dlo_t, dhi_t = torch.from_numpy(lo_t).to(dev), torch.from_numpy(hi_t).to(dev)
+        tot = torch.zeros(qpc, dtype=torch.int64, device=dev)
+        for c in full + [part]:
+            if c not in dcl:
+                dcl[c] = torch.from_numpy(cl[c]).to(dev)
+            rows_c = dcl[c] if c != part else dcl[c][:ins]
+            cnt = torch.zeros(qpc, dtype=torch.int64, device=dev)
+            K.kde_count_in_box_dev(rows_c, dlo_t, dhi_t, cnt)
+            tot += cnt
         torch.cuda.synchronize()
-        p[sel] = ((c0 + c1).double() / (n0 + ins)).cpu().numpy()
-    del dbase
-    # replacement pool: rows of the current database
-    pool = np.concatenate([base[synth.rng(14).integers(0, n0, size=1 << 17)], new_rows[:chunk]])
+        p[i * qpc:(i + 1) * qpc] = (tot.double() / (len(full) * rows + ins)).cpu().numpy()
+    del dcl
+    # karma replacement pool: rows of the live database at the cycle boundary
+    g = synth.rng(14)
+    pool = np.concatenate([cl[c][g.integers(0, rows, size=1 << 15)] for c in (1, 2, 3)] +
+                          [chunk_rows(ts[-1])[: 1 << 15]])
     d_pool = torch.from_numpy(pool).to(dev)
     npool = len(pool) - cap
+    stream = torch.cuda.Stream(device=dev)
     d_lo, d_hi = torch.from_numpy(Qlo).to(dev), torch.from_numpy(Qhi).to(dev)
     d_true = torch.from_numpy(p).to(dev)
     kp = K.karma_params(loss=K.LOSS_ABSOLUTE, threshold=-1.0 / (N - 1), k_max=4.0)
@@ -576,14 +606,13 @@ def run_stream(args, cfg, dev):
     d_cnt = torch.zeros(1, dtype=torch.int64, device=dev)
     d_est = torch.zeros(1, dtype=torch.float64, device=dev)
     d_dpdh = torch.zeros(d, dtype=torch.float64, device=dev)
-    state = {"n_seen": n0, "written": []}
 
     def query(qi):
         off = (qi * 977) % npool
         K.kde_stream_step_dev(m.handle, d_lo[qi:qi + 1], d_hi[qi:qi + 1], d_true[qi:qi + 1], kp, op, d_idx, d_cnt,
                               d_pool[off:off + cap], d_est, d_dpdh, stream=stream)
 
-    # the chunk's 16 queries: one CUDA graph per chunk (launch-bound multi-kernel steps)
+    # launch statistics of one query step (libkde's counters), then one CUDA graph per chunk
     K.kde_set_profiling(m.handle, True)
     with torch.cuda.stream(stream):
         for qi in range(min(P * qpc, 64)):
@@ -594,32 +623,43 @@ def run_stream(args, cfg, dev):
     K.kde_set_profiling(m.handle, False)
     graphs = []
     if not args.no_graph:
-        for t in range(P):
-            g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g, stream=stream):
-                for qi in range(t * qpc, (t + 1) * qpc):
+        for i in range(P):
+            gr = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(gr, stream=stream):
+                for qi in range(i * qpc, (i + 1) * qpc):
                     query(qi)
-            graphs.append(g)
+            graphs.append(gr)
         with torch.cuda.stream(stream):
-            for g in graphs:
-                g.replay()
+            for gr in graphs:
+                gr.replay()
         torch.cuda.synchronize()
 
+    split_ev = []
+
     def step(i):
-        t = i % P
-        rows_t = new_rows[t * chunk:(t + 1) * chunk]
-        n_seen, nw = m.insert_rows(rows_t, res_seed, state["n_seen"])  # host decision, accepted rows only
+        i = i % P
+        # host reservoir decision, only accepted rows cross PCIe; the deletion of a cluster
+        # at a cycle boundary changes only the database (true selectivities), not the sample
+        t_ins = time.perf_counter()
+        n_seen, nw = m.insert_rows(chunk_rows(ts[i]), res_seed, state["n_seen"])
         state["n_seen"] = n_seen
         state["written"].append(nw)
+        ev = torch.cuda.Event(enable_timing=True)
+        ev.record(stream)  # the queries' share of the step starts here
+        split_ev.append((time.perf_counter() - t_ins, ev))
         if graphs:
-            graphs[t].replay()
+            graphs[i].replay()
         else:
-            for qi in range(t * qpc, (t + 1) * qpc):
+            for qi in range(i * qpc, (i + 1) * qpc):
                 query(qi)
 
     T = timed_steps(step, args.steps, args.warmup, stream, m, K, None, None, 0)
     ms_per_step = sum(T["step_ms"]) / args.steps
     value = N * qpc / (ms_per_step * 1e-3)
+    # breakdown of the timed steps: host insert call (wall) and the queries' device time
+    timed = split_ev[args.warmup:args.warmup + args.steps]
+    ins_ms = 1e3 * float(np.mean([w for w, _ in timed]))
+    q_ms = float(np.mean([ev.elapsed_time(T["events"][k][1]) for k, (_, ev) in enumerate(timed)]))
     launches = T["launches"] + int(round(prof_pre[2] / n_pre * qpc * args.steps)) if graphs else T["launches"]
     avg_scan_ms = prof_pre[0] / max(prof_pre[1], 1)
     written = float(np.mean(state["written"])) if state["written"] else 0.0
@@ -630,10 +670,9 @@ def run_stream(args, cfg, dev):
     torch.cuda.synchronize()
     t0 = time.perf_counter()
     for i in range(e2e_steps):
-        t = i % P
-        ns, _ = m.insert_rows(new_rows[t * chunk:(t + 1) * chunk], res_seed, state["n_seen"])
+        ns, _ = m.insert_rows(chunk_rows(ts[i % P]), res_seed, state["n_seen"])
         state["n_seen"] = ns
-        for qi in range(t * qpc, (t + 1) * qpc):
+        for qi in range((i % P) * qpc, (i % P + 1) * qpc):
             m.estimate(Qlo[qi:qi + 1], Qhi[qi:qi + 1], grad=True)
             idx, nf, _ = m.karma_update(Qlo[qi], Qhi[qi], p[qi], kp, cap=cap)
             m.online_update(Qlo[qi], Qhi[qi], p[qi], op)
@@ -658,14 +697,18 @@ def run_stream(args, cfg, dev):
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": cfg["desc"], "d": d, "n_per_gpu": N, "n_global": N, "q": qpc,
-                   "insert_chunk": chunk, "database_rows": n0 + P * chunk, "cuda_graph": bool(graphs),
-                   "l2": "sample larger than L2",
+                   "insert_chunk": chunk, "chunks_per_cycle": per_cycle,
+                   "timed_chunks": f"global chunks {ts[0]}..{ts[-1]} (cycle boundary, delete of cluster 0, "
+                                   f"after chunk {per_cycle - 1})",
+                   "cuda_graph": bool(graphs), "l2": "sample larger than L2",
                    "cull": "off" if args.no_cull else "on (DESIGN R15)",
                    "clock_sampling": "nvidia-smi every 100 ms over the timed steps"
                                      + (f" + {T['soak']} identical untimed soak steps" if T["soak"] else "")},
         "estimates_per_s": qpc / (ms_per_step * 1e-3),
         "stream": {"queries_per_s": qpc * 1e3 / ms_per_step, "inserts_per_s": chunk * 1e3 / ms_per_step,
-                   "rows_written_per_chunk": written, "mean_flagged_per_query_e2e": mean_flag},
+                   "rows_written_per_chunk": written, "mean_flagged_per_query_e2e": mean_flag,
+                   "insert_call_ms": ins_ms, "queries_device_ms": q_ms,
+                   "us_per_query_device": 1e3 * q_ms / qpc},
         "e2e": {"value": N * qpc * e2e_steps / e2e_s, "unit": "point·query evals/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": e2e_steps,
                 "queries_per_s": qpc * e2e_steps / e2e_s},

@@ -679,7 +679,7 @@ __global__ void online_update_kernel(const double* __restrict__ ret, const doubl
 #define KDE_TUNE_COOP_THREADS 256
 #endif
 #ifndef KDE_TUNE_COOP_MINB
-#define KDE_TUNE_COOP_MINB 4  // 64 registers, 4 CTAs per SM
+#define KDE_TUNE_COOP_MINB 2  // 128 registers, 2 CTAs per SM (room for PB = 4)
 #endif
 constexpr int kCoopThreads = KDE_TUNE_COOP_THREADS;
 constexpr int kCoopPass = kCoopThreads * kKarmaKV;  // points per pass (kCoopThreads / 8 bitmap words)
@@ -731,7 +731,7 @@ __global__ void __launch_bounds__(kCoopThreads, KDE_TUNE_COOP_MINB) karma_coop_k
   // ---------------- phase 1: karma + flags
   int32_t my = 0;
 #ifndef KDE_TUNE_COOP_PB
-#define KDE_TUNE_COOP_PB 2
+#define KDE_TUNE_COOP_PB 4  // 4 passes of loads in flight (ncu: 25.3 vs 27.6 us at 2^22 with 2, profiles/r02_experiments.md)
 #endif
   constexpr int PB = KDE_TUNE_COOP_PB;  // passes whose loads are in flight together
 #pragma unroll 1

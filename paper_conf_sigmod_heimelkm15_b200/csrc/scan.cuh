@@ -513,6 +513,9 @@ __device__ __forceinline__ void batched_tile_compute(const float* tl, int npts, 
 // time (the warp iterates max over its lanes -- boxes are sorted by their kept
 // fraction within the CTA, see the kernel) with lane-varying LDS gathers from the tile.
 constexpr int kTileWords = kTilePts / 32;
+#ifndef KDE_TUNE_BATCHED_LINF
+#define KDE_TUNE_BATCHED_LINF 0
+#endif
 
 // phase / R: with R threads per box (small batches) the thread owns the words w = phase (mod R)
 template <int D, bool EPAN>
@@ -531,7 +534,12 @@ __device__ __forceinline__ void cull_tile_mask(const float* tl, int npts, const 
 #pragma unroll
       for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * kTilePts + 2 * pp);
       // kept <=> score - limit < 0: the sign bits are the mask bits (finite scores, exact sign)
-      const float2 u = __fadd2_rn(cull_score<D, EPAN>(t, ap, cb), f2(-cull_limit<EPAN>()));
+      // KDE_TUNE_BATCHED_LINF: Gaussian classification by max_j o_j >= sqrt(64.5) (sound: it implies
+      // sum_j o_j^2 >= 64.5) -- 2 FMA-pipe + 1 ALU op per pair-dimension instead of 4 FMA-pipe ops,
+      // at the price of evaluating points the L2 test would cull (A/B experiment)
+      constexpr bool kMax = EPAN || KDE_TUNE_BATCHED_LINF;
+      const float lim = EPAN ? cull_limit<true>() : (KDE_TUNE_BATCHED_LINF ? 8.0311892f : cull_limit<false>());
+      const float2 u = __fadd2_rn(cull_score<D, kMax>(t, ap, cb), f2(-lim));
       m |= (__float_as_uint(u.x) >> 31) << (2 * q);
       m |= (__float_as_uint(u.y) >> 31) << (2 * q + 1);
     }

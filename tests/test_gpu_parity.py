@@ -436,7 +436,7 @@ def test_c3_full_size_single_and_batched_sampled():
     h = m.bandwidth
     lo, hi = synth.mixed_workload(S, 4096, seed=28)
     est, g = m.estimate(lo, hi, grad=True)
-    pick = np.array([0, 1, 1000, 4095])
+    pick = np.unique(np.concatenate([[0, 1, 1000, 4095], np.linspace(0, 4095, 60).astype(int)]))  # 64 boxes
     est_o, g_o = oracle.estimate_grad(S, h, lo[pick], hi[pick])
     mabs = oracle.grad_abs_scale(S, h, lo[pick], hi[pick])
     sel_ok(est[pick], est_o)
@@ -449,7 +449,7 @@ def test_c3_full_size_single_and_batched_sampled():
 
 def test_c2_full_size_loss_grad_sampled():
     """configs[1]: d=3, N=2^20, 10k boxes: loss/grad consistent with the per-box
-    estimates; a 64-box subset matches the oracle's loss and gradient."""
+    estimates; a 512-box subset matches the oracle's estimates, loss and gradient."""
     n, d = 1 << 20, 3
     S = synth.make_data("gauss", n, d, seed=29)
     lo, hi = synth.mixed_workload(S, 10000, seed=30)
@@ -458,13 +458,30 @@ def test_c2_full_size_loss_grad_sampled():
     h = m.bandwidth
     L, g, est = m.loss_and_grad(lo, hi, p, K.LOSS_SQUARED, 0.0, False, return_est=True)
     assert abs(L - np.mean((est - p) ** 2)) <= 1e-12 * max(L, 1e-30) + 1e-18
-    sub = np.arange(0, 10000, 157)[:64]
+    sub = np.linspace(0, 9999, 512).astype(int)
     L_o, g_o, est_o = oracle.loss_and_grad(S, h, lo[sub], hi[sub], p[sub], 0, 0.0, False)
     sel_ok(est[sub], est_o)
     Ls, gs = m.loss_and_grad(lo[sub], hi[sub], p[sub], K.LOSS_SQUARED, 0.0, False)
     dL = 2 * np.abs(est_o - p[sub])
     mabs = oracle.grad_abs_scale(S, h, lo[sub], hi[sub])
     grad_ok(gs, g_o, (dL[:, None] * mabs).mean(axis=0), h, np.mean(dL))
+
+
+def test_c4_shard_size_batched_sampled():
+    """configs[3] per-GPU shard: d = 8, 2^25 rows (one of eight 2^28-row shards), a 4096-box batch
+    (estimate + gradient, the culled batched scan at d = 8) sampled against the oracle."""
+    n, d = 1 << 25, 8
+    S = synth.gaussian_clusters_rows(1 << 28, d, 7, 0, n)
+    m = model(S)
+    h = m.bandwidth
+    lo, hi = synth.mixed_workload(S[: 1 << 20], 4096, seed=33)
+    est, g = m.estimate(lo, hi, grad=True)
+    pick = np.linspace(0, 4095, 8).astype(int)
+    est_o, g_o = oracle.estimate_grad(S, h, lo[pick], hi[pick])
+    mabs = oracle.grad_abs_scale(S, h, lo[pick], hi[pick])
+    sel_ok(est[pick], est_o)
+    grad_ok(g[pick], g_o, mabs, h)
+    assert np.all(est >= 0) and np.all(est <= 1.0 + 1e-12)
 
 
 # ------------------------------------------------------------------ device-resident streaming step
