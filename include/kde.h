@@ -23,6 +23,11 @@
  *    stream (cudaStream_t passed as void*, NULL = the model's own stream);
  *    they only enqueue work: results are valid once that stream reaches the
  *    end of the enqueued work.  Device buffers must stay alive until then.
+ *    Every call that uses the model's own stream (all host-pointer calls,
+ *    getters, setters) is ordered after the work of the _dev calls issued
+ *    before it (an event recorded at the end of each _dev call, also inside
+ *    CUDA-graph capture); ordering between _dev calls on DIFFERENT caller
+ *    streams is the caller's job.
  *  - Box queries are hyper-rectangles Omega = (l_1,u_1) x ... x (l_d,u_d)
  *    over real-valued attributes, passed as row-major fp32 arrays
  *    lo[q][d], hi[q][d].  lo <= hi is required (lo == hi gives 0);

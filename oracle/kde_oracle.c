@@ -91,8 +91,7 @@ typedef struct { double s, c; } nsum_t;
 static void nsum_add(nsum_t *a, double x)
 {
     double t = a->s + x;
-    if (fabs(a->s) >= fabs(x)) a->c += (a->s - t) + x;
-    else                       a->c += (x - t) + a->s;
+    a->c += fabs(a->s) >= fabs(x) ? (a->s - t) + x : (x - t) + a->s;
     a->s = t;
 }
 
@@ -138,17 +137,17 @@ static void point_terms(const float *t, int32_t d, const double *h, const float 
     }
 }
 
-/* Driver shared by eq. (2) and eq. (17): sums[qq][0..d] = index-order Neumaier
- * sums of the per-point terms.  Many small queries run one query per thread;
- * a large sample is cut into fixed point chunks whose terms are computed by
- * all threads and then added sequentially in index order, so every result is
- * identical for any thread count. */
-#define OR_CHUNK 65536
+/* Driver shared by eq. (2) and eq. (17): sums[qq][0..d] = Neumaier-compensated sums of the
+ * per-point terms.  Many small queries run one query per thread, each summed in index order.  A
+ * large sample is cut into fixed 8192-point chunks ("OpenMP over (query, fixed
+ * sample chunk), partials combined in chunk order"): every chunk is summed in index order, the
+ * chunk partials are then added in chunk order -- the result does not depend on the thread count. */
+#define OR_CHUNK 8192
 static void scan_queries(const float *sample, int64_t n, int32_t d, const double *h,
                          const float *lo, const float *hi, int64_t q, int mode, double *sums)
 {
     const int32_t na = 1 + d;
-    if (n < OR_CHUNK) {
+    if (n < 4 * OR_CHUNK) {
         #pragma omp parallel for schedule(dynamic, 1)
         for (int64_t qq = 0; qq < q; ++qq) {
             nsum_t acc[65];
@@ -162,21 +161,36 @@ static void scan_queries(const float *sample, int64_t n, int32_t d, const double
         }
         return;
     }
-    double *buf = (double *)malloc(sizeof(double) * (size_t)OR_CHUNK * (size_t)na);
-    for (int64_t qq = 0; qq < q; ++qq) {
-        nsum_t acc[65];
-        for (int32_t k = 0; k < na; ++k) acc[k].s = acc[k].c = 0.0;
-        for (int64_t c0 = 0; c0 < n; c0 += OR_CHUNK) {
-            const int64_t m = n - c0 < OR_CHUNK ? n - c0 : OR_CHUNK;
-            #pragma omp parallel for schedule(static)
-            for (int64_t i = 0; i < m; ++i)
-                point_terms(sample + (c0 + i) * d, d, h, lo + qq * d, hi + qq * d, mode, buf + i * na);
-            for (int64_t i = 0; i < m; ++i)
-                for (int32_t k = 0; k < na; ++k) nsum_add(&acc[k], buf[i * na + k]);
+    const int64_t nch = (n + OR_CHUNK - 1) / OR_CHUNK;
+    const int64_t QB = 64;  /* queries per block of (query, chunk) work items */
+    nsum_t *part = (nsum_t *)malloc(sizeof(nsum_t) * (size_t)QB * (size_t)nch * (size_t)na);
+    for (int64_t q0 = 0; q0 < q; q0 += QB) {
+        const int64_t qn = q - q0 < QB ? q - q0 : QB;
+        #pragma omp parallel for collapse(2) schedule(dynamic, 1)
+        for (int64_t qq = 0; qq < qn; ++qq)
+            for (int64_t c = 0; c < nch; ++c) {
+                nsum_t acc[65];
+                double term[65];
+                for (int32_t k = 0; k < na; ++k) acc[k].s = acc[k].c = 0.0;
+                const int64_t i1 = (c + 1) * OR_CHUNK < n ? (c + 1) * OR_CHUNK : n;
+                for (int64_t i = c * OR_CHUNK; i < i1; ++i) {
+                    point_terms(sample + i * d, d, h, lo + (q0 + qq) * d, hi + (q0 + qq) * d, mode, term);
+                    for (int32_t k = 0; k < na; ++k) nsum_add(&acc[k], term[k]);
+                }
+                for (int32_t k = 0; k < na; ++k) part[(qq * nch + c) * na + k] = acc[k];
+            }
+        for (int64_t qq = 0; qq < qn; ++qq) {
+            nsum_t tot[65];
+            for (int32_t k = 0; k < na; ++k) tot[k].s = tot[k].c = 0.0;
+            for (int64_t c = 0; c < nch; ++c)
+                for (int32_t k = 0; k < na; ++k) {
+                    nsum_add(&tot[k], part[(qq * nch + c) * na + k].s);
+                    nsum_add(&tot[k], part[(qq * nch + c) * na + k].c);
+                }
+            for (int32_t k = 0; k < na; ++k) sums[(q0 + qq) * na + k] = nsum_get(&tot[k]);
         }
-        for (int32_t k = 0; k < na; ++k) sums[qq * na + k] = nsum_get(&acc[k]);
     }
-    free(buf);
+    free(part);
 }
 
 /* ---------------------------------------------------------------------

@@ -92,6 +92,8 @@ struct kde_model {
   void* rbuf = nullptr;              // replacement staging (idx + rows), grow-only
   size_t rbuf_cap = 0;
   std::vector<int32_t> ins_last;     // kde_insert_rows: last arrival of a chunk per local slot (-1 = none)
+  cudaEvent_t dev_done = nullptr;    // recorded on the caller's stream at the end of every _dev call
+  bool dev_pending = false;          // some _dev call enqueued work on a stream other than m->stream
   void* kbuf = nullptr;              // sharded karma gather: counts + index lists, grow-only
   size_t kbuf_cap = 0;
 
@@ -169,6 +171,32 @@ struct DeviceGuard {
     if (prev >= 0) cudaSetDevice(prev);
   }
 };
+
+// Ordering between the two call styles.  _dev calls enqueue on the caller's stream; host-pointer
+// calls run on the model's stream and are synchronous.  Every _dev call records dev_done on its
+// stream (an external event node when the stream is being captured into a CUDA graph); every call
+// that works on the model's stream first waits for it, so e.g. kde_insert_rows after a replayed
+// streaming step never overlaps that step's scan / karma / replacement.
+static kde_status mark_dev(kde_model* m, cudaStream_t s) {
+  if (s == m->stream) return KDE_OK;
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  CU(cudaStreamIsCapturing(s, &cs));
+  if (cs == cudaStreamCaptureStatusActive)
+    CU(cudaEventRecordWithFlags(m->dev_done, s, cudaEventRecordExternal));
+  else
+    CU(cudaEventRecord(m->dev_done, s));
+  m->dev_pending = true;
+  return KDE_OK;
+}
+static kde_status wait_dev(kde_model* m) {
+  if (m->dev_pending) CU(cudaStreamWaitEvent(m->stream, m->dev_done, 0));
+  return KDE_OK;
+}
+#define WAIT_DEV(m)                        \
+  do {                                     \
+    kde_status wst_ = wait_dev(m);         \
+    if (wst_ != KDE_OK) return wst_;       \
+  } while (0)
 
 static bool h_ok(double h) { return std::isfinite(h) && h >= 1e-30 && h <= 1e30; }
 
@@ -452,6 +480,7 @@ static void free_model(kde_model* m) {
     cudaFree(m->pa_dev);
   }
   cudaFree(m->kbuf);
+  if (m->dev_done) cudaEventDestroy(m->dev_done);
   if (m->stream) cudaStreamDestroy(m->stream);
   delete m;
 }
@@ -541,6 +570,7 @@ static kde_status create_impl(const float* rows, int64_t n_local, int64_t row_of
                        cudaGetErrorString(e_)));                                                    \
   } while (0)
   CUB(cudaStreamCreateWithFlags(&m->stream, cudaStreamNonBlocking));
+  CUB(cudaEventCreateWithFlags(&m->dev_done, cudaEventDisableTiming));
   CUB(cudaMalloc(&m->cols, sizeof(float) * (size_t)d * m->ld));
   CUB(cudaMalloc(&m->karma, sizeof(double) * (size_t)m->ld));  // padded: 128-bit karma loads
   CUB(cudaMalloc(&m->cret, sizeof(float) * (size_t)m->ld));
@@ -725,6 +755,7 @@ extern "C" kde_status kde_get_bandwidth(kde_model* m, double* h) {
   CHECK_MODEL(m);
   if (!h) return fail(KDE_EINVAL, "h is NULL");
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   DevConsts c;
   CU(cudaMemcpyAsync(&c, m->consts, sizeof(DevConsts), cudaMemcpyDeviceToHost, m->stream));
   CU(cudaStreamSynchronize(m->stream));
@@ -738,6 +769,7 @@ extern "C" kde_status kde_set_bandwidth(kde_model* m, const double* h) {
   for (int j = 0; j < m->d; ++j)
     if (!h_ok(h[j])) return fail(KDE_EINVAL, "h[%d] = %g not finite in [1e-30, 1e30]", j, h[j]);
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   CUL(launch_set_consts(h, m->d, m->consts, m->stream));
   CU(cudaStreamSynchronize(m->stream));
   ++m->gen;
@@ -749,6 +781,7 @@ extern "C" kde_status kde_set_kernel(kde_model* m, int32_t kernel) {
   if (kernel != KDE_KERNEL_GAUSSIAN && kernel != KDE_KERNEL_EPANECHNIKOV)
     return fail(KDE_EINVAL, "unknown kernel %d", kernel);
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   CUL(launch_set_kernel_type(kernel, m->d, m->consts, m->stream));
   CU(cudaStreamSynchronize(m->stream));
   m->kernel = kernel;
@@ -783,6 +816,7 @@ extern "C" kde_status kde_get_cull(const kde_model* m, int32_t* on) {
 extern "C" kde_status kde_synchronize(kde_model* m) {
   CHECK_MODEL(m);
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   CU(cudaStreamSynchronize(m->stream));
   return KDE_OK;
 }
@@ -819,6 +853,7 @@ extern "C" kde_status kde_estimate_batch(kde_model* m, const float* lo, const fl
   if (q > 0 && !est) return fail(KDE_EINVAL, "est is NULL");
   if (q == 0) return KDE_OK;
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   st = stage_bounds(m, lo, hi, q);
   if (st != KDE_OK) return st;
   const float* d_lo = m->qbuf;
@@ -853,7 +888,9 @@ extern "C" kde_status kde_estimate_batch_dev(kde_model* m, const float* d_lo, co
   DeviceGuard g(m->device);
   cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
   m->ret_valid = false;  // bounds are device-side; no retained-state bookkeeping
-  return estimate_dev(m, d_lo, d_hi, q, d_est, d_dest_dh, s, m->retain && q == 1);
+  kde_status rst = estimate_dev(m, d_lo, d_hi, q, d_est, d_dest_dh, s, m->retain && q == 1);
+  if (rst != KDE_OK) return rst;
+  return mark_dev(m, s);
 }
 
 static kde_status loss_grad_dev_impl(kde_model* m, const float* d_lo, const float* d_hi, const double* d_true,
@@ -886,6 +923,7 @@ extern "C" kde_status kde_loss_and_grad(kde_model* m, const float* lo, const flo
   for (int64_t k = 0; k < q; ++k)
     if (!(true_sel[k] >= 0.0 && true_sel[k] <= 1.0)) return fail(KDE_EINVAL, "true_sel[%lld] outside [0, 1]", (long long)k);
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   st = stage_bounds(m, lo, hi, q);
   if (st != KDE_OK) return st;
   CU(cudaMemcpyAsync(o_true(m), true_sel, sizeof(double) * q, cudaMemcpyHostToDevice, m->stream));
@@ -912,7 +950,9 @@ extern "C" kde_status kde_loss_and_grad_dev(kde_model* m, const float* d_lo, con
   DeviceGuard g(m->device);
   cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
   m->ret_valid = false;
-  return loss_grad_dev_impl(m, d_lo, d_hi, d_true_sel, q, loss, lambda, log_bandwidth, d_loss, d_grad, d_est, s);
+  kde_status rst = loss_grad_dev_impl(m, d_lo, d_hi, d_true_sel, q, loss, lambda, log_bandwidth, d_loss, d_grad, d_est, s);
+  if (rst != KDE_OK) return rst;
+  return mark_dev(m, s);
 }
 
 // ------------------------------------------------------------------ feedback parameter checks
@@ -995,6 +1035,7 @@ extern "C" kde_status kde_karma_update(kde_model* m, const float* lo, const floa
   if (st != KDE_OK) return st;
   if (std::isnan(kp->k_max) || std::isnan(kp->threshold)) return fail(KDE_EINVAL, "NaN k_max / threshold");
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   st = ensure_retained(m, lo, hi, true, false);
   if (st != KDE_OK) return st;
   // index output buffer: local flags at most n
@@ -1081,6 +1122,7 @@ extern "C" kde_status kde_online_update(kde_model* m, const float* lo, const flo
   if (st != KDE_OK) return st;
   if (!(true_sel >= 0.0 && true_sel <= 1.0)) return fail(KDE_EINVAL, "true_sel outside [0, 1]");
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   OnlineParamsDev od;
   st = online_params_dev(m, op, &od, m->stream);
   if (st != KDE_OK) return st;
@@ -1144,6 +1186,7 @@ extern "C" kde_status kde_replace_points(kde_model* m, const int64_t* idx, const
   for (int64_t e = 0; e < k * m->d; ++e)
     if (!std::isfinite(rows[e])) return fail(KDE_EINVAL, "non-finite value in replacement rows");
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   return replace_impl(m, idx, rows, k, k_init);
 }
 
@@ -1193,6 +1236,7 @@ extern "C" kde_status kde_insert_rows(kde_model* m, const float* rows, int64_t k
     if (slot[r] >= 0 && i >= 0 && i < m->n) m->ins_last[(size_t)i] = -1;
   }
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   kde_status st = idx.empty() ? KDE_OK : replace_impl(m, idx.data(), sel.data(), (int64_t)idx.size(), k_init);
   if (st != KDE_OK) return st;
   ++m->gen;
@@ -1218,7 +1262,7 @@ extern "C" kde_status kde_karma_update_dev(kde_model* m, const float* d_lo, cons
   CUL(launch_karma(m->cret, m->karma, m->n, (double)m->n_global, m->ret, d_true_sel, kd, d_lo, d_hi, m->d,
                    m->consts, m->bitmap, m->block_counts, m->block_offsets, m->done, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
                    StreamTail{}, s));
-  return KDE_OK;
+  return mark_dev(m, s);
 }
 
 extern "C" kde_status kde_online_update_dev(kde_model* m, const double* d_true_sel, const kde_online_params* op,
@@ -1233,7 +1277,7 @@ extern "C" kde_status kde_online_update_dev(kde_model* m, const double* d_true_s
   if (st != KDE_OK) return st;
   CUL(launch_online_update(m->ret, d_true_sel, od, m->d, m->online, m->consts, s));
   ++m->gen;
-  return KDE_OK;
+  return mark_dev(m, s);
 }
 
 extern "C" kde_status kde_replace_points_dev(kde_model* m, const int64_t* d_idx, const float* d_rows,
@@ -1248,7 +1292,7 @@ extern "C" kde_status kde_replace_points_dev(kde_model* m, const int64_t* d_idx,
   CUL(launch_scatter_rows_dev(d_idx, d_rows, d_k, cap, m->d, m->cols, m->ld, m->n, m->row_offset, m->karma, k_init,
                               m->range_enc, m->consts, s));
   ++m->gen;
-  return KDE_OK;
+  return mark_dev(m, s);
 }
 
 // One device-resident streaming step in three kernels: the
@@ -1298,7 +1342,7 @@ extern "C" kde_status kde_stream_step_dev(kde_model* m, const float* d_lo, const
                    m->consts, m->bitmap, m->block_counts, m->block_offsets, m->done, m->row_offset, d_idx_out, idx_cap, d_n_flagged,
                    tail, s));
   ++m->gen;
-  return KDE_OK;
+  return mark_dev(m, s);
 }
 
 // ------------------------------------------------------------------ inspection
@@ -1306,6 +1350,7 @@ extern "C" kde_status kde_get_karma(kde_model* m, double* karma) {
   CHECK_MODEL(m);
   if (!karma) return fail(KDE_EINVAL, "NULL karma");
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   CU(cudaStreamSynchronize(m->stream));
   CU(cudaMemcpy(karma, m->karma, sizeof(double) * m->n, cudaMemcpyDeviceToHost));
   return KDE_OK;
@@ -1317,6 +1362,7 @@ extern "C" kde_status kde_set_karma(kde_model* m, const double* karma) {
   for (int64_t i = 0; i < m->n; ++i)
     if (std::isnan(karma[i])) return fail(KDE_EINVAL, "NaN karma");
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   CU(cudaStreamSynchronize(m->stream));
   CU(cudaMemcpy(m->karma, karma, sizeof(double) * m->n, cudaMemcpyHostToDevice));
   return KDE_OK;
@@ -1326,6 +1372,7 @@ extern "C" kde_status kde_get_sample(kde_model* m, float* rows) {
   CHECK_MODEL(m);
   if (!rows) return fail(KDE_EINVAL, "NULL rows");
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   float* d_rows = nullptr;
   CU(cudaMalloc(&d_rows, sizeof(float) * (size_t)m->n * m->d));
   CUL(launch_cols_to_rows(m->cols, m->ld, m->n, m->d, d_rows, m->stream));
@@ -1340,6 +1387,7 @@ extern "C" kde_status kde_get_contributions(kde_model* m, float* c) {
   if (!c) return fail(KDE_EINVAL, "NULL c");
   if (!m->ret_valid || !m->ret_has_c) return fail(KDE_ESTATE, "no retained contributions");
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   CU(cudaStreamSynchronize(m->stream));
   CU(cudaMemcpy(c, m->cret, sizeof(float) * m->n, cudaMemcpyDeviceToHost));
   return KDE_OK;
@@ -1349,6 +1397,7 @@ extern "C" kde_status kde_get_online_state(kde_model* m, double* acc, double* ms
                                            int32_t* count) {
   CHECK_MODEL(m);
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   OnlineState s;
   CU(cudaStreamSynchronize(m->stream));
   CU(cudaMemcpy(&s, m->online, sizeof(s), cudaMemcpyDeviceToHost));
@@ -1366,6 +1415,7 @@ extern "C" kde_status kde_set_online_state(kde_model* m, const double* acc, cons
   CHECK_MODEL(m);
   if (!acc || !ms || !lr || !gprev || count < 0) return fail(KDE_EINVAL, "bad online state");
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   OnlineState s;
   memset(&s, 0, sizeof(s));
   const size_t b = sizeof(double) * m->d;
@@ -1392,6 +1442,7 @@ extern "C" kde_status kde_set_profiling(kde_model* m, int32_t on) {
 extern "C" kde_status kde_get_profile(kde_model* m, double* scan_ms, int64_t* scan_launches, int64_t* launches) {
   CHECK_MODEL(m);
   DeviceGuard g(m->device);
+  WAIT_DEV(m);
   CU(cudaDeviceSynchronize());
   double tot = 0.0;
   for (size_t i = 0; i + 1 < m->ev_used; i += 2) {
