@@ -344,7 +344,7 @@ def roofline_batched(cfg, args, n_local, q, avg_ms, sms, config_name):
                 "peak_source": f"FP32 ceiling {sms} SMs x 128 lanes x {SM_MAX_MHZ:.0f} MHz / (6d)"}
     peak = sms * MUFU_PER_SM_CLK * SM_MAX_MHZ * 1e6 / (2 * d) / 1e9
     return {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gpt·q/s", "frac": achieved / peak,
-            "traffic": _traffic(config_name),
+            "traffic": _traffic(config_name), "ncu_pipes": _pipes(config_name),
             "kernel": f"scan_batched_kernel<{d},grad>{'' if args.no_cull else ' (culled)'}",
             "algorithmic": f"{n_local} points x {q} boxes per launch (per GPU); 2d MUFU.EX2 per point*box"
                            + ("" if args.no_cull else " (brute-force count: culled pairs are counted as "
@@ -358,7 +358,7 @@ def roofline_single(d, n_local, grad, retain, avg_ms, cull, config_name):
     achieved = alg_bytes / (avg_ms * 1e-3) / 1e9
     peak = _measured_hbm()
     return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-            "traffic": _traffic(config_name),
+            "traffic": _traffic(config_name), "ncu_pipes": _pipes(config_name),
             "kernel": (f"scan_single_tma_kernel<{d},{'grad' if grad else 'est'},cull>" if cull else
                        f"{'scan_single_tma_kernel' if d <= 8 else 'scan_single_kernel'}<{d},{'grad' if grad else 'est'}>"),
             "algorithmic": f"4*d bytes/point{' + 4 B/point retained' if retain else ''} x {n_local} points per launch",
@@ -723,6 +723,15 @@ def _measured_hbm():
         return float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"])
     except Exception:
         return 6650.0  # B200_PROFILING.md fallback
+
+
+def _pipes(config):
+    """ncu pipe utilisation of the dominant kernel from the committed capture, if any."""
+    try:
+        t = json.load(open(os.path.join(ROOT, "profiles", "ncu_pipes.json")))
+        return t.get(config)
+    except Exception:
+        return None
 
 
 def _traffic(config):
