@@ -235,6 +235,24 @@ kde_status kde_set_retain(kde_model *m, int32_t on);
 kde_status kde_set_cull(kde_model *m, int32_t on);
 kde_status kde_get_cull(const kde_model *m, int32_t *on);
 
+/* kde_set_cells / kde_get_cells -- on != 0 (the default): the culled batched
+ * scan (q > 1, culling on, batches that fill 256-box CTAs) visits a spatially
+ * ordered COPY of the local sample instead of the sample itself (R16):
+ * points sorted by a 32-bit Morton key over the column range, cut into cells of
+ * 256 points with their bounding boxes.  A (box, cell) pair whose bounding box
+ * lies >= 8 scaled bandwidths outside the box is skipped as a whole (every point
+ * in it obeys the R15 bound above); a cell inside the box's kept region is
+ * evaluated without per-point classification.  The estimator is a sum over an
+ * unordered set (eq. 2), so only the summation order changes; results
+ * stay deterministic.  The copy (d x ld fp32, device) and its cell boxes are
+ * built on the model's stream at the first such call and rebuilt after any call
+ * that changes sample rows (replace / insert / streaming step); the sample, its
+ * karma and retained contributions keep their original order.
+ * builds: number of index builds so far (may be NULL).
+ * Errors: KDE_EINVAL for a NULL model / on. */
+kde_status kde_set_cells(kde_model *m, int32_t on);
+kde_status kde_get_cells(const kde_model *m, int32_t *on, int64_t *builds);
+
 /* ---------------------------------------------------------------- hot path */
 /* kde_estimate_batch -- selectivity estimates for q boxes, eq. (2)+(13):
  *   est[k]        = p_hat_H(Omega_k) = (1/s) sum_i prod_j [Phi((u_kj - t_ij)/h_j) - Phi((l_kj - t_ij)/h_j)]

@@ -37,7 +37,8 @@ ABI_SYMBOLS = (
     "kde_get_karma", "kde_set_karma", "kde_get_sample", "kde_get_contributions", "kde_get_online_state",
     "kde_set_online_state", "kde_synchronize", "kde_count_in_box_dev", "kde_set_profiling", "kde_get_profile",
     "kde_karma_update_dev", "kde_online_update_dev", "kde_replace_points_dev", "kde_stream_step_dev",
-    "kde_set_kernel", "kde_get_kernel", "kde_set_cull", "kde_get_cull", "kde_reservoir_select", "kde_insert_rows",
+    "kde_set_kernel", "kde_get_kernel", "kde_set_cull", "kde_get_cull", "kde_set_cells", "kde_get_cells",
+    "kde_reservoir_select", "kde_insert_rows",
     "kde_create_sharded_peer", "kde_peer_handle", "kde_peer_attach",
 )
 
@@ -109,6 +110,8 @@ def lib() -> ctypes.CDLL:
         "kde_get_kernel": (ctypes.c_int, [P, P]),
         "kde_set_cull": (ctypes.c_int, [P, i32]),
         "kde_get_cull": (ctypes.c_int, [P, P]),
+        "kde_set_cells": (ctypes.c_int, [P, i32]),
+        "kde_get_cells": (ctypes.c_int, [P, P, P]),
         "kde_estimate_batch": (ctypes.c_int, [P, P, P, i64, P, P]),
         "kde_estimate_batch_dev": (ctypes.c_int, [P, P, P, i64, P, P, P]),
         "kde_loss_and_grad": (ctypes.c_int, [P, P, P, P, i64, i32, f64, i32, P, P, P]),
@@ -291,6 +294,18 @@ def kde_get_cull(m) -> bool:
     k = ctypes.c_int32()
     _check(lib().kde_get_cull(m, ctypes.byref(k)))
     return bool(k.value)
+
+
+def kde_set_cells(m, on: bool):
+    _check(lib().kde_set_cells(m, int(bool(on))))
+
+
+def kde_get_cells(m):
+    """(on, index builds so far)"""
+    k = ctypes.c_int32()
+    b = ctypes.c_int64()
+    _check(lib().kde_get_cells(m, ctypes.byref(k), ctypes.byref(b)))
+    return bool(k.value), b.value
 
 
 def kde_set_retain(m, on: bool):
@@ -565,6 +580,15 @@ class KDEModel:
     @cull.setter
     def cull(self, on):
         kde_set_cull(self.handle, on)
+
+    @property
+    def cells(self):
+        """culled batched scan over the spatially ordered copy of the sample (default on, DESIGN R16)"""
+        return kde_get_cells(self.handle)[0]
+
+    @cells.setter
+    def cells(self, on):
+        kde_set_cells(self.handle, on)
 
     def estimate(self, lo, hi, grad=False):
         return kde_estimate_batch(self.handle, lo, hi, self.d, grad)

@@ -120,7 +120,34 @@ struct ScanBatchedArgs {
   const int* perm;        // nullable: CTA slot order -> box index (boxes sorted by their probed kept fraction)
 };
 
+// culled batched scan over the spatially ordered copy of the sample (scan_cells.cuh, reading R16):
+// cells of kCellPts consecutive points in Morton order, each with its bounding box; a CTA owns a
+// group of boxes (dealt from the probe order so groups and warps get similar cost) and the cells
+// split, split + nsplit, ... (strided over the whole curve, so every CTA sees every region).
+constexpr int kCellPts = 256;  // points per cell (= the batched scan's tile)
+struct ScanCellsArgs {
+  const float* ccols;     // [d][ld] ordered copy of the sample (cells.cu)
+  int64_t ld;             // padded column length
+  int64_t n;              // valid points
+  int64_t ncells;         // ceil(n / kCellPts)
+  const float* cbb;       // [ncells][d][2] per-cell (min, max) of the raw coordinates
+  const float* lo;        // device [q][d]
+  const float* hi;        // device [q][d]
+  int64_t q;
+  const DevConsts* consts;
+  const int* perm;        // nullable: sorted position -> box index (probe order, cull_order.cu)
+  double* partials;       // [nsplit][1+d][q]
+};
+
+// spatial index of the sample (cells.cu): Morton keys over the column range, stable radix sort,
+// gathered ordered copy (padding points 0) and per-cell bounding boxes
+size_t cells_scratch_bytes(int64_t n);
+cudaError_t launch_cells_build(const float* cols, int64_t ld, int64_t n, int d, const DevConsts* c, void* scratch,
+                               size_t scratch_bytes, float* ccols, float* cbb, cudaStream_t s);
+
 // host-side launchers (scan_inst_*.cu)
+cudaError_t launch_scan_cells(int d, bool grad, const ScanCellsArgs& a, int num_sms, int* splits_out, cudaStream_t s,
+                              bool dry_run);
 cudaError_t launch_scan_single(int d, bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s);
 cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int num_sms, int* splits_out,
                                 cudaStream_t s, bool dry_run);

@@ -75,6 +75,16 @@ struct kde_model {
   size_t partials_cap = 0;           // bytes
   void* order = nullptr;             // culled batched scan: box-order scratch (cull_order.cu)
   size_t order_cap = 0;              // bytes
+  // spatial index for the culled batched scan (cells.cu, reading R16): ordered copy + cell boxes,
+  // rebuilt lazily when the sample changed since it was built (sgen != cells_gen)
+  bool cells_on = true;              // KDE_CELLS=0: the unordered culled batched scan instead
+  float* ccols = nullptr;            // [d][ld]
+  float* cbb = nullptr;              // [ncells][d][2]
+  void* cscratch = nullptr;          // build scratch (keys, indices, radix-sort temp)
+  size_t cscratch_cap = 0;
+  uint64_t sgen = 1;                 // bumped whenever the sample's rows change
+  uint64_t cells_gen = 0;            // sgen the index was built at (0: none)
+  int64_t cells_builds = 0;          // index builds so far (kde_get_profile_counters)
   double* gather = nullptr;          // [world][q][1+d]
   size_t gather_cap = 0;
   uint32_t* bitmap = nullptr;
@@ -102,7 +112,7 @@ struct kde_model {
   bool cull = true;  // kde_set_cull: skip points whose contribution is provably < 2^-64 (single-box scan)
   bool ret_valid = false, ret_has_c = false, ret_has_grad = false;
   float ret_lo[kMaxDim], ret_hi[kMaxDim];
-  uint64_t gen = 1;      // bumped whenever h or the sample changes
+  uint64_t gen = 1;      // bumped whenever h or the sample changes (sgen: the sample only)
   uint64_t ret_gen = 0;
   bool online_init = false;
   int32_t kernel = 0;  // KDE_KERNEL_GAUSSIAN
@@ -310,6 +320,25 @@ static kde_status check_peer(kde_model* m) {
 }
 
 // ------------------------------------------------------------------ scans
+// The spatial index of the local shard (cells.cu), rebuilt when the sample changed since the last
+// build.  Stream-ordered: the build reads m->cols on s, after every write enqueued before it.
+static kde_status ensure_cells(kde_model* m, cudaStream_t s) {
+  if (m->cells_gen == m->sgen && m->ccols) return KDE_OK;
+  const int64_t ncells = (m->n + kCellPts - 1) / kCellPts;
+  if (!m->ccols) {
+    CU(cudaMalloc(&m->ccols, sizeof(float) * (size_t)m->d * m->ld));
+    CU(cudaMalloc(&m->cbb, sizeof(float) * 2 * (size_t)m->d * (size_t)(ncells > 0 ? ncells : 1)));
+  }
+  kde_status st = ensure_bytes(&m->cscratch, &m->cscratch_cap, cells_scratch_bytes(m->n));
+  if (st != KDE_OK) return st;
+  m->launches += 3;  // keys, gather, boxes (+ the radix sort's own kernels, library code)
+  CU(launch_cells_build(m->cols, m->ld, m->n, m->d, m->consts, m->cscratch, m->cscratch_cap, m->ccols, m->cbb, s));
+  if (debug_sync()) CU(cudaDeviceSynchronize());
+  m->cells_gen = m->sgen;
+  ++m->cells_builds;
+  return KDE_OK;
+}
+
 // Raw sums for q boxes (device bounds) -> sums[q][na] combined over ranks.
 // For q == 1 also retains c (if c_out) and writes the finalised values to fin.
 static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, int64_t q, bool grad, float* c_out,
@@ -357,7 +386,10 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     a.hi = d_hi;
     a.q = q;
     a.consts = m->consts;
-    a.cull = (m->cull && batched_culls(q)) ? 1 : 0;  // full CTAs only (measured: phased culling gains nothing)
+    static const bool env_cells = !(getenv("KDE_CELLS") && atoi(getenv("KDE_CELLS")) == 0);  // A/B switch
+    const bool cells = m->cull && m->cells_on && env_cells;
+    // unordered sample: culling for full 256-box CTAs only (measured: phased culling gains nothing)
+    a.cull = (m->cull && (cells || batched_culls(q))) ? 1 : 0;
     a.split_len = 0;
     a.partials = nullptr;
     a.perm = nullptr;
@@ -368,6 +400,34 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
       int* perm = nullptr;
       CUL(launch_cull_order(m->cols, m->ld, m->n, d, d_lo, d_hi, q, m->consts, m->order, m->order_cap, &perm, s));
       a.perm = perm;
+    }
+    if (cells) {  // the ordered copy: cell-level skipping (scan_cells.cuh), any batch size
+      kde_status st = ensure_cells(m, s);
+      if (st != KDE_OK) return st;
+      ScanCellsArgs c;
+      c.ccols = m->ccols;
+      c.ld = m->ld;
+      c.n = m->n;
+      c.ncells = (m->n + kCellPts - 1) / kCellPts;
+      c.cbb = m->cbb;
+      c.lo = d_lo;
+      c.hi = d_hi;
+      c.q = q;
+      c.consts = m->consts;
+      c.perm = a.perm;
+      c.partials = nullptr;
+      int splits = 1;
+      CU(launch_scan_cells(d, grad, c, m->num_sms, &splits, s, true));
+      st = ensure_bytes((void**)&m->partials, &m->partials_cap, sizeof(double) * (size_t)splits * na * q);
+      if (st != KDE_OK) return st;
+      c.partials = m->partials;
+      cudaEvent_t e1 = nullptr, e2 = nullptr;
+      st = prof_begin(m, s, &e1, &e2);
+      if (st != KDE_OK) return st;
+      CUL(launch_scan_cells(d, grad, c, m->num_sms, &splits, s, false));
+      if (e2) CU(cudaEventRecord(e2, s));
+      CUL(launch_reduce_splits(m->partials, splits, q, na, d_sums, fused, s));
+      goto exchange;
     }
     int splits = 1;
     CU(launch_scan_batched(d, grad, a, m->num_sms, &splits, s, true));
@@ -381,6 +441,7 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     if (e2) CU(cudaEventRecord(e2, s));
     CUL(launch_reduce_splits(m->partials, splits, q, na, d_sums, fused, s));
   }
+exchange:
   if (fused) {
     CUL(launch_peer_combine(d_sums, q * na, m->pa, m->num_sms, s));
   } else if (m->world > 1) {
@@ -447,6 +508,9 @@ static void free_model(kde_model* m) {
   DeviceGuard g(m->device);
   if (m->stream) cudaStreamSynchronize(m->stream);
   cudaFree(m->cols);
+  cudaFree(m->ccols);
+  cudaFree(m->cbb);
+  cudaFree(m->cscratch);
   cudaFree(m->karma);
   cudaFree(m->cret);
   cudaFree(m->consts);
@@ -813,6 +877,19 @@ extern "C" kde_status kde_get_cull(const kde_model* m, int32_t* on) {
   return KDE_OK;
 }
 
+extern "C" kde_status kde_set_cells(kde_model* m, int32_t on) {
+  CHECK_MODEL(m);
+  m->cells_on = on != 0;
+  return KDE_OK;
+}
+
+extern "C" kde_status kde_get_cells(const kde_model* m, int32_t* on, int64_t* builds) {
+  if (!m || !on) return fail(KDE_EINVAL, "NULL argument");
+  *on = m->cells_on ? 1 : 0;
+  if (builds) *builds = m->cells_builds;
+  return KDE_OK;
+}
+
 extern "C" kde_status kde_synchronize(kde_model* m) {
   CHECK_MODEL(m);
   DeviceGuard g(m->device);
@@ -1163,6 +1240,7 @@ static kde_status replace_impl(kde_model* m, const int64_t* idx, const float* ro
     CUL(launch_row_range((const float*)((char*)m->rbuf + ib), kl, m->d, m->range_enc, m->consts, m->stream));
     CUL(launch_scatter_rows((const int64_t*)m->rbuf, (const float*)((char*)m->rbuf + ib), kl, m->d, m->cols, m->ld,
                            m->karma, k_init, m->stream));
+    ++m->sgen;
     CU(cudaStreamSynchronize(m->stream));  // the pinned staging buffer is reused by the next call
   }
   ++m->gen;
@@ -1291,6 +1369,7 @@ extern "C" kde_status kde_replace_points_dev(kde_model* m, const int64_t* d_idx,
   ++m->launches;
   CUL(launch_scatter_rows_dev(d_idx, d_rows, d_k, cap, m->d, m->cols, m->ld, m->n, m->row_offset, m->karma, k_init,
                               m->range_enc, m->consts, s));
+  ++m->sgen;
   ++m->gen;
   return mark_dev(m, s);
 }
@@ -1330,6 +1409,7 @@ extern "C" kde_status kde_stream_step_dev(kde_model* m, const float* d_lo, const
   if (d_rows && idx_cap > 0) {
     tail.rows = d_rows;
     tail.cols = m->cols;
+    ++m->sgen;  // the tail may replace flagged rows
     tail.ld = m->ld;
     tail.karma = m->karma;
     tail.k_init = k_init;

@@ -450,6 +450,17 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity)
       "r"(parity)
       : "memory");
 }
+// as mbar_wait_parity, but a waiting warp is suspended (up to the hint, woken early by the phase
+// flip) instead of spinning on issue slots that the computing warps of the SM need
+__device__ __forceinline__ void mbar_wait_parity_suspend(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "KDE_WAITS_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
+      "@!p bra KDE_WAITS_%=;\n\t}" ::"r"(smem_u32(bar)),
+      "r"(parity), "r"(1000000u)
+      : "memory");
+}
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   asm volatile(
       "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(dst)),
@@ -993,9 +1004,11 @@ cudaError_t launch_batched_t(bool grad, const ScanBatchedArgs& a_in, int num_sms
 }  // namespace kde
 
 #include "scan_single_tma.cuh"
+#include "scan_cells.cuh"
 
 #define KDE_INSTANTIATE_SCAN(D)                                                                              \
   namespace kde {                                                                                            \
   template cudaError_t launch_single_t<D>(bool, const ScanSingleArgs&, int, cudaStream_t);                   \
   template cudaError_t launch_batched_t<D>(bool, const ScanBatchedArgs&, int, int*, cudaStream_t, bool);     \
+  template cudaError_t launch_cells_t<D>(bool, const ScanCellsArgs&, int, int*, cudaStream_t, bool);         \
   }

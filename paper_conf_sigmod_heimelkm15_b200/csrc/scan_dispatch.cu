@@ -5,7 +5,8 @@ namespace kde {
 
 #define KDE_DECL(D)                                                                                    \
   extern template cudaError_t launch_single_t<D>(bool, const ScanSingleArgs&, int, cudaStream_t);      \
-  extern template cudaError_t launch_batched_t<D>(bool, const ScanBatchedArgs&, int, int*, cudaStream_t, bool);
+  extern template cudaError_t launch_batched_t<D>(bool, const ScanBatchedArgs&, int, int*, cudaStream_t, bool); \
+  extern template cudaError_t launch_cells_t<D>(bool, const ScanCellsArgs&, int, int*, cudaStream_t, bool);
 KDE_DECL(1) KDE_DECL(2) KDE_DECL(3) KDE_DECL(4) KDE_DECL(5) KDE_DECL(6) KDE_DECL(7) KDE_DECL(8)
 KDE_DECL(9) KDE_DECL(10) KDE_DECL(11) KDE_DECL(12) KDE_DECL(13) KDE_DECL(14) KDE_DECL(15) KDE_DECL(16)
 #undef KDE_DECL
@@ -25,6 +26,16 @@ cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int 
                                 cudaStream_t s, bool dry_run) {
   switch (d) {
 #define X(D) case D: return launch_batched_t<D>(grad, a, num_sms, splits_out, s, dry_run);
+    KDE_CASES(X)
+#undef X
+  }
+  return cudaErrorInvalidValue;
+}
+
+cudaError_t launch_scan_cells(int d, bool grad, const ScanCellsArgs& a, int num_sms, int* splits_out, cudaStream_t s,
+                              bool dry_run) {
+  switch (d) {
+#define X(D) case D: return launch_cells_t<D>(grad, a, num_sms, splits_out, s, dry_run);
     KDE_CASES(X)
 #undef X
   }
