@@ -315,11 +315,13 @@ def timed_steps(step, steps, warmup, stream, m, K, flush=None, barrier=None, clo
         barrier()
     torch.cuda.synchronize()
     scan_ms, scan_launches, launches = K.kde_get_profile(m.handle)
+    cstats = K.kde_get_cells(m.handle, stats=True)[2]  # cells-scan counters (zeros when not used)
     K.kde_set_profiling(m.handle, False)
     frac = steps / max(steps + soak, 1)  # the soak launched the same kernels: keep the timed steps' share
     step_ms = [a.elapsed_time(b) for a, b in evs]
     return dict(step_ms=step_ms, scan_ms=scan_ms * frac, scan_launches=int(round(scan_launches * frac)),
-                launches=int(round(launches * frac)), clocks=clk.summary(), soak=soak, events=evs)
+                launches=int(round(launches * frac)), clocks=clk.summary(), soak=soak, events=evs,
+                cells_stats=[c / max(scan_launches, 1) for c in cstats])  # per scan launch
 
 
 def max_over_ranks(x, world, dev):
@@ -333,22 +335,35 @@ def max_over_ranks(x, world, dev):
     return float(t.item())
 
 
-def roofline_batched(cfg, args, n_local, q, avg_ms, sms, config_name):
+def roofline_batched(cfg, args, n_local, q, avg_ms, sms, config_name, cells_stats=None):
     d = cfg["d"]
     achieved = n_local * q / (avg_ms * 1e-3) / 1e9
+    cells = bool(cells_stats and cells_stats[0] > 0)
+    kname = (f"scan_cells_kernel<{d},grad> (culled, ordered copy)" if cells else
+             f"scan_batched_kernel<{d},grad>{'' if args.no_cull else ' (culled)'}")
+    extra = {}
+    if cells:  # what the culled scan actually evaluated (kde_get_cells profiling counters)
+        ev = cells_stats[2] / (n_local * q)
+        extra = {"evaluated_pairs_frac": ev, "classified_pairs_frac": cells_stats[3] / (n_local * q),
+                 "items_per_launch": cells_stats[0], "full_items_frac": cells_stats[1] / max(cells_stats[0], 1)}
     if cfg.get("kernel") == "epan":
         peak = sms * 128 * SM_MAX_MHZ * 1e6 / (6 * d) / 1e9
         return {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gpt·q/s", "frac": achieved / peak,
-                "traffic": _traffic(config_name), "kernel": f"scan_batched_kernel<{d},grad> (Epanechnikov)",
+                "traffic": _traffic(config_name), "kernel": kname + " (Epanechnikov)", **extra,
                 "algorithmic": f"{n_local} points x {q} boxes per launch; 6d FP32 ops per point*box",
                 "peak_source": f"FP32 ceiling {sms} SMs x 128 lanes x {SM_MAX_MHZ:.0f} MHz / (6d)"}
     peak = sms * MUFU_PER_SM_CLK * SM_MAX_MHZ * 1e6 / (2 * d) / 1e9
     return {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "Gpt·q/s", "frac": achieved / peak,
             "traffic": _traffic(config_name), "ncu_pipes": _pipes(config_name),
-            "kernel": f"scan_batched_kernel<{d},grad>{'' if args.no_cull else ' (culled)'}",
+            "kernel": kname,
             "algorithmic": f"{n_local} points x {q} boxes per launch (per GPU); 2d MUFU.EX2 per point*box"
                            + ("" if args.no_cull else " (brute-force count: culled pairs are counted as "
-                              "evaluated, so frac is throughput against the unculled SFU ceiling)"),
+                              "evaluated, so frac is throughput against the unculled SFU ceiling; "
+                              "evaluated_pairs_frac x frac is the fraction of the ceiling the pairs that "
+                              "reached eq. 13 alone use)"),
+            **extra,
+            **({"evaluated_work_frac": achieved * extra["evaluated_pairs_frac"] /
+                (sms * MUFU_PER_SM_CLK * SM_MAX_MHZ * 1e6 / (2 * d) / 1e9)} if extra else {}),
             "peak_source": f"SFU ceiling {sms} SMs x {MUFU_PER_SM_CLK} MUFU/clk x {SM_MAX_MHZ:.0f} MHz / (2d) "
                            "(guide unit counts; 16/clk/SM re-measured by tools/pipe_rates.cu)"}
 
@@ -419,8 +434,25 @@ def run_cuda(args, cfg, rank, world, local_rank):
             K.kde_loss_and_grad_dev(m.handle, d_lo, d_hi, d_true, d_loss, d_grad, K.LOSS_SQUARED, 0.0, False,
                                     stream=stream)
 
+    first_ms = None
+    if cfg["path"] != "single":  # the first culled batched call builds the ordered copy (cells.cu)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        with torch.cuda.stream(stream):
+            step(0)
+        torch.cuda.synchronize()
+        first_ms = (time.perf_counter() - t0) * 1e3
     T = timed_steps(step, args.steps, args.warmup, stream, m, K, flush, barrier, gpu)
     ms_per_step = max_over_ranks(sum(T["step_ms"]), world, dev) / args.steps
+    cells_info = None
+    if first_ms is not None:
+        on, builds = K.kde_get_cells(m.handle)
+        if on and builds:
+            cells_info = {"builds": builds, "first_call_ms": first_ms,
+                          "build_ms_approx": max(first_ms - ms_per_step, 0.0),
+                          "note": "the Morton-ordered copy of the sample is built by the first culled batched "
+                                  "call (before the timed region; the sample does not change between steps) "
+                                  "and rebuilt after any call that changes sample rows"}
     units_per_step = n_global * q
     value = units_per_step / (ms_per_step * 1e-3)
 
@@ -480,7 +512,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
         roof = roofline_single(d, n_local, cfg.get("grad"), cfg.get("retain"), avg_scan_ms, not args.no_cull,
                                args.config)
     else:
-        roof = roofline_batched(cfg, args, n_local, q, avg_scan_ms, sms, args.config)
+        roof = roofline_batched(cfg, args, n_local, q, avg_scan_ms, sms, args.config, T.get("cells_stats"))
     if clocks.get("sm_mhz"):
         roof["frac_at_measured_clock"] = roof["frac"] * SM_MAX_MHZ / clocks["sm_mhz"] if roof["bound"] == "alu" \
             else roof["frac"]
@@ -504,7 +536,8 @@ def run_cuda(args, cfg, rank, world, local_rank):
                    "clock_sampling": "nvidia-smi every 100 ms over the timed steps"
                                      + (f" + {T['soak']} identical untimed soak steps (timed region < 1 s)"
                                         if T["soak"] else ""),
-                   "accumulation": "fp32 per <=32 points, fp64 above"},
+                   "accumulation": ("fp32 per (box, 256-point cell) item, fp64 above" if cells_info else
+                                    "fp32 per <=32 points, fp64 above")},
         "estimates_per_s": q / (ms_per_step * 1e-3),
         "e2e": {"value": units_per_step * e2e_steps / e2e_s, "unit": "point·query evals/s",
                 "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "steps": e2e_steps},
@@ -512,6 +545,8 @@ def run_cuda(args, cfg, rank, world, local_rank):
         "roofline": roof, "cpu_baseline": cpu, "clocks": clocks,
         "step_ms": {"min": min(T["step_ms"]), "median": statistics.median(T["step_ms"]), "max": max(T["step_ms"])},
     }
+    if cells_info is not None:
+        line["cells_index"] = cells_info
     if single is not None:
         line["single_query"] = single
     print(json.dumps(line), flush=True)

@@ -237,7 +237,7 @@ kde_status kde_get_cull(const kde_model *m, int32_t *on);
 
 /* kde_set_cells / kde_get_cells -- on != 0 (the default): the culled batched
  * scan (q > 1, culling on, batches that fill 256-box CTAs) visits a spatially
- * ordered COPY of the local sample instead of the sample itself (R16):
+ * ordered COPY of the local sample instead of the sample itself (R17):
  * points sorted by a 32-bit Morton key over the column range, cut into cells of
  * 256 points with their bounding boxes.  A (box, cell) pair whose bounding box
  * lies >= 8 scaled bandwidths outside the box is skipped as a whole (every point
@@ -249,9 +249,14 @@ kde_status kde_get_cull(const kde_model *m, int32_t *on);
  * that changes sample rows (replace / insert / streaming step); the sample, its
  * karma and retained contributions keep their original order.
  * builds: number of index builds so far (may be NULL).
- * Errors: KDE_EINVAL for a NULL model / on. */
+ * stats: NULL or 4 int64 -- while profiling is on (kde_set_profiling), the cells
+ * scans' (box, cell) items, items evaluated without classification, points
+ * evaluated (point x box pairs that reached eq. 13) and points classified, summed
+ * since the previous read or kde_set_profiling call (reading resets them; zeros
+ * when profiling is off).  Synchronises the model's stream when stats != NULL.
+ * Errors: KDE_EINVAL for a NULL model / on; KDE_ECUDA. */
 kde_status kde_set_cells(kde_model *m, int32_t on);
-kde_status kde_get_cells(const kde_model *m, int32_t *on, int64_t *builds);
+kde_status kde_get_cells(kde_model *m, int32_t *on, int64_t *builds, int64_t *stats);
 
 /* ---------------------------------------------------------------- hot path */
 /* kde_estimate_batch -- selectivity estimates for q boxes, eq. (2)+(13):

@@ -111,7 +111,7 @@ def lib() -> ctypes.CDLL:
         "kde_set_cull": (ctypes.c_int, [P, i32]),
         "kde_get_cull": (ctypes.c_int, [P, P]),
         "kde_set_cells": (ctypes.c_int, [P, i32]),
-        "kde_get_cells": (ctypes.c_int, [P, P, P]),
+        "kde_get_cells": (ctypes.c_int, [P, P, P, P]),
         "kde_estimate_batch": (ctypes.c_int, [P, P, P, i64, P, P]),
         "kde_estimate_batch_dev": (ctypes.c_int, [P, P, P, i64, P, P, P]),
         "kde_loss_and_grad": (ctypes.c_int, [P, P, P, P, i64, i32, f64, i32, P, P, P]),
@@ -300,12 +300,14 @@ def kde_set_cells(m, on: bool):
     _check(lib().kde_set_cells(m, int(bool(on))))
 
 
-def kde_get_cells(m):
-    """(on, index builds so far)"""
+def kde_get_cells(m, stats=False):
+    """(on, index builds so far[, profiling counters: items, full items, points evaluated,
+    points classified -- read and reset])"""
     k = ctypes.c_int32()
     b = ctypes.c_int64()
-    _check(lib().kde_get_cells(m, ctypes.byref(k), ctypes.byref(b)))
-    return bool(k.value), b.value
+    st = (ctypes.c_int64 * 4)()
+    _check(lib().kde_get_cells(m, ctypes.byref(k), ctypes.byref(b), st if stats else None))
+    return (bool(k.value), b.value, list(st)) if stats else (bool(k.value), b.value)
 
 
 def kde_set_retain(m, on: bool):
@@ -583,7 +585,7 @@ class KDEModel:
 
     @property
     def cells(self):
-        """culled batched scan over the spatially ordered copy of the sample (default on, DESIGN R16)"""
+        """culled batched scan over the spatially ordered copy of the sample (default on, DESIGN R17)"""
         return kde_get_cells(self.handle)[0]
 
     @cells.setter

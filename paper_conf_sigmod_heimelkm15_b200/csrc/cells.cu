@@ -1,4 +1,4 @@
-// cells.cu -- spatial index of the sample for the culled batched scan (reading R16).
+// cells.cu -- spatial index of the sample for the culled batched scan (reading R17).
 //
 // The sample is an unordered set (the estimator is a sum over its points), so the batched
 // scan may visit it in any order.  For large batches it visits an ordered COPY: points sorted by a

@@ -102,6 +102,11 @@ struct ScanSingleArgs {
   double n_global;        // s (results are divided by s, so s ones give exactly 1)
   int cull;               // 1: skip points whose contribution is provably < 2^-64 (scan_single_tma.cuh)
   const PeerArgs* peer;   // nullable (device): the last block pushes sums_out into every rank's window
+  // nullable: the spatially ordered copy (cells.cu, reading R17) -- with cull on and no c_out the
+  // scan visits cells and skips those whose bounding box is >= 8 bandwidths outside the box
+  const float* ccols;     // [d][ld]
+  const float* cbb;       // [ncells][d][2]
+  int64_t ncells;
 };
 
 // scan for many boxes: sample tiles staged in shared memory by TMA bulk
@@ -120,7 +125,7 @@ struct ScanBatchedArgs {
   const int* perm;        // nullable: CTA slot order -> box index (boxes sorted by their probed kept fraction)
 };
 
-// culled batched scan over the spatially ordered copy of the sample (scan_cells.cuh, reading R16):
+// culled batched scan over the spatially ordered copy of the sample (scan_cells.cuh, reading R17):
 // cells of kCellPts consecutive points in Morton order, each with its bounding box; a CTA owns a
 // group of boxes (dealt from the probe order so groups and warps get similar cost) and the cells
 // split, split + nsplit, ... (strided over the whole curve, so every CTA sees every region).
@@ -137,6 +142,7 @@ struct ScanCellsArgs {
   const DevConsts* consts;
   const int* perm;        // nullable: sorted position -> box index (probe order, cull_order.cu)
   double* partials;       // [nsplit][1+d][q]
+  unsigned long long* stats;  // nullable (profiling): += items, full items, points evaluated, points classified
 };
 
 // spatial index of the sample (cells.cu): Morton keys over the column range, stable radix sort,

@@ -75,7 +75,7 @@ struct kde_model {
   size_t partials_cap = 0;           // bytes
   void* order = nullptr;             // culled batched scan: box-order scratch (cull_order.cu)
   size_t order_cap = 0;              // bytes
-  // spatial index for the culled batched scan (cells.cu, reading R16): ordered copy + cell boxes,
+  // spatial index for the culled batched scan (cells.cu, reading R17): ordered copy + cell boxes,
   // rebuilt lazily when the sample changed since it was built (sgen != cells_gen)
   bool cells_on = true;              // KDE_CELLS=0: the unordered culled batched scan instead
   float* ccols = nullptr;            // [d][ld]
@@ -84,7 +84,8 @@ struct kde_model {
   size_t cscratch_cap = 0;
   uint64_t sgen = 1;                 // bumped whenever the sample's rows change
   uint64_t cells_gen = 0;            // sgen the index was built at (0: none)
-  int64_t cells_builds = 0;          // index builds so far (kde_get_profile_counters)
+  int64_t cells_builds = 0;          // index builds so far (kde_get_cells)
+  unsigned long long* cstats = nullptr;  // device [4] cells-scan counters while profiling (kde_get_cells)
   double* gather = nullptr;          // [world][q][1+d]
   size_t gather_cap = 0;
   uint32_t* bitmap = nullptr;
@@ -371,7 +372,21 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     a.dpdh_out = m->world == 1 ? d_dpdh : nullptr;
     a.n_global = (double)m->n_global;
     a.cull = m->cull ? 1 : 0;
-    const int grid = scan_single_grid(d, grad, m->n, m->num_sms, m->cull);
+    a.ccols = nullptr;
+    a.cbb = nullptr;
+    a.ncells = 0;
+    int grid = scan_single_grid(d, grad, m->n, m->num_sms, m->cull);
+    // the ordered copy, when current (built by a culled batched call since the last sample change):
+    // cells far from the box are not read at all (scan_cells.cuh); not for retained contributions,
+    // which are per point in the sample's own order
+    static const bool env_cells1 = !(getenv("KDE_CELLS") && atoi(getenv("KDE_CELLS")) == 0);
+    if (m->cull && m->cells_on && env_cells1 && !c_out && m->ccols && m->cells_gen == m->sgen) {
+      a.ccols = m->ccols;
+      a.cbb = m->cbb;
+      a.ncells = (m->n + kCellPts - 1) / kCellPts;
+      const int64_t want = (a.ncells + 7) / 8;  // at least one cell per warp
+      grid = (int)std::min<int64_t>((int64_t)m->num_sms * 4, std::max<int64_t>(want, 1));  // <= 8 CTAs/SM (block_partials)
+    }
     cudaEvent_t e1 = nullptr, e2 = nullptr;
     kde_status pst = prof_begin(m, s, &e1, &e2);
     if (pst != KDE_OK) return pst;
@@ -416,6 +431,14 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
       c.consts = m->consts;
       c.perm = a.perm;
       c.partials = nullptr;
+      c.stats = nullptr;
+      if (m->prof) {  // evaluated-pair counters for the bench's roofline (kde_get_cells)
+        if (!m->cstats) {
+          CU(cudaMalloc(&m->cstats, 4 * sizeof(unsigned long long)));
+          CU(cudaMemsetAsync(m->cstats, 0, 4 * sizeof(unsigned long long), s));
+        }
+        c.stats = m->cstats;
+      }
       int splits = 1;
       CU(launch_scan_cells(d, grad, c, m->num_sms, &splits, s, true));
       st = ensure_bytes((void**)&m->partials, &m->partials_cap, sizeof(double) * (size_t)splits * na * q);
@@ -511,6 +534,7 @@ static void free_model(kde_model* m) {
   cudaFree(m->ccols);
   cudaFree(m->cbb);
   cudaFree(m->cscratch);
+  cudaFree(m->cstats);
   cudaFree(m->karma);
   cudaFree(m->cret);
   cudaFree(m->consts);
@@ -883,10 +907,21 @@ extern "C" kde_status kde_set_cells(kde_model* m, int32_t on) {
   return KDE_OK;
 }
 
-extern "C" kde_status kde_get_cells(const kde_model* m, int32_t* on, int64_t* builds) {
+extern "C" kde_status kde_get_cells(kde_model* m, int32_t* on, int64_t* builds, int64_t* stats) {
   if (!m || !on) return fail(KDE_EINVAL, "NULL argument");
   *on = m->cells_on ? 1 : 0;
   if (builds) *builds = m->cells_builds;
+  if (stats) {
+    unsigned long long h[4] = {0, 0, 0, 0};
+    if (m->cstats) {
+      DeviceGuard g(m->device);
+      WAIT_DEV(m);
+      CU(cudaStreamSynchronize(m->stream));
+      CU(cudaMemcpy(h, m->cstats, sizeof(h), cudaMemcpyDeviceToHost));
+      CU(cudaMemset(m->cstats, 0, sizeof(h)));  // counters run from one read to the next
+    }
+    for (int i = 0; i < 4; ++i) stats[i] = (int64_t)h[i];
+  }
   return KDE_OK;
 }
 
@@ -1513,6 +1548,11 @@ extern "C" kde_status kde_set_online_state(kde_model* m, const double* acc, cons
 extern "C" kde_status kde_set_profiling(kde_model* m, int32_t on) {
   CHECK_MODEL(m);
   m->prof = on != 0;
+  if (m->cstats) {
+    DeviceGuard g(m->device);
+    WAIT_DEV(m);
+    CU(cudaMemset(m->cstats, 0, 4 * sizeof(unsigned long long)));
+  }
   m->ev_used = 0;
   m->scan_launches = 0;
   m->launches = 0;

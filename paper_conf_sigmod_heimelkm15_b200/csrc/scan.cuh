@@ -881,7 +881,9 @@ __global__ void __launch_bounds__(kBatchedThreads, MINB) scan_batched_kernel(con
 }
 
 // ---------------------------------------------------------------- launchers
-// forward declaration (scan_single_tma.cuh, included below)
+// forward declarations (scan_single_tma.cuh, scan_cells.cuh, included below)
+template <int D>
+cudaError_t launch_cells_single_t(bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s);
 template <int D, bool GRAD, int TILE, int STAGES, int OCC, bool CULL>
 cudaError_t launch_single_tma_variant(const ScanSingleArgs& a, int grid, cudaStream_t s);
 
@@ -908,6 +910,7 @@ __host__ __device__ constexpr int cull_occ(int d) { return KDE_TUNE_CULL_OCC(d);
 // d > 8: register-streaming variant (measured faster or equal there).
 template <int D>
 cudaError_t launch_single_t(bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s) {
+  if (a.cull && a.ccols && !a.c_out) return launch_cells_single_t<D>(grad, a, grid, s);  // scan_cells.cuh
   if (a.cull) {
     return grad ? launch_single_tma_variant<D, true, cull_tile(D), cull_stages(D), cull_occ(D), true>(a, grid, s)
                 : launch_single_tma_variant<D, false, cull_tile(D), cull_stages(D), cull_occ(D), true>(a, grid, s);

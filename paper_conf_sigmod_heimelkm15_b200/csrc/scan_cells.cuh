@@ -1,5 +1,5 @@
 // scan_cells.cuh -- the culled batched scan over the spatially ordered copy of the sample
-// (reading R16; included by scan.cuh, which provides the TMA / mbarrier helpers, point_box2 and
+// (reading R17; included by scan.cuh, which provides the TMA / mbarrier helpers, point_box2 and
 // the cull helpers of phi.cuh).
 //
 // Per box the scan computes the same sums as scan_batched_kernel (eq. 2 + 13 and the eq. 17 terms,
@@ -59,7 +59,7 @@ __host__ __device__ constexpr int cells_stages(int d) {
 // CTAs per resident slot (waves): several smaller CTAs per SM slot even out the work of the
 // strided cell sets and box groups (the hardware starts a new CTA where one finished)
 #ifndef KDE_TUNE_CELLS_WAVES
-#define KDE_TUNE_CELLS_WAVES 1
+#define KDE_TUNE_CELLS_WAVES 16
 #endif
 // point pairs per lane and iteration of a full item (kCellPts / 64 must be a multiple)
 #ifndef KDE_TUNE_CELLS_PU
@@ -161,9 +161,10 @@ __device__ __forceinline__ void cells_boxdims(const float4* tb, const float* hdb
   }
 }
 
-// One (box, cell) item: the lanes hold point pairs.  Adds the item's sums into acc[0..NA).
+// One (box, cell) item: the lanes hold point pairs.  Adds the item's sums into acc[0..NA) and
+// returns the number of points evaluated (all of a full cell, the kept ones of a partial cell).
 template <int D, bool GRAD, int MODE>
-__device__ __forceinline__ void cells_item(const float* tl, int npts, bool full, const float4* tb, const float* hdb,
+__device__ __forceinline__ int cells_item(const float* tl, int npts, bool full, const float4* tb, const float* hdb,
                                            unsigned nm, const float (&ap)[D], double* acc, unsigned char* list,
                                            int lane) {
   constexpr int NA = GRAD ? D + 1 : 1;
@@ -173,6 +174,7 @@ __device__ __forceinline__ void cells_item(const float* tl, int npts, bool full,
   for (int k = 0; k < NA; ++k) s[k] = f2(0.0f);
   constexpr int kRounds = kCellPts / 64;  // point pairs per lane
   const int rounds = (npts + 63) >> 6;
+  int ev = npts;
   if (full) {
     for (int r = 0; r < rounds; r += KDE_TUNE_CELLS_PU) {  // PU independent pairs per iteration (ILP)
 #pragma unroll
@@ -208,7 +210,8 @@ __device__ __forceinline__ void cells_item(const float* tl, int npts, bool full,
       }
     }
     const int m = (int)__reduce_add_sync(0xffffffffu, (unsigned)__popc(kb));
-    if (m == 0) return;
+    if (m == 0) return 0;
+    ev = m;
     if (m > KDE_TUNE_CELLS_DENSE) {  // many kept: masked evaluation of the rounds that hold any
       for (int r = 0; r < rounds; ++r) {
         const unsigned v = (kb >> (2 * r)) & 3u;
@@ -253,6 +256,7 @@ __device__ __forceinline__ void cells_item(const float* tl, int npts, bool full,
 #pragma unroll
   for (int k = 0; k < NA; ++k) v[k] = s[k].x + s[k].y;
   warp_sum_scatter<NA>(v, acc, lane);
+  return ev;
 }
 
 template <int D, bool GRAD>
@@ -335,6 +339,9 @@ __global__ void __launch_bounds__(kCellsThreads, CellsMinB<D>::value) scan_cells
   const float2* cbb2 = reinterpret_cast<const float2*>(a.cbb);
   float2 bbn = make_float2(0.0f, 0.0f);  // the next cell's bounding box (lane j: dimension j), prefetched
   if (lane < D && ntiles > 0) bbn = __ldg(cbb2 + (int64_t)split * D + lane);
+  __shared__ unsigned long long wstats[4 * kCellsWarps];  // a.stats (profiling)
+  if (lane < 4) wstats[4 * warp + lane] = 0ull;
+  __syncwarp();
   for (int k = 0; k < ntiles; ++k) {
     const int st = k % S;
     const int64_t cell = split + (int64_t)k * nsplit;
@@ -393,12 +400,20 @@ __global__ void __launch_bounds__(kCellsThreads, CellsMinB<D>::value) scan_cells
         const float4* tb = tab + slot * D;
         const float* hb = hdt + slot * D;
         double* ac = acc + (size_t)slot * NA;
+        int ev;
         if (epan)
-          cells_item<D, GRAD, 2>(tl, npts, fl, tb, hb, f, ap, ac, list, lane);
+          ev = cells_item<D, GRAD, 2>(tl, npts, fl, tb, hb, f, ap, ac, list, lane);
         else if (f & ((1u << D) - 1u))
-          cells_item<D, GRAD, 1>(tl, npts, fl, tb, hb, f, ap, ac, list, lane);
+          ev = cells_item<D, GRAD, 1>(tl, npts, fl, tb, hb, f, ap, ac, list, lane);
         else
-          cells_item<D, GRAD, 0>(tl, npts, fl, tb, hb, f, ap, ac, list, lane);
+          ev = cells_item<D, GRAD, 0>(tl, npts, fl, tb, hb, f, ap, ac, list, lane);
+        if (a.stats && lane == 0) {  // per-warp counters in shared memory (no registers held)
+          unsigned long long* c4 = wstats + 4 * warp;
+          c4[0] += 1;
+          c4[1] += fl ? 1 : 0;
+          c4[2] += (unsigned long long)ev;
+          c4[3] += fl ? 0 : (unsigned long long)npts;
+        }
       }
     }
     __syncwarp();
@@ -410,6 +425,7 @@ __global__ void __launch_bounds__(kCellsThreads, CellsMinB<D>::value) scan_cells
       }
     }
   }
+  if (a.stats && lane < 4) atomicAdd(a.stats + lane, wstats[4 * warp + lane]);  // per-warp totals
   __syncthreads();
   for (int i = tid; i < QG; i += kCellsThreads) {
     const int64_t pos = (int64_t)g + (int64_t)ngroups * i;
@@ -452,6 +468,146 @@ cudaError_t launch_cells_t(bool grad, const ScanCellsArgs& a, int num_sms, int* 
   if (dry_run) return cudaSuccess;
   dim3 grid((unsigned)nsplit, (unsigned)ngroups);
   return grad ? launch_cells_tg<D, true>(a, grid, s) : launch_cells_tg<D, false>(a, grid, s);
+}
+
+// ---------------------------------------------------------------- one box (q == 1, no retain)
+// The same cell test for a single box: every warp walks cells gw, gw + W, ... (W = all warps of the
+// grid); a skipped cell is never read (HBM traffic drops to the cells near the box), a full cell is
+// evaluated without classification, a partial cell round by round with a per-point mask.  Loads are
+// plain coalesced LDG.64 (lane = point pair), two rounds in flight per warp; fp32 sums per cell (8
+// points per lane), fp64 per lane across cells, then the block reduction + deterministic last-block
+// pass of the other single-box scans (single_reduce_finalize).
+__host__ __device__ constexpr int cells_single_occ(int d) { return d <= 3 ? 4 : (d <= 6 ? 3 : 2); }
+template <int D, bool GRAD, int MODE>
+__device__ __forceinline__ void cells_single_body(const ScanSingleArgs& a, const float4* smc, const float2* scb,
+                                                  bool keep_all, double* acc) {
+  constexpr int NA = GRAD ? D + 1 : 1;
+  constexpr bool EPAN = MODE == 2;
+  const int lane = threadIdx.x & 31;
+  const int64_t W = (int64_t)gridDim.x * (kCellsThreads / 32);
+  const int64_t gw = (int64_t)blockIdx.x * (kCellsThreads / 32) + (threadIdx.x >> 5);
+  float ap[D];
+#pragma unroll
+  for (int j = 0; j < D; ++j) ap[j] = smc[j].w;
+  const float apj = lane < D ? smc[lane].w : 0.0f;
+  const float2 cbj = lane < D ? scb[lane] : make_float2(0.0f, 0.0f);
+  const float2* cbb2 = reinterpret_cast<const float2*>(a.cbb);
+  constexpr float kEps = 1.0f / (1 << 20);
+  float2 bbn = make_float2(0.0f, 0.0f);
+  if (lane < D && gw < a.ncells) bbn = __ldg(cbb2 + gw * D + lane);
+  for (int64_t c = gw; c < a.ncells; c += W) {
+    const float2 bb = bbn;
+    if (lane < D && c + W < a.ncells) bbn = __ldg(cbb2 + (c + W) * D + lane);
+    // lane j < D: this dimension's smallest / largest distance of the cell outside the box
+    float nr = EPAN ? -INFINITY : 0.0f, fr = nr;  // neutral for the max (EPAN) / sum over the lanes
+    if (lane < D) {
+      const float cc = fmaf(0.5f, bb.x, 0.5f * bb.y) * apj, chw = (0.5f * bb.y - 0.5f * bb.x) * apj;
+      const float dc = fabsf(cc - cbj.x);
+      const float err = kEps * (fabsf(cc) + chw + fabsf(cbj.x) + cbj.y);
+      nr = dc - chw - cbj.y - err;
+      fr = dc + chw - cbj.y;
+      if (!EPAN) {
+        nr = fmaxf(nr, 0.0f);
+        fr = fmaxf(fr, 0.0f);
+        nr *= nr;
+        fr *= fr;
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+      const float x = __shfl_xor_sync(0xffffffffu, nr, o), y = __shfl_xor_sync(0xffffffffu, fr, o);
+      nr = EPAN ? fmaxf(nr, x) : nr + x;
+      fr = EPAN ? fmaxf(fr, y) : fr + y;
+    }
+    const bool skip = !keep_all && (EPAN ? nr >= 1.0f : nr >= kCullY2);
+    if (skip) continue;  // warp-uniform
+    const bool full = keep_all || (EPAN ? fr < 1.0f : fr < kCullY2);
+    const int npts = (int)min((int64_t)kCellPts, a.n - c * kCellPts);
+    const float* cp = a.ccols + c * kCellPts;
+    float2 s[NA];
+#pragma unroll
+    for (int k = 0; k < NA; ++k) s[k] = f2(0.0f);
+    for (int r0 = 0; 64 * r0 < npts; r0 += 2) {
+      float2 t2[2][D];
+#pragma unroll
+      for (int u = 0; u < 2; ++u)
+#pragma unroll
+        for (int j = 0; j < D; ++j)
+          t2[u][j] = __ldcs(reinterpret_cast<const float2*>(cp + (int64_t)j * a.ld + 64 * (r0 + u) + 2 * lane));
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const int p = 64 * (r0 + u) + 2 * lane;
+        if (64 * (r0 + u) >= npts) break;  // warp-uniform
+        float2 valid = make_float2(p < npts ? 1.0f : 0.0f, p + 1 < npts ? 1.0f : 0.0f);
+        if (!full) {
+          float2 cb[D];
+#pragma unroll
+          for (int j = 0; j < D; ++j) cb[j] = scb[j];
+          const float2 sc = __fadd2_rn(cull_score<D, EPAN>(t2[u], ap, cb), f2(-cull_limit<EPAN>()));
+          valid.x = (__float_as_uint(sc.x) >> 31) ? valid.x : 0.0f;
+          valid.y = (__float_as_uint(sc.y) >> 31) ? valid.y : 0.0f;
+          if (!__any_sync(0xffffffffu, valid.x + valid.y > 0.0f)) continue;
+        }
+        BoxDim bd[D];
+#pragma unroll
+        for (int j = 0; j < D; ++j) {
+          const float4 v = cells_lds4(smc + j);
+          bd[j].b = make_float2(v.x, v.y);
+          bd[j].hd = v.z;
+        }
+        point_box2<D, GRAD, MODE>(bd, t2[u], ap, s, valid);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < NA; ++k) acc[k] += (double)s[k].x + (double)s[k].y;
+  }
+}
+
+template <int D, bool GRAD>
+__global__ void __launch_bounds__(kCellsThreads, cells_single_occ(D)) scan_cells_single_kernel(const ScanSingleArgs a) {
+  constexpr int NA = GRAD ? D + 1 : 1;
+  __shared__ float4 smc[D];  // (b.x, b.y, hd, ap)
+  __shared__ float2 scb[D];  // cull box
+  __shared__ int narrow_s, nocull_s;
+  const int tid = threadIdx.x;
+  if (tid == 0) {
+    narrow_s = 0;
+    nocull_s = 0;
+  }
+  __syncthreads();
+  const bool epan = a.consts->kernel == kEpanechnikov;
+  if (tid < D) {
+    const int j = tid;
+    const float ap = a.consts->ap[j];
+    const float l = __ldg(a.lo + j), u = __ldg(a.hi + j);
+    const unsigned rmin = a.consts->renc[2 * j], rmax = a.consts->renc[2 * j + 1];
+    const BoxDim bd = epan ? make_boxdim<kEpanechnikov>(l, u, ap, rmin, rmax) : make_boxdim(l, u, ap, rmin, rmax);
+    smc[j] = make_float4(bd.b.x, bd.b.y, bd.hd, ap);
+    if (!epan && bd.hd > 0.0f) atomicOr(&narrow_s, 1);
+    scb[j] = make_cullbox(l, u, ap, rmin, rmax);
+    if (!cullbox_ok(scb[j])) atomicOr(&nocull_s, 1);
+  }
+  __syncthreads();
+  double acc[NA];
+#pragma unroll
+  for (int k = 0; k < NA; ++k) acc[k] = 0.0;
+  const bool keep_all = nocull_s != 0;
+  if (epan)
+    cells_single_body<D, GRAD, 2>(a, smc, scb, keep_all, acc);
+  else if (narrow_s)
+    cells_single_body<D, GRAD, 1>(a, smc, scb, keep_all, acc);
+  else
+    cells_single_body<D, GRAD, 0>(a, smc, scb, keep_all, acc);
+  single_reduce_finalize<NA, kCellsThreads>(a, acc);
+}
+
+template <int D>
+cudaError_t launch_cells_single_t(bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s) {
+  if (grad)
+    scan_cells_single_kernel<D, true><<<grid, kCellsThreads, 0, s>>>(a);
+  else
+    scan_cells_single_kernel<D, false><<<grid, kCellsThreads, 0, s>>>(a);
+  return cudaGetLastError();
 }
 
 }  // namespace kde

@@ -1,5 +1,5 @@
 """GPU parity of the culled batched scan over the spatially ordered copy of the sample
-(scan_cells.cuh, R16) against the fp64 oracle, through the C ABI.
+(scan_cells.cuh, R17) against the fp64 oracle, through the C ABI.
 
 The ordered copy only changes the order in which the (unordered, eq. 2 / P:L98) sum over the
 sample is taken and which far (point, box) pairs are skipped as whole cells; the tolerances are
@@ -151,4 +151,57 @@ def test_cells_loss_and_grad_all_losses(kind):
     grad_ok(g_g, g_o, (dL[:, None] * mabs).mean(axis=0) * h, h, np.mean(dL) * h)
     Ltol = np.mean(dL * (1e-7 + 1e-5 * np.abs(est_o))) * 2 + 1e-12
     assert abs(L_g - L_o) <= Ltol + 1e-9 * abs(L_o)
+    m.close()
+
+
+@pytest.mark.parametrize("kernel,d,n", [("gauss", 2, 30011), ("gauss", 5, 70001), ("gauss", 10, 9001),
+                                        ("gauss", 16, 3001), ("epan", 4, 30011)])
+def test_cells_single_box_matches_oracle(kernel, d, n):
+    """q == 1 over the ordered copy (built by a batched call): far cells are not read; every special
+    box (unbounded, empty, far, narrow) and a few mixed ones, with and without the gradient.  With
+    retained contributions or a stale index the scan falls back to the TMA scan of the sample."""
+    S = synth.make_data("gauss", n, d, seed=100 + d)
+    lo, hi = _boxes(S, 300, seed=101 + d)
+    m = K.KDEModel.create(S)
+    if kernel == "epan":
+        m.set_kernel("epan")
+        m.bandwidth = m.bandwidth * np.sqrt(5.0)
+    h = m.bandwidth
+    est_o, g_o, mabs = _ref(S, h, lo, hi, kernel)
+    m.estimate(lo, hi)                                  # builds the index
+    assert K.kde_get_cells(m.handle)[1] == 1
+    ks = list(range(len(lo) - 12, len(lo))) + [0, 1, 2, 3, 50, 100]
+    for k in ks:
+        e1, g1 = m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+        sel_ok(e1, est_o[k:k + 1])
+        grad_ok(g1, g_o[k:k + 1], mabs[k:k + 1], h)
+        sel_ok(m.estimate(lo[k:k + 1], hi[k:k + 1]), est_o[k:k + 1])
+    e1 = m.estimate(lo[5:6], hi[5:6])
+    assert np.array_equal(e1, m.estimate(lo[5:6], hi[5:6]))  # deterministic
+    m.set_retain(True)                                  # retained p^(i): the sample-order scan
+    e2 = m.estimate(lo[5:6], hi[5:6])
+    sel_ok(e2, est_o[5:6])
+    c = m.contributions()
+    assert np.isclose(c.sum() / n, e2[0], rtol=1e-5, atol=1e-9)
+    m.close()
+
+
+def test_cells_single_box_stale_index_falls_back():
+    d, n = 3, 40000
+    S = synth.make_data("gauss", n, d, seed=110)
+    lo, hi = _boxes(S, 256, seed=111)
+    m = K.KDEModel.create(S)
+    h = m.bandwidth
+    m.estimate(lo, hi)
+    idx = np.arange(0, n, 7, dtype=np.int64)
+    rows = synth.make_data("rect", len(idx), d, seed=112)
+    m.replace_points(idx, rows)                         # index now stale: q == 1 must see the new rows
+    S2 = S.copy()
+    S2[idx] = rows
+    est_o, g_o, mabs = _ref(S2, h, lo, hi, "gauss")
+    for k in (0, 9, 77, len(lo) - 1):
+        e1, g1 = m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+        sel_ok(e1, est_o[k:k + 1])
+        grad_ok(g1, g_o[k:k + 1], mabs[k:k + 1], h)
+    assert K.kde_get_cells(m.handle)[1] == 1            # single-box calls do not rebuild
     m.close()
