@@ -368,16 +368,26 @@ def roofline_batched(cfg, args, n_local, q, avg_ms, sms, config_name, cells_stat
                            "(guide unit counts; 16/clk/SM re-measured by tools/pipe_rates.cu)"}
 
 
-def roofline_single(d, n_local, grad, retain, avg_ms, cull, config_name):
+def roofline_single(d, n_local, grad, retain, avg_ms, cull, config_name, cells_stats=None):
     alg_bytes = n_local * d * 4 + (n_local * 4 if retain else 0)  # 4d B/point read (+4 B/point retained c)
     achieved = alg_bytes / (avg_ms * 1e-3) / 1e9
     peak = _measured_hbm()
-    return {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-            "traffic": _traffic(config_name), "ncu_pipes": _pipes(config_name),
-            "kernel": (f"scan_single_tma_kernel<{d},{'grad' if grad else 'est'},cull>" if cull else
-                       f"{'scan_single_tma_kernel' if d <= 8 else 'scan_single_kernel'}<{d},{'grad' if grad else 'est'}>"),
-            "algorithmic": f"4*d bytes/point{' + 4 B/point retained' if retain else ''} x {n_local} points per launch",
-            "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
+    cells = bool(cells_stats and cells_stats[0] > 0)
+    g = 'grad' if grad else 'est'
+    out = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+           "traffic": None if cells else _traffic(config_name), "ncu_pipes": None if cells else _pipes(config_name),
+           "kernel": (f"scan_cells_single_kernel<{d},{g}> (ordered copy: far cells not read)" if cells else
+                      f"scan_single_tma_kernel<{d},{g},cull>" if cull else
+                      f"{'scan_single_tma_kernel' if d <= 8 else 'scan_single_kernel'}<{d},{g}>"),
+           "algorithmic": f"4*d bytes/point{' + 4 B/point retained' if retain else ''} x {n_local} points per launch",
+           "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
+    if cells:  # kde_get_cells counters: the cells actually read (effective vs read bandwidth)
+        read = cells_stats[0] * 256 / n_local
+        out.update({"sample_read_frac": read, "read_bytes_GBps": achieved * read, "read_frac": achieved * read / peak,
+                    "points_evaluated_frac": cells_stats[2] / n_local,
+                    "note": "frac counts the whole sample as read (effective); read_frac is the bandwidth of the "
+                            "cells actually read"})
+    return out
 
 
 def run_cuda(args, cfg, rank, world, local_rank):
@@ -408,8 +418,13 @@ def run_cuda(args, cfg, rank, world, local_rank):
         m.bandwidth = m.bandwidth * np.sqrt(5.0)  # variance-matched to Scott's Gaussian bandwidth
     h = m.bandwidth
     m.cull = not args.no_cull
+    m.cells = not args.no_cells
     if cfg.get("retain"):
         m.set_retain(True)
+    if cfg["path"] == "single" and not args.no_cull and not args.no_cells and not cfg.get("retain"):
+        # the ordered copy is a property of the sample version: build it once (one culled batched
+        # call, untimed) so single-box estimates read only the cells near the box (DESIGN R17)
+        m.estimate(lo[:1].repeat(2, axis=0), hi[:1].repeat(2, axis=0))
 
     stream = torch.cuda.Stream(device=dev)
     d_lo, d_hi = torch.from_numpy(lo).to(dev), torch.from_numpy(hi).to(dev)
@@ -493,7 +508,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
             m.estimate(lo1[i % len(lo1):i % len(lo1) + 1], hi1[i % len(lo1):i % len(lo1) + 1])
         e2e1 = max_over_ranks(time.perf_counter() - t0, world, dev)
         avg1 = T1["scan_ms"] / max(T1["scan_launches"], 1)
-        roof1 = roofline_single(d, n_local, False, False, avg1, not args.no_cull, "c3s")
+        roof1 = roofline_single(d, n_local, False, False, avg1, not args.no_cull, "c3s", T1.get("cells_stats"))
         single = {"workload": "configs[2] single DT box per step, estimate (kde_estimate_batch_dev, q = 1)",
                   "value": n_global / (ms1 * 1e-3), "unit": "point·query evals/s",
                   "estimates_per_s": 1e3 / ms1, "ms_per_step": ms1, "steps": len(T1["step_ms"]),
@@ -510,7 +525,7 @@ def run_cuda(args, cfg, rank, world, local_rank):
     sms = torch.cuda.get_device_properties(dev).multi_processor_count
     if cfg["path"] == "single":
         roof = roofline_single(d, n_local, cfg.get("grad"), cfg.get("retain"), avg_scan_ms, not args.no_cull,
-                               args.config)
+                               args.config, T.get("cells_stats"))
     else:
         roof = roofline_batched(cfg, args, n_local, q, avg_scan_ms, sms, args.config, T.get("cells_stats"))
     if clocks.get("sm_mhz"):
@@ -798,6 +813,8 @@ def main():
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline leg")
     ap.add_argument("--no-cull", action="store_true",
                     help="evaluate every (point, box) pair (kde_set_cull(0)); default culls provably < 2^-64")
+    ap.add_argument("--no-cells", action="store_true",
+                    help="culled scans over the sample's own order instead of the Morton-ordered copy (A/B)")
     ap.add_argument("--no-graph", action="store_true", help="stream configs: launch eagerly instead of CUDA graphs")
     ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of all-core oracle work")
     ap.add_argument("--rows", type=int, default=0,

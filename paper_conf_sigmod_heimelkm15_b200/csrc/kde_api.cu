@@ -354,7 +354,7 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
                               ? m->pa_dev
                               : nullptr;
   if (q == 1) {
-    ScanSingleArgs a;
+    ScanSingleArgs a{};
     a.peer = fused;
     a.cols = m->cols;
     a.ld = m->ld;
@@ -375,6 +375,7 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     a.ccols = nullptr;
     a.cbb = nullptr;
     a.ncells = 0;
+    a.stats = nullptr;
     int grid = scan_single_grid(d, grad, m->n, m->num_sms, m->cull);
     // the ordered copy, when current (built by a culled batched call since the last sample change):
     // cells far from the box are not read at all (scan_cells.cuh); not for retained contributions,
@@ -384,6 +385,13 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
       a.ccols = m->ccols;
       a.cbb = m->cbb;
       a.ncells = (m->n + kCellPts - 1) / kCellPts;
+      if (m->prof) {
+        if (!m->cstats) {
+          CU(cudaMalloc(&m->cstats, 4 * sizeof(unsigned long long)));
+          CU(cudaMemsetAsync(m->cstats, 0, 4 * sizeof(unsigned long long), s));
+        }
+        a.stats = m->cstats;
+      }
       const int64_t want = (a.ncells + 7) / 8;  // at least one cell per warp
       grid = (int)std::min<int64_t>((int64_t)m->num_sms * 4, std::max<int64_t>(want, 1));  // <= 8 CTAs/SM (block_partials)
     }

@@ -734,6 +734,9 @@ __global__ void __launch_bounds__(kCoopThreads, KDE_TUNE_COOP_MINB) karma_coop_k
 #define KDE_TUNE_COOP_PB 4  // 4 passes of loads in flight (ncu: 25.3 vs 27.6 us at 2^22 with 2, profiles/r02_experiments.md)
 #endif
   constexpr int PB = KDE_TUNE_COOP_PB;  // passes whose loads are in flight together
+#if KDE_TUNE_L2KEEP
+  const uint64_t pol_keep = l2_policy_evict_last();  // K and p^(i) stay in L2 across queries
+#endif
 #pragma unroll 1
   for (int64_t q0 = p0; q0 < p1; q0 += PB) {
     float4 cv[PB];
@@ -742,9 +745,15 @@ __global__ void __launch_bounds__(kCoopThreads, KDE_TUNE_COOP_MINB) karma_coop_k
     for (int r = 0; r < PB; ++r) {
       const int64_t i = (q0 + r) * kCoopPass + (int64_t)tid * kKarmaKV;
       if (q0 + r < p1 && i < n) {  // i is a multiple of 4; c and K are padded past n
+#if KDE_TUNE_L2KEEP
+        cv[r] = ld_keep_f4(a.cvals + i, pol_keep);
+        kv[r][0] = ld_keep_d2(a.karma + i, pol_keep);
+        kv[r][1] = ld_keep_d2(a.karma + i + 2, pol_keep);
+#else
         cv[r] = __ldcs(reinterpret_cast<const float4*>(a.cvals + i));
         kv[r][0] = __ldcs(reinterpret_cast<const double2*>(a.karma + i));
         kv[r][1] = __ldcs(reinterpret_cast<const double2*>(a.karma + i + 2));
+#endif
       } else {
         cv[r] = make_float4(0.f, 0.f, 0.f, 0.f);
         kv[r][0] = kv[r][1] = make_double2(0.0, 0.0);
@@ -769,8 +778,13 @@ __global__ void __launch_bounds__(kCoopThreads, KDE_TUNE_COOP_MINB) karma_coop_k
         }
       }
       if (i < n) {
+#if KDE_TUNE_L2KEEP
+        st_keep_d2(a.karma + i, make_double2(kk[0], kk[1]), pol_keep);
+        st_keep_d2(a.karma + i + 2, make_double2(kk[2], kk[3]), pol_keep);
+#else
         __stcs(reinterpret_cast<double2*>(a.karma + i), make_double2(kk[0], kk[1]));
         __stcs(reinterpret_cast<double2*>(a.karma + i + 2), make_double2(kk[2], kk[3]));
+#endif
       }
       unsigned word = nib << (4 * (lane & 7));  // word of 32 points = nibbles of 8 lanes
       word |= __shfl_xor_sync(0xffffffffu, word, 1);

@@ -450,6 +450,14 @@ __device__ __forceinline__ void mbar_wait_parity(uint64_t* bar, uint32_t parity)
       "r"(parity)
       : "memory");
 }
+// bulk copy with an L2 eviction policy (createpolicy), for streams that should not displace others
+__device__ __forceinline__ void bulk_g2s_hint(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+      : "memory");
+}
 // as mbar_wait_parity, but a waiting warp is suspended (up to the hint, woken early by the phase
 // flip) instead of spinning on issue slots that the computing warps of the SM need
 __device__ __forceinline__ void mbar_wait_parity_suspend(uint64_t* bar, uint32_t parity) {

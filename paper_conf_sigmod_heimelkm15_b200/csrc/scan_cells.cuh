@@ -480,7 +480,7 @@ cudaError_t launch_cells_t(bool grad, const ScanCellsArgs& a, int num_sms, int* 
 __host__ __device__ constexpr int cells_single_occ(int d) { return d <= 3 ? 4 : (d <= 6 ? 3 : 2); }
 template <int D, bool GRAD, int MODE>
 __device__ __forceinline__ void cells_single_body(const ScanSingleArgs& a, const float4* smc, const float2* scb,
-                                                  bool keep_all, double* acc) {
+                                                  bool keep_all, double* acc, unsigned long long* wst) {
   constexpr int NA = GRAD ? D + 1 : 1;
   constexpr bool EPAN = MODE == 2;
   const int lane = threadIdx.x & 31;
@@ -523,6 +523,13 @@ __device__ __forceinline__ void cells_single_body(const ScanSingleArgs& a, const
     if (skip) continue;  // warp-uniform
     const bool full = keep_all || (EPAN ? fr < 1.0f : fr < kCullY2);
     const int npts = (int)min((int64_t)kCellPts, a.n - c * kCellPts);
+    if (a.stats && lane == 0) {  // per-warp counters in shared memory (profiling)
+      unsigned long long* c4 = wst + 4 * (threadIdx.x >> 5);
+      c4[0] += 1;
+      c4[1] += full ? 1 : 0;
+      c4[2] += full ? (unsigned long long)npts : 0ull;
+      c4[3] += full ? 0ull : (unsigned long long)npts;
+    }
     const float* cp = a.ccols + c * kCellPts;
     float2 s[NA];
 #pragma unroll
@@ -546,6 +553,10 @@ __device__ __forceinline__ void cells_single_body(const ScanSingleArgs& a, const
           const float2 sc = __fadd2_rn(cull_score<D, EPAN>(t2[u], ap, cb), f2(-cull_limit<EPAN>()));
           valid.x = (__float_as_uint(sc.x) >> 31) ? valid.x : 0.0f;
           valid.y = (__float_as_uint(sc.y) >> 31) ? valid.y : 0.0f;
+          if (a.stats) {
+            const unsigned kept = __reduce_add_sync(0xffffffffu, (unsigned)(valid.x + valid.y));
+            if (lane == 0) wst[4 * (threadIdx.x >> 5) + 2] += kept;
+          }
           if (!__any_sync(0xffffffffu, valid.x + valid.y > 0.0f)) continue;
         }
         BoxDim bd[D];
@@ -592,12 +603,23 @@ __global__ void __launch_bounds__(kCellsThreads, cells_single_occ(D)) scan_cells
 #pragma unroll
   for (int k = 0; k < NA; ++k) acc[k] = 0.0;
   const bool keep_all = nocull_s != 0;
+  __shared__ unsigned long long wst[4 * (kCellsThreads / 32)];
+  if (tid < 4 * (kCellsThreads / 32)) wst[tid] = 0ull;
+  __syncthreads();
   if (epan)
-    cells_single_body<D, GRAD, 2>(a, smc, scb, keep_all, acc);
+    cells_single_body<D, GRAD, 2>(a, smc, scb, keep_all, acc, wst);
   else if (narrow_s)
-    cells_single_body<D, GRAD, 1>(a, smc, scb, keep_all, acc);
+    cells_single_body<D, GRAD, 1>(a, smc, scb, keep_all, acc, wst);
   else
-    cells_single_body<D, GRAD, 0>(a, smc, scb, keep_all, acc);
+    cells_single_body<D, GRAD, 0>(a, smc, scb, keep_all, acc, wst);
+  if (a.stats) {
+    __syncthreads();
+    if (tid < 4) {
+      unsigned long long t = 0ull;
+      for (int w = 0; w < kCellsThreads / 32; ++w) t += wst[4 * w + tid];
+      atomicAdd(a.stats + tid, t);
+    }
+  }
   single_reduce_finalize<NA, kCellsThreads>(a, acc);
 }
 

@@ -171,6 +171,9 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
     load_cb();
   }
   const unsigned lt = (1u << lane) - 1u;
+#if KDE_TUNE_L2KEEP
+  const uint64_t pol_keep = l2_policy_evict_last();  // retained p^(i): read by the karma pass next
+#endif
   unsigned head = 0, tail = 0;  // warp-uniform ring positions (head is a multiple of 64)
   int nproc = 0;
   float2 s[NA];
@@ -197,8 +200,13 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
       c = point_box2<D, GRAD, MODE>(bd, t, ap, s, vv);
     if (a.c_out) {
       const int2 ix = *reinterpret_cast<const int2*>(qi + e);
+#if KDE_TUNE_L2KEEP
+      if (v0) st_keep_f1(a.c_out + c0 + ix.x, c.x, pol_keep);
+      if (v1) st_keep_f1(a.c_out + c0 + ix.y, c.y, pol_keep);
+#else
       if (v0) __stcs(a.c_out + c0 + ix.x, c.x);
       if (v1) __stcs(a.c_out + c0 + ix.y, c.y);
+#endif
     }
     head += 64;
     if (++nproc == kCullFlushChunks) {
@@ -231,10 +239,17 @@ __device__ __forceinline__ void scan_single_cull_body(const ScanSingleArgs& a, c
       const bool al0 = val0 && (keep_all || o2.x < cull_limit<MODE == 2>()),
                  al1 = val1 && (keep_all || o2.y < cull_limit<MODE == 2>());
       if (a.c_out) {  // culled points retain 0; kept points are overwritten after evaluation (same warp, synced)
+#if KDE_TUNE_L2KEEP
+        if (val1)
+          st_keep_f2(a.c_out + base + 2 * pp, f2(0.0f), pol_keep);
+        else if (val0)
+          st_keep_f1(a.c_out + base + 2 * pp, 0.0f, pol_keep);
+#else
         if (val1)
           __stcs(reinterpret_cast<float2*>(a.c_out + base + 2 * pp), f2(0.0f));
         else if (val0)
           __stcs(a.c_out + base + 2 * pp, 0.0f);
+#endif
       }
       __syncwarp();  // the previous chunk's ring reads are done before these writes
       // Branch-free compaction of the 64 candidates: the kept ones go to [tail, tail + nkeep)
@@ -310,6 +325,16 @@ __global__ void __launch_bounds__(single_tma_threads<D, CULL>(), OCC) scan_singl
     const int64_t nb = c0 + (int64_t)k * TILE;
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
     mbar_arrive_expect_tx(&full[st], (uint32_t)(D * TILE * sizeof(float)));
+#if KDE_TUNE_L2KEEP
+    if (a.c_out) {  // streaming step: the sample must not displace K and p^(i) from L2
+      const uint64_t pol = l2_policy_evict_first();
+#pragma unroll
+      for (int j = 0; j < D; ++j)
+        bulk_g2s_hint(tiles + ((size_t)st * D + j) * TILE, a.cols + (int64_t)j * a.ld + nb,
+                      (uint32_t)(TILE * sizeof(float)), &full[st], pol);
+      return;
+    }
+#endif
 #pragma unroll
     for (int j = 0; j < D; ++j)
       bulk_g2s(tiles + ((size_t)st * D + j) * TILE, a.cols + (int64_t)j * a.ld + nb, (uint32_t)(TILE * sizeof(float)),
