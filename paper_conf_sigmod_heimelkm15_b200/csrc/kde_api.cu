@@ -393,7 +393,9 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
         a.stats = m->cstats;
       }
       const int64_t want = (a.ncells + 7) / 8;  // at least one cell per warp
-      grid = (int)std::min<int64_t>((int64_t)m->num_sms * 4, std::max<int64_t>(want, 1));  // <= 8 CTAs/SM (block_partials)
+      // CTAs per SM (waves of the 2 resident ones; KDE_CELLS1_CTAS tunes, <= 8 for block_partials)
+      static const int per_sm = getenv("KDE_CELLS1_CTAS") ? std::max(1, std::min(8, atoi(getenv("KDE_CELLS1_CTAS")))) : 2;
+      grid = (int)std::min<int64_t>((int64_t)m->num_sms * per_sm, std::max<int64_t>(want, 1));
     }
     cudaEvent_t e1 = nullptr, e2 = nullptr;
     kde_status pst = prof_begin(m, s, &e1, &e2);

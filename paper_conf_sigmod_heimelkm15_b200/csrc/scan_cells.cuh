@@ -81,7 +81,6 @@ constexpr size_t cells_smem_bytes() {
   return (size_t)cells_stages(D) * D * kCellPts * sizeof(float)  // tile ring
          + (size_t)QG * D * sizeof(float4)                     // (b.x, b.y, cb.x, cb.y) per box and dim
          + (size_t)QG * NA * sizeof(double)                    // fp64 accumulators
-         + (size_t)QG * D * sizeof(float)                      // hd per box and dim
          + (size_t)cells_stages(D) * (sizeof(uint64_t) + sizeof(int))  // full barriers, arrival counters
          + (size_t)QG * sizeof(unsigned)                       // per-box flags
          + (size_t)kCellsWarps * kCellPts;                     // per-warp kept-point lists (uint8)
@@ -146,17 +145,22 @@ __device__ __forceinline__ float cells_lds1(const float* p) {
   return *p;
 #endif
 }
+// Box table entry per dimension: (b.x, b.y, cb.x, cb.y).  A narrow dimension (MODE 1, bit j of nm)
+// has b = (l, l) and keeps its half-width hd in the .y slot; an Epanechnikov dimension (MODE 2)
+// recomputes Delta = (b.x - b.y) ap -- the same fp32 operations as make_boxdim when the bounds are
+// not clamped, and unused by phi_epan2 when they are (every point is then >= 2h outside the
+// clamped bound, so |v| > 1 and the clamped difference is taken).
 template <int D, int MODE>
-__device__ __forceinline__ void cells_boxdims(const float4* tb, const float* hdb, unsigned nm, BoxDim (&bd)[D]) {
+__device__ __forceinline__ void cells_boxdims(const float4* tb, const float (&ap)[D], unsigned nm, BoxDim (&bd)[D]) {
 #pragma unroll
   for (int j = 0; j < D; ++j) {
     const float4 v = cells_lds4(tb + j);
     if (MODE == 1 && ((nm >> j) & 1u)) {
       bd[j].b = make_float2(v.x, v.x);
-      bd[j].hd = cells_lds1(hdb + j);
+      bd[j].hd = v.y;
     } else {
       bd[j].b = make_float2(v.x, v.y);
-      bd[j].hd = MODE == 2 ? cells_lds1(hdb + j) : 0.0f;
+      bd[j].hd = MODE == 2 ? (v.x - v.y) * ap[j] : 0.0f;
     }
   }
 }
@@ -164,7 +168,7 @@ __device__ __forceinline__ void cells_boxdims(const float4* tb, const float* hdb
 // One (box, cell) item: the lanes hold point pairs.  Adds the item's sums into acc[0..NA) and
 // returns the number of points evaluated (all of a full cell, the kept ones of a partial cell).
 template <int D, bool GRAD, int MODE>
-__device__ __forceinline__ int cells_item(const float* tl, int npts, bool full, const float4* tb, const float* hdb,
+__device__ __forceinline__ int cells_item(const float* tl, int npts, bool full, const float4* tb,
                                            unsigned nm, const float (&ap)[D], double* acc, unsigned char* list,
                                            int lane) {
   constexpr int NA = GRAD ? D + 1 : 1;
@@ -184,7 +188,7 @@ __device__ __forceinline__ int cells_item(const float* tl, int npts, bool full, 
 #pragma unroll
         for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * kCellPts + p);
         BoxDim bd[D];
-        cells_boxdims<D, MODE>(tb, hdb, nm, bd);
+        cells_boxdims<D, MODE>(tb, ap, nm, bd);
         point_box2<D, GRAD, MODE>(bd, t, ap, s, make_float2(p < npts ? 1.0f : 0.0f, p + 1 < npts ? 1.0f : 0.0f));
       }
     }
@@ -221,7 +225,7 @@ __device__ __forceinline__ int cells_item(const float* tl, int npts, bool full, 
 #pragma unroll
         for (int j = 0; j < D; ++j) t[j] = *reinterpret_cast<const float2*>(tl + j * kCellPts + p);
         BoxDim bd[D];
-        cells_boxdims<D, MODE>(tb, hdb, nm, bd);
+        cells_boxdims<D, MODE>(tb, ap, nm, bd);
         point_box2<D, GRAD, MODE>(bd, t, ap, s, make_float2((float)(v & 1u), (float)(v >> 1)));
       }
     } else {  // few kept: compact their indices (round-major, lane order), evaluate 64 at a time
@@ -245,7 +249,7 @@ __device__ __forceinline__ int cells_item(const float* tl, int npts, bool full, 
 #pragma unroll
         for (int j = 0; j < D; ++j) t[j] = make_float2(tl[j * kCellPts + i0], tl[j * kCellPts + i1]);
         BoxDim bd[D];
-        cells_boxdims<D, MODE>(tb, hdb, nm, bd);
+        cells_boxdims<D, MODE>(tb, ap, nm, bd);
         point_box2<D, GRAD, MODE>(bd, t, ap, s, make_float2(v0 ? 1.0f : 0.0f, v1 ? 1.0f : 0.0f));
       }
       __syncwarp();  // the list is rewritten by the next item
@@ -269,8 +273,7 @@ __global__ void __launch_bounds__(kCellsThreads, CellsMinB<D>::value) scan_cells
   float* tile = reinterpret_cast<float*>(smem_raw);                           // [S][D][kCellPts]
   float4* tab = reinterpret_cast<float4*>(tile + (size_t)S * D * kCellPts);  // [QG][D]
   double* acc = reinterpret_cast<double*>(tab + (size_t)QG * D);             // [QG][NA]
-  float* hdt = reinterpret_cast<float*>(acc + (size_t)QG * NA);              // [QG][D]
-  uint64_t* bar = reinterpret_cast<uint64_t*>(hdt + (size_t)QG * D);         // [S] (8-aligned: QG*D even)
+  uint64_t* bar = reinterpret_cast<uint64_t*>(acc + (size_t)QG * NA);       // [S]
   int* cnt = reinterpret_cast<int*>(bar + S);                                // [S]
   unsigned* flags = reinterpret_cast<unsigned*>(cnt + S);                    // [QG]
   unsigned char* lists = reinterpret_cast<unsigned char*>(flags + QG);       // [warps][kCellPts]
@@ -296,8 +299,7 @@ __global__ void __launch_bounds__(kCellsThreads, CellsMinB<D>::value) scan_cells
         const BoxDim bd = epan ? make_boxdim<kEpanechnikov>(l, u, ap[j], rmin, rmax) : make_boxdim(l, u, ap[j], rmin, rmax);
         const float2 cb = make_cullbox(l, u, ap[j], rmin, rmax);
         const bool nar = !epan && bd.hd > 0.0f;
-        tab[i * D + j] = make_float4(bd.b.x, bd.b.y, cb.x, cb.y);
-        hdt[i * D + j] = bd.hd;
+        tab[i * D + j] = make_float4(bd.b.x, nar ? bd.hd : bd.b.y, cb.x, cb.y);  // see cells_boxdims
         if (nar) f |= 1u << j;
         if (!cullbox_ok(cb)) f |= kCellsKeepAll;
       }
@@ -398,15 +400,14 @@ __global__ void __launch_bounds__(kCellsThreads, CellsMinB<D>::value) scan_cells
         const bool fl = (fullm[kk] >> b) & 1u;
         const unsigned f = flags[slot];
         const float4* tb = tab + slot * D;
-        const float* hb = hdt + slot * D;
         double* ac = acc + (size_t)slot * NA;
         int ev;
         if (epan)
-          ev = cells_item<D, GRAD, 2>(tl, npts, fl, tb, hb, f, ap, ac, list, lane);
+          ev = cells_item<D, GRAD, 2>(tl, npts, fl, tb, f, ap, ac, list, lane);
         else if (f & ((1u << D) - 1u))
-          ev = cells_item<D, GRAD, 1>(tl, npts, fl, tb, hb, f, ap, ac, list, lane);
+          ev = cells_item<D, GRAD, 1>(tl, npts, fl, tb, f, ap, ac, list, lane);
         else
-          ev = cells_item<D, GRAD, 0>(tl, npts, fl, tb, hb, f, ap, ac, list, lane);
+          ev = cells_item<D, GRAD, 0>(tl, npts, fl, tb, f, ap, ac, list, lane);
         if (a.stats && lane == 0) {  // per-warp counters in shared memory (no registers held)
           unsigned long long* c4 = wstats + 4 * warp;
           c4[0] += 1;
@@ -471,164 +472,197 @@ cudaError_t launch_cells_t(bool grad, const ScanCellsArgs& a, int num_sms, int* 
 }
 
 // ---------------------------------------------------------------- one box (q == 1, no retain)
-// The same cell test for a single box: every warp walks cells gw, gw + W, ... (W = all warps of the
-// grid); a skipped cell is never read (HBM traffic drops to the cells near the box), a full cell is
-// evaluated without classification, a partial cell round by round with a per-point mask.  Loads are
-// plain coalesced LDG.64 (lane = point pair), two rounds in flight per warp; fp32 sums per cell (8
-// points per lane), fp64 per lane across cells, then the block reduction + deterministic last-block
-// pass of the other single-box scans (single_reduce_finalize).
-__host__ __device__ constexpr int cells_single_occ(int d) { return d <= 3 ? 4 : (d <= 6 ? 3 : 2); }
+// The same cell test for a single box.  Warp gw owns the cells gw, gw + W, ... (W = all warps of the
+// grid; at most 32 per warp for the sizes the grid is chosen for, else in batches of 32): one
+// batched test (lane k: candidate k) gives the warp its touched cells, which it then streams
+// through two per-warp shared-memory buffers with cp.async (the next touched cell loads while the
+// current one is evaluated).  A skipped cell is never read.  Each touched cell is one cells_item
+// (full / classified, compacted or masked) added into the warp's fp64 accumulator; the warps'
+// accumulators are summed in warp order, then the block reduction + deterministic last-block pass
+// of the other single-box scans (single_reduce_finalize).
+__host__ __device__ constexpr int cells_single_occ(int d) { return d <= 5 ? 2 : 1; }
+template <int D>
+__host__ __device__ constexpr int cells_single_nbuf() { return D <= 12 ? 2 : 1; }  // shared-memory budget
+template <int D>
+__host__ __device__ constexpr size_t cells_single_smem() {
+  return (size_t)(kCellsThreads / 32) * cells_single_nbuf<D>() * D * kCellPts * sizeof(float);  // per-warp buffers
+}
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(dst))),
+               "l"(src)
+               : "memory");
+}
+
 template <int D, bool GRAD, int MODE>
-__device__ __forceinline__ void cells_single_body(const ScanSingleArgs& a, const float4* smc, const float2* scb,
-                                                  bool keep_all, double* acc, unsigned long long* wst) {
-  constexpr int NA = GRAD ? D + 1 : 1;
-  constexpr bool EPAN = MODE == 2;
-  const int lane = threadIdx.x & 31;
+__device__ __forceinline__ void cells_single_body(const ScanSingleArgs& a, const float4* tab, unsigned nm, bool keep_all,
+                                                  const float (&ap)[D], float* wbuf, unsigned char* list, double* wacc,
+                                                  unsigned long long* wst) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int64_t W = (int64_t)gridDim.x * (kCellsThreads / 32);
-  const int64_t gw = (int64_t)blockIdx.x * (kCellsThreads / 32) + (threadIdx.x >> 5);
-  float ap[D];
-#pragma unroll
-  for (int j = 0; j < D; ++j) ap[j] = smc[j].w;
-  const float apj = lane < D ? smc[lane].w : 0.0f;
-  const float2 cbj = lane < D ? scb[lane] : make_float2(0.0f, 0.0f);
-  const float2* cbb2 = reinterpret_cast<const float2*>(a.cbb);
+  const int64_t gw = (int64_t)blockIdx.x * (kCellsThreads / 32) + warp;
+  constexpr bool EPAN = MODE == 2;
   constexpr float kEps = 1.0f / (1 << 20);
-  float2 bbn = make_float2(0.0f, 0.0f);
-  if (lane < D && gw < a.ncells) bbn = __ldg(cbb2 + gw * D + lane);
-  for (int64_t c = gw; c < a.ncells; c += W) {
-    const float2 bb = bbn;
-    if (lane < D && c + W < a.ncells) bbn = __ldg(cbb2 + (c + W) * D + lane);
-    // lane j < D: this dimension's smallest / largest distance of the cell outside the box
-    float nr = EPAN ? -INFINITY : 0.0f, fr = nr;  // neutral for the max (EPAN) / sum over the lanes
-    if (lane < D) {
-      const float cc = fmaf(0.5f, bb.x, 0.5f * bb.y) * apj, chw = (0.5f * bb.y - 0.5f * bb.x) * apj;
-      const float dc = fabsf(cc - cbj.x);
-      const float err = kEps * (fabsf(cc) + chw + fabsf(cbj.x) + cbj.y);
-      nr = dc - chw - cbj.y - err;
-      fr = dc + chw - cbj.y;
-      if (!EPAN) {
-        nr = fmaxf(nr, 0.0f);
-        fr = fmaxf(fr, 0.0f);
-        nr *= nr;
-        fr *= fr;
+  const float2* cbb2 = reinterpret_cast<const float2*>(a.cbb);
+  for (int64_t base = gw; base < a.ncells; base += 32 * W) {  // batches of 32 candidate cells
+    // lane k tests candidate base + k W against the box (all dimensions)
+    const int64_t cand = base + (int64_t)lane * W;
+    float nr = 0.0f, fr = 0.0f;  // EPAN: max_j; Gaussian: sum_j relu^2
+    if (cand < a.ncells) {
+      if (EPAN) nr = fr = -INFINITY;
+#pragma unroll
+      for (int j = 0; j < D; ++j) {
+        const float2 bb = __ldg(cbb2 + cand * D + j);
+        const float4 tb = tab[j];
+        const float cc = fmaf(0.5f, bb.x, 0.5f * bb.y) * ap[j], chw = (0.5f * bb.y - 0.5f * bb.x) * ap[j];
+        const float dc = fabsf(cc - tb.z);
+        const float err = kEps * (fabsf(cc) + chw + fabsf(tb.z) + tb.w);
+        const float near = dc - chw - tb.w - err, far = dc + chw - tb.w;
+        if (EPAN) {
+          nr = fmaxf(nr, near);
+          fr = fmaxf(fr, far);
+        } else {
+          const float n2 = fmaxf(near, 0.0f), f2v = fmaxf(far, 0.0f);
+          nr = fmaf(n2, n2, nr);
+          fr = fmaf(f2v, f2v, fr);
+        }
       }
     }
+    const bool touched = cand < a.ncells && (keep_all || (EPAN ? nr < 1.0f : nr < kCullY2));
+    const bool isfull = touched && (keep_all || (EPAN ? fr < 1.0f : fr < kCullY2));
+    unsigned tm = __ballot_sync(0xffffffffu, touched);
+    const unsigned fm = __ballot_sync(0xffffffffu, isfull);
+    auto load = [&](int k, int buf) {  // cell base + k W -> buffer buf (cp.async, one group)
+      const float* src = a.ccols + (base + (int64_t)k * W) * kCellPts;
+      float* dst = wbuf + (size_t)buf * D * kCellPts;
 #pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-      const float x = __shfl_xor_sync(0xffffffffu, nr, o), y = __shfl_xor_sync(0xffffffffu, fr, o);
-      nr = EPAN ? fmaxf(nr, x) : nr + x;
-      fr = EPAN ? fmaxf(fr, y) : fr + y;
+      for (int j = 0; j < D; ++j)
+#pragma unroll
+        for (int h = 0; h < kCellPts / 128; ++h)
+          cp_async16(dst + j * kCellPts + 128 * h + 4 * lane, src + (int64_t)j * a.ld + 128 * h + 4 * lane);
+      asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    int cur = tm ? __ffs(tm) - 1 : -1;
+    if (cur >= 0) {
+      tm &= tm - 1u;
+      load(cur, 0);
     }
-    const bool skip = !keep_all && (EPAN ? nr >= 1.0f : nr >= kCullY2);
-    if (skip) continue;  // warp-uniform
-    const bool full = keep_all || (EPAN ? fr < 1.0f : fr < kCullY2);
-    const int npts = (int)min((int64_t)kCellPts, a.n - c * kCellPts);
-    if (a.stats && lane == 0) {  // per-warp counters in shared memory (profiling)
-      unsigned long long* c4 = wst + 4 * (threadIdx.x >> 5);
-      c4[0] += 1;
-      c4[1] += full ? 1 : 0;
-      c4[2] += full ? (unsigned long long)npts : 0ull;
-      c4[3] += full ? 0ull : (unsigned long long)npts;
-    }
-    const float* cp = a.ccols + c * kCellPts;
-    float2 s[NA];
-#pragma unroll
-    for (int k = 0; k < NA; ++k) s[k] = f2(0.0f);
-    for (int r0 = 0; 64 * r0 < npts; r0 += 2) {
-      float2 t2[2][D];
-#pragma unroll
-      for (int u = 0; u < 2; ++u)
-#pragma unroll
-        for (int j = 0; j < D; ++j)
-          t2[u][j] = __ldcs(reinterpret_cast<const float2*>(cp + (int64_t)j * a.ld + 64 * (r0 + u) + 2 * lane));
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const int p = 64 * (r0 + u) + 2 * lane;
-        if (64 * (r0 + u) >= npts) break;  // warp-uniform
-        float2 valid = make_float2(p < npts ? 1.0f : 0.0f, p + 1 < npts ? 1.0f : 0.0f);
-        if (!full) {
-          float2 cb[D];
-#pragma unroll
-          for (int j = 0; j < D; ++j) cb[j] = scb[j];
-          const float2 sc = __fadd2_rn(cull_score<D, EPAN>(t2[u], ap, cb), f2(-cull_limit<EPAN>()));
-          valid.x = (__float_as_uint(sc.x) >> 31) ? valid.x : 0.0f;
-          valid.y = (__float_as_uint(sc.y) >> 31) ? valid.y : 0.0f;
-          if (a.stats) {
-            const unsigned kept = __reduce_add_sync(0xffffffffu, (unsigned)(valid.x + valid.y));
-            if (lane == 0) wst[4 * (threadIdx.x >> 5) + 2] += kept;
-          }
-          if (!__any_sync(0xffffffffu, valid.x + valid.y > 0.0f)) continue;
-        }
-        BoxDim bd[D];
-#pragma unroll
-        for (int j = 0; j < D; ++j) {
-          const float4 v = cells_lds4(smc + j);
-          bd[j].b = make_float2(v.x, v.y);
-          bd[j].hd = v.z;
-        }
-        point_box2<D, GRAD, MODE>(bd, t2[u], ap, s, valid);
+    constexpr int NB = cells_single_nbuf<D>();
+    int buf = 0;
+    while (cur >= 0) {
+      const int nxt = tm ? __ffs(tm) - 1 : -1;
+      if (nxt >= 0) tm &= tm - 1u;
+      if (NB == 2 && nxt >= 0) {
+        load(nxt, buf ^ 1);
+        asm volatile("cp.async.wait_group 1;" ::: "memory");
+      } else {
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
       }
+      __syncwarp();
+      const int64_t cell = base + (int64_t)cur * W;
+      const int npts = (int)min((int64_t)kCellPts, a.n - cell * kCellPts);
+      const bool fl = (fm >> cur) & 1u;
+      const int ev = cells_item<D, GRAD, MODE>(wbuf + (size_t)buf * D * kCellPts, npts, fl, tab, nm, ap, wacc, list, lane);
+      if (a.stats && lane == 0) {
+        unsigned long long* c4 = wst + 4 * warp;
+        c4[0] += 1;
+        c4[1] += fl ? 1 : 0;
+        c4[2] += (unsigned long long)ev;
+        c4[3] += fl ? 0ull : (unsigned long long)npts;
+      }
+      __syncwarp();  // the buffer is refilled NB cells later
+      if (NB == 2) {
+        buf ^= 1;
+      } else if (nxt >= 0) {
+        load(nxt, 0);
+      }
+      cur = nxt;
     }
-#pragma unroll
-    for (int k = 0; k < NA; ++k) acc[k] += (double)s[k].x + (double)s[k].y;
   }
 }
 
 template <int D, bool GRAD>
 __global__ void __launch_bounds__(kCellsThreads, cells_single_occ(D)) scan_cells_single_kernel(const ScanSingleArgs a) {
   constexpr int NA = GRAD ? D + 1 : 1;
-  __shared__ float4 smc[D];  // (b.x, b.y, hd, ap)
-  __shared__ float2 scb[D];  // cull box
-  __shared__ int narrow_s, nocull_s;
-  const int tid = threadIdx.x;
+  constexpr int NW = kCellsThreads / 32;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  float* wbufs = reinterpret_cast<float*>(smem_raw);  // [NW][2][D][kCellPts]
+  __shared__ float4 tab[D];                           // cells_boxdims encoding (b.x, b.y | hd, cb.x, cb.y)
+  __shared__ unsigned nm_s, nocull_s;
+  __shared__ double wacc[NW][NA];
+  __shared__ unsigned long long wst[4 * NW];
+  __shared__ __align__(16) unsigned char lists[NW][kCellPts];
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid == 0) {
-    narrow_s = 0;
-    nocull_s = 0;
+    nm_s = 0u;
+    nocull_s = 0u;
   }
+  if (tid < NW * NA) wacc[tid / NA][tid % NA] = 0.0;
+  if (tid < 4 * NW) wst[tid] = 0ull;
   __syncthreads();
   const bool epan = a.consts->kernel == kEpanechnikov;
   if (tid < D) {
     const int j = tid;
-    const float ap = a.consts->ap[j];
+    const float apj = a.consts->ap[j];
     const float l = __ldg(a.lo + j), u = __ldg(a.hi + j);
     const unsigned rmin = a.consts->renc[2 * j], rmax = a.consts->renc[2 * j + 1];
-    const BoxDim bd = epan ? make_boxdim<kEpanechnikov>(l, u, ap, rmin, rmax) : make_boxdim(l, u, ap, rmin, rmax);
-    smc[j] = make_float4(bd.b.x, bd.b.y, bd.hd, ap);
-    if (!epan && bd.hd > 0.0f) atomicOr(&narrow_s, 1);
-    scb[j] = make_cullbox(l, u, ap, rmin, rmax);
-    if (!cullbox_ok(scb[j])) atomicOr(&nocull_s, 1);
+    const BoxDim bd = epan ? make_boxdim<kEpanechnikov>(l, u, apj, rmin, rmax) : make_boxdim(l, u, apj, rmin, rmax);
+    const float2 cb = make_cullbox(l, u, apj, rmin, rmax);
+    const bool nar = !epan && bd.hd > 0.0f;
+    tab[j] = make_float4(bd.b.x, nar ? bd.hd : bd.b.y, cb.x, cb.y);
+    if (nar) atomicOr(&nm_s, 1u << j);
+    if (!cullbox_ok(cb)) atomicOr(&nocull_s, 1u);
   }
+  __syncthreads();
+  float ap[D];
+#pragma unroll
+  for (int j = 0; j < D; ++j) ap[j] = a.consts->ap[j];
+  const unsigned nm = nm_s;
+  const bool keep_all = nocull_s != 0u;
+  float* wbuf = wbufs + (size_t)warp * cells_single_nbuf<D>() * D * kCellPts;
+  if (epan)
+    cells_single_body<D, GRAD, 2>(a, tab, nm, keep_all, ap, wbuf, lists[warp], wacc[warp], wst);
+  else if (nm)
+    cells_single_body<D, GRAD, 1>(a, tab, nm, keep_all, ap, wbuf, lists[warp], wacc[warp], wst);
+  else
+    cells_single_body<D, GRAD, 0>(a, tab, nm, keep_all, ap, wbuf, lists[warp], wacc[warp], wst);
   __syncthreads();
   double acc[NA];
 #pragma unroll
-  for (int k = 0; k < NA; ++k) acc[k] = 0.0;
-  const bool keep_all = nocull_s != 0;
-  __shared__ unsigned long long wst[4 * (kCellsThreads / 32)];
-  if (tid < 4 * (kCellsThreads / 32)) wst[tid] = 0ull;
-  __syncthreads();
-  if (epan)
-    cells_single_body<D, GRAD, 2>(a, smc, scb, keep_all, acc, wst);
-  else if (narrow_s)
-    cells_single_body<D, GRAD, 1>(a, smc, scb, keep_all, acc, wst);
-  else
-    cells_single_body<D, GRAD, 0>(a, smc, scb, keep_all, acc, wst);
-  if (a.stats) {
-    __syncthreads();
-    if (tid < 4) {
-      unsigned long long t = 0ull;
-      for (int w = 0; w < kCellsThreads / 32; ++w) t += wst[4 * w + tid];
-      atomicAdd(a.stats + tid, t);
-    }
+  for (int k = 0; k < NA; ++k) {
+    double t = 0.0;
+    if (tid == 0)
+      for (int w = 0; w < NW; ++w) t += wacc[w][k];  // warp order: deterministic
+    acc[k] = t;
   }
+  if (a.stats && tid < 4) {
+    unsigned long long t = 0ull;
+    for (int w = 0; w < NW; ++w) t += wst[4 * w + tid];
+    atomicAdd(a.stats + tid, t);
+  }
+  (void)lane;
   single_reduce_finalize<NA, kCellsThreads>(a, acc);
 }
 
 template <int D>
 cudaError_t launch_cells_single_t(bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s) {
+  constexpr size_t smem = cells_single_smem<D>();
+  static_assert(smem + 8 * 1024 <= 227 * 1024, "single-box cells scan shared memory");
+  static std::atomic<unsigned long long> attr_set{0ull};  // per device ordinal
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  const unsigned long long bit = 1ull << (dev & 63);
+  if (!(attr_set.load(std::memory_order_acquire) & bit)) {
+    e = cudaFuncSetAttribute(scan_cells_single_kernel<D, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(scan_cells_single_kernel<D, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr_set.fetch_or(bit, std::memory_order_acq_rel);
+  }
   if (grad)
-    scan_cells_single_kernel<D, true><<<grid, kCellsThreads, 0, s>>>(a);
+    scan_cells_single_kernel<D, true><<<grid, kCellsThreads, smem, s>>>(a);
   else
-    scan_cells_single_kernel<D, false><<<grid, kCellsThreads, 0, s>>>(a);
+    scan_cells_single_kernel<D, false><<<grid, kCellsThreads, smem, s>>>(a);
   return cudaGetLastError();
 }
 

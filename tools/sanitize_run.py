@@ -65,6 +65,18 @@ def run(d, n, q, kernel="gauss"):
     # reservoir inserts (host decision, accepted rows only)
     m.insert_rows(S[: min(n, 3000)][::-1].copy(), seed=5, n_seen=n)
     m.estimate(lo[:1], hi[:1], grad=True)
+    # the ordered copy (cells.cu, scan_cells.cuh): rebuilt by this batch after the row changes above,
+    # then single-box estimates without retained contributions read it too
+    m.set_retain(False)
+    m.estimate(lo, hi, grad=True)
+    for k in (0, 3, len(lo) - 1):
+        m.estimate(lo[k:k + 1], hi[k:k + 1], grad=True)
+        m.estimate(lo[k:k + 1], hi[k:k + 1])
+    K.kde_set_profiling(m.handle, True)                 # cells-scan counters
+    m.estimate(lo, hi)
+    m.estimate(lo[:1], hi[:1])
+    K.kde_get_cells(m.handle, stats=True)
+    K.kde_set_profiling(m.handle, False)
     torch.cuda.synchronize()
     m.close()
 
