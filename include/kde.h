@@ -342,6 +342,20 @@ kde_status kde_reservoir_select(uint64_t seed, int64_t n_sample, int64_t n_seen,
 kde_status kde_insert_rows(kde_model *m, const float *rows, int64_t k, uint64_t seed, int64_t *n_seen,
                            double k_init, int64_t *n_written);
 
+/* kde_insert_rows_async -- kde_insert_rows whose device work (the H2D copy of the
+ * accepted rows, the column-range update and the scatter) is enqueued on `stream`
+ * (NULL: the model's stream) without waiting for it: the host decides the next
+ * chunk while the device still runs the previous queries (the host makes
+ * the reservoir decisions, only accepted rows cross PCIe).  The rows are copied
+ * into one of two pinned staging buffers before the call returns (the caller may
+ * reuse `rows`); a call waits only for the copy out of the buffer it reuses (two
+ * calls back).  Later work on `stream` sees the new rows in stream order; other
+ * calls of the library order themselves after it as after any _dev call.  Use one
+ * stream for a model's async inserts.  Single-GPU (world == 1).
+ * Errors: as kde_insert_rows; KDE_EINVAL for world > 1. */
+kde_status kde_insert_rows_async(kde_model *m, const float *rows, int64_t k, uint64_t seed, int64_t *n_seen,
+                                 double k_init, int64_t *n_written, void *stream);
+
 /* ---------------------------------------------------------------- device-resident feedback loop
  * Single-GPU (world == 1) device-pointer variants of the feedback calls, so a
  * whole streaming step (estimate -> karma -> bandwidth -> replacement) runs

@@ -38,7 +38,7 @@ ABI_SYMBOLS = (
     "kde_set_online_state", "kde_synchronize", "kde_count_in_box_dev", "kde_set_profiling", "kde_get_profile",
     "kde_karma_update_dev", "kde_online_update_dev", "kde_replace_points_dev", "kde_stream_step_dev",
     "kde_set_kernel", "kde_get_kernel", "kde_set_cull", "kde_get_cull", "kde_set_cells", "kde_get_cells",
-    "kde_reservoir_select", "kde_insert_rows",
+    "kde_reservoir_select", "kde_insert_rows", "kde_insert_rows_async",
     "kde_create_sharded_peer", "kde_peer_handle", "kde_peer_attach",
 )
 
@@ -121,6 +121,7 @@ def lib() -> ctypes.CDLL:
         "kde_replace_points": (ctypes.c_int, [P, P, P, i64, f64]),
         "kde_reservoir_select": (ctypes.c_int, [ctypes.c_uint64, i64, i64, i64, P]),
         "kde_insert_rows": (ctypes.c_int, [P, P, i64, ctypes.c_uint64, P, f64, P]),
+        "kde_insert_rows_async": (ctypes.c_int, [P, P, i64, ctypes.c_uint64, P, f64, P, P]),
         "kde_get_karma": (ctypes.c_int, [P, P]),
         "kde_set_karma": (ctypes.c_int, [P, P]),
         "kde_get_sample": (ctypes.c_int, [P, P]),
@@ -442,6 +443,16 @@ def kde_insert_rows(m, rows, seed: int, n_seen: int, k_init=0.0):
     nw = ctypes.c_int64()
     _check(lib().kde_insert_rows(m, _p(rows), rows.shape[0], seed, ctypes.byref(ns), float(k_init),
                                  ctypes.byref(nw)))
+    return ns.value, nw.value
+
+
+def kde_insert_rows_async(m, rows, seed: int, n_seen: int, k_init=0.0, stream=None):
+    """kde_insert_rows with the device work enqueued on `stream` (no wait); returns (new n_seen, slots written)."""
+    rows = _f32(rows)
+    ns = ctypes.c_int64(n_seen)
+    nw = ctypes.c_int64()
+    _check(lib().kde_insert_rows_async(m, _p(rows), rows.shape[0], seed, ctypes.byref(ns), float(k_init),
+                                       ctypes.byref(nw), _stream_ptr(stream)))
     return ns.value, nw.value
 
 

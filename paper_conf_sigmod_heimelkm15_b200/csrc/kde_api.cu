@@ -100,9 +100,12 @@ struct kde_model {
   double* scal = nullptr;            // [8] device scalars (true selectivity staging)
   void* pinned = nullptr;            // pinned host staging
   size_t pinned_cap = 0;
+  void* apin[2] = {nullptr, nullptr};  // kde_insert_rows_async: double-buffered pinned staging
+  size_t apin_cap[2] = {0, 0};
+  cudaEvent_t apin_ev[2] = {nullptr, nullptr};  // recorded after the H2D copy out of apin[b]
+  int apin_next = 0;
   void* rbuf = nullptr;              // replacement staging (idx + rows), grow-only
   size_t rbuf_cap = 0;
-  std::vector<int32_t> ins_last;     // kde_insert_rows: last arrival of a chunk per local slot (-1 = none)
   cudaEvent_t dev_done = nullptr;    // recorded on the caller's stream at the end of every _dev call
   bool dev_pending = false;          // some _dev call enqueued work on a stream other than m->stream
   void* kbuf = nullptr;              // sharded karma gather: counts + index lists, grow-only
@@ -232,6 +235,10 @@ static kde_status validate_loss(int32_t loss, double lambda) {
 static kde_status ensure_pinned(kde_model* m, size_t bytes) {
   if (m->pinned_cap >= bytes) return KDE_OK;
   if (m->pinned) cudaFreeHost(m->pinned);
+  for (int b = 0; b < 2; ++b) {
+    if (m->apin[b]) cudaFreeHost(m->apin[b]);
+    if (m->apin_ev[b]) cudaEventDestroy(m->apin_ev[b]);
+  }
   m->pinned = nullptr;
   m->pinned_cap = 0;
   size_t cap = std::max<size_t>(bytes, 1 << 16);
@@ -1262,7 +1269,8 @@ extern "C" kde_status kde_online_update(kde_model* m, const float* lo, const flo
 
 // Rows owned by this shard -> device staging (grow-only buffer, no per-call allocation) -> scatter.
 // idx are validated GLOBAL indices, unique; rows host row-major k x d.
-static kde_status replace_impl(kde_model* m, const int64_t* idx, const float* rows, int64_t k, double k_init) {
+static kde_status replace_impl(kde_model* m, const int64_t* idx, const float* rows, int64_t k, double k_init,
+                               cudaStream_t as = nullptr) {
   std::vector<int64_t> li;
   std::vector<float> lr;
   for (int64_t r = 0; r < k; ++r) {
@@ -1275,18 +1283,39 @@ static kde_status replace_impl(kde_model* m, const int64_t* idx, const float* ro
   const int64_t kl = (int64_t)li.size();
   if (kl > 0) {
     const size_t ib = sizeof(int64_t) * kl, rb = sizeof(float) * kl * m->d;
-    kde_status st = ensure_pinned(m, ib + rb);
+    cudaStream_t s = as ? as : m->stream;
+    void* pin = nullptr;
+    int b = 0;
+    if (as) {  // async: the staging buffer of two calls ago is free once its copy completed
+      b = m->apin_next;
+      m->apin_next ^= 1;
+      if (!m->apin_ev[b]) CU(cudaEventCreateWithFlags(&m->apin_ev[b], cudaEventDisableTiming));
+      CU(cudaEventSynchronize(m->apin_ev[b]));
+      if (m->apin_cap[b] < ib + rb) {
+        if (m->apin[b]) cudaFreeHost(m->apin[b]);
+        m->apin[b] = nullptr;
+        m->apin_cap[b] = 0;
+        const size_t cap = std::max<size_t>(ib + rb, (size_t)1 << 20);
+        if (cudaMallocHost(&m->apin[b], cap) != cudaSuccess) return fail(KDE_ENOMEM, "pinned staging of %zu bytes", cap);
+        m->apin_cap[b] = cap;
+      }
+      pin = m->apin[b];
+    } else {
+      kde_status st = ensure_pinned(m, ib + rb);
+      if (st != KDE_OK) return st;
+      pin = m->pinned;
+    }
+    kde_status st = ensure_bytes(&m->rbuf, &m->rbuf_cap, ib + rb);  // (a reallocation synchronises the device)
     if (st != KDE_OK) return st;
-    st = ensure_bytes(&m->rbuf, &m->rbuf_cap, ib + rb);
-    if (st != KDE_OK) return st;
-    memcpy(m->pinned, li.data(), ib);
-    memcpy((char*)m->pinned + ib, lr.data(), rb);
-    CU(cudaMemcpyAsync(m->rbuf, m->pinned, ib + rb, cudaMemcpyHostToDevice, m->stream));
-    CUL(launch_row_range((const float*)((char*)m->rbuf + ib), kl, m->d, m->range_enc, m->consts, m->stream));
+    memcpy(pin, li.data(), ib);
+    memcpy((char*)pin + ib, lr.data(), rb);
+    CU(cudaMemcpyAsync(m->rbuf, pin, ib + rb, cudaMemcpyHostToDevice, s));
+    if (as) CU(cudaEventRecord(m->apin_ev[b], s));
+    CUL(launch_row_range((const float*)((char*)m->rbuf + ib), kl, m->d, m->range_enc, m->consts, s));
     CUL(launch_scatter_rows((const int64_t*)m->rbuf, (const float*)((char*)m->rbuf + ib), kl, m->d, m->cols, m->ld,
-                           m->karma, k_init, m->stream));
+                           m->karma, k_init, s));
     ++m->sgen;
-    CU(cudaStreamSynchronize(m->stream));  // the pinned staging buffer is reused by the next call
+    if (!as) CU(cudaStreamSynchronize(m->stream));  // the pinned staging buffer is reused by the next call
   }
   ++m->gen;
   return KDE_OK;
@@ -1323,10 +1352,29 @@ extern "C" kde_status kde_reservoir_select(uint64_t seed, int64_t n_sample, int6
   return KDE_OK;
 }
 
+static kde_status insert_impl(kde_model* m, const float* rows, int64_t k, uint64_t seed, int64_t* n_seen,
+                              double k_init, int64_t* n_written, cudaStream_t as);
+
 extern "C" kde_status kde_insert_rows(kde_model* m, const float* rows, int64_t k, uint64_t seed, int64_t* n_seen,
                                       double k_init, int64_t* n_written) {
   KDE_RANGE();
   CHECK_MODEL(m);
+  return insert_impl(m, rows, k, seed, n_seen, k_init, n_written, nullptr);
+}
+
+extern "C" kde_status kde_insert_rows_async(kde_model* m, const float* rows, int64_t k, uint64_t seed,
+                                            int64_t* n_seen, double k_init, int64_t* n_written, void* stream) {
+  KDE_RANGE();
+  CHECK_MODEL(m);
+  if (m->world != 1) return fail(KDE_EINVAL, "kde_insert_rows_async is single-GPU (world == 1)");
+  cudaStream_t s = stream ? (cudaStream_t)stream : m->stream;
+  kde_status st = insert_impl(m, rows, k, seed, n_seen, k_init, n_written, s);
+  if (st != KDE_OK) return st;
+  return mark_dev(m, s);
+}
+
+static kde_status insert_impl(kde_model* m, const float* rows, int64_t k, uint64_t seed, int64_t* n_seen,
+                              double k_init, int64_t* n_written, cudaStream_t as) {
   if (k < 0 || !n_seen || *n_seen < 0 || *n_seen > INT64_MAX - k) return fail(KDE_EINVAL, "bad k / n_seen");
   if (k > 0 && !rows) return fail(KDE_EINVAL, "rows is NULL");
   if (!std::isfinite(k_init)) return fail(KDE_EINVAL, "k_init not finite");
@@ -1339,28 +1387,41 @@ extern "C" kde_status kde_insert_rows(kde_model* m, const float* rows, int64_t k
   std::vector<int64_t> slot((size_t)k);
   reservoir_slots(seed, m->n_global, *n_seen, k, slot.data());
   // several arrivals of one chunk may take the same slot: the last one wins (sequential semantics);
-  // only this shard's winners are transferred.  O(k) with a per-shard last-writer table.
-  if (m->ins_last.size() != (size_t)m->n) m->ins_last.assign((size_t)m->n, -1);
-  std::vector<int64_t> idx;
-  std::vector<float> sel;
+  // only this shard's winners are transferred.  O(k): the accepted arrivals of this shard
+  // (a small fraction of k once the stream is long) are walked newest first through an
+  // open-addressing set of their slots sized to that count, so the host touches a few cache-resident
+  // kilobytes instead of an n-entry table.
+  std::vector<int32_t> acc;  // accepted arrivals of this shard, in arrival order
   for (int64_t r = 0; r < k; ++r) {
     const int64_t i = slot[r] - m->row_offset;
-    if (slot[r] >= 0 && i >= 0 && i < m->n) m->ins_last[(size_t)i] = (int32_t)r;
+    if (slot[r] >= 0 && i >= 0 && i < m->n) acc.push_back((int32_t)r);
   }
-  for (int64_t r = 0; r < k; ++r) {
-    const int64_t i = slot[r] - m->row_offset;
-    if (slot[r] >= 0 && i >= 0 && i < m->n && m->ins_last[(size_t)i] == (int32_t)r) {
-      idx.push_back(slot[r]);
-      sel.insert(sel.end(), rows + r * m->d, rows + (r + 1) * m->d);
+  size_t cap = 16;
+  while (cap < 2 * acc.size()) cap <<= 1;
+  std::vector<int64_t> set(cap, -1);
+  std::vector<char> win(acc.size(), 0);
+  for (size_t a = acc.size(); a-- > 0;) {
+    const int64_t sl = slot[(size_t)acc[a]];
+    size_t hsh = (size_t)((uint64_t)sl * 0x9E3779B97F4A7C15ull >> 20) & (cap - 1);
+    while (set[hsh] >= 0 && set[hsh] != sl) hsh = (hsh + 1) & (cap - 1);
+    if (set[hsh] < 0) {  // newest arrival for this slot
+      set[hsh] = sl;
+      win[a] = 1;
     }
   }
-  for (int64_t r = 0; r < k; ++r) {  // reset the touched entries
-    const int64_t i = slot[r] - m->row_offset;
-    if (slot[r] >= 0 && i >= 0 && i < m->n) m->ins_last[(size_t)i] = -1;
-  }
+  std::vector<int64_t> idx;
+  std::vector<float> sel;
+  idx.reserve(acc.size());
+  sel.reserve(acc.size() * (size_t)m->d);
+  for (size_t a = 0; a < acc.size(); ++a)
+    if (win[a]) {
+      const int64_t r = acc[a];
+      idx.push_back(slot[(size_t)r]);
+      sel.insert(sel.end(), rows + r * m->d, rows + (r + 1) * m->d);
+    }
   DeviceGuard g(m->device);
-  WAIT_DEV(m);
-  kde_status st = idx.empty() ? KDE_OK : replace_impl(m, idx.data(), sel.data(), (int64_t)idx.size(), k_init);
+  if (!as) WAIT_DEV(m);
+  kde_status st = idx.empty() ? KDE_OK : replace_impl(m, idx.data(), sel.data(), (int64_t)idx.size(), k_init, as);
   if (st != KDE_OK) return st;
   ++m->gen;
   *n_seen += k;

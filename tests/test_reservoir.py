@@ -64,3 +64,43 @@ def test_insert_rows_follow_the_oracle_reservoir():
     est_o = oracle.estimate(expect, h, lo, hi)
     est = m.estimate(lo, hi)
     assert np.all(np.abs(est - est_o) <= 1e-7 + 1e-5 * np.abs(est_o))
+
+
+@pytest.mark.gpu
+def test_insert_rows_async_matches_sync_and_orders_with_stream_work():
+    """kde_insert_rows_async: the same slots and rows as the synchronous call (the host decision is
+    identical), the device work in stream order -- a _dev estimate enqueued right after it on the
+    same stream sees the inserted rows -- and the caller may overwrite its rows buffer at once."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    n, d, seed = 5000, 3, 99
+    S0 = synth.make_data("gauss", n, d, seed=70)
+    arrivals = synth.make_data("rect", 60000, d, seed=71)
+    ma, ms = K.KDEModel.create(S0), K.KDEModel.create(S0)
+    h = ma.bandwidth
+    s = torch.cuda.Stream()
+    lo, hi = synth.mixed_workload(S0, 8, seed=72)
+    dlo, dhi = torch.from_numpy(lo).cuda(), torch.from_numpy(hi).cuda()
+    est = torch.zeros(8, dtype=torch.float64, device="cuda")
+    na = nsy = n
+    outs = []
+    for k in (1000, 20000, 39000):
+        buf = arrivals[na - n:na - n + k].copy()
+        na2, nwa = K.kde_insert_rows_async(ma.handle, buf, seed, na, k_init=-2.0, stream=s)
+        buf[:] = np.nan                                   # the call copied the rows before returning
+        with torch.cuda.stream(s):
+            K.kde_estimate_batch_dev(ma.handle, dlo, dhi, est, None, stream=s)
+            outs.append(est.clone())                      # on s: after the estimate
+        nsy2, nws = ms.insert_rows(arrivals[nsy - n:nsy - n + k], seed, nsy, k_init=-2.0)
+        assert (na2, nwa) == (nsy2, nws)
+        na, nsy = na2, nsy2
+        s.synchronize()
+        cur = ms.sample
+        est_o = oracle.estimate(cur, h, lo, hi)
+        assert np.all(np.abs(outs[-1].cpu().numpy() - est_o) <= 1e-7 + 1e-5 * np.abs(est_o))
+    torch.cuda.synchronize()
+    assert np.array_equal(ma.sample, ms.sample)
+    assert np.array_equal(ma.karma, ms.karma)
+    ma.close()
+    ms.close()
