@@ -672,3 +672,40 @@ def test_reservoir_slots_follow_algorithm_r():
                 content[j] = a
         n_seen += k
     assert np.array_equal(content, oracle.reservoir_run(seed, Ns, n_seen))
+
+
+@pytest.mark.parametrize("d", [2, 5, 8])
+def test_r17_cell_skip_implies_r15_bound_for_every_point(d):
+    """DESIGN R17: the cells scan skips a (box, cell) pair when, from the cell's bounding box alone,
+    sum_j max(|c_cell - c_box| - hw_cell - hw_box, 0)^2 >= 64.5 in y' units (centres and half-widths
+    scaled by ap_j = sqrt(log2 e) / (sqrt2 h_j)).  Every point inside the bounding box is then at
+    least that far outside the box, so each one obeys the R15 bound on the fp64 oracle: p^(i) <= 2^-64
+    and |d p^(i) / d h_j| <= 2^-60 gconst_j.  Cells are Morton-ordered chunks of a clustered sample;
+    boxes anywhere, so both skipped and kept cells occur."""
+    import synth
+    n, C = 1 << 14, 256
+    S = synth.make_data("gauss", n, d, seed=1700 + d)
+    h = oracle.scott(S) * 0.5
+    ap = math.sqrt(math.log2(math.e)) / (math.sqrt(2.0) * h)
+    key = np.lexsort(tuple(np.floor((S[:, j] - S[:, j].min()) / (np.ptp(S[:, j]) + 1e-30) * 15.999).astype(int)
+                           for j in range(d)))
+    X = S[key].reshape(n // C, C, d).astype(np.float64)
+    mn, mx = X.min(1), X.max(1)
+    lo, hi = synth.random_boxes(S, 12, seed=1701 + d)
+    gconst = 1.0 / (math.sqrt(math.pi) * math.sqrt(math.log2(math.e)) * h)
+    skipped = 0
+    for b in range(len(lo)):
+        cb, hwb = 0.5 * (lo[b].astype(np.float64) + hi[b]) * ap, 0.5 * (hi[b].astype(np.float64) - lo[b]) * ap
+        cc, chw = 0.5 * (mn + mx) * ap, 0.5 * (mx - mn) * ap
+        o = np.maximum(np.abs(cc - cb) - chw - hwb, 0.0)
+        skip = (o ** 2).sum(axis=1) >= 64.5
+        for c in np.nonzero(skip)[0][:6]:
+            skipped += 1
+            pts = X[c].astype(np.float32)
+            assert np.all(_outside_sq(pts, h, lo[b], hi[b]) >= 64.0)
+            cv = oracle.contributions(pts, h, lo[b], hi[b])
+            assert np.all(cv <= 2.0 ** -64 * (1 + 1e-12))
+            for i in range(8):  # |d p^(i) / d h_j| of single points (grad_abs_scale of a one-point sample)
+                t = oracle.grad_abs_scale(pts[i:i + 1], h, lo[b], hi[b])[0]
+                assert np.all(t <= 2.0 ** -60 * gconst * (1 + 1e-9) + 1e-300)
+    assert skipped >= 6
