@@ -279,7 +279,11 @@ static kde_status ensure_bytes(void** p, size_t* cap, size_t bytes) {
   if (*p) cudaFree(*p);
   *p = nullptr;
   *cap = 0;
-  if (cudaMalloc(p, bytes) != cudaSuccess) return fail(KDE_ENOMEM, "device allocation of %zu bytes failed", bytes);
+  if (cudaMalloc(p, bytes) != cudaSuccess) {
+    *p = nullptr;
+    cudaGetLastError();  // not sticky: later launch checks must not see this error
+    return fail(KDE_ENOMEM, "device allocation of %zu bytes failed", bytes);
+  }
   *cap = bytes;
   return KDE_OK;
 }
@@ -333,9 +337,21 @@ static kde_status check_peer(kde_model* m) {
 static kde_status ensure_cells(kde_model* m, cudaStream_t s) {
   if (m->cells_gen == m->sgen && m->ccols) return KDE_OK;
   const int64_t ncells = (m->n + kCellPts - 1) / kCellPts;
-  if (!m->ccols) {
-    CU(cudaMalloc(&m->ccols, sizeof(float) * (size_t)m->d * m->ld));
-    CU(cudaMalloc(&m->cbb, sizeof(float) * 2 * (size_t)m->d * (size_t)(ncells > 0 ? ncells : 1)));
+  if (!m->ccols || !m->cbb) {  // both or neither (a failed allocation leaves neither behind)
+    float* cc = nullptr;
+    float* bb = nullptr;
+    cudaError_t e = cudaMalloc(&cc, sizeof(float) * (size_t)m->d * m->ld);
+    if (e == cudaSuccess) e = cudaMalloc(&bb, sizeof(float) * 2 * (size_t)m->d * (size_t)(ncells > 0 ? ncells : 1));
+    if (e != cudaSuccess) {
+      cudaFree(cc);
+      cudaGetLastError();  // clear the allocation error: the model stays usable without the copy
+      return fail(KDE_ENOMEM, "ordered copy of the sample: %s (kde_set_cells(m, 0) scans the sample itself)",
+                  cudaGetErrorString(e));
+    }
+    cudaFree(m->ccols);
+    cudaFree(m->cbb);
+    m->ccols = cc;
+    m->cbb = bb;
   }
   kde_status st = ensure_bytes(&m->cscratch, &m->cscratch_cap, cells_scratch_bytes(m->n));
   if (st != KDE_OK) return st;
