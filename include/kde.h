@@ -247,7 +247,9 @@ kde_status kde_get_cull(const kde_model *m, int32_t *on);
  * stay deterministic.  The copy (d x ld fp32, device) and its cell boxes are
  * built on the model's stream at the first such call and rebuilt after any call
  * that changes sample rows (replace / insert / streaming step); the sample, its
- * karma and retained contributions keep their original order.
+ * karma and retained contributions keep their original order.  When the device
+ * memory for the copy (d x ld fp32 + 16 B/point of build scratch) cannot be
+ * allocated, the call scans the sample itself and the setting turns off.
  * builds: number of index builds so far (may be NULL).
  * stats: NULL or 4 int64 -- while profiling is on (kde_set_profiling), the cells
  * scans' (box, cell) items, items evaluated without classification, points

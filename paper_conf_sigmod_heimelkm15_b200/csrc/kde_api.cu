@@ -435,7 +435,16 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
     a.q = q;
     a.consts = m->consts;
     static const bool env_cells = !(getenv("KDE_CELLS") && atoi(getenv("KDE_CELLS")) == 0);  // A/B switch
-    const bool cells = m->cull && m->cells_on && env_cells;
+    bool cells = m->cull && m->cells_on && env_cells;
+    if (cells) {  // build (or reuse) the ordered copy first; without the memory for it, scan the sample itself
+      const kde_status cst = ensure_cells(m, s);
+      if (cst == KDE_ENOMEM) {
+        m->cells_on = false;  // do not retry every call (kde_set_cells(m, 1) re-enables)
+        cells = false;
+      } else if (cst != KDE_OK) {
+        return cst;
+      }
+    }
     // unordered sample: culling for full 256-box CTAs only (measured: phased culling gains nothing)
     a.cull = (m->cull && (cells || batched_culls(q))) ? 1 : 0;
     a.split_len = 0;
@@ -450,8 +459,7 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
       a.perm = perm;
     }
     if (cells) {  // the ordered copy: cell-level skipping (scan_cells.cuh), any batch size
-      kde_status st = ensure_cells(m, s);
-      if (st != KDE_OK) return st;
+      kde_status st = KDE_OK;
       ScanCellsArgs c;
       c.ccols = m->ccols;
       c.ld = m->ld;
