@@ -20,7 +20,9 @@
  *    caller-allocated buffers; the caller keeps ownership of everything.
  *    Host-pointer calls are synchronous (they return after results landed).
  *  - "_dev" variants take DEVICE pointers (on the model's device) and a CUDA
- *    stream (cudaStream_t passed as void*, NULL = the model's own stream);
+ *    stream (cudaStream_t passed as void*, NULL = the model's own stream; the
+ *    legacy default stream is passed as cudaStreamLegacy -- the Python binding
+ *    maps torch's default stream, whose handle is 0, to it);
  *    they only enqueue work: results are valid once that stream reaches the
  *    end of the enqueued work.  Device buffers must stay alive until then.
  *    Every call that uses the model's own stream (all host-pointer calls,

@@ -199,10 +199,16 @@ def _bounds(d_lo, d_hi, d, q=None):
     return d_lo.numel() // d
 
 
+_CUDA_STREAM_LEGACY = 1  # cudaStreamLegacy: the C ABI reads a NULL stream as "the model's own stream"
+
+
 def _stream_ptr(stream):
+    """None -> NULL (the model's stream); a torch stream -> its handle, the default (legacy) stream,
+    whose handle is 0, as cudaStreamLegacy so that the work is ordered with torch's default stream."""
     if stream is None:
         return None
-    return ctypes.c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
+    h = stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+    return ctypes.c_void_p(h if h else _CUDA_STREAM_LEGACY)
 
 
 # ---------------------------------------------------------------- C-ABI mirrors

@@ -104,3 +104,25 @@ def test_insert_rows_async_matches_sync_and_orders_with_stream_work():
     assert np.array_equal(ma.karma, ms.karma)
     ma.close()
     ms.close()
+
+
+@pytest.mark.gpu
+def test_default_torch_stream_orders_dev_calls():
+    """torch's default stream (handle 0) reaches the library as cudaStreamLegacy, not as NULL (= the
+    model's own stream): a _dev estimate on it is ordered with torch work and CUDA events on it."""
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    S = synth.make_data("gauss", 1 << 18, 4, seed=80)
+    lo, hi = synth.mixed_workload(S, 300, seed=81)
+    m = K.KDEModel.create(S)
+    ref = m.estimate(lo, hi)
+    dlo, dhi = torch.from_numpy(lo).cuda(), torch.from_numpy(hi).cuda()
+    est = torch.full((300,), -1.0, dtype=torch.float64, device="cuda")
+    s0 = torch.cuda.current_stream()
+    assert s0.cuda_stream == 0
+    K.kde_estimate_batch_dev(m.handle, dlo, dhi, est, None, stream=s0)
+    got = est.clone()  # torch work on the default stream, after the estimate in stream order
+    torch.cuda.synchronize()
+    assert np.array_equal(got.cpu().numpy(), ref)
+    m.close()
