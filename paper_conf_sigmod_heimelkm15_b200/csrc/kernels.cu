@@ -266,6 +266,41 @@ __global__ void reduce_splits_kernel(const double* __restrict__ partials, int sp
   }
 }
 
+// The same sums for few outputs and many splits (small batches over the cells scan: q x na outputs,
+// thousands of splits): one warp per output, lane l sums the splits s = l (mod 32) in increasing order,
+// then a fixed butterfly -- deterministic, and ~32x shorter dependent load chains than a thread per
+// output.
+__global__ void reduce_splits_wide_kernel(const double* __restrict__ partials, int splits, int64_t q, int na,
+                                          double* __restrict__ sums, const PeerArgs* __restrict__ peer) {
+  const int64_t o = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;  // output = qi * na + k
+  const int lane = threadIdx.x & 31;
+  const uint64_t pe = peer ? peer_next_epoch(*peer) : 0;
+  if (o < q * na) {  // warp-uniform
+    const int64_t qi = o / na;
+    const int k = (int)(o % na);
+    double t = 0.0;
+    for (int s = lane; s < splits; s += 32) t += partials[((int64_t)s * na + k) * q + qi];
+#pragma unroll
+    for (int w = 16; w > 0; w >>= 1) t += __shfl_xor_sync(0xffffffffu, t, w);
+    if (lane == 0) {
+      if (peer)
+        peer_store(*peer, pe, qi * na + k, t);
+      else
+        sums[qi * na + k] = t;
+    }
+  }
+  if (!peer) return;
+  __shared__ bool last_s;
+  __threadfence_system();
+  __syncthreads();
+  if (threadIdx.x == 0) last_s = atomicAdd(peer->count + 2, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (last_s && threadIdx.x == 0) {
+    peer->count[2] = 0u;
+    peer_release(*peer, pe);
+  }
+}
+
 // gathered[r][q][na] summed in rank order -> sums[q][na]
 __global__ void combine_ranks_kernel(const double* __restrict__ gathered, int world, int64_t q, int na,
                                      double* __restrict__ sums) {
@@ -1020,7 +1055,12 @@ cudaError_t launch_set_consts(const double* h, int d, DevConsts* c, cudaStream_t
 }
 cudaError_t launch_reduce_splits(const double* partials, int splits, int64_t q, int na, double* sums,
                                  const PeerArgs* peer, cudaStream_t s) {
-  reduce_splits_kernel<<<(unsigned)((q + 255) / 256), 256, 0, s>>>(partials, splits, q, na, sums, peer);
+  if (splits >= 64 && q * na <= 16384) {  // few outputs, long chains: a warp per output
+    const int64_t threads = q * na * 32;
+    reduce_splits_wide_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, s>>>(partials, splits, q, na, sums, peer);
+  } else {
+    reduce_splits_kernel<<<(unsigned)((q + 255) / 256), 256, 0, s>>>(partials, splits, q, na, sums, peer);
+  }
   KDE_LAUNCH_CHECK();
 }
 cudaError_t launch_combine_ranks(const double* gathered, int world, int64_t q, int na, double* sums,

@@ -458,6 +458,9 @@ __device__ __forceinline__ void bulk_g2s_hint(void* dst, const void* src, uint32
       "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
       : "memory");
 }
+#ifndef KDE_TUNE_SUSPEND_NS
+#define KDE_TUNE_SUSPEND_NS 1000000
+#endif
 // as mbar_wait_parity, but a waiting warp is suspended (up to the hint, woken early by the phase
 // flip) instead of spinning on issue slots that the computing warps of the SM need
 __device__ __forceinline__ void mbar_wait_parity_suspend(uint64_t* bar, uint32_t parity) {
@@ -466,7 +469,7 @@ __device__ __forceinline__ void mbar_wait_parity_suspend(uint64_t* bar, uint32_t
       "KDE_WAITS_%=:\n\t"
       "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
       "@!p bra KDE_WAITS_%=;\n\t}" ::"r"(smem_u32(bar)),
-      "r"(parity), "r"(1000000u)
+      "r"(parity), "r"((uint32_t)KDE_TUNE_SUSPEND_NS)
       : "memory");
 }
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
