@@ -1055,7 +1055,7 @@ cudaError_t launch_set_consts(const double* h, int d, DevConsts* c, cudaStream_t
 }
 cudaError_t launch_reduce_splits(const double* partials, int splits, int64_t q, int na, double* sums,
                                  const PeerArgs* peer, cudaStream_t s) {
-  if (splits >= 64 && q * na <= 16384) {  // few outputs, long chains: a warp per output
+  if (splits >= 64 && q * na <= 65536) {  // few outputs, long chains: a warp per output
     const int64_t threads = q * na * 32;
     reduce_splits_wide_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, s>>>(partials, splits, q, na, sums, peer);
   } else {
