@@ -205,3 +205,17 @@ def test_cells_single_box_stale_index_falls_back():
         grad_ok(g1, g_o[k:k + 1], mabs[k:k + 1], h)
     assert K.kde_get_cells(m.handle)[1] == 1            # single-box calls do not rebuild
     m.close()
+
+
+def test_cells_rebuild_is_deterministic():
+    """A rebuild of an unchanged sample (one row rewritten with itself) reproduces the ordered copy
+    exactly: the stable radix sort and the fixed reduction order give bitwise-equal estimates."""
+    S = synth.make_data("gauss", 70001, 5, seed=120)
+    lo, hi = _boxes(S, 600, seed=121)
+    m = K.KDEModel.create(S)
+    e1, g1 = m.estimate(lo, hi, grad=True)
+    m.replace_points(np.array([123], np.int64), S[123:124].copy())
+    e2, g2 = m.estimate(lo, hi, grad=True)
+    assert K.kde_get_cells(m.handle)[1] == 2
+    assert np.array_equal(e1, e2) and np.array_equal(g1, g2)
+    m.close()
