@@ -480,9 +480,15 @@ cudaError_t launch_cells_t(bool grad, const ScanCellsArgs& a, int num_sms, int* 
 // (full / classified, compacted or masked) added into the warp's fp64 accumulator; the warps'
 // accumulators are summed in warp order, then the block reduction + deterministic last-block pass
 // of the other single-box scans (single_reduce_finalize).
-__host__ __device__ constexpr int cells_single_occ(int d) { return d <= 5 ? 2 : 1; }
+#ifndef KDE_TUNE_CELLS1_OCC
+#define KDE_TUNE_CELLS1_OCC(d) ((d) <= 5 ? 2 : 1)
+#endif
+#ifndef KDE_TUNE_CELLS1_NBUF
+#define KDE_TUNE_CELLS1_NBUF(d) ((d) <= 12 ? 2 : 1)
+#endif
+__host__ __device__ constexpr int cells_single_occ(int d) { return KDE_TUNE_CELLS1_OCC(d); }
 template <int D>
-__host__ __device__ constexpr int cells_single_nbuf() { return D <= 12 ? 2 : 1; }  // shared-memory budget
+__host__ __device__ constexpr int cells_single_nbuf() { return KDE_TUNE_CELLS1_NBUF(D); }  // shared-memory budget
 template <int D>
 __host__ __device__ constexpr size_t cells_single_smem() {
   return (size_t)(kCellsThreads / 32) * cells_single_nbuf<D>() * D * kCellPts * sizeof(float);  // per-warp buffers
