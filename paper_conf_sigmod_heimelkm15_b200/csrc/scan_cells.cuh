@@ -59,7 +59,7 @@ __host__ __device__ constexpr int cells_stages(int d) {
 // CTAs per resident slot (waves): several smaller CTAs per SM slot even out the work of the
 // strided cell sets and box groups (the hardware starts a new CTA where one finished)
 #ifndef KDE_TUNE_CELLS_WAVES
-#define KDE_TUNE_CELLS_WAVES 16
+#define KDE_TUNE_CELLS_WAVES 32
 #endif
 // point pairs per lane and iteration of a full item (kCellPts / 64 must be a multiple)
 #ifndef KDE_TUNE_CELLS_PU
