@@ -184,7 +184,8 @@ struct ScanCellsArgs {
   int64_t q;
   const DevConsts* consts;
   const int* perm;        // nullable: sorted position -> box index (probe order, cull_order.cu)
-  double* partials;       // [nsplit][1+d][q]
+  double* partials;       // [nsplit][1+d][qpad], row entry r = g * QG + slot (coalesced per CTA)
+  int64_t qpad;           // ngroups * QG (cells_layout)
   unsigned long long* stats;  // nullable (profiling): += items, full items, points evaluated, points classified
 };
 
@@ -197,6 +198,8 @@ cudaError_t launch_cells_build(const float* cols, int64_t ld, int64_t n, int d, 
 // host-side launchers (scan_inst_*.cu)
 cudaError_t launch_scan_cells(int d, bool grad, const ScanCellsArgs& a, int num_sms, int* splits_out, cudaStream_t s,
                               bool dry_run);
+// boxes per CTA group of the cells scan for dimension d (the partials' row layout, reduce_splits_mapped)
+int cells_group_boxes(int d);
 cudaError_t launch_scan_single(int d, bool grad, const ScanSingleArgs& a, int grid, cudaStream_t s);
 cudaError_t launch_scan_batched(int d, bool grad, const ScanBatchedArgs& a, int num_sms, int* splits_out,
                                 cudaStream_t s, bool dry_run);

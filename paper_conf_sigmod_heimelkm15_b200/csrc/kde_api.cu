@@ -482,7 +482,10 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
       }
       int splits = 1;
       CU(launch_scan_cells(d, grad, c, m->num_sms, &splits, s, true));
-      st = ensure_bytes((void**)&m->partials, &m->partials_cap, sizeof(double) * (size_t)splits * na * q);
+      const int qg = cells_group_boxes(d);
+      const int64_t ngroups = (q + qg - 1) / qg;
+      c.qpad = ngroups * qg;
+      st = ensure_bytes((void**)&m->partials, &m->partials_cap, sizeof(double) * (size_t)splits * na * c.qpad);
       if (st != KDE_OK) return st;
       c.partials = m->partials;
       cudaEvent_t e1 = nullptr, e2 = nullptr;
@@ -490,7 +493,7 @@ static kde_status scan_sums(kde_model* m, const float* d_lo, const float* d_hi, 
       if (st != KDE_OK) return st;
       CUL(launch_scan_cells(d, grad, c, m->num_sms, &splits, s, false));
       if (e2) CU(cudaEventRecord(e2, s));
-      CUL(launch_reduce_splits(m->partials, splits, q, na, d_sums, fused, s));
+      CUL(launch_reduce_splits_mapped(m->partials, splits, c.qpad, q, na, qg, (int)ngroups, c.perm, d_sums, fused, s));
       goto exchange;
     }
     int splits = 1;

@@ -301,6 +301,63 @@ __global__ void reduce_splits_wide_kernel(const double* __restrict__ partials, i
   }
 }
 
+// The cells scan's partials: row entry r = g * QG + i holds the box at probe-sorted position
+// pos = g + ngroups * i (perm[pos], or pos itself); entries with pos >= q are padding.
+__device__ __forceinline__ int64_t cells_entry_box(int64_t r, int qg, int ngroups, int64_t q, const int* perm) {
+  const int64_t g = r / qg, i = r % qg;
+  const int64_t pos = g + (int64_t)ngroups * i;
+  if (pos >= q) return -1;
+  return perm ? (int64_t)perm[pos] : pos;
+}
+__global__ void reduce_splits_mapped_kernel(const double* __restrict__ partials, int splits, int64_t qpad, int64_t q,
+                                            int na, int qg, int ngroups, const int* __restrict__ perm,
+                                            double* __restrict__ sums, const PeerArgs* __restrict__ peer, int wide) {
+  const uint64_t pe = peer ? peer_next_epoch(*peer) : 0;
+  if (wide) {  // a warp per (entry, component): lanes over splits, fixed butterfly
+    const int64_t o = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (o < qpad * na) {
+      const int64_t r = o / na;
+      const int k = (int)(o % na);
+      const int64_t qi = cells_entry_box(r, qg, ngroups, q, perm);
+      if (qi >= 0) {  // warp-uniform
+        double t = 0.0;
+        for (int s = lane; s < splits; s += 32) t += partials[((int64_t)s * na + k) * qpad + r];
+#pragma unroll
+        for (int w = 16; w > 0; w >>= 1) t += __shfl_xor_sync(0xffffffffu, t, w);
+        if (lane == 0) {
+          if (peer)
+            peer_store(*peer, pe, qi * na + k, t);
+          else
+            sums[qi * na + k] = t;
+        }
+      }
+    }
+  } else {  // a thread per entry (coalesced across entries)
+    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t qi = r < qpad ? cells_entry_box(r, qg, ngroups, q, perm) : -1;
+    if (qi >= 0)
+      for (int k = 0; k < na; ++k) {
+        double t = 0.0;
+        for (int s = 0; s < splits; ++s) t += partials[((int64_t)s * na + k) * qpad + r];
+        if (peer)
+          peer_store(*peer, pe, qi * na + k, t);
+        else
+          sums[qi * na + k] = t;
+      }
+  }
+  if (!peer) return;
+  __shared__ bool last_s;
+  __threadfence_system();
+  __syncthreads();
+  if (threadIdx.x == 0) last_s = atomicAdd(peer->count + 2, 1u) == gridDim.x - 1;
+  __syncthreads();
+  if (last_s && threadIdx.x == 0) {
+    peer->count[2] = 0u;
+    peer_release(*peer, pe);
+  }
+}
+
 // gathered[r][q][na] summed in rank order -> sums[q][na]
 __global__ void combine_ranks_kernel(const double* __restrict__ gathered, int world, int64_t q, int na,
                                      double* __restrict__ sums) {
@@ -1061,6 +1118,15 @@ cudaError_t launch_reduce_splits(const double* partials, int splits, int64_t q, 
   } else {
     reduce_splits_kernel<<<(unsigned)((q + 255) / 256), 256, 0, s>>>(partials, splits, q, na, sums, peer);
   }
+  KDE_LAUNCH_CHECK();
+}
+cudaError_t launch_reduce_splits_mapped(const double* partials, int splits, int64_t qpad, int64_t q, int na, int qg,
+                                        int ngroups, const int* perm, double* sums, const PeerArgs* peer,
+                                        cudaStream_t s) {
+  const int wide = (splits >= 64 && qpad * na <= 65536) ? 1 : 0;
+  const int64_t threads = wide ? qpad * na * 32 : qpad;
+  reduce_splits_mapped_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, s>>>(partials, splits, qpad, q, na, qg,
+                                                                                ngroups, perm, sums, peer, wide);
   KDE_LAUNCH_CHECK();
 }
 cudaError_t launch_combine_ranks(const double* gathered, int world, int64_t q, int na, double* sums,

@@ -62,6 +62,10 @@ cudaError_t launch_cull_order(const float* cols, int64_t ld, int64_t n, int d, c
 // exchange) <- the fixed-order sum over splits
 cudaError_t launch_reduce_splits(const double* partials, int splits, int64_t q, int na, double* sums,
                                  const PeerArgs* peer, cudaStream_t s);
+// the cells scan's partials (row entry g * QG + slot, see scan_cells.cuh) -> sums[box][na], split order
+cudaError_t launch_reduce_splits_mapped(const double* partials, int splits, int64_t qpad, int64_t q, int na, int qg,
+                                        int ngroups, const int* perm, double* sums, const PeerArgs* peer,
+                                        cudaStream_t s);
 cudaError_t launch_combine_ranks(const double* gathered, int world, int64_t q, int na, double* sums,
                                  cudaStream_t s);
 cudaError_t launch_finalize(const double* sums, int64_t q, int d, int na, const DevConsts* c, double n_global,

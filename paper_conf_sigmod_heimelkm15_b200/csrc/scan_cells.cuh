@@ -278,8 +278,10 @@ __global__ void __launch_bounds__(kCellsThreads, CellsMinB<D>::value) scan_cells
   unsigned* flags = reinterpret_cast<unsigned*>(cnt + S);                    // [QG]
   unsigned char* lists = reinterpret_cast<unsigned char*>(flags + QG);       // [warps][kCellPts]
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int split = blockIdx.x, nsplit = gridDim.x;
-  const int g = blockIdx.y, ngroups = gridDim.y;
+  // x = box group, y = cell set: the groups of one cell set are launched together and share its
+  // tiles through L2 (the sample is read from HBM about once, not once per group)
+  const int g = blockIdx.x, ngroups = gridDim.x;
+  const int split = blockIdx.y, nsplit = gridDim.y;
 
   float ap[D];
 #pragma unroll
@@ -428,12 +430,14 @@ __global__ void __launch_bounds__(kCellsThreads, CellsMinB<D>::value) scan_cells
   }
   if (a.stats && lane < 4) atomicAdd(a.stats + lane, wstats[4 * warp + lane]);  // per-warp totals
   __syncthreads();
+  // partials row entry g * QG + slot: consecutive threads write consecutive doubles (the reduction
+  // maps entries back to boxes, reduce_splits_mapped)
   for (int i = tid; i < QG; i += kCellsThreads) {
     const int64_t pos = (int64_t)g + (int64_t)ngroups * i;
     if (pos >= a.q) continue;
-    const int64_t qi = a.perm ? a.perm[pos] : pos;
 #pragma unroll
-    for (int k = 0; k < NA; ++k) a.partials[((int64_t)split * NA + k) * a.q + qi] = acc[(size_t)i * NA + k];
+    for (int k = 0; k < NA; ++k)
+      a.partials[((int64_t)split * NA + k) * a.qpad + (int64_t)g * QG + i] = acc[(size_t)i * NA + k];
   }
 }
 
@@ -461,13 +465,14 @@ cudaError_t launch_cells_t(bool grad, const ScanCellsArgs& a, int num_sms, int* 
                            bool dry_run) {
   constexpr int QG = cells_qg<D>();
   const int64_t ngroups = (a.q + QG - 1) / QG;
-  if (ngroups > 65535) return cudaErrorInvalidValue;
+  if (ngroups > 0x7fffffff) return cudaErrorInvalidValue;
   int64_t nsplit = ((int64_t)num_sms * CellsMinB<D>::value * KDE_TUNE_CELLS_WAVES + ngroups - 1) / ngroups;
   if (nsplit > a.ncells) nsplit = a.ncells;
   if (nsplit < 1) nsplit = 1;
+  if (nsplit > 65535) nsplit = 65535;  // grid y
   if (splits_out) *splits_out = (int)nsplit;
   if (dry_run) return cudaSuccess;
-  dim3 grid((unsigned)nsplit, (unsigned)ngroups);
+  dim3 grid((unsigned)ngroups, (unsigned)nsplit);
   return grad ? launch_cells_tg<D, true>(a, grid, s) : launch_cells_tg<D, false>(a, grid, s);
 }
 

@@ -42,6 +42,15 @@ cudaError_t launch_scan_cells(int d, bool grad, const ScanCellsArgs& a, int num_
   return cudaErrorInvalidValue;
 }
 
+int cells_group_boxes(int d) {
+  switch (d) {
+#define X(D) case D: return cells_qg<D>();
+    KDE_CASES(X)
+#undef X
+  }
+  return 0;
+}
+
 // the batched scan culls (and wants the probe order) when a CTA holds 256 boxes (one thread per box)
 bool batched_culls(int64_t q) { return batched_qb(q) == kBatchedThreads; }
 
